@@ -1,0 +1,87 @@
+"""In-tree build of the native libraries (sm_100a only).
+
+libagnn.so    — the product: C-ABI (include/agnn.h) + hand-written CUDA kernels.
+libagnngen.so — seeded input generators (host + device), shared test/bench infra.
+
+Both are built with explicit ``nvcc -gencode arch=compute_100a,code=sm_100a``;
+the .so files land next to their sources so they travel with gpurun snapshots.
+"""
+from __future__ import annotations
+
+import glob
+import os
+import subprocess
+import sys
+
+PKG = os.path.dirname(os.path.abspath(__file__))
+ROOT = os.path.dirname(PKG)
+INCLUDE = os.path.join(ROOT, "include")
+NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
+ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
+
+GEN_DIR = os.path.join(PKG, "gen")
+GEN_SO = os.path.join(GEN_DIR, "libagnngen.so")
+CSRC = os.path.join(PKG, "csrc")
+AGNN_SO = os.path.join(PKG, "libagnn.so")
+
+
+def _nccl_dirs():
+    try:
+        import nvidia.nccl as nn  # the NCCL torch itself loads (2.28.x)
+        base = os.path.dirname(nn.__file__) if nn.__file__ else list(nn.__path__)[0]
+        inc, libd = os.path.join(base, "include"), os.path.join(base, "lib")
+        if os.path.exists(os.path.join(inc, "nccl.h")):
+            return inc, libd
+    except Exception:
+        pass
+    return "/usr/include", "/usr/lib/x86_64-linux-gnu"
+
+
+def _stale(target, sources):
+    if not os.path.exists(target):
+        return True
+    t = os.path.getmtime(target)
+    return any(os.path.getmtime(s) > t for s in sources)
+
+
+def _run(cmd):
+    print("[build]", " ".join(cmd), file=sys.stderr)
+    subprocess.check_call(cmd)
+
+
+def build_gen(force: bool = False) -> str:
+    srcs = [os.path.join(GEN_DIR, "gen.cu"), os.path.join(GEN_DIR, "agnn_gen.h")]
+    if force or _stale(GEN_SO, srcs):
+        _run([NVCC, *ARCH, "-O3", "-std=c++17", "-lineinfo", "-shared", "-Xcompiler", "-fPIC,-fopenmp",
+              "-o", GEN_SO, srcs[0], "-lgomp"])
+    return GEN_SO
+
+
+def agnn_sources():
+    return sorted(glob.glob(os.path.join(CSRC, "*.cu")))
+
+
+def agnn_deps():
+    return agnn_sources() + sorted(glob.glob(os.path.join(CSRC, "*.cuh"))) + \
+        sorted(glob.glob(os.path.join(INCLUDE, "*.h")))
+
+
+def build_agnn(force: bool = False, verbose_ptxas: bool = False) -> str:
+    if force or _stale(AGNN_SO, agnn_deps()):
+        nccl_inc, nccl_lib = _nccl_dirs()
+        cmd = [NVCC, *ARCH, "-O3", "-std=c++17", "-lineinfo", "-shared", "-Xcompiler", "-fPIC",
+               "--expt-relaxed-constexpr", "-I", INCLUDE, "-I", CSRC, "-I", nccl_inc,
+               "-o", AGNN_SO, *agnn_sources(), "-L", nccl_lib, "-l:libnccl.so.2",
+               "-Xlinker", "-rpath," + nccl_lib, "-lcuda"]
+        if verbose_ptxas:
+            cmd.insert(1, "-Xptxas=-v")
+        _run(cmd)
+    return AGNN_SO
+
+
+def build_all(force: bool = False):
+    return build_gen(force), build_agnn(force)
+
+
+if __name__ == "__main__":
+    build_all(force="--force" in sys.argv)
