@@ -1,0 +1,366 @@
+#!/usr/bin/env python
+"""bench.py — GAT/AGNN/VA layer fwd+bwd edges/s on B200 (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C5] [--impl ours|reference]
+
+A "step" is one pass of the whole hot path over the synthetic workload: the
+L-layer forward (projection GEMM, fused SDDMM -> edge softmax -> SpMM, sigma)
+followed by the L-layer backward (prologue, fused recompute backward, weight-
+gradient and dH GEMMs, and at N > 1 the NCCL exchanges).  edges/s = L * m / T
+(m = nnz after preprocessing, global).
+
+Default workload: C5 = GAT, 4 heads, k = 128, Kronecker n = 2^24 / ~1.0e9
+edges, 1 layer — the north_star target (fits one B200).  Inputs (8.6 GB per
+feature matrix) are far larger than the 126 MB L2, so no explicit flush.
+
+Multi-GPU: launched by torch.distributed.run, one rank per GPU; 1D row blocks,
+NCCL all-gather of P / G and all-reduce of dW, da inside libagnn.so; rank 0
+prints the JSON line; time = max over ranks of CUDA-event time.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "GAT layer fwd+bwd edges/s"
+UNIT = "edges/s"
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=10)
+    p.add_argument("--warmup", type=int, default=3)
+    p.add_argument("--config", default="C5")
+    p.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--cpu-sample-scale", type=int, default=17,
+                   help="log2 n of the bounded oracle sample (same recipe as the workload)")
+    return p.parse_args()
+
+
+# ----------------------------------------------------------------------------- clocks
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index):
+        self.gpu, self.rows, self.proc = gpu_index, [], None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.Q}",
+                 "--format=csv,noheader,nounits", "-lms", "200"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except FileNotFoundError:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def stop(self):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+        sms = [float(r[0]) for r in self.rows if r and r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if len(r) > 1 and r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = set()
+        for r in self.rows:
+            for i, nm in enumerate(names):
+                if len(r) > 4 + i and r[4 + i].lower().startswith("active"):
+                    reasons.add(nm)
+        sms.sort()
+        return {"sm_mhz": sms[len(sms) // 2] if sms else None,
+                "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sms)}
+
+
+def measured_peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        return {}
+
+
+# ----------------------------------------------------------------------------- CPU oracle
+def oracle_sample(w, scale):
+    """A bounded sample of the same workload recipe (Kronecker at 2^scale, same ef/k/heads)."""
+    from paper_conf_sc_bestarglzcgssci23_b200 import gen
+    ef = max(1, w.n_samples // w.n)
+    n = 1 << scale if w.graph != "er" else min(w.n, 1 << scale)
+    return gen.Workload(f"{w.name}-sample-2^{scale}", w.model, w.graph, scale, n, ef * n, w.k,
+                        w.heads, w.layers, w.seed, w.act, w.slope, w.beta, w.eps)
+
+
+def time_oracle(w, scale, reps=1):
+    sys.path.insert(0, os.path.join(ROOT, "oracle"))
+    sys.path.insert(0, os.path.join(ROOT, "tests"))
+    import oracle
+    import parity_utils as pu
+    ws = oracle_sample(w, scale)
+    src, dst = ws.host_edges()
+    rp, ci = oracle.csr_build(ws.n, src, dst)
+    H, Ws, As, R = ws.host_inputs()
+    times = []
+    for _ in range(reps):
+        t0 = time.perf_counter()
+        pu.oracle_step(ws, rp, ci, H, Ws, As, R)
+        times.append(time.perf_counter() - t0)
+    cores = len(os.sched_getaffinity(0))
+    return ws, len(ci), times, cores
+
+
+def cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return "unknown"
+
+
+def run_reference(args):
+    """--impl reference: the FP64 oracle (this tier's reference arm) on host cores."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    from paper_conf_sc_bestarglzcgssci23_b200 import gen
+    w = gen.CONFIGS[args.config]
+    ws = oracle_sample(w, args.cpu_sample_scale)
+    sys.path.insert(0, os.path.join(ROOT, "oracle"))
+    sys.path.insert(0, os.path.join(ROOT, "tests"))
+    import oracle
+    import parity_utils as pu
+    src, dst = ws.host_edges()
+    rp, ci = oracle.csr_build(ws.n, src, dst)
+    H, Ws, As, R = ws.host_inputs()
+    for _ in range(args.warmup):
+        pu.oracle_step(ws, rp, ci, H, Ws, As, R)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        pu.oracle_step(ws, rp, ci, H, Ws, As, R)
+    T = (time.perf_counter() - t0) / args.steps
+    m = len(ci)
+    val = ws.layers * m / T
+    cores = len(os.sched_getaffinity(0))
+    sample = (f"oracle (C, FP64, OpenMP) on {gen.describe(ws)}, m={m} — a bounded sample of "
+              f"{args.config} ({gen.describe(w)})")
+    line = {"impl": "reference", "metric": METRIC, "value": val, "unit": UNIT, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": T * 1e3,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic",
+            "config": {"workload": args.config, "model": w.model, "graph": w.graph,
+                       "n": ws.n, "edges": m, "k": w.k, "heads": w.heads, "layers": w.layers,
+                       "sample_of": gen.describe(w)},
+            "cpu_baseline": {"value": val, "unit": UNIT, "cores": cores, "kind": "oracle",
+                             "sample": sample, "cpu": cpu_model()},
+            "e2e": {"value": val, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+# ----------------------------------------------------------------------------- ours
+def algorithmic_bytes(w, m, n):
+    """Bytes the dominant kernel must move per launch.
+
+    GAT backward sparse kernel, per stored edge: 4 B column index + the gathered
+    rows P_i and G_i (2 k' f) + the neighbour record {s,m,1/l,delta} (16 h) and
+    t_i (4 h); per row: P_j, G_j read, dP_j written (3 k' f) + own record/t
+    (20 h) + row_ptr (8 B).  AGNN/VA backward: per edge 4 + 2 k f (+16 AGNN
+    record); per row H_j, M_j read, dH_j written (3 k f) (+16) + 8.
+    """
+    f = 4
+    if w.model == "gat":
+        per_edge = 4 + 2 * w.k * f + 20 * w.heads
+        per_row = 3 * w.k * f + 20 * w.heads + 8
+    else:
+        rec = 16 if w.model == "agnn" else 0
+        per_edge = 4 + 2 * w.k * f + rec
+        per_row = 3 * w.k * f + rec + 8
+    return per_edge * m + per_row * n, per_edge, per_row
+
+
+DOMINANT = {"gat": "gat_bwd_kernel", "agnn": "av_bwd_kernel", "va": "av_bwd_kernel"}
+
+
+def run_ours(args):
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_sc_bestarglzcgssci23_b200 import agnn, gen, runner
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if not torch.cuda.is_available():
+        raise RuntimeError("bench.py needs CUDA GPUs (no CPU fallback)")
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        dist.init_process_group("nccl", device_id=dev)
+    w = gen.CONFIGS[args.config]
+    agnn.lib()
+    uid = None
+    if world > 1:
+        obj = [agnn.nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        uid = obj[0]
+
+    t_setup = time.perf_counter()
+    st = runner.Stack(w, dev, rank=rank, world=world, nccl_uid=uid)
+    torch.cuda.synchronize()
+    setup_s = time.perf_counter() - t_setup
+    m, n = st.graph.nnz, w.n
+    stream = st.stream
+
+    def barrier():
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    for _ in range(args.warmup):
+        st.step()
+    barrier()
+
+    # ---- device-resident timed region -----------------------------------------
+    clocks = ClockSampler(local)
+    clocks.start()
+    agnn.profile_enable(True)
+    agnn.profile_reset()
+    launches0 = agnn.launch_count()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    barrier()
+    e0.record(stream)
+    for _ in range(args.steps):
+        st.step()
+    e1.record(stream)
+    barrier()
+    launches = agnn.launch_count() - launches0
+    prof = agnn.profile_report()
+    agnn.profile_enable(False)
+    ck = clocks.stop()
+    ms = e0.elapsed_time(e1)
+    if world > 1:
+        t = torch.tensor([ms], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    T = ms / 1e3 / args.steps
+    value = w.layers * m / T
+
+    # ---- roofline of the dominant kernel ----------------------------------------
+    peaks = measured_peaks()
+    hbm = peaks.get("hbm_gbs")
+    peak_src = "measured (MEASURED_PEAKS.json hbm_gbs)" if hbm else "fallback (B200_PROFILING.md)"
+    hbm = hbm or 6650.0
+    dom = DOMINANT[w.model]
+    cnt, tot = prof.get(dom, (0, 0.0))
+    alg, per_edge, per_row = algorithmic_bytes(w, st.nnz_local, st.n_local)
+    dom_ms = tot / cnt if cnt else None
+    achieved = (alg * w.layers / (dom_ms / 1e3) / 1e9 / w.layers) if dom_ms else None
+    # one launch per layer per step: alg bytes per launch over the mean launch time
+    achieved = (alg / (dom_ms / 1e3) / 1e9) if dom_ms else None
+    step_ms_prof = sum(v[1] for v in prof.values()) / args.steps
+    roof = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": hbm, "unit": "GB/s",
+            "frac": (achieved / hbm) if achieved else None, "traffic": None,
+            "peak_source": peak_src, "algorithmic_bytes_per_launch": alg,
+            "bytes_per_edge": per_edge, "bytes_per_row": per_row,
+            "launch_ms": dom_ms, "share_of_step": (tot / args.steps / step_ms_prof)
+            if step_ms_prof else None}
+    kernels = {k: {"launches": v[0], "ms_per_step": v[1] / args.steps} for k, v in prof.items()}
+
+    # ---- end-to-end through the C ABI with host buffers -------------------------
+    e2e = None
+    if not args.no_e2e:
+        nl, k = st.n_local, w.k
+        h_H = torch.empty((nl, k), dtype=torch.float32, pin_memory=True)
+        h_R = torch.empty((nl, k), dtype=torch.float32, pin_memory=True)
+        h_dH = torch.empty((nl, k), dtype=torch.float32, pin_memory=True)
+        h_dW = [torch.empty_like(x, device="cpu").pin_memory() for x in st.dW]
+        h_da = [torch.empty_like(x, device="cpu").pin_memory() for x in st.da if x is not None]
+        h_H.copy_(st.H[0].cpu())
+        h_R.copy_(st.dH[w.layers].cpu())
+        barrier()
+        e2, e3 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e2.record(stream)
+        for _ in range(args.steps):
+            st.H[0].copy_(h_H, non_blocking=True)
+            st.dH[w.layers].copy_(h_R, non_blocking=True)
+            st.step()
+            h_dH.copy_(st.dH[0], non_blocking=True)
+            for hw_, dw_ in zip(h_dW, st.dW):
+                hw_.copy_(dw_, non_blocking=True)
+            for ha_, da_ in zip(h_da, [x for x in st.da if x is not None]):
+                ha_.copy_(da_, non_blocking=True)
+        e3.record(stream)
+        barrier()
+        ms2 = e2.elapsed_time(e3)
+        if world > 1:
+            t = torch.tensor([ms2], device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ms2 = float(t.item())
+        T2 = ms2 / 1e3 / args.steps
+        h2d = 2 * nl * k * 4
+        d2h = nl * k * 4 + sum(x.numel() * 4 for x in h_dW) + sum(x.numel() * 4 for x in h_da)
+        e2e = {"value": w.layers * m / T2, "unit": UNIT, "h2d_bytes_per_step": h2d * world,
+               "d2h_bytes_per_step": d2h * world, "ms_per_step": T2 * 1e3,
+               "api": "agnn_forward/agnn_backward via paper_conf_sc_bestarglzcgssci23_b200.runner"}
+
+    # ---- CPU oracle baseline (rank 0, N = 1 only) ------------------------------
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        ws_, m_s, times, cores = time_oracle(w, args.cpu_sample_scale)
+        t_med = sorted(times)[len(times) // 2]
+        cpu = {"value": ws_.layers * m_s / t_med, "unit": UNIT, "cores": cores, "kind": "oracle",
+               "sample": f"FP64 C oracle fwd+bwd on {gen.describe(ws_)} (m={m_s}), same recipe "
+                         f"as {args.config} at 2^{args.cpu_sample_scale} vertices; "
+                         f"{t_med:.1f} s", "cpu": cpu_model()}
+
+    if rank == 0:
+        line = {"metric": METRIC if w.model == "gat" else f"{w.model.upper()} layer fwd+bwd edges/s",
+                "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": T * 1e3, "higher_is_better": True,
+                "scaling": "weak" if world == 1 else "strong", "vs_baseline": None,
+                "dtype": "f32", "data": "synthetic",
+                "config": {"workload": args.config, "model": w.model, "graph": w.graph,
+                           "n": n, "edges": m, "k": w.k, "heads": w.heads, "layers": w.layers,
+                           "parallelism": f"1d-rowblock{world}", "l2_flush": "inputs > L2 (126 MB)",
+                           "setup_s": setup_s},
+                "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
+                "clocks": ck, "kernels": kernels}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,198 @@
+/*
+ * agnn.h — C ABI of the B200-native A-GNN layer hot path (libagnn.so).
+ *
+ * One layer of an attentional GNN in the paper's global tensor formulation
+ * (Besta et al., SC'23, Eq. 1):
+ *     H^{l+1} = sigma(Z^l),  Z^l = (Phi o (+))(Psi(A, H^l), H^l)
+ * for the three models of PAPER.md:169-177:
+ *     AGNN_VA   Psi = A (.) (H H^T)                         (Eq. 7 at :262)
+ *     AGNN_AGNN Psi = sm(beta A (.) (H_x (/) n n^T))        (reading A8)
+ *     AGNN_GAT  Psi = sm(A (.) LReLU(C)), C = s 1^T + 1 t^T
+ * with the graph softmax sm over the stored entries of each row
+ * and the backward pass of PAPER.md:221-298
+ * (Eq. 2-13; readings A11/A12 in DESIGN.md §2).  The dense n x n virtual
+ * matrices are never materialised.
+ *
+ * Conventions
+ *  - Every pointer argument of agnn_forward / agnn_backward / agnn_debug_*
+ *    is a DEVICE pointer unless marked "host".  Floating data are fp32,
+ *    row-major, 16-byte aligned, rows contiguous (leading dimension = width).
+ *  - H_in: [n_local x k_in]; W: [k_in x k_out]; GAT a: [heads][2d] with
+ *    a1 = a[h][0:d] (centre vertex = row i), a2 = a[h][d:2d] (neighbour =
+ *    column j), d = k_out/heads; H_out, dH_out: [n_local x k_out];
+ *    dH_in: [n_local x k_in]; dW: [k_in x k_out]; da: [heads][2d].
+ *  - The CSR lists, for every local row i, the vertices i aggregates from
+ *    (N^(i)), by GLOBAL column id, strictly ascending.
+ *    The library computes on exactly this pattern: it never adds self-loops
+ *    or symmetrises (use agnn_csr_build for the paper's preprocessing).
+ *    The backward's single-pass kernel requires a symmetric pattern
+ *    (AGNN_CSR_SYMMETRIC, "for undirected graphs A = A^T");
+ *    unsymmetric patterns are rejected with AGNN_EUNSUPPORTED by agnn_backward.
+ *
+ * Ownership
+ *  - The caller owns every feature, weight, gradient, `saved` and
+ *    `workspace` buffer (sizes from agnn_saved_bytes / agnn_workspace_bytes).
+ *    The plan owns only derived metadata (work lists, NCCL communicator);
+ *    the model owns nothing on the device.
+ *  - agnn_forward / agnn_backward never allocate, never synchronise the
+ *    host and only enqueue work on `stream`: they are CUDA-graph capturable
+ *    when world == 1.
+ *
+ * Errors
+ *  - Every call returns an agnn_status; C++ exceptions never cross the ABI.
+ *    agnn_last_error() returns a thread-local message for the last failure.
+ *  - Descriptor / argument checks on the host return AGNN_EINVAL (e.g.
+ *    k_out % heads != 0, unsupported widths, misaligned pointers).
+ *  - CSR content errors (non-monotone row_ptr, column out of range,
+ *    unsorted or duplicate columns) are detected on the device and surface
+ *    ONLY from agnn_plan_create (the one call that synchronises).
+ *  - CUDA launch failures return AGNN_ECUDA, NCCL failures AGNN_ENCCL.
+ *  - With world > 1 every rank must call forward/backward in the same order.
+ */
+#ifndef AGNN_H
+#define AGNN_H
+
+#include <stddef.h>
+#include <stdint.h>
+#include <cuda_runtime.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  AGNN_OK = 0,
+  AGNN_EINVAL = 1,
+  AGNN_ECUDA = 2,
+  AGNN_ENCCL = 3,
+  AGNN_ENOMEM = 4,
+  AGNN_EUNSUPPORTED = 5,
+  AGNN_ESTATE = 6
+} agnn_status;
+
+typedef enum { AGNN_VA = 0, AGNN_AGNN = 1, AGNN_GAT = 2 } agnn_kind;
+
+/* sigma; reading A6: ReLU with sigma'(0) = 0, ELU(alpha = 1) */
+typedef enum { AGNN_ACT_NONE = 0, AGNN_ACT_RELU = 1, AGNN_ACT_ELU = 2 } agnn_act;
+
+/* arithmetic of the dense projection; sparse passes are always fp32 */
+typedef enum {
+  AGNN_PREC_FP32 = 0,    /* fp32 FFMA, or 3xTF32 on tcgen05 (fp32-accurate)  */
+  AGNN_PREC_TF32X3 = 1   /* force the tcgen05 3xTF32 path                      */
+} agnn_prec;
+
+enum { AGNN_CSR_SYMMETRIC = 1u };
+
+typedef struct {
+  int64_t n;               /* global vertex count                                  */
+  int64_t row_begin;       /* this rank owns global rows [row_begin, row_end)      */
+  int64_t row_end;
+  const int64_t* row_ptr;  /* device, [row_end - row_begin + 1], row_ptr[0] == 0   */
+  const int32_t* col_idx;  /* device, [row_ptr[n_local]], global ids, ascending    */
+  uint32_t flags;          /* AGNN_CSR_SYMMETRIC                                   */
+} agnn_csr;
+
+typedef struct {
+  int rank, world;
+  const void* nccl_unique_id; /* host, 128 bytes (ncclUniqueId); NULL iff world == 1 */
+  const int64_t* bounds;      /* host, [world + 1] row bounds (agnn_partition)      */
+} agnn_dist;
+
+typedef struct {
+  agnn_kind kind;
+  int k_in, k_out, heads;  /* GAT: heads >= 1, k_out % heads == 0; AGNN/VA: heads == 1 */
+  agnn_act act;
+  agnn_prec prec;
+  float negative_slope;    /* GAT LeakyReLU slope lambda (reading A5), 0.2          */
+  float beta;              /* AGNN temperature (reading A8), 1.0, not trained        */
+  float eps;               /* AGNN norm floor nu_i = max(||h_i||, eps), 1e-12        */
+} agnn_layer_desc;
+
+typedef struct agnn_plan_s* agnn_plan_t;
+typedef struct agnn_model_s* agnn_model_t;
+
+/* 1D row-block partition (reading A20; the paper's own scheme is 2D,
+ * PAPER.md:321).  Pure host function, bit-exact with the oracle:
+ * w(r) = row_ptr[r] + c_v * r, bounds[0] = 0, bounds[world] = n,
+ * bounds[p] = min{ r : w(r) >= ceil(p * w(n) / world) }.  row_ptr is host. */
+agnn_status agnn_partition(int64_t n, const int64_t* row_ptr_host, int world, int64_t c_v,
+                           int64_t* bounds_host);
+
+/* Validate the CSR on the device, build the work lists (light rows + heavy-row
+ * chunks), and (world > 1) create the NCCL communicator.  Synchronises once. */
+agnn_status agnn_plan_create(const agnn_csr* csr, const agnn_dist* dist /* NULL => 1 GPU */,
+                             cudaStream_t stream, agnn_plan_t* out);
+agnn_status agnn_plan_destroy(agnn_plan_t plan);
+/* host-side statistics: [0]=n_local [1]=nnz_local [2]=light rows [3]=heavy rows
+ * [4]=heavy chunks [5]=chunk size [6]=max degree [7]=n (global)            */
+agnn_status agnn_plan_info(agnn_plan_t plan, int64_t* info8);
+
+agnn_status agnn_model_create(agnn_plan_t plan, int n_layers, const agnn_layer_desc* descs,
+                              agnn_model_t* out);
+agnn_status agnn_model_destroy(agnn_model_t model);
+
+/* bytes of the per-layer `saved` buffer (intermediates kept for backward)
+ * and of the scratch `workspace` shared by forward and backward.            */
+agnn_status agnn_saved_bytes(agnn_model_t model, int layer, size_t* bytes);
+agnn_status agnn_workspace_bytes(agnn_model_t model, int layer, size_t* bytes);
+
+/* Layer forward: H_out = sigma(Z).  saved == NULL => inference mode (nothing
+ * kept, PAPER.md:623/:636 --inference); otherwise `saved` receives what
+ * agnn_backward needs.  Enqueued on `stream`.                              */
+agnn_status agnn_forward(agnn_model_t model, int layer, const float* W, const float* a,
+                         const float* H_in, float* H_out, void* saved, void* workspace,
+                         cudaStream_t stream);
+
+/* Layer backward (Eq. 6): from dH_out = dL/dH^{l+1} computes
+ * dH_in = Gamma = dL/dH^l (nullable: skipped), dW = Y^l, and for GAT
+ * da = dL/da (reading A12; NULL for VA/AGNN).  `saved` is the buffer filled
+ * by the matching agnn_forward; H_in is the same layer input.              */
+agnn_status agnn_backward(agnn_model_t model, int layer, const float* W, const float* a,
+                          const float* H_in, const void* saved, const float* dH_out,
+                          float* dH_in, float* dW, float* da, void* workspace,
+                          cudaStream_t stream);
+
+/* Test-only export (excluded from timing): recompute the attention
+ * coefficients alpha of `count` stored entries (positions into the LOCAL
+ * col_idx) from the saved row statistics.  alpha_out: [count x heads].
+ * GAT/AGNN give the softmax alpha_ij, VA the raw score S_ij.  H_in is the
+ * layer input (needed by AGNN/VA on one GPU; ignored for GAT).             */
+agnn_status agnn_debug_attention(agnn_model_t model, int layer, const void* saved,
+                                 const float* H_in, const int64_t* edge_pos, int64_t count,
+                                 float* alpha_out, cudaStream_t stream);
+
+/* Number of kernels this library launched since load (all entry points).   */
+uint64_t agnn_launch_count(void);
+
+/* Live per-kernel timing for the bench (off by default).  When enabled, a CUDA
+ * event is recorded on the launch stream after every kernel (and at the start
+ * of each forward/backward call); a kernel's time is the gap to the previous
+ * event on that stream.  report() synchronises on the recorded events and
+ * writes "name launches total_ms" lines into buf (host, len bytes).        */
+agnn_status agnn_profile_enable(int on);
+agnn_status agnn_profile_report(char* buf, size_t len);
+agnn_status agnn_profile_reset(void);
+/* ncclGetUniqueId for the multi-GPU plan (host, 128 bytes).                 */
+agnn_status agnn_nccl_unique_id(void* out128);
+
+/* ---- utilities (harness / tests; not on the timed path) ---------------- */
+enum { AGNN_BUILD_SYMMETRIZE = 1u, AGNN_BUILD_SELF_LOOPS = 2u, AGNN_BUILD_CONNECT_ISOLATED = 4u };
+
+/* Canonical CSR (readings A1-A3, A21) from n_pairs device edge samples:
+ * drop self-pairs, optionally symmetrise, dedup, optionally connect every
+ * vertex without a non-self neighbour to (v+1) mod n (both directions),
+ * optionally add (v,v) for all v.  row_ptr: device [n+1], caller-allocated;
+ * *col_idx: device, allocated by the library (free with agnn_free);
+ * *nnz_out: host.  Uses device radix sort; synchronises.                   */
+agnn_status agnn_csr_build(int64_t n, const uint32_t* src, const uint32_t* dst, int64_t n_pairs,
+                           uint32_t build_flags, int64_t* row_ptr, int32_t** col_idx,
+                           int64_t* nnz_out, cudaStream_t stream);
+void agnn_free(void* device_ptr);
+
+const char* agnn_status_string(agnn_status status);
+const char* agnn_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* AGNN_H */

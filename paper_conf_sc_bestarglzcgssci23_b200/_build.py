@@ -67,15 +67,28 @@ def agnn_deps():
 
 
 def build_agnn(force: bool = False, verbose_ptxas: bool = False) -> str:
-    if force or _stale(AGNN_SO, agnn_deps()):
-        nccl_inc, nccl_lib = _nccl_dirs()
-        cmd = [NVCC, *ARCH, "-O3", "-std=c++17", "-lineinfo", "-shared", "-Xcompiler", "-fPIC",
-               "--expt-relaxed-constexpr", "-I", INCLUDE, "-I", CSRC, "-I", nccl_inc,
-               "-o", AGNN_SO, *agnn_sources(), "-L", nccl_lib, "-l:libnccl.so.2",
-               "-Xlinker", "-rpath," + nccl_lib, "-lcuda"]
-        if verbose_ptxas:
-            cmd.insert(1, "-Xptxas=-v")
-        _run(cmd)
+    """Compile every csrc/*.cu to an object (in parallel) and link libagnn.so."""
+    if not (force or _stale(AGNN_SO, agnn_deps())):
+        return AGNN_SO
+    nccl_inc, nccl_lib = _nccl_dirs()
+    objdir = os.path.join(ROOT, "build", "agnn")
+    os.makedirs(objdir, exist_ok=True)
+    headers = [d for d in agnn_deps() if not d.endswith(".cu")]
+    flags = [*ARCH, "-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC",
+             "--expt-relaxed-constexpr", "-I", INCLUDE, "-I", CSRC, "-I", nccl_inc]
+    if verbose_ptxas:
+        flags.append("-Xptxas=-v")
+    jobs = []
+    for src in agnn_sources():
+        obj = os.path.join(objdir, os.path.basename(src)[:-3] + ".o")
+        if force or _stale(obj, [src] + headers):
+            jobs.append([NVCC, *flags, "-c", src, "-o", obj])
+    from concurrent.futures import ThreadPoolExecutor
+    with ThreadPoolExecutor(max_workers=max(1, min(8, os.cpu_count() or 1))) as ex:
+        list(ex.map(_run, jobs))
+    objs = [os.path.join(objdir, os.path.basename(s)[:-3] + ".o") for s in agnn_sources()]
+    _run([NVCC, *ARCH, "-shared", "-o", AGNN_SO, *objs, "-L", nccl_lib, "-l:libnccl.so.2",
+          "-Xlinker", "-rpath," + nccl_lib])
     return AGNN_SO
 
 

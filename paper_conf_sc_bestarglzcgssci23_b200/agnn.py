@@ -1,0 +1,250 @@
+"""Thin Python binding of libagnn.so (include/agnn.h) — argument marshalling only.
+
+Every step of the layer runs in the library's CUDA kernels; this module only
+turns torch tensors into device pointers and streams into handles.  There is
+no CPU or PyTorch fallback: if libagnn.so is missing or no CUDA device is
+present, the calls raise.  The names mirror the C ABI (agnn_plan / agnn_forward
+/ agnn_backward, Eq. 1 and :250-254 Eq. 6).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+from . import _build
+
+VA, AGNN, GAT = 0, 1, 2
+KIND = {"va": VA, "agnn": AGNN, "gat": GAT}
+ACT = {"none": 0, "relu": 1, "elu": 2}
+PREC_FP32, PREC_TF32X3 = 0, 1
+CSR_SYMMETRIC = 1
+BUILD_SYMMETRIZE, BUILD_SELF_LOOPS, BUILD_CONNECT_ISOLATED = 1, 2, 4
+BUILD_PAPER = BUILD_SYMMETRIZE | BUILD_SELF_LOOPS | BUILD_CONNECT_ISOLATED
+
+STATUS = {0: "AGNN_OK", 1: "AGNN_EINVAL", 2: "AGNN_ECUDA", 3: "AGNN_ENCCL", 4: "AGNN_ENOMEM",
+          5: "AGNN_EUNSUPPORTED", 6: "AGNN_ESTATE"}
+
+# every symbol include/agnn.h declares (tests check the .so exports all of them)
+EXPORTS = ("agnn_partition", "agnn_plan_create", "agnn_plan_destroy", "agnn_plan_info",
+           "agnn_model_create", "agnn_model_destroy", "agnn_saved_bytes", "agnn_workspace_bytes",
+           "agnn_forward", "agnn_backward", "agnn_debug_attention", "agnn_launch_count",
+           "agnn_profile_enable", "agnn_profile_report", "agnn_profile_reset",
+           "agnn_nccl_unique_id", "agnn_csr_build", "agnn_free", "agnn_status_string",
+           "agnn_last_error")
+
+
+class AgnnError(RuntimeError):
+    def __init__(self, status, msg):
+        super().__init__(f"{STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+class CSR(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_int64), ("row_begin", ctypes.c_int64), ("row_end", ctypes.c_int64),
+                ("row_ptr", ctypes.c_void_p), ("col_idx", ctypes.c_void_p),
+                ("flags", ctypes.c_uint32)]
+
+
+class Dist(ctypes.Structure):
+    _fields_ = [("rank", ctypes.c_int), ("world", ctypes.c_int),
+                ("nccl_unique_id", ctypes.c_void_p), ("bounds", ctypes.c_void_p)]
+
+
+class LayerDesc(ctypes.Structure):
+    _fields_ = [("kind", ctypes.c_int), ("k_in", ctypes.c_int), ("k_out", ctypes.c_int),
+                ("heads", ctypes.c_int), ("act", ctypes.c_int), ("prec", ctypes.c_int),
+                ("negative_slope", ctypes.c_float), ("beta", ctypes.c_float),
+                ("eps", ctypes.c_float)]
+
+
+_lib = None
+
+
+def lib(build: bool = True):
+    """Load libagnn.so (building it in-tree if stale).  Raises if unavailable."""
+    global _lib
+    if _lib is None:
+        so = _build.build_agnn() if build else _build.AGNN_SO
+        if not os.path.exists(so):
+            raise RuntimeError(f"libagnn.so not found at {so}; run __graft_entry__.build()")
+        L = ctypes.CDLL(so)
+        L.agnn_status_string.restype = ctypes.c_char_p
+        L.agnn_last_error.restype = ctypes.c_char_p
+        L.agnn_launch_count.restype = ctypes.c_uint64
+        for name in EXPORTS:
+            fn = getattr(L, name)
+            if name not in ("agnn_status_string", "agnn_last_error", "agnn_launch_count",
+                            "agnn_free"):
+                fn.restype = ctypes.c_int
+        _lib = L
+    return _lib
+
+
+def _check(rc):
+    if rc != 0:
+        raise AgnnError(rc, lib().agnn_last_error().decode(errors="replace"))
+
+
+def _ptr(t):
+    return ctypes.c_void_p(0 if t is None else t.data_ptr())
+
+
+def _stream(stream):
+    if stream is None:
+        import torch
+        stream = torch.cuda.current_stream()
+    return ctypes.c_void_p(stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream))
+
+
+def launch_count() -> int:
+    return int(lib().agnn_launch_count())
+
+
+def profile_enable(on: bool = True):
+    _check(lib().agnn_profile_enable(ctypes.c_int(1 if on else 0)))
+
+
+def profile_reset():
+    _check(lib().agnn_profile_reset())
+
+
+def profile_report() -> dict:
+    """{kernel name: (launches, total_ms)} accumulated since the last reset (synchronises)."""
+    buf = ctypes.create_string_buffer(1 << 16)
+    _check(lib().agnn_profile_report(buf, ctypes.c_size_t(len(buf))))
+    out = {}
+    for line in buf.value.decode().splitlines():
+        name, cnt, ms = line.rsplit(" ", 2)
+        out[name] = (int(cnt), float(ms))
+    return out
+
+
+def nccl_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(128)
+    _check(lib().agnn_nccl_unique_id(buf))
+    return buf.raw
+
+
+def partition(row_ptr_host, world: int, c_v: int = 4):
+    """agnn_partition on a host int64 row_ptr (numpy); returns numpy bounds[world+1]."""
+    import numpy as np
+    rp = np.ascontiguousarray(row_ptr_host, dtype=np.int64)
+    b = np.zeros(world + 1, dtype=np.int64)
+    _check(lib().agnn_partition(ctypes.c_int64(len(rp) - 1), rp.ctypes.data_as(ctypes.c_void_p),
+                                ctypes.c_int(world), ctypes.c_int64(c_v),
+                                b.ctypes.data_as(ctypes.c_void_p)))
+    return b
+
+
+class _DeviceArray:
+    """Library-allocated device buffer exposed to torch via __cuda_array_interface__."""
+
+    def __init__(self, ptr, n, typestr):
+        self.ptr, self.n = ptr, n
+        self.__cuda_array_interface__ = {"shape": (n,), "typestr": typestr,
+                                         "data": (ptr, False), "version": 3, "strides": None}
+
+    def __del__(self):
+        if self.ptr and _lib is not None:
+            _lib.agnn_free(ctypes.c_void_p(self.ptr))
+            self.ptr = 0
+
+
+def csr_build(n: int, src, dst, flags: int = BUILD_PAPER, stream=None):
+    """agnn_csr_build on device uint32 edge samples -> (row_ptr int64[n+1], col_idx int32)."""
+    import torch
+    row_ptr = torch.empty(n + 1, dtype=torch.int64, device=src.device)
+    col = ctypes.c_void_p(0)
+    nnz = ctypes.c_int64(0)
+    _check(lib().agnn_csr_build(ctypes.c_int64(n), _ptr(src), _ptr(dst), ctypes.c_int64(src.numel()),
+                                ctypes.c_uint32(flags), _ptr(row_ptr), ctypes.byref(col),
+                                ctypes.byref(nnz), _stream(stream)))
+    holder = _DeviceArray(col.value or 0, nnz.value, "<i4")
+    col_t = torch.as_tensor(holder, device=src.device) if nnz.value > 0 else \
+        torch.empty(0, dtype=torch.int32, device=src.device)
+    col_t._agnn_holder = holder  # keep the allocation alive with the tensor
+    return row_ptr, col_t
+
+
+class Plan:
+    """agnn_plan_create: validated CSR + work lists (+ NCCL communicator when world > 1)."""
+
+    def __init__(self, row_ptr, col_idx, n, row_begin=0, row_end=None, symmetric=True,
+                 rank=0, world=1, nccl_unique_id: bytes | None = None, bounds=None, stream=None):
+        self.row_ptr, self.col_idx = row_ptr, col_idx  # keep the caller's CSR alive
+        row_end = n if row_end is None else row_end
+        self._csr = CSR(n, row_begin, row_end, row_ptr.data_ptr(), col_idx.data_ptr(),
+                        CSR_SYMMETRIC if symmetric else 0)
+        dist = None
+        if world > 1:
+            import numpy as np
+            self._bounds = np.ascontiguousarray(bounds, dtype=np.int64)
+            self._uid = ctypes.create_string_buffer(bytes(nccl_unique_id), 128)
+            dist = Dist(rank, world, ctypes.cast(self._uid, ctypes.c_void_p),
+                        self._bounds.ctypes.data_as(ctypes.c_void_p))
+        h = ctypes.c_void_p()
+        _check(lib().agnn_plan_create(ctypes.byref(self._csr),
+                                      ctypes.byref(dist) if dist is not None else None,
+                                      _stream(stream), ctypes.byref(h)))
+        self.handle = h
+        self.n, self.row_begin, self.row_end = n, row_begin, row_end
+        self.n_local = row_end - row_begin
+
+    def info(self) -> dict:
+        a = (ctypes.c_int64 * 8)()
+        _check(lib().agnn_plan_info(self.handle, a))
+        keys = ("n_local", "nnz", "light_rows", "heavy_rows", "heavy_chunks", "chunk", "max_degree",
+                "n")
+        return dict(zip(keys, list(a)))
+
+    def __del__(self):
+        if getattr(self, "handle", None) and _lib is not None:
+            _lib.agnn_plan_destroy(self.handle)
+            self.handle = None
+
+
+def layer_desc(kind, k_in, k_out, heads=1, act="relu", prec=PREC_FP32, negative_slope=0.2,
+               beta=1.0, eps=1e-12) -> LayerDesc:
+    return LayerDesc(KIND[kind] if isinstance(kind, str) else kind, k_in, k_out, heads,
+                     ACT[act] if isinstance(act, str) else act, prec, negative_slope, beta, eps)
+
+
+class Model:
+    """agnn_model_create over a plan; forward/backward are the C entry points."""
+
+    def __init__(self, plan: Plan, descs):
+        self.plan = plan
+        self.descs = list(descs)
+        arr = (LayerDesc * len(self.descs))(*self.descs)
+        h = ctypes.c_void_p()
+        _check(lib().agnn_model_create(plan.handle, len(self.descs), arr, ctypes.byref(h)))
+        self.handle = h
+
+    def saved_bytes(self, layer: int) -> int:
+        b = ctypes.c_size_t(0)
+        _check(lib().agnn_saved_bytes(self.handle, layer, ctypes.byref(b)))
+        return b.value
+
+    def workspace_bytes(self, layer: int) -> int:
+        b = ctypes.c_size_t(0)
+        _check(lib().agnn_workspace_bytes(self.handle, layer, ctypes.byref(b)))
+        return b.value
+
+    def forward(self, layer, W, a, H_in, H_out, saved, workspace, stream=None):
+        _check(lib().agnn_forward(self.handle, layer, _ptr(W), _ptr(a), _ptr(H_in), _ptr(H_out),
+                                  _ptr(saved), _ptr(workspace), _stream(stream)))
+
+    def backward(self, layer, W, a, H_in, saved, dH_out, dH_in, dW, da, workspace, stream=None):
+        _check(lib().agnn_backward(self.handle, layer, _ptr(W), _ptr(a), _ptr(H_in), _ptr(saved),
+                                   _ptr(dH_out), _ptr(dH_in), _ptr(dW), _ptr(da), _ptr(workspace),
+                                   _stream(stream)))
+
+    def debug_attention(self, layer, saved, H_in, edge_pos, out, stream=None):
+        _check(lib().agnn_debug_attention(self.handle, layer, _ptr(saved), _ptr(H_in),
+                                          _ptr(edge_pos), ctypes.c_int64(edge_pos.numel()),
+                                          _ptr(out), _stream(stream)))
+
+    def __del__(self):
+        if getattr(self, "handle", None) and _lib is not None:
+            _lib.agnn_model_destroy(self.handle)
+            self.handle = None

@@ -1,0 +1,169 @@
+// common.cuh — shared device helpers and internal structures of libagnn.so.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+#include <string>
+
+#include "agnn.h"
+
+namespace agnn {
+
+constexpr float kLog2e = 1.4426950408889634f;
+constexpr int kNumSMs = 148;
+
+// ---- error plumbing (host) -------------------------------------------------
+void set_error(const std::string& msg);
+agnn_status fail(agnn_status st, const std::string& msg);
+agnn_status cuda_status(cudaError_t e, const char* what);
+void count_launch(int n = 1);
+// live per-kernel timing (agnn_profile_*): an event is recorded on the launch
+// stream after every kernel; a kernel's time is the gap to the previous marker.
+extern bool g_profiling;
+void prof_mark(const char* name, cudaStream_t s);
+
+#define AGNN_CUDA_TRY(expr)                                            \
+  do {                                                                 \
+    cudaError_t _e = (expr);                                           \
+    if (_e != cudaSuccess) return ::agnn::cuda_status(_e, #expr);      \
+  } while (0)
+
+// (expects the launch stream in a variable named `s`)
+#define AGNN_LAUNCH_CHECK(name)                                        \
+  do {                                                                 \
+    ::agnn::count_launch();                                            \
+    cudaError_t _e = cudaGetLastError();                               \
+    if (_e != cudaSuccess) return ::agnn::cuda_status(_e, name);       \
+    if (::agnn::g_profiling) ::agnn::prof_mark(name, s);               \
+  } while (0)
+
+// ---- device helpers ----------------------------------------------------------
+__device__ __forceinline__ float ex2(float x) {
+  float y;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
+
+__device__ __forceinline__ float4 ldg4(const float* p) {
+  return __ldg(reinterpret_cast<const float4*>(p));
+}
+// streaming (read-once) load: do not allocate in L1
+__device__ __forceinline__ float4 ld_stream4(const float* p) {
+  float4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
+               : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w)
+               : "l"(p));
+  return r;
+}
+__device__ __forceinline__ void st4(float* p, float4 v) { *reinterpret_cast<float4*>(p) = v; }
+
+__device__ __forceinline__ float dot4(float4 a, float4 b) {
+  return fmaf(a.x, b.x, fmaf(a.y, b.y, fmaf(a.z, b.z, a.w * b.w)));
+}
+__device__ __forceinline__ float4 f4(float v) { return make_float4(v, v, v, v); }
+__device__ __forceinline__ float4 fma4(float s, float4 x, float4 y) {  // s*x + y
+  return make_float4(fmaf(s, x.x, y.x), fmaf(s, x.y, y.y), fmaf(s, x.z, y.z), fmaf(s, x.w, y.w));
+}
+__device__ __forceinline__ float4 mul4(float s, float4 x) {
+  return make_float4(s * x.x, s * x.y, s * x.z, s * x.w);
+}
+__device__ __forceinline__ float4 add4(float4 a, float4 b) {
+  return make_float4(a.x + b.x, a.y + b.y, a.z + b.z, a.w + b.w);
+}
+
+__device__ __forceinline__ float act_fwd(int act, float z) {
+  if (act == AGNN_ACT_RELU) return z > 0.f ? z : 0.f;
+  if (act == AGNN_ACT_ELU) return z > 0.f ? z : expm1f(z);
+  return z;
+}
+__device__ __forceinline__ float act_grad(int act, float z) {
+  if (act == AGNN_ACT_RELU) return z > 0.f ? 1.f : 0.f;
+  if (act == AGNN_ACT_ELU) return z > 0.f ? 1.f : expf(z);
+  return 1.f;
+}
+__device__ __forceinline__ float4 act_fwd4(int act, float4 z) {
+  return make_float4(act_fwd(act, z.x), act_fwd(act, z.y), act_fwd(act, z.z), act_fwd(act, z.w));
+}
+
+// ---- lane layout of one feature row over a group of lanes -------------------
+// A row of K fp32 features is held by LANES lanes, VPL float4 each; the v-th
+// float4 of lane q covers columns c = v*LANES*4 + q*4 .. +3 (coalesced).
+template <int K, int NH>
+struct RowLayout {
+  static_assert(K % 16 == 0 && K >= 16 && K <= 256, "K must be 16..256, multiple of 16");
+  static constexpr int LANES = (K / 4 >= 32) ? 32 : K / 4;
+  static constexpr int VPL = K / (4 * LANES);
+  static constexpr int GROUPS = 32 / LANES;
+  static constexpr int D = K / NH;  // head width
+  static_assert(K % NH == 0 && D % 4 == 0, "head width must be a multiple of 4");
+  // lanes sharing one head inside one float4 slot
+  static constexpr int HL = (D / 4 < LANES) ? D / 4 : LANES;
+  // consecutive v slots spanned by one head (D > 4*LANES)
+  static constexpr int VS = (D > 4 * LANES) ? D / (4 * LANES) : 1;
+  __device__ static __forceinline__ int col(int v, int q) { return v * LANES * 4 + q * 4; }
+  __device__ static __forceinline__ int head(int v, int q) { return col(v, q) / D; }
+  // sum x over the lanes of one head (xor butterfly inside aligned HL groups)
+  __device__ static __forceinline__ float head_sum(float x) {
+#pragma unroll
+    for (int o = HL / 2; o > 0; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
+    return x;
+  }
+  // per-slot partial dot products -> full per-head dot product in every slot
+  __device__ static __forceinline__ void head_reduce(float (&x)[VPL]) {
+    if constexpr (VS > 1) {
+#pragma unroll
+      for (int v0 = 0; v0 < VPL; v0 += VS) {
+        float t = 0.f;
+#pragma unroll
+        for (int v = 0; v < VS; ++v) t += x[v0 + v];
+#pragma unroll
+        for (int v = 0; v < VS; ++v) x[v0 + v] = t;
+      }
+    }
+#pragma unroll
+    for (int v = 0; v < VPL; ++v) x[v] = head_sum(x[v]);
+  }
+};
+
+// ---- plan / model (host structures) ------------------------------------------
+struct Plan {
+  int64_t n = 0, row_begin = 0, row_end = 0, n_local = 0, nnz = 0;
+  const int64_t* row_ptr = nullptr;   // caller-owned, local rows
+  const int32_t* col_idx = nullptr;   // caller-owned
+  uint32_t flags = 0;
+  int64_t max_deg = 0;
+  // work lists (device, plan-owned)
+  int chunk = 2048;
+  int64_t n_light = 0, n_heavy = 0, n_chunks = 0;
+  int32_t* light_rows = nullptr;      // [n_light]
+  int32_t* chunk_row = nullptr;       // [n_chunks]
+  int32_t* chunk_idx = nullptr;       // [n_chunks] chunk ordinal within its row
+  int32_t* heavy_rows = nullptr;      // [n_heavy]
+  int32_t* heavy_off = nullptr;       // [n_heavy+1] chunk ranges
+  void* meta_block = nullptr;         // single allocation backing the lists
+  // distribution
+  int rank = 0, world = 1;
+  int64_t* bounds = nullptr;          // host [world+1]
+  void* nccl = nullptr;               // ncclComm_t
+};
+
+struct Model {
+  Plan* plan = nullptr;
+  int n_layers = 0;
+  agnn_layer_desc* descs = nullptr;
+};
+
+// byte layout helpers (aligned sub-buffers inside saved / workspace)
+struct Carver {
+  char* base;
+  size_t off = 0;
+  explicit Carver(void* b) : base(static_cast<char*>(b)) {}
+  template <typename T>
+  T* take(size_t count) {
+    off = (off + 255) & ~size_t(255);
+    T* p = base ? reinterpret_cast<T*>(base + off) : nullptr;
+    off += count * sizeof(T);
+    return p;
+  }
+};
+
+}  // namespace agnn

@@ -1,0 +1,70 @@
+// internal.cuh — launcher prototypes shared between the .cu files of libagnn.so
+#pragma once
+#include "common.cuh"
+
+namespace agnn {
+
+// ---- work items (plan) ---------------------------------------------------------
+struct Items {
+  const int64_t* row_ptr;     // local rows
+  const int32_t* col;         // global column ids
+  const int32_t* light_rows;  // local row ids
+  int64_t n_light;
+  const int32_t* chunk_row;
+  const int32_t* chunk_idx;
+  int64_t n_chunks;
+  int chunk;
+  const int32_t* heavy_rows;
+  const int32_t* heavy_off;
+  int64_t n_heavy;
+  int64_t row_begin;          // global id of local row 0
+  int64_t n_local;
+};
+Items items_of(const Plan& p);
+
+// persistent sparse-kernel grid: 256-thread blocks, SMs x resident blocks of `func`
+constexpr int kSparseThreads = 256;
+constexpr int kMaxSparseBlocks = kNumSMs * 8;
+int persistent_blocks(const void* func);
+template <typename F>
+inline int grid_of(F* func) { return persistent_blocks(reinterpret_cast<const void*>(func)); }
+
+// ---- GEMMs (gemm_simt.cu) -----------------------------------------------------
+// C[M x N] = A[M x K] * op(B);  op(B) = B ([K x N], ldb=N) or B^T (B is [N x K]).
+// Columns [0, n_split) go to C0 (ld = n_split), [n_split, N) to C1 (ld = N - n_split).
+// If Cact != NULL, sigma(C) (act) is also written to Cact (layout of C0); C0 may be NULL.
+agnn_status gemm_rows(const float* A, int64_t M, int K, const float* B, bool b_trans, int N,
+                      float* C0, int n_split, float* C1, cudaStream_t s, float* Cact = nullptr,
+                      int act = 0);
+// C[K1 x N] = A^T B over M rows (A [M x K1], B [M x N]); deterministic split-M with
+// partials in `ws` (gemm_tn_ws_floats) and an ordered reduction.  If accumulate,
+// C += result.
+size_t gemm_tn_ws_floats(int K1, int N);
+agnn_status gemm_tn(const float* A, int64_t M, int K1, const float* B, int N, float* C,
+                    float* ws, cudaStream_t s);
+
+// ---- GAT (gat.cu) ---------------------------------------------------------------
+struct GatShape {
+  int k_in, k_out, heads;
+  float slope;
+  int act;
+};
+size_t gat_saved_bytes(const Plan& p, const GatShape& g);
+size_t gat_workspace_bytes(const Plan& p, const GatShape& g);
+agnn_status gat_forward(const Plan& p, const GatShape& g, const float* W, const float* a,
+                        const float* H_in, float* H_out, void* saved, void* ws, cudaStream_t s);
+agnn_status gat_backward(const Plan& p, const GatShape& g, const float* W, const float* a,
+                         const float* H_in, const void* saved, const float* dH_out,
+                         float* dH_in, float* dW, float* da, void* ws, cudaStream_t s);
+agnn_status gat_debug_alpha(const Plan& p, const GatShape& g, const void* saved,
+                            const int64_t* edge_pos, int64_t count, float* out, cudaStream_t s);
+
+// ---- multi-GPU exchange (comm.cu) -------------------------------------------------
+// all-gather of row blocks: rows [bounds[r], bounds[r+1]) of `full` (row width
+// `width` floats) are broadcast from rank r; in place.
+agnn_status allgather_rows(const Plan& p, float* full, int64_t width, cudaStream_t s);
+agnn_status allreduce_sum(const Plan& p, float* buf, int64_t count, cudaStream_t s);
+agnn_status comm_init(Plan& p, const void* unique_id);
+void comm_destroy(Plan& p);
+
+}  // namespace agnn

@@ -1,0 +1,100 @@
+"""Shared helpers for the GPU parity tests (CUDA path vs the FP64 oracle)."""
+from __future__ import annotations
+
+import numpy as np
+import torch
+
+import oracle
+from paper_conf_sc_bestarglzcgssci23_b200 import agnn, gen, runner
+
+TOL_FP32 = 1e-5  # north_star: "within 1e-5 relative in FP32" (normwise, SURVEY §8(c) parity protocol)
+
+
+def rel(x, y):
+    x = np.asarray(x, np.float64)
+    y = np.asarray(y, np.float64)
+    ny = np.linalg.norm(y)
+    return float(np.linalg.norm(x - y) / (ny if ny > 0 else 1.0))
+
+
+def host_graph(w: gen.Workload):
+    src, dst = w.host_edges()
+    rp, ci = oracle.csr_build(w.n, src, dst)
+    return src, dst, rp, ci
+
+
+def device_graph(w: gen.Workload, src, dst):
+    s = torch.from_numpy(src.view(np.int32)).cuda()
+    d = torch.from_numpy(dst.view(np.int32)).cuda()
+    rp, ci = agnn.csr_build(w.n, s, d, agnn.BUILD_PAPER)
+    return runner.Graph(w.n, rp, ci, int(ci.numel()))
+
+
+def oracle_step(w: gen.Workload, rp, ci, H, Ws, As, R):
+    """L-layer forward then backward with the oracle; returns per-layer outputs."""
+    Hs, fwd = [np.asarray(H, np.float64)], []
+    for l in range(w.layers):
+        f, _ = oracle.layer(w.model, rp, ci, Hs[-1], Ws[l], As[l], w.heads, act=w.act,
+                            slope=w.slope, beta=w.beta, eps=w.eps)
+        fwd.append(f)
+        Hs.append(f["Hout"])
+    dHs = [None] * (w.layers + 1)
+    dHs[w.layers] = np.asarray(R, np.float64)
+    dWs, das = [None] * w.layers, [None] * w.layers
+    for l in reversed(range(w.layers)):
+        if w.model == "gat":
+            b = oracle.gat_backward(rp, ci, Hs[l], Ws[l], As[l], w.heads, fwd[l], dHs[l + 1],
+                                    w.slope, w.act)
+            das[l] = b["da"]
+        elif w.model == "agnn":
+            b = oracle.agnn_backward(rp, ci, Hs[l], Ws[l], fwd[l], dHs[l + 1], w.beta, w.eps, w.act)
+        else:
+            b = oracle.va_backward(rp, ci, Hs[l], Ws[l], fwd[l], dHs[l + 1], w.act)
+        dHs[l], dWs[l] = b["dH"], b["dW"]
+    return {"H": Hs, "fwd": fwd, "dH": dHs, "dW": dWs, "da": das}
+
+
+def gpu_step(w: gen.Workload, graph=None):
+    st = runner.Stack(w, "cuda", graph=graph)
+    st.step()
+    torch.cuda.synchronize()
+    return st
+
+
+def compare(w, st, ref, tol=TOL_FP32):
+    """Normwise parity of every output of the step; returns the error table."""
+    errs = {}
+    for l in range(1, w.layers + 1):
+        errs[f"H{l}"] = rel(st.H[l].cpu().numpy(), ref["H"][l])
+    for l in range(w.layers + 1):
+        errs[f"dH{l}"] = rel(st.dH[l].cpu().numpy(), ref["dH"][l])
+    for l in range(w.layers):
+        errs[f"dW{l}"] = rel(st.dW[l].cpu().numpy(), ref["dW"][l])
+        if w.model == "gat":
+            errs[f"da{l}"] = rel(st.da[l].cpu().numpy(), ref["da"][l])
+    bad = {k: v for k, v in errs.items() if not (v <= tol)}
+    assert not bad, f"parity failures (tol {tol}): {bad}; all: {errs}"
+    return errs
+
+
+def compare_attention(w, st, ref, layer=0, n_samples=4096, seed=0):
+    """Elementwise alpha (or VA score) on sampled stored entries via agnn_debug_attention."""
+    nnz = st.nnz_local
+    rng = np.random.default_rng(seed)
+    pos = np.unique(rng.integers(0, nnz, min(n_samples, nnz))).astype(np.int64)
+    pos_t = torch.from_numpy(pos).cuda()
+    heads = w.heads if w.model == "gat" else 1
+    out = torch.empty(len(pos) * heads, dtype=torch.float32, device="cuda")
+    st.model.debug_attention(layer, st.saved[layer], st.H[layer], pos_t, out)
+    torch.cuda.synchronize()
+    got = out.cpu().numpy().reshape(len(pos), heads)
+    f = ref["fwd"][layer]
+    exp = f["alpha"][pos] if w.model != "va" else f["S"][pos][:, None]
+    exp = exp.reshape(len(pos), heads)
+    if w.model == "va":
+        err = np.abs(got - exp) / (np.abs(exp) + 1e-3)
+        assert err.max() < 1e-4, err.max()
+    else:
+        err = np.abs(got - exp) - (1e-5 * exp + 1e-9)
+        assert err.max() <= 0, f"alpha mismatch, worst excess {err.max()}"
+    return float(np.max(np.abs(got - exp)))

@@ -1,0 +1,169 @@
+"""GPU parity: the CUDA path (through the C ABI) against the FP64 oracle.
+
+Inputs are the seeded synthetic workloads (paper_conf_sc_bestarglzcgssci23_b200.gen)
+at sizes the oracle finishes in seconds that still span many tiles, heavy-row
+chunks (degree > 2048) and ragged tails.  Bars (north_star / SURVEY §8(c)):
+  * CSR metadata bit-exact with the oracle's host builder;
+  * every float output normwise <= 1e-5 relative (FP32);
+  * attention alpha elementwise |a - a_ref| <= 1e-5 a_ref + 1e-9.
+"""
+from __future__ import annotations
+
+import dataclasses
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+
+pytestmark = [pytest.mark.gpu,
+              pytest.mark.skipif(not torch.cuda.is_available(), reason="needs a CUDA device")]
+
+import oracle  # noqa: E402
+import parity_utils as pu  # noqa: E402
+from paper_conf_sc_bestarglzcgssci23_b200 import agnn, gen, runner  # noqa: E402
+
+
+def W(model, graph, scale, ef, k, heads=1, layers=1, act="relu", n=None, samples=None, **kw):
+    n = n or (1 << scale)
+    return gen.Workload(f"{model}-{graph}{scale}-k{k}h{heads}L{layers}", model, graph, scale, n,
+                        samples if samples is not None else ef * n, k, heads, layers, act=act, **kw)
+
+
+# ------------------------------------------------------------------ CSR metadata
+@pytest.mark.parametrize("w", [gen.CONFIGS["C1"], W("gat", "kron", 14, 8, 16),
+                               W("gat", "rmat", 13, 16, 16), W("gat", "er", 0, 0, 16, n=3000,
+                                                               samples=20000)],
+                         ids=lambda w: w.name)
+def test_csr_build_bit_exact(w):
+    src, dst, rp, ci = pu.host_graph(w)
+    g = pu.device_graph(w, src, dst)
+    np.testing.assert_array_equal(g.row_ptr.cpu().numpy(), rp)
+    np.testing.assert_array_equal(g.col_idx.cpu().numpy(), ci)
+
+
+def test_device_generators_match_host():
+    w = gen.CONFIGS["C2"]
+    s = torch.empty(w.n_samples, dtype=torch.int32, device="cuda")
+    d = torch.empty_like(s)
+    gen.edges_device(w.kind, w.seed, w.scale, w.n, w.n_samples, s.data_ptr(), d.data_ptr())
+    hs, hd = w.host_edges()
+    np.testing.assert_array_equal(s.cpu().numpy().view(np.uint32), hs)
+    np.testing.assert_array_equal(d.cpu().numpy().view(np.uint32), hd)
+    H = torch.empty(1000, 64, device="cuda")
+    gen.fill_device(1, gen.STREAM_W(0), H.numel(), gen.glorot_bound(64, 64), H.data_ptr(),
+                    offset=0)
+    np.testing.assert_array_equal(H.cpu().numpy(), gen.fill(1, gen.STREAM_W(0), (1000, 64),
+                                                            gen.glorot_bound(64, 64)))
+
+
+def test_plan_info_and_heavy_rows():
+    w = W("gat", "kron", 16, 8, 64)
+    src, dst, rp, ci = pu.host_graph(w)
+    g = pu.device_graph(w, src, dst)
+    plan = agnn.Plan(g.row_ptr, g.col_idx, w.n)
+    info = plan.info()
+    deg = np.diff(rp)
+    assert info["nnz"] == len(ci) and info["max_degree"] == deg.max()
+    assert info["heavy_rows"] == int((deg > info["chunk"]).sum()) > 0
+    assert info["heavy_chunks"] == int(np.ceil(deg[deg > info["chunk"]] / info["chunk"]).sum())
+    assert info["light_rows"] + info["heavy_rows"] == w.n
+
+
+# ------------------------------------------------------------------ layer parity
+CASES = [
+    gen.CONFIGS["C1"],                                    # GAT ER 1024, k=16
+    dataclasses.replace(gen.CONFIGS["C2"]),               # GAT Kron 2^16 ef8, k=64, 2 layers
+    W("gat", "kron", 15, 8, 128, heads=4),                # C5 shape (k=128, 4 heads), heavy rows
+    W("gat", "kron", 13, 8, 32, heads=8, act="elu"),
+    W("gat", "er", 0, 0, 256, heads=2, n=2000, samples=12000, act="none"),
+    W("gat", "rmat", 14, 8, 64, heads=1, layers=2),
+    W("agnn", "rmat", 14, 16, 128, layers=2),             # C3 shape (R-MAT, k=128)
+    W("agnn", "kron", 13, 8, 64, act="elu"),
+    W("agnn", "er", 0, 0, 256, n=1500, samples=9000, act="none", beta=1.5),
+    W("agnn", "er", 0, 0, 16, n=1024, samples=7680),
+    W("va", "kron", 13, 8, 256, act="none"),              # C4 shape (VA, k=256)
+    W("va", "kron", 14, 8, 128),
+    W("va", "er", 0, 0, 32, n=1024, samples=7680, act="elu"),
+]
+
+
+@pytest.mark.parametrize("w", CASES, ids=lambda w: w.name)
+def test_layer_parity(w):
+    src, dst, rp, ci = pu.host_graph(w)
+    g = pu.device_graph(w, src, dst)
+    np.testing.assert_array_equal(g.col_idx.cpu().numpy(), ci)
+    st = pu.gpu_step(w, graph=g)
+    H, Ws, As, R = w.host_inputs()
+    np.testing.assert_array_equal(st.H[0].cpu().numpy(), H)
+    ref = pu.oracle_step(w, rp, ci, H, Ws, As, R)
+    pu.compare(w, st, ref)
+    pu.compare_attention(w, st, ref)
+
+
+def test_inference_mode_matches_training_forward():
+    w = W("gat", "kron", 13, 8, 64, heads=2)
+    st = runner.Stack(w, "cuda")
+    st.forward()
+    out_train = st.H[1].clone()
+    st.H[1].zero_()
+    st.forward(inference=True)
+    torch.cuda.synchronize()
+    assert torch.equal(out_train, st.H[1])
+
+
+@pytest.mark.parametrize("model", ["gat", "agnn", "va"])
+def test_run_to_run_bitwise_determinism(model):
+    w = W(model, "kron", 14, 8, 128, heads=4 if model == "gat" else 1)
+    st = runner.Stack(w, "cuda")
+    st.step()
+    a = [t.clone() for t in (st.H[1], st.dH[0], st.dW[0])]
+    st.step()
+    torch.cuda.synchronize()
+    for x, y in zip(a, (st.H[1], st.dH[0], st.dW[0])):
+        assert torch.equal(x, y)
+
+
+def test_empty_rows_and_no_self_loops():
+    """Rows without stored entries give zero output / gradient (reading A7)."""
+    n, k = 50, 16
+    rng = np.random.default_rng(3)
+    A = rng.random((n, n)) < 0.1
+    A = A | A.T
+    np.fill_diagonal(A, False)
+    A[7, :] = A[:, 7] = False      # isolated vertex, empty row
+    rp = np.concatenate([[0], np.cumsum(A.sum(1))]).astype(np.int64)
+    ci = np.concatenate([np.nonzero(A[i])[0] for i in range(n)]).astype(np.int32)
+    for model, heads in (("gat", 2), ("agnn", 1), ("va", 1)):
+        w = gen.Workload("edge", model, "er", 0, n, 0, k, heads, 1, act="none")
+        g = runner.Graph(n, torch.from_numpy(rp).cuda(), torch.from_numpy(ci).cuda(), len(ci))
+        st = pu.gpu_step(w, graph=g)
+        H, Ws, As, R = w.host_inputs()
+        ref = pu.oracle_step(w, rp, ci, H, Ws, As, R)
+        pu.compare(w, st, ref)
+        assert torch.all(st.H[1][7] == 0) and torch.all(st.dH[0][7] == 0)
+
+
+@pytest.mark.parametrize("bad", ["unsorted", "duplicate", "range", "rowptr"])
+def test_invalid_csr_rejected_at_plan(bad):
+    rp = np.array([0, 2, 4, 6], np.int64)
+    ci = np.array([0, 1, 0, 2, 1, 2], np.int32)
+    if bad == "unsorted":
+        ci[[2, 3]] = ci[[3, 2]]
+    elif bad == "duplicate":
+        ci[3] = 0
+    elif bad == "range":
+        ci[5] = 3
+    else:
+        rp[2] = 1
+    with pytest.raises(agnn.AgnnError) as e:
+        agnn.Plan(torch.from_numpy(rp).cuda(), torch.from_numpy(ci).cuda(), 3)
+    assert e.value.status == 1
+
+
+def test_launch_count_increases():
+    w = gen.CONFIGS["C1"]
+    st = runner.Stack(w, "cuda")
+    c0 = agnn.launch_count()
+    st.step()
+    assert agnn.launch_count() > c0
