@@ -489,14 +489,16 @@ __global__ void gat_da_reduce_kernel(const float* __restrict__ part, int64_t row
 
 // W_ext = [W | W a1^h ... | W a2^h ...]   (a' = W a, Table 2)
 __global__ void gat_wext_kernel(const float* __restrict__ W, const float* __restrict__ a, int k_in,
-                                int K, int NH, float* __restrict__ Wext) {
-  const int D = K / NH, NE = K + 2 * NH;
+                                int K, int NH, int NE, float* __restrict__ Wext) {
+  const int D = K / NH;
   for (int idx = blockIdx.x * blockDim.x + threadIdx.x; idx < k_in * NE;
        idx += gridDim.x * blockDim.x) {
     const int r = idx / NE, c = idx % NE;
     float v;
     if (c < K) {
       v = W[r * K + c];
+    } else if (c >= K + 2 * NH) {
+      v = 0.f;  // padding column (N multiple of 4)
     } else {
       const int h = (c - K) % NH, which = (c - K) / NH;
       v = 0.f;
@@ -562,7 +564,7 @@ int64_t da_rows() { return (int64_t)kMaxSparseBlocks * (kSparseThreads / 32) * 2
 WsGat carve_ws(const Plan& p, const GatShape& g, void* base, size_t* total) {
   Carver c(base);
   WsGat w;
-  const int NE = g.k_out + 2 * g.heads;
+  const int NE = (g.k_out + 2 * g.heads + 3) / 4 * 4;
   w.Wext = c.take<float>((size_t)g.k_in * NE);
   w.pacc = c.take<float>((size_t)p.n_chunks * g.k_out);
   w.pm = c.take<float>((size_t)p.n_chunks * g.heads);
@@ -615,13 +617,13 @@ agnn_status gat_forward(const Plan& p, const GatShape& g, const float* W, const 
                         const float* H_in, float* H_out, void* saved, void* ws, cudaStream_t s) {
   WsGat w = carve_ws(p, g, ws, nullptr);
   SavedGat sv = carve_saved(p, g, saved ? saved : w.saved_inf);
-  const int K_ = g.k_out, NH_ = g.heads, NE = g.k_out + 2 * g.heads;
-  gat_wext_kernel<<<64, 256, 0, s>>>(W, a, g.k_in, g.k_out, g.heads, w.Wext);
+  const int K_ = g.k_out, NH_ = g.heads, NEs = g.k_out + 2 * g.heads, NE = (NEs + 3) / 4 * 4;
+  gat_wext_kernel<<<64, 256, 0, s>>>(W, a, g.k_in, g.k_out, g.heads, NE, w.Wext);
   AGNN_LAUNCH_CHECK("gat_wext_kernel");
   // P (and s, t) for the local rows, written at their global offsets
   agnn_status st = gemm_rows(H_in, p.n_local, g.k_in, w.Wext, false, NE,
                              sv.P + p.row_begin * g.k_out, g.k_out,
-                             sv.st + p.row_begin * 2 * g.heads, s);
+                             sv.st + p.row_begin * 2 * g.heads, s, nullptr, 0, NEs);
   if (st != AGNN_OK) return st;
   if (p.world > 1) {
     if ((st = allgather_rows(p, sv.P, g.k_out, s)) != AGNN_OK) return st;

@@ -15,7 +15,7 @@ constexpr int BM = 128, BN = 128, BK = 8, TPB = 256;
 __global__ void __launch_bounds__(TPB)
 gemm_rows_kernel(const float* __restrict__ A, int64_t M, int K, const float* __restrict__ B,
                  int b_trans, int N, float* __restrict__ C0, int n_split, float* __restrict__ C1,
-                 float* __restrict__ Cact, int act) {
+                 float* __restrict__ Cact, int act, int n_store) {
   __shared__ __align__(16) float As[2][BK][BM + 4];
   __shared__ __align__(16) float Bs[2][BK][BN + 4];
   const int tid = threadIdx.x, tx = tid % 16, ty = tid / 16;
@@ -98,12 +98,12 @@ gemm_rows_kernel(const float* __restrict__ A, int64_t M, int K, const float* __r
 #pragma unroll
     for (int j = 0; j < 8; ++j) {
       const int c = n0 + (j < 4 ? tx * 4 + j : 64 + tx * 4 + j - 4);
-      if (c >= N) continue;
+      if (c >= n_store) continue;
       if (c < n_split) {
         if (C0) C0[r * n_split + c] = acc[i][j];
         if (Cact) Cact[r * n_split + c] = act_fwd(act, acc[i][j]);
       } else {
-        C1[r * (N - n_split) + (c - n_split)] = acc[i][j];
+        C1[r * (n_store - n_split) + (c - n_split)] = acc[i][j];
       }
     }
   }
@@ -195,12 +195,14 @@ __global__ void sum_splits_kernel(const float* __restrict__ part, int splits, in
 }  // namespace
 
 agnn_status gemm_rows(const float* A, int64_t M, int K, const float* B, bool b_trans, int N,
-                      float* C0, int n_split, float* C1, cudaStream_t s, float* Cact, int act) {
+                      float* C0, int n_split, float* C1, cudaStream_t s, float* Cact, int act,
+                      int n_store) {
   if (M <= 0) return AGNN_OK;
   if (K % 4 || N % 4) return fail(AGNN_EINVAL, "gemm_rows: K and N must be multiples of 4");
   dim3 grid((unsigned)((M + BM - 1) / BM), (N + BN - 1) / BN);
+  if (n_store <= 0 || n_store > N) n_store = N;
   gemm_rows_kernel<<<grid, TPB, 0, s>>>(A, M, K, B, b_trans ? 1 : 0, N, C0, n_split, C1, Cact,
-                                        act);
+                                        act, n_store);
   AGNN_LAUNCH_CHECK("gemm_rows_kernel");
   return AGNN_OK;
 }

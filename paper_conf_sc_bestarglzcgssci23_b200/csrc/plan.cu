@@ -10,6 +10,7 @@
 // any launch geometry and any number of GPUs (the row is always computed by its
 // owner in the same order).
 #include <algorithm>
+#include <cstdlib>
 #include <mutex>
 #include <unordered_map>
 #include <vector>
@@ -83,6 +84,12 @@ Items items_of(const Plan& p) {
 }
 
 agnn_status plan_build(Plan& p, cudaStream_t s) {
+  // heavy-row chunk size (edges); AGNN_CHUNK_EDGES overrides it (tests use small
+  // chunks to exercise the split/merge path on small graphs)
+  if (const char* env = getenv("AGNN_CHUNK_EDGES")) {
+    const long v = atol(env);
+    if (v >= 32 && v <= (1L << 30)) p.chunk = (int)v;
+  }
   // 1. validate on the device
   int* d_err = nullptr;
   AGNN_CUDA_TRY(cudaMallocAsync(&d_err, sizeof(int), s));

@@ -30,6 +30,25 @@ def device_graph(w: gen.Workload, src, dst):
     return runner.Graph(w.n, rp, ci, int(ci.numel()))
 
 
+def relu_kink_mask(w: gen.Workload, Z_last, R, rel_tau=1e-5):
+    """Zero the upstream gradient where the oracle's last-layer Z is within
+    rel_tau * rms(Z) of the ReLU kink.
+
+    sigma'(z) = [z > 0] is a discontinuous decision: an fp32 Z of ~1e-7 relative
+    size can fall on either side of 0 between two correct implementations, and a
+    single flipped element moves dH by ~1e-4 normwise.  Masking R there (decided
+    by the oracle, not the CUDA path) removes the decision from the comparison;
+    it touches ~1e-5 of the entries (reading A6').
+    """
+    if w.act != "relu":
+        return R
+    Z = np.asarray(Z_last, np.float64)
+    tau = rel_tau * np.sqrt(np.mean(Z * Z))
+    R = np.array(R, copy=True)
+    R[np.abs(Z) < tau] = 0.0
+    return R
+
+
 def oracle_step(w: gen.Workload, rp, ci, H, Ws, As, R):
     """L-layer forward then backward with the oracle; returns per-layer outputs."""
     Hs, fwd = [np.asarray(H, np.float64)], []
@@ -54,8 +73,10 @@ def oracle_step(w: gen.Workload, rp, ci, H, Ws, As, R):
     return {"H": Hs, "fwd": fwd, "dH": dHs, "dW": dWs, "da": das}
 
 
-def gpu_step(w: gen.Workload, graph=None):
+def gpu_step(w: gen.Workload, graph=None, R=None):
     st = runner.Stack(w, "cuda", graph=graph)
+    if R is not None:
+        st.dH[w.layers].copy_(torch.from_numpy(np.ascontiguousarray(R, np.float32)))
     st.step()
     torch.cuda.synchronize()
     return st
@@ -92,8 +113,10 @@ def compare_attention(w, st, ref, layer=0, n_samples=4096, seed=0):
     exp = f["alpha"][pos] if w.model != "va" else f["S"][pos][:, None]
     exp = exp.reshape(len(pos), heads)
     if w.model == "va":
-        err = np.abs(got - exp) / (np.abs(exp) + 1e-3)
-        assert err.max() < 1e-4, err.max()
+        # raw dot products S_ij = H_i . H_j can cancel; bound by k * eps32 * |H_i||H_j|
+        scale = np.sqrt(w.k) * np.sqrt(np.mean(f["S"] ** 2)) + 1e-30
+        err = np.abs(got - exp) / (1e-6 * scale + 1e-5 * np.abs(exp))
+        assert err.max() <= 1.0, err.max()
     else:
         err = np.abs(got - exp) - (1e-5 * exp + 1e-9)
         assert err.max() <= 0, f"alpha mismatch, worst excess {err.max()}"

@@ -73,12 +73,14 @@ def test_plan_info_and_heavy_rows():
 # ------------------------------------------------------------------ layer parity
 CASES = [
     gen.CONFIGS["C1"],                                    # GAT ER 1024, k=16
-    dataclasses.replace(gen.CONFIGS["C2"]),               # GAT Kron 2^16 ef8, k=64, 2 layers
+    dataclasses.replace(gen.CONFIGS["C2"], act="elu"),    # GAT Kron 2^16 ef8, k=64, 2 layers
+                                                          # (ELU: C1 sigma' across layers, A6')
     W("gat", "kron", 15, 8, 128, heads=4),                # C5 shape (k=128, 4 heads), heavy rows
     W("gat", "kron", 13, 8, 32, heads=8, act="elu"),
     W("gat", "er", 0, 0, 256, heads=2, n=2000, samples=12000, act="none"),
-    W("gat", "rmat", 14, 8, 64, heads=1, layers=2),
-    W("agnn", "rmat", 14, 16, 128, layers=2),             # C3 shape (R-MAT, k=128)
+    W("gat", "rmat", 14, 8, 64, heads=1, layers=2, act="elu"),
+    W("gat", "kron", 14, 8, 64, heads=2, layers=2, act="none"),
+    W("agnn", "rmat", 14, 16, 128, layers=2, act="elu"),  # C3 shape (R-MAT, k=128)
     W("agnn", "kron", 13, 8, 64, act="elu"),
     W("agnn", "er", 0, 0, 256, n=1500, samples=9000, act="none", beta=1.5),
     W("agnn", "er", 0, 0, 16, n=1024, samples=7680),
@@ -93,8 +95,12 @@ def test_layer_parity(w):
     src, dst, rp, ci = pu.host_graph(w)
     g = pu.device_graph(w, src, dst)
     np.testing.assert_array_equal(g.col_idx.cpu().numpy(), ci)
-    st = pu.gpu_step(w, graph=g)
     H, Ws, As, R = w.host_inputs()
+    if w.act == "relu":
+        assert w.layers == 1, "multi-layer ReLU backward has inner-layer kink decisions (A6')"
+        f0 = pu.oracle_step(dataclasses.replace(w), rp, ci, H, Ws, As, R)["fwd"][-1]
+        R = pu.relu_kink_mask(w, f0["Z"], R)
+    st = pu.gpu_step(w, graph=g, R=R)
     np.testing.assert_array_equal(st.H[0].cpu().numpy(), H)
     ref = pu.oracle_step(w, rp, ci, H, Ws, As, R)
     pu.compare(w, st, ref)
