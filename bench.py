@@ -43,6 +43,8 @@ def parse():
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--scale", type=int, default=None,
+                   help="override log2 n of the workload (same recipe and edge factor)")
     p.add_argument("--cpu-sample-scale", type=int, default=17,
                    help="log2 n of the bounded oracle sample (same recipe as the workload)")
     return p.parse_args()
@@ -139,13 +141,24 @@ def cpu_model():
     return "unknown"
 
 
+def workload(args):
+    from paper_conf_sc_bestarglzcgssci23_b200 import gen
+    w = gen.CONFIGS[args.config]
+    if args.scale is not None and w.graph != "er":
+        ef = w.n_samples // w.n
+        w = gen.Workload(f"{w.name}@2^{args.scale}", w.model, w.graph, args.scale, 1 << args.scale,
+                         ef << args.scale, w.k, w.heads, w.layers, w.seed, w.act, w.slope, w.beta,
+                         w.eps)
+    return w
+
+
 def run_reference(args):
     """--impl reference: the FP64 oracle (this tier's reference arm) on host cores."""
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
     from paper_conf_sc_bestarglzcgssci23_b200 import gen
-    w = gen.CONFIGS[args.config]
+    w = workload(args)
     ws = oracle_sample(w, args.cpu_sample_scale)
     sys.path.insert(0, os.path.join(ROOT, "oracle"))
     sys.path.insert(0, os.path.join(ROOT, "tests"))
@@ -219,7 +232,7 @@ def run_ours(args):
     if world > 1:
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
         dist.init_process_group("nccl", device_id=dev)
-    w = gen.CONFIGS[args.config]
+    w = workload(args)
     agnn.lib()
     uid = None
     if world > 1:

@@ -140,6 +140,8 @@ struct Plan {
   int32_t* heavy_rows = nullptr;      // [n_heavy]
   int32_t* heavy_off = nullptr;       // [n_heavy+1] chunk ranges
   void* meta_block = nullptr;         // single allocation backing the lists
+  int32_t* empty_rows = nullptr;      // [n_empty] local rows without stored entries
+  int64_t n_empty = 0;
   // distribution
   int rank = 0, world = 1;
   int64_t* bounds = nullptr;          // host [world+1]

@@ -22,7 +22,7 @@
 // result does not depend on launch geometry or on the number of GPUs.
 #include <cfloat>
 
-#include "internal.cuh"
+#include "gat_args.cuh"
 
 namespace agnn {
 
@@ -31,21 +31,13 @@ namespace {
 constexpr unsigned FULL = 0xffffffffu;
 constexpr float NEG_INF = -INFINITY;
 
-struct FwdOut {
-  float* Z;      // [n_local x K]   nullable (inference)
-  float* Hout;   // [n_local x K]
-  float* m;      // [n_local x NH]  nullable
-  float* l;      // [n_local x NH]  nullable
-  float* pacc;   // [n_chunks x K]
-  float* pm;     // [n_chunks x NH]
-  float* pl;     // [n_chunks x NH]
-};
+using FwdOut = GatFwdOut;
 
 __device__ __forceinline__ void merge_softmax(float& m, float& l, float4& acc, float m2, float l2,
                                               float4 acc2) {
   const float mn = fmaxf(m, m2);
   if (mn == NEG_INF) return;
-  const float x = ex2((m - mn) * kLog2e), y = ex2((m2 - mn) * kLog2e);
+  const float x = ex2(m - mn), y = ex2(m2 - mn);
   l = l * x + l2 * y;
   acc = make_float4(fmaf(acc.x, x, acc2.x * y), fmaf(acc.y, x, acc2.y * y),
                     fmaf(acc.z, x, acc2.z * y), fmaf(acc.w, x, acc2.w * y));
@@ -144,13 +136,13 @@ gat_fwd_kernel(Items it, const float* __restrict__ P, const float* __restrict__ 
             if (val[u]) mn = fmaxf(mn, ev[u]);
           }
           if (mn != NEG_INF) {
-            const float sc = ex2((m[v] - mn) * kLog2e);
+            const float sc = ex2(m[v] - mn);
             l[v] *= sc;
             acc[v] = mul4(sc, acc[v]);
 #pragma unroll
             for (int u = 0; u < U; ++u) {
               if (val[u]) {
-                const float p = ex2((ev[u] - mn) * kLog2e);
+                const float p = ex2(ev[u] - mn);
                 l[v] += p;
                 acc[v] = fma4(p, pj[u][v], acc[v]);
               }
@@ -230,21 +222,7 @@ gat_fwd_merge_kernel(Items it, int act, FwdOut o) {
 }
 
 // ---------------------------------------------------------------- backward
-struct BwdArgs {
-  const float* P;      // [n_tot x K]
-  const float* st;     // [n_tot x 2NH]   (s | t)
-  const float* G;      // [n_tot x K]
-  const float4* rec;   // [n_tot x NH]    {s, m, 1/l, delta}
-  const float* a;      // [NH x 2D]
-  float slope;
-  float* dP;           // [n_local x K]
-  float* pacc;         // [n_chunks x K]
-  float* pds;          // [n_chunks x NH]
-  float* pdt;          // [n_chunks x NH]
-  float* da_part;      // [warps x 2K]
-  float* ds_out;       // [n_local x NH] nullable
-  float* dt_out;       // [n_local x NH] nullable
-};
+using BwdArgs = GatBwdArgs;
 
 template <int K, int NH>
 __device__ __forceinline__ void bwd_finish(const BwdArgs& A, int64_t row, int64_t grow, int q,
@@ -342,12 +320,12 @@ gat_bwd_kernel(Items it, BwdArgs A) {
               // row role: entry (j,i) of row j, centre j
               const float pre = rj[v].x + ti[u][v];
               const float e = pre > 0.f ? pre : slope * pre;
-              const float aji = ex2((e - rj[v].y) * kLog2e) * rj[v].z;
+              const float aji = ex2(e - rj[v].y) * rj[v].z;
               ds[v] = fmaf(aji * (pre > 0.f ? 1.f : slope), d1[v] - rj[v].w, ds[v]);
               // column role: entry (i,j) of row i, centre i
               const float pre2 = ri[u][v].x + tj[v];
               const float e2 = pre2 > 0.f ? pre2 : slope * pre2;
-              const float aij = ex2((e2 - ri[u][v].y) * kLog2e) * ri[u][v].z;
+              const float aij = ex2(e2 - ri[u][v].y) * ri[u][v].z;
               dt[v] = fmaf(aij * (pre2 > 0.f ? 1.f : slope), d2[v] - ri[u][v].w, dt[v]);
               acc[v] = fma4(aij, Gi[u][v], acc[v]);
             }
@@ -487,7 +465,9 @@ __global__ void gat_da_reduce_kernel(const float* __restrict__ part, int64_t row
   da[h * 2 * D + (c2 >= K ? D : 0) + cc] = s;
 }
 
-// W_ext = [W | W a1^h ... | W a2^h ...]   (a' = W a, Table 2)
+// W_ext = [W | log2e W a1^h ... | log2e W a2^h ...]   (a' = W a, Table 2).
+// The scores s, t (and the saved row maxima m) are stored in log2 units so every
+// exponential is a single ex2; LReLU commutes with the positive scale.
 __global__ void gat_wext_kernel(const float* __restrict__ W, const float* __restrict__ a, int k_in,
                                 int K, int NH, int NE, float* __restrict__ Wext) {
   const int D = K / NH;
@@ -503,6 +483,7 @@ __global__ void gat_wext_kernel(const float* __restrict__ W, const float* __rest
       const int h = (c - K) % NH, which = (c - K) / NH;
       v = 0.f;
       for (int x = 0; x < D; ++x) v = fmaf(W[r * K + h * D + x], a[h * 2 * D + which * D + x], v);
+      v *= kLog2e;  // scores are kept in log2 units: e2 = LReLU(s2 + t2) = log2(e) * e_nat
     }
     Wext[idx] = v;
   }
@@ -527,7 +508,7 @@ __global__ void gat_debug_alpha_kernel(const int64_t* __restrict__ rp, int64_t n
   const int64_t j = col[e];
   const float pre = st[(row_begin + lo) * 2 * NH + h] + st[j * 2 * NH + NH + h];
   const float x = pre > 0.f ? pre : slope * pre;
-  out[t] = expf(x - mrow[lo * NH + h]) / lrow[lo * NH + h];
+  out[t] = exp2f(x - mrow[lo * NH + h]) / lrow[lo * NH + h];
 }
 
 // ---------------------------------------------------------------- layout
@@ -632,7 +613,9 @@ agnn_status gat_forward(const Plan& p, const GatShape& g, const float* W, const 
   Items it = items_of(p);
   FwdOut o{saved ? sv.Z : nullptr, H_out, saved ? sv.m : nullptr, saved ? sv.l : nullptr,
            w.pacc, w.pm, w.pl};
-  if (it.n_chunks + it.n_light > 0) {
+  if (gat_k128_supported(g.k_out, g.heads)) {
+    if ((st = gat_fwd_k128(it, g.heads, sv.P, sv.st, g.slope, g.act, o, s)) != AGNN_OK) return st;
+  } else if (it.n_chunks + it.n_light > 0) {
     AGNN_GAT_DISPATCH(K_, NH_, (gat_fwd_kernel<K, NH, fwd_unroll<K>()>
                                 <<<grid_of(gat_fwd_kernel<K, NH, fwd_unroll<K>()>), kSparseThreads,
                                    0, s>>>(it, sv.P, sv.st, g.slope, g.act, o)));
@@ -670,20 +653,25 @@ agnn_status gat_backward(const Plan& p, const GatShape& g, const float* W, const
   BwdArgs A{sv.P, sv.st, w.G, w.rec, a, g.slope, w.dP, w.pacc, w.pm, w.pl, w.da_part,
             nullptr, nullptr};
   int64_t main_warps = 0, merge_warps = 0;
-  AGNN_GAT_DISPATCH(K_, NH_, (main_warps = (int64_t)grid_of(gat_bwd_kernel<K, NH, bwd_unroll<K>()>) *
-                                           (kSparseThreads / 32),
-                              merge_warps = (int64_t)grid_of(gat_bwd_merge_kernel<K, NH>) *
+  if (gat_k128_supported(g.k_out, g.heads)) {
+    if ((st = gat_bwd_k128(it, g.heads, A, &main_warps, s)) != AGNN_OK) return st;
+  } else {
+    AGNN_GAT_DISPATCH(K_, NH_, (main_warps = (int64_t)grid_of(gat_bwd_kernel<K, NH, bwd_unroll<K>()>) *
+                                             (kSparseThreads / 32)));
+    AGNN_GAT_DISPATCH(K_, NH_, (gat_bwd_kernel<K, NH, bwd_unroll<K>()>
+                                <<<(unsigned)(main_warps / 8), kSparseThreads, 0, s>>>(it, A)));
+    AGNN_LAUNCH_CHECK("gat_bwd_kernel");
+  }
+  AGNN_GAT_DISPATCH(K_, NH_, (merge_warps = (int64_t)grid_of(gat_bwd_merge_kernel<K, NH>) *
                                             (kSparseThreads / 32)));
-  AGNN_GAT_DISPATCH(K_, NH_, (gat_bwd_kernel<K, NH, bwd_unroll<K>()>
-                              <<<(unsigned)(main_warps / 8), kSparseThreads, 0, s>>>(it, A)));
-  AGNN_LAUNCH_CHECK("gat_bwd_kernel");
   AGNN_GAT_DISPATCH(K_, NH_, (gat_bwd_merge_kernel<K, NH>
                               <<<(unsigned)(merge_warps / 8), kSparseThreads, 0, s>>>(it, A,
                                                                                      main_warps)));
   AGNN_LAUNCH_CHECK("gat_bwd_merge_kernel");
+  const int64_t da_rows_used = main_warps + merge_warps;
   if (da) {
     gat_da_reduce_kernel<<<(2 * g.k_out + 127) / 128, 128, 0, s>>>(
-        w.da_part, main_warps + merge_warps, g.k_out, g.k_out / g.heads, da);
+        w.da_part, da_rows_used, g.k_out, g.k_out / g.heads, da);
     AGNN_LAUNCH_CHECK("gat_da_reduce_kernel");
     if (p.world > 1 && (st = allreduce_sum(p, da, 2 * (int64_t)g.k_out, s)) != AGNN_OK) return st;
   }

@@ -1,0 +1,40 @@
+// gat_args.cuh — argument blocks shared by the GAT sparse kernels (gat.cu, gat_k128.cu)
+#pragma once
+#include "internal.cuh"
+
+namespace agnn {
+
+struct GatFwdOut {
+  float* Z;      // [n_local x K]   nullable (inference)
+  float* Hout;   // [n_local x K]
+  float* m;      // [n_local x NH]  nullable
+  float* l;      // [n_local x NH]  nullable
+  float* pacc;   // [n_chunks x K]
+  float* pm;     // [n_chunks x NH]
+  float* pl;     // [n_chunks x NH]
+};
+
+struct GatBwdArgs {
+  const float* P;      // [n_tot x K]
+  const float* st;     // [n_tot x 2NH]   (s | t)
+  const float* G;      // [n_tot x K]
+  const float4* rec;   // [n_tot x NH]    {s, m, 1/l, delta}
+  const float* a;      // [NH x 2D]
+  float slope;
+  float* dP;           // [n_local x K]
+  float* pacc;         // [n_chunks x K]
+  float* pds;          // [n_chunks x NH]
+  float* pdt;          // [n_chunks x NH]
+  float* da_part;      // [warps x 2K]
+  float* ds_out;       // [n_local x NH] nullable
+  float* dt_out;       // [n_local x NH] nullable
+};
+
+// k' = 128 kernels (gat_k128.cu): lane-parallel scalar work, warp-parallel rows
+bool gat_k128_supported(int k_out, int heads);
+agnn_status gat_fwd_k128(const Items& it, int heads, const float* P, const float* st, float slope,
+                         int act, const GatFwdOut& o, cudaStream_t s);
+agnn_status gat_bwd_k128(const Items& it, int heads, const GatBwdArgs& A, int64_t* warps,
+                         cudaStream_t s);
+
+}  // namespace agnn

@@ -22,6 +22,7 @@ struct Items {
 };
 Items items_of(const Plan& p);
 
+
 // persistent sparse-kernel grid: 256-thread blocks, SMs x resident blocks of `func`
 constexpr int kSparseThreads = 256;
 constexpr int kMaxSparseBlocks = kNumSMs * 8;

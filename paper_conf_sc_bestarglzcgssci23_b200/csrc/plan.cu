@@ -116,12 +116,13 @@ agnn_status plan_build(Plan& p, cudaStream_t s) {
   }
   p.nnz = rp[(size_t)p.n_local];
   // 3. work lists
-  std::vector<int32_t> light, chunk_row, chunk_idx, heavy, heavy_off{0};
+  std::vector<int32_t> light, chunk_row, chunk_idx, heavy, heavy_off{0}, empty;
   light.reserve((size_t)p.n_local);
   int64_t maxdeg = 0;
   for (int64_t i = 0; i < p.n_local; ++i) {
     const int64_t d = rp[(size_t)i + 1] - rp[(size_t)i];
     maxdeg = std::max(maxdeg, d);
+    if (d == 0) empty.push_back((int32_t)i);
     if (d > p.chunk) {
       const int64_t c = (d + p.chunk - 1) / p.chunk;
       heavy.push_back((int32_t)i);
@@ -138,7 +139,9 @@ agnn_status plan_build(Plan& p, cudaStream_t s) {
   p.n_light = (int64_t)light.size();
   p.n_heavy = (int64_t)heavy.size();
   p.n_chunks = (int64_t)chunk_row.size();
-  const size_t total = light.size() + 2 * chunk_row.size() + heavy.size() + heavy_off.size() + 128;
+  p.n_empty = (int64_t)empty.size();
+  const size_t total = light.size() + 2 * chunk_row.size() + heavy.size() + heavy_off.size() +
+                       empty.size() + 160;
   AGNN_CUDA_TRY(cudaMalloc(&p.meta_block, sizeof(int32_t) * total));
   int32_t* b = static_cast<int32_t*>(p.meta_block);
   auto put = [&](std::vector<int32_t>& v, int32_t*& dst) -> cudaError_t {
@@ -152,6 +155,7 @@ agnn_status plan_build(Plan& p, cudaStream_t s) {
   AGNN_CUDA_TRY(put(chunk_idx, p.chunk_idx));
   AGNN_CUDA_TRY(put(heavy, p.heavy_rows));
   AGNN_CUDA_TRY(put(heavy_off, p.heavy_off));
+  AGNN_CUDA_TRY(put(empty, p.empty_rows));
   AGNN_CUDA_TRY(cudaStreamSynchronize(s));
   return AGNN_OK;
 }
