@@ -547,7 +547,7 @@ WsGat carve_ws(const Plan& p, const GatShape& g, void* base, size_t* total) {
   WsGat w;
   const int NE = (g.k_out + 2 * g.heads + 3) / 4 * 4;
   w.Wext = c.take<float>((size_t)g.k_in * NE);
-  w.pacc = c.take<float>((size_t)p.n_chunks * g.k_out);
+  w.pacc = c.take<float>((size_t)p.n_chunks * 3 * g.k_out);
   w.pm = c.take<float>((size_t)p.n_chunks * g.heads);
   w.pl = c.take<float>((size_t)p.n_chunks * g.heads);
   w.G = c.take<float>((size_t)p.n * g.k_out);

@@ -22,7 +22,7 @@ struct GatBwdArgs {
   const float* a;      // [NH x 2D]
   float slope;
   float* dP;           // [n_local x K]
-  float* pacc;         // [n_chunks x K]
+  float* pacc;         // [n_chunks x 3K] heavy-row chunk partials
   float* pds;          // [n_chunks x NH]
   float* pdt;          // [n_chunks x NH]
   float* da_part;      // [warps x 2K]

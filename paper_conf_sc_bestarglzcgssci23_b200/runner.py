@@ -37,6 +37,19 @@ def build_graph(w: gen.Workload, device, stream=None) -> Graph:
     return Graph(w.n, rp, ci, int(ci.numel()))
 
 
+def row_block(row_ptr_host, world: int, rank: int, c_v: int = 4):
+    """1D row-block of `rank` (reading A20): (bounds, row_begin, row_end, edge_begin, edge_end).
+
+    Pure host logic (agnn_partition from libagnn.so on the host row_ptr); the
+    rank keeps rows [row_begin, row_end) and stored entries [edge_begin, edge_end)
+    of the global CSR, with its local row_ptr = row_ptr[row_begin:row_end+1] - edge_begin.
+    """
+    rp = np.ascontiguousarray(row_ptr_host, dtype=np.int64)
+    bounds = agnn.partition(rp, world, c_v) if world > 1 else np.array([0, len(rp) - 1], np.int64)
+    b0, b1 = int(bounds[rank]), int(bounds[rank + 1])
+    return bounds, b0, b1, int(rp[b0]), int(rp[b1])
+
+
 class Stack:
     """Buffers + plan + model for one workload on this rank."""
 
@@ -47,10 +60,7 @@ class Stack:
         g = graph or build_graph(w, self.device)
         self.graph = g
         if world > 1:
-            rp_host = g.row_ptr.cpu().numpy()
-            self.bounds = agnn.partition(rp_host, world, c_v)
-            b0, b1 = int(self.bounds[rank]), int(self.bounds[rank + 1])
-            e0, e1 = int(rp_host[b0]), int(rp_host[b1])
+            self.bounds, b0, b1, e0, e1 = row_block(g.row_ptr.cpu().numpy(), world, rank, c_v)
             self.row_ptr = (g.row_ptr[b0:b1 + 1] - e0).contiguous()
             self.col_idx = g.col_idx[e0:e1].contiguous()
         else:
