@@ -161,6 +161,12 @@ agnn_status agnn_debug_attention(agnn_model_t model, int layer, const void* save
                                  const float* H_in, const int64_t* edge_pos, int64_t count,
                                  float* alpha_out, cudaStream_t stream);
 
+/* Test-only export: C[M x N] = A[M x K] B^T with B given as [N x K], through the
+ * same dense-projection path the layers use (tcgen05 3xTF32 when the shape has
+ * an instantiation, else fp32 FFMA).  Device pointers, row-major.          */
+agnn_status agnn_debug_gemm(const float* A, int64_t M, int K, const float* B, int N, float* C,
+                            cudaStream_t stream);
+
 /* Number of kernels this library launched since load (all entry points).   */
 uint64_t agnn_launch_count(void);
 

@@ -27,7 +27,8 @@ STATUS = {0: "AGNN_OK", 1: "AGNN_EINVAL", 2: "AGNN_ECUDA", 3: "AGNN_ENCCL", 4: "
 # every symbol include/agnn.h declares (tests check the .so exports all of them)
 EXPORTS = ("agnn_partition", "agnn_plan_create", "agnn_plan_destroy", "agnn_plan_info",
            "agnn_model_create", "agnn_model_destroy", "agnn_saved_bytes", "agnn_workspace_bytes",
-           "agnn_forward", "agnn_backward", "agnn_debug_attention", "agnn_launch_count",
+           "agnn_forward", "agnn_backward", "agnn_debug_attention", "agnn_debug_gemm",
+           "agnn_launch_count",
            "agnn_profile_enable", "agnn_profile_report", "agnn_profile_reset",
            "agnn_nccl_unique_id", "agnn_csr_build", "agnn_free", "agnn_status_string",
            "agnn_last_error")
@@ -117,6 +118,12 @@ def profile_report() -> dict:
         name, cnt, ms = line.rsplit(" ", 2)
         out[name] = (int(cnt), float(ms))
     return out
+
+
+def debug_gemm(A, B, C, stream=None):
+    """C = A @ B.T through the library's projection GEMM (test-only)."""
+    _check(lib().agnn_debug_gemm(_ptr(A), ctypes.c_int64(A.shape[0]), ctypes.c_int(A.shape[1]),
+                                 _ptr(B), ctypes.c_int(B.shape[0]), _ptr(C), _stream(stream)))
 
 
 def nccl_unique_id() -> bytes:

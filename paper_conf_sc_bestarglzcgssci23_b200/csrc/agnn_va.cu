@@ -427,7 +427,7 @@ SavedAv carve_saved(const Plan& p, const agnn_layer_desc& d, void* base, size_t*
 }
 
 struct WsAv {
-  float *pacc, *pl, *G, *M, *gemm;
+  float *pacc, *pl, *G, *M, *gemm, *WT;
   float4* rec;
   void* saved_inf;
 };
@@ -442,6 +442,7 @@ WsAv carve_ws(const Plan& p, const agnn_layer_desc& d, void* base, size_t* total
   w.M = c.take<float>((size_t)p.n * d.k_in);
   w.rec = c.take<float4>(d.kind == AGNN_AGNN ? (size_t)p.n : 0);
   w.gemm = c.take<float>(gemm_tn_ws_floats(d.k_in, d.k_out));
+  w.WT = c.take<float>((size_t)d.k_in * d.k_out);
   w.saved_inf = c.take<char>(sv);
   if (total) *total = c.off + 256;
   return w;
@@ -511,8 +512,9 @@ agnn_status av_forward(const Plan& p, const agnn_layer_desc& d, const float* W, 
                                <<<kNumSMs * 2, kSparseThreads, 0, s>>>(it, A)));
     AGNN_LAUNCH_CHECK("av_fwd_merge_kernel");
   }
-  // Z = X W ; H_out = sigma(Z)
-  return gemm_rows(sv.X, p.n_local, d.k_in, W, false, d.k_out, saved ? sv.Z : nullptr, d.k_out,
+  // Z = X W ; H_out = sigma(Z)   (B = W^T as [k_out x k_in] for the tensor-core path)
+  if ((st = transpose(W, d.k_in, d.k_out, w.WT, s)) != AGNN_OK) return st;
+  return gemm_rows(sv.X, p.n_local, d.k_in, w.WT, true, d.k_out, saved ? sv.Z : nullptr, d.k_out,
                    nullptr, s, H_out, (int)d.act);
 }
 

@@ -154,6 +154,13 @@ const char* agnn_last_error(void) { return g_last_error.c_str(); }
 
 uint64_t agnn_launch_count(void) { return g_launches.load(); }
 
+agnn_status agnn_debug_gemm(const float* A, int64_t M, int K, const float* B, int N, float* C,
+                            cudaStream_t s) {
+  if (!A || !B || !C || M < 0 || K <= 0 || N <= 0)
+    return fail(AGNN_EINVAL, "agnn_debug_gemm: bad arguments");
+  return gemm_rows(A, M, K, B, true, N, C, N, nullptr, s);
+}
+
 agnn_status agnn_profile_enable(int on) {
   std::lock_guard<std::mutex> lock(g_prof_mu);
   g_profiling = on != 0;

@@ -469,11 +469,11 @@ __global__ void gat_da_reduce_kernel(const float* __restrict__ part, int64_t row
 // The scores s, t (and the saved row maxima m) are stored in log2 units so every
 // exponential is a single ex2; LReLU commutes with the positive scale.
 __global__ void gat_wext_kernel(const float* __restrict__ W, const float* __restrict__ a, int k_in,
-                                int K, int NH, int NE, float* __restrict__ Wext) {
+                                int K, int NH, int NE, float* __restrict__ WextT) {
   const int D = K / NH;
   for (int idx = blockIdx.x * blockDim.x + threadIdx.x; idx < k_in * NE;
        idx += gridDim.x * blockDim.x) {
-    const int r = idx / NE, c = idx % NE;
+    const int c = idx / k_in, r = idx % k_in;  // output [NE x k_in] (B given as [N x K])
     float v;
     if (c < K) {
       v = W[r * K + c];
@@ -485,7 +485,7 @@ __global__ void gat_wext_kernel(const float* __restrict__ W, const float* __rest
       for (int x = 0; x < D; ++x) v = fmaf(W[r * K + h * D + x], a[h * 2 * D + which * D + x], v);
       v *= kLog2e;  // scores are kept in log2 units: e2 = LReLU(s2 + t2) = log2(e) * e_nat
     }
-    Wext[idx] = v;
+    WextT[idx] = v;
   }
 }
 
@@ -602,7 +602,7 @@ agnn_status gat_forward(const Plan& p, const GatShape& g, const float* W, const 
   gat_wext_kernel<<<64, 256, 0, s>>>(W, a, g.k_in, g.k_out, g.heads, NE, w.Wext);
   AGNN_LAUNCH_CHECK("gat_wext_kernel");
   // P (and s, t) for the local rows, written at their global offsets
-  agnn_status st = gemm_rows(H_in, p.n_local, g.k_in, w.Wext, false, NE,
+  agnn_status st = gemm_rows(H_in, p.n_local, g.k_in, w.Wext, true, NE,
                              sv.P + p.row_begin * g.k_out, g.k_out,
                              sv.st + p.row_begin * 2 * g.heads, s, nullptr, 0, NEs);
   if (st != AGNN_OK) return st;

@@ -183,6 +183,12 @@ gemm_tn_kernel(const float* __restrict__ A, int64_t M, int K1, const float* __re
   }
 }
 
+__global__ void transpose_kernel(const float* __restrict__ X, int rows, int cols,
+                                 float* __restrict__ Y) {
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < rows * cols; i += gridDim.x * blockDim.x)
+    Y[(i % cols) * rows + i / cols] = X[i];
+}
+
 __global__ void sum_splits_kernel(const float* __restrict__ part, int splits, int64_t count,
                                   float* __restrict__ C) {
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -194,16 +200,30 @@ __global__ void sum_splits_kernel(const float* __restrict__ part, int splits, in
 
 }  // namespace
 
+agnn_status gemm_tc(const float* A, int64_t M, int K, const float* B, int n_real, float* C0,
+                    int n_split, float* C1, int n_store, float* Cact, int act, cudaStream_t s);
+
 agnn_status gemm_rows(const float* A, int64_t M, int K, const float* B, bool b_trans, int N,
                       float* C0, int n_split, float* C1, cudaStream_t s, float* Cact, int act,
                       int n_store) {
   if (M <= 0) return AGNN_OK;
+  if (b_trans) {  // tcgen05 3xTF32 path when the shape has an instantiation
+    const int ns = (n_store <= 0 || n_store > N) ? N : n_store;
+    const agnn_status st = gemm_tc(A, M, K, B, ns, C0, n_split, C1, ns, Cact, act, s);
+    if (st != AGNN_EUNSUPPORTED) return st;
+  }
   if (K % 4 || N % 4) return fail(AGNN_EINVAL, "gemm_rows: K and N must be multiples of 4");
   dim3 grid((unsigned)((M + BM - 1) / BM), (N + BN - 1) / BN);
   if (n_store <= 0 || n_store > N) n_store = N;
   gemm_rows_kernel<<<grid, TPB, 0, s>>>(A, M, K, B, b_trans ? 1 : 0, N, C0, n_split, C1, Cact,
                                         act, n_store);
   AGNN_LAUNCH_CHECK("gemm_rows_kernel");
+  return AGNN_OK;
+}
+
+agnn_status transpose(const float* X, int rows, int cols, float* Y, cudaStream_t s) {
+  transpose_kernel<<<64, 256, 0, s>>>(X, rows, cols, Y);
+  AGNN_LAUNCH_CHECK("transpose_kernel");
   return AGNN_OK;
 }
 

@@ -42,6 +42,8 @@ agnn_status gemm_rows(const float* A, int64_t M, int K, const float* B, bool b_t
 // partials in `ws` (gemm_tn_ws_floats) and an ordered reduction.  If accumulate,
 // C += result.
 size_t gemm_tn_ws_floats(int K1, int N);
+// Y[cols x rows] = X[rows x cols]^T (small weight matrices)
+agnn_status transpose(const float* X, int rows, int cols, float* Y, cudaStream_t s);
 agnn_status gemm_tn(const float* A, int64_t M, int K1, const float* B, int N, float* C,
                     float* ws, cudaStream_t s);
 

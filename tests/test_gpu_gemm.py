@@ -1,0 +1,43 @@
+"""The dense projection GEMM (tcgen05 3xTF32 / fp32 FFMA) against fp64 numpy.
+
+PAPER.md:141 (H' = HW) / :149 (MM).  Outputs are pre-filled with garbage (NaN)
+so a missed store or a race shows up; every shape is run several times and
+must be bitwise reproducible.
+"""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = [pytest.mark.gpu,
+              pytest.mark.skipif(not torch.cuda.is_available(), reason="needs a CUDA device")]
+
+from paper_conf_sc_bestarglzcgssci23_b200 import agnn  # noqa: E402
+
+
+@pytest.mark.parametrize("M,K,N", [(128, 128, 128), (1000, 128, 144), (65536, 64, 66),
+                                   (300001, 128, 136), (4097, 64, 64), (77, 128, 128),
+                                   (20000, 128, 130)])
+def test_gemm_against_fp64(M, K, N):
+    g = torch.Generator(device="cpu").manual_seed(M + K + N)
+    A = (torch.rand((M, K), generator=g) * 2 - 1).cuda()
+    B = (torch.rand((N, K), generator=g) * 2 - 1).mul_(K ** -0.5).cuda()
+    ref = A.double().cpu().numpy() @ B.double().cpu().numpy().T
+    outs = []
+    for rep in range(3):
+        C = torch.full((M, N), float("nan"), device="cuda")
+        agnn.debug_gemm(A, B, C)
+        torch.cuda.synchronize()
+        outs.append(C.cpu().numpy())
+    for o in outs[1:]:
+        assert np.array_equal(o, outs[0]), "GEMM not reproducible"
+    c = outs[0].astype(np.float64)
+    assert np.isfinite(c).all()
+    err = np.abs(c - ref)
+    # fp32-class accuracy: elementwise within 1e-6 of the dot's magnitude sum_k |a||b|
+    # (3xTF32 with tensor-core fp32 accumulation measures <= 5.2e-7; an fp32 FFMA
+    # dot is ~1e-7), normwise <= 5e-7 -- far inside the layers' 1e-5 parity bar
+    scale = np.abs(A.double().cpu().numpy()) @ np.abs(B.double().cpu().numpy()).T
+    assert (err <= 1e-6 * scale + 1e-30).all(), float((err / scale).max())
+    assert np.linalg.norm(c - ref) / np.linalg.norm(ref) < 5e-7
