@@ -614,7 +614,7 @@ agnn_status gat_forward(const Plan& p, const GatShape& g, const float* W, const 
   FwdOut o{saved ? sv.Z : nullptr, H_out, saved ? sv.m : nullptr, saved ? sv.l : nullptr,
            w.pacc, w.pm, w.pl};
   if (gat_k128_supported(g.k_out, g.heads)) {
-    if ((st = gat_fwd_k128(it, g.heads, sv.P, sv.st, g.slope, g.act, o, s)) != AGNN_OK) return st;
+    if ((st = gat_fwd_k128(it, g.heads, sv.P, sv.st, g.slope, g.act, o, p.n, s)) != AGNN_OK) return st;
   } else if (it.n_chunks + it.n_light > 0) {
     AGNN_GAT_DISPATCH(K_, NH_, (gat_fwd_kernel<K, NH, fwd_unroll<K>()>
                                 <<<grid_of(gat_fwd_kernel<K, NH, fwd_unroll<K>()>), kSparseThreads,

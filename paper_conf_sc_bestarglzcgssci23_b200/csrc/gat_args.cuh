@@ -33,7 +33,7 @@ struct GatBwdArgs {
 // k' = 128 kernels (gat_k128.cu): lane-parallel scalar work, warp-parallel rows
 bool gat_k128_supported(int k_out, int heads);
 agnn_status gat_fwd_k128(const Items& it, int heads, const float* P, const float* st, float slope,
-                         int act, const GatFwdOut& o, cudaStream_t s);
+                         int act, const GatFwdOut& o, int64_t n_rows, cudaStream_t s);
 agnn_status gat_bwd_k128(const Items& it, int heads, const GatBwdArgs& A, int64_t* warps,
                          cudaStream_t s);
 
