@@ -411,8 +411,15 @@ struct Transpose {
   }
 };
 
-template <int NH, int B>
-__global__ void __launch_bounds__(256, 3)
+template <int B>
+struct BwdBatch {  // operands of one batch of B edges held by one lane
+  float4 Pi[B], Gi[B];
+  float4 ri;
+  float ti;
+};
+
+template <int NH, int B, int MINB>
+__global__ void __launch_bounds__(256, MINB)
 gat_bwd_k128_kernel(Items it, GatBwdArgs A) {
   constexpr int D = K / NH, HL = D / 4;
   static_assert(B <= HL && (B & (B - 1)) == 0, "B edges per batch, at most one per head lane");
@@ -425,6 +432,8 @@ gat_bwd_k128_kernel(Items it, GatBwdArgs A) {
   const int64_t nitems = it.n_chunks + it.n_light;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const float* Pl = A.P + cq;
+  const float* Gl = A.G + cq;
   float4 da1 = f4(0.f), da2 = f4(0.f);
 
   for (int64_t w = gw; w < nitems; w += nw) {
@@ -437,48 +446,44 @@ gat_bwd_k128_kernel(Items it, GatBwdArgs A) {
     const float tj = __ldg(A.st + grow * (2 * NH) + NH + hv);
     float4 acc = f4(0.f);
     float dsp = 0.f, dtp = 0.f;
-    int cidx = 0;
-    for (int64_t b0 = beg; b0 < end; b0 += B) {
-      const int off32 = (int)((b0 - beg) & 31);
-      if (off32 == 0) {
-        const int64_t e = b0 + lane;
-        cidx = e < end ? __ldg(it.col + e) : 0;
-      }
-      const int cnt = (int)(end - b0 < B ? end - b0 : B);
-      float4 Pi[B], Gi[B];
+    // gathers of batch (window offset off, cnt valid edges): rows i of P, G and the
+    // record of the edge this lane owns after the reduction
+    auto load = [&](BwdBatch<B>& q, int cidx, int off, int cnt) {
 #pragma unroll
       for (int b = 0; b < B; ++b) {
-        const int64_t i = __shfl_sync(FULL, cidx, off32 + b);
+        const uint32_t i = (uint32_t)__shfl_sync(FULL, cidx, off + b);
         if (b < cnt) {
-          Pi[b] = ldg4(A.P + i * K + cq);
-          Gi[b] = ldg4(A.G + i * K + cq);
+          q.Pi[b] = ldg4(Pl + (int64_t)i * K);
+          q.Gi[b] = ldg4(Gl + (int64_t)i * K);
         } else {
-          Pi[b] = Gi[b] = f4(0.f);
+          q.Pi[b] = q.Gi[b] = f4(0.f);
         }
       }
-      // scalar operands of the edge this lane will own after the reduction
-      const int64_t im = __shfl_sync(FULL, cidx, off32 + my_b);
+      const uint32_t im = (uint32_t)__shfl_sync(FULL, cidx, off + my_b);
       const bool vm = my_b < cnt;
-      const float4 ri = vm ? __ldg(A.rec + im * NH + hv) : f4(0.f);
-      const float ti = vm ? __ldg(A.st + im * (2 * NH) + NH + hv) : 0.f;
+      q.ri = vm ? __ldg(A.rec + (int64_t)im * NH + hv) : f4(0.f);
+      q.ti = vm ? __ldg(A.st + (int64_t)im * (2 * NH) + NH + hv) : 0.f;
+    };
+    auto body = [&](const BwdBatch<B>& q, int cnt) {
       float x1[B], x2[B];
 #pragma unroll
       for (int b = 0; b < B; ++b) {
-        x1[b] = dot4(Gj, Pi[b]);  // G_j . P_i  (row role)
-        x2[b] = dot4(Gi[b], Pj);  // G_i . P_j  (column role)
+        x1[b] = dot4(Gj, q.Pi[b]);  // G_j . P_i  (row role)
+        x2[b] = dot4(q.Gi[b], Pj);  // G_i . P_j  (column role)
       }
       TR::template reduce<HL>(x1, lane);
       TR::template reduce<HL>(x2, lane);
+      const bool vm = my_b < cnt;
       // row role: entry (j,i) of row j
-      const float pre = rj.x + ti;
+      const float pre = rj.x + q.ti;
       const float e = fmaxf(pre, slope * pre);
       const float aji = ex2(e - rj.y) * rj.z;
       const float dcji = aji * (pre > 0.f ? 1.f : slope) * (x1[0] - rj.w);
       // column role: entry (i,j) of row i
-      const float pre2 = ri.x + tj;
+      const float pre2 = q.ri.x + tj;
       const float e2 = fmaxf(pre2, slope * pre2);
-      float aij = ex2(e2 - ri.y) * ri.z;
-      const float dcij = aij * (pre2 > 0.f ? 1.f : slope) * (x2[0] - ri.w);
+      float aij = ex2(e2 - q.ri.y) * q.ri.z;
+      const float dcij = aij * (pre2 > 0.f ? 1.f : slope) * (x2[0] - q.ri.w);
       if (vm && owner) {
         dsp += dcji;
         dtp += dcij;
@@ -487,7 +492,30 @@ gat_bwd_k128_kernel(Items it, GatBwdArgs A) {
 #pragma unroll
       for (int b = 0; b < B; ++b) {
         const float ab = __shfl_sync(FULL, aij, gbase + TR::lane_of(b));
-        acc = fma4(ab, Gi[b], acc);
+        acc = fma4(ab, q.Gi[b], acc);
+      }
+    };
+    for (int64_t w0 = beg; w0 < end; w0 += 32) {
+      const int wcnt = (int)(end - w0 < 32 ? end - w0 : 32);
+      const int cidx = lane < wcnt ? __ldg(it.col + w0 + lane) : 0;
+      if (wcnt == 32) {
+        // full window: 32/B batches, the next batch's gathers in flight during this one
+        BwdBatch<B> qa, qb;
+        load(qa, cidx, 0, B);
+#pragma unroll
+        for (int bb = 0; bb < 32 / B; bb += 2) {
+          load(qb, cidx, (bb + 1) * B, B);
+          body(qa, B);
+          if (bb + 2 < 32 / B) load(qa, cidx, (bb + 2) * B, B);
+          body(qb, B);
+        }
+      } else {
+        for (int off = 0; off < wcnt; off += B) {
+          BwdBatch<B> q;
+          const int cnt = wcnt - off < B ? wcnt - off : B;
+          load(q, cidx, off, cnt);
+          body(q, cnt);
+        }
       }
     }
     // per-head row sums ds_j, dt_j: every lane of the head group ends with the total
@@ -621,10 +649,21 @@ agnn_status gat_fwd_k128(const Items& it, int heads, const float* P, const float
 agnn_status gat_bwd_k128(const Items& it, int heads, const GatBwdArgs& A, int64_t* warps,
                          cudaStream_t s) {
   *warps = 0;
+  static int minb = -1;
+  if (minb < 0) {
+    const char* e = getenv("AGNN_BWD_MINB");
+    minb = e ? atoi(e) : 2;
+  }
   AGNN_K128_DISPATCH(heads, ({
     constexpr int B = bwd_batch<NH>();
-    const int grid = grid_for(gat_bwd_k128_kernel<NH, B>);
-    gat_bwd_k128_kernel<NH, B><<<grid, 256, 0, s>>>(it, A);
+    int grid;
+    if (minb == 3) {
+      grid = grid_for(gat_bwd_k128_kernel<NH, B, 3>);
+      gat_bwd_k128_kernel<NH, B, 3><<<grid, 256, 0, s>>>(it, A);
+    } else {
+      grid = grid_for(gat_bwd_k128_kernel<NH, B, 2>);
+      gat_bwd_k128_kernel<NH, B, 2><<<grid, 256, 0, s>>>(it, A);
+    }
     AGNN_LAUNCH_CHECK("gat_bwd_kernel");
     *warps = (int64_t)grid * 8;
   }));
