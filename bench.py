@@ -295,8 +295,16 @@ def run_ours(args):
     # one launch per layer per step: alg bytes per launch over the mean launch time
     achieved = (alg / (dom_ms / 1e3) / 1e9) if dom_ms else None
     step_ms_prof = sum(v[1] for v in prof.values()) / args.steps
+    traffic = None
+    try:  # ncu DRAM bytes per launch of the same kernel on the same workload (committed)
+        tr = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))
+        if args.scale is None and world == 1:
+            traffic = tr.get(args.config, {}).get(dom)
+    except Exception:
+        traffic = None
     roof = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": hbm, "unit": "GB/s",
-            "frac": (achieved / hbm) if achieved else None, "traffic": None,
+            "frac": (achieved / hbm) if achieved else None, "traffic": traffic,
+            "dram_frac": (traffic / (dom_ms / 1e3) / 1e9 / hbm) if (traffic and dom_ms) else None,
             "peak_source": peak_src, "algorithmic_bytes_per_launch": alg,
             "bytes_per_edge": per_edge, "bytes_per_row": per_row,
             "launch_ms": dom_ms, "share_of_step": (tot / args.steps / step_ms_prof)

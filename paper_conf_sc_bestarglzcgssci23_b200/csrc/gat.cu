@@ -455,14 +455,29 @@ gat_bwd_prologue_kernel(int64_t n_local, int64_t row_begin, const float* __restr
 }
 
 // da[h][0:D] = sum_w part[w][c], da[h][D:2D] = sum_w part[w][K + c]   (fixed order)
-__global__ void gat_da_reduce_kernel(const float* __restrict__ part, int64_t rows, int K, int D,
-                                     float* __restrict__ da) {
-  const int c2 = blockIdx.x * blockDim.x + threadIdx.x;
-  if (c2 >= 2 * K) return;
+__global__ void __launch_bounds__(1024)
+gat_da_reduce_kernel(const float* __restrict__ part, int64_t rows, int K, int D,
+                     float* __restrict__ da) {
+  // block: 32 columns x 32 row-lanes; each row-lane sums a strided subset, then a
+  // fixed-order tree over the row-lanes (deterministic)
+  __shared__ float red[32][33];
+  const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;
+  const int c2 = blockIdx.x * 32 + tx;
   float s = 0.f;
-  for (int64_t r = 0; r < rows; ++r) s += part[r * 2 * K + c2];
-  const int c = c2 % K, h = c / D, cc = c % D;
-  da[h * 2 * D + (c2 >= K ? D : 0) + cc] = s;
+  if (c2 < 2 * K) {
+#pragma unroll 8
+    for (int64_t r = ty; r < rows; r += 32) s += part[r * 2 * K + c2];
+  }
+  red[ty][tx] = s;
+  __syncthreads();
+  for (int o = 16; o > 0; o >>= 1) {
+    if (ty < o) red[ty][tx] += red[ty + o][tx];
+    __syncthreads();
+  }
+  if (ty == 0 && c2 < 2 * K) {
+    const int c = c2 % K, h = c / D, cc = c % D;
+    da[h * 2 * D + (c2 >= K ? D : 0) + cc] = red[0][tx];
+  }
 }
 
 // W_ext = [W | log2e W a1^h ... | log2e W a2^h ...]   (a' = W a, Table 2).
@@ -670,7 +685,7 @@ agnn_status gat_backward(const Plan& p, const GatShape& g, const float* W, const
   AGNN_LAUNCH_CHECK("gat_bwd_merge_kernel");
   const int64_t da_rows_used = main_warps + merge_warps;
   if (da) {
-    gat_da_reduce_kernel<<<(2 * g.k_out + 127) / 128, 128, 0, s>>>(
+    gat_da_reduce_kernel<<<(2 * g.k_out + 31) / 32, 1024, 0, s>>>(
         w.da_part, da_rows_used, g.k_out, g.k_out / g.heads, da);
     AGNN_LAUNCH_CHECK("gat_da_reduce_kernel");
     if (p.world > 1 && (st = allreduce_sum(p, da, 2 * (int64_t)g.k_out, s)) != AGNN_OK) return st;
