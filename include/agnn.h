@@ -167,6 +167,13 @@ agnn_status agnn_debug_attention(agnn_model_t model, int layer, const void* save
 agnn_status agnn_debug_gemm(const float* A, int64_t M, int K, const float* B, int N, float* C,
                             cudaStream_t stream);
 
+/* Test-only export: C[K1 x N] = A^T B over the M rows of A [M x K1] and
+ * B [M x N] (the weight-gradient contraction, Eq. 5), with the
+ * split partials in `ws` (agnn_debug_gemm_tn_ws_bytes bytes, device).       */
+agnn_status agnn_debug_gemm_tn(const float* A, int64_t M, int K1, const float* B, int N, float* C,
+                               float* ws, cudaStream_t stream);
+size_t agnn_debug_gemm_tn_ws_bytes(int K1, int N);
+
 /* Number of kernels this library launched since load (all entry points).   */
 uint64_t agnn_launch_count(void);
 

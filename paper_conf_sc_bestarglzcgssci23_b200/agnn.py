@@ -28,6 +28,7 @@ STATUS = {0: "AGNN_OK", 1: "AGNN_EINVAL", 2: "AGNN_ECUDA", 3: "AGNN_ENCCL", 4: "
 EXPORTS = ("agnn_partition", "agnn_plan_create", "agnn_plan_destroy", "agnn_plan_info",
            "agnn_model_create", "agnn_model_destroy", "agnn_saved_bytes", "agnn_workspace_bytes",
            "agnn_forward", "agnn_backward", "agnn_debug_attention", "agnn_debug_gemm",
+           "agnn_debug_gemm_tn", "agnn_debug_gemm_tn_ws_bytes",
            "agnn_launch_count",
            "agnn_profile_enable", "agnn_profile_report", "agnn_profile_reset",
            "agnn_nccl_unique_id", "agnn_csr_build", "agnn_free", "agnn_status_string",
@@ -72,10 +73,11 @@ def lib(build: bool = True):
         L.agnn_status_string.restype = ctypes.c_char_p
         L.agnn_last_error.restype = ctypes.c_char_p
         L.agnn_launch_count.restype = ctypes.c_uint64
+        L.agnn_debug_gemm_tn_ws_bytes.restype = ctypes.c_size_t
         for name in EXPORTS:
             fn = getattr(L, name)
             if name not in ("agnn_status_string", "agnn_last_error", "agnn_launch_count",
-                            "agnn_free"):
+                            "agnn_free", "agnn_debug_gemm_tn_ws_bytes"):
                 fn.restype = ctypes.c_int
         _lib = L
     return _lib
@@ -124,6 +126,16 @@ def debug_gemm(A, B, C, stream=None):
     """C = A @ B.T through the library's projection GEMM (test-only)."""
     _check(lib().agnn_debug_gemm(_ptr(A), ctypes.c_int64(A.shape[0]), ctypes.c_int(A.shape[1]),
                                  _ptr(B), ctypes.c_int(B.shape[0]), _ptr(C), _stream(stream)))
+
+
+def debug_gemm_tn(A, B, C, stream=None):
+    """C = A.T @ B through the library's weight-gradient GEMM (test-only)."""
+    import torch
+    nbytes = lib().agnn_debug_gemm_tn_ws_bytes(ctypes.c_int(A.shape[1]), ctypes.c_int(B.shape[1]))
+    ws = torch.empty(nbytes // 4 + 1, dtype=torch.float32, device=A.device)
+    _check(lib().agnn_debug_gemm_tn(_ptr(A), ctypes.c_int64(A.shape[0]), ctypes.c_int(A.shape[1]),
+                                    _ptr(B), ctypes.c_int(B.shape[1]), _ptr(C), _ptr(ws),
+                                    _stream(stream)))
 
 
 def nccl_unique_id() -> bytes:

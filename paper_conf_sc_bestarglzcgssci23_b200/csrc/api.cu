@@ -154,6 +154,15 @@ const char* agnn_last_error(void) { return g_last_error.c_str(); }
 
 uint64_t agnn_launch_count(void) { return g_launches.load(); }
 
+agnn_status agnn_debug_gemm_tn(const float* A, int64_t M, int K1, const float* B, int N,
+                               float* C, float* ws, cudaStream_t s) {
+  if (!A || !B || !C || !ws || M < 0 || K1 <= 0 || N <= 0)
+    return fail(AGNN_EINVAL, "agnn_debug_gemm_tn: bad arguments");
+  return gemm_tn(A, M, K1, B, N, C, ws, s);
+}
+
+size_t agnn_debug_gemm_tn_ws_bytes(int K1, int N) { return gemm_tn_ws_floats(K1, N) * sizeof(float); }
+
 agnn_status agnn_debug_gemm(const float* A, int64_t M, int K, const float* B, int N, float* C,
                             cudaStream_t s) {
   if (!A || !B || !C || M < 0 || K <= 0 || N <= 0)

@@ -227,10 +227,21 @@ agnn_status transpose(const float* X, int rows, int cols, float* Y, cudaStream_t
   return AGNN_OK;
 }
 
-size_t gemm_tn_ws_floats(int K1, int N) { return (size_t)tn_splits(K1, N) * K1 * N; }
+size_t gemm_tn_ws_floats(int K1, int N) {
+  const size_t simt = (size_t)tn_splits(K1, N) * K1 * N;
+  const size_t tc = (size_t)kNumSMs * K1 * N;  // one partial per SM (gemm_tn_tc)
+  return simt > tc ? simt : tc;
+}
+
+agnn_status gemm_tn_tc(const float* A, int64_t M, int K1, const float* B, int N, float* C,
+                       float* ws, cudaStream_t s);
 
 agnn_status gemm_tn(const float* A, int64_t M, int K1, const float* B, int N, float* C, float* ws,
                     cudaStream_t s) {
+  {
+    const agnn_status st = gemm_tn_tc(A, M, K1, B, N, C, ws, s);
+    if (st != AGNN_EUNSUPPORTED) return st;
+  }
   if (K1 % 4 || N % 4) return fail(AGNN_EINVAL, "gemm_tn: widths must be multiples of 4");
   const int S = tn_splits(K1, N);
   int64_t rps = (M + S - 1) / S;

@@ -292,6 +292,152 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const float* __restrict_
                  : "memory");
 }
 
+// ---------------------------------------------------------------- C = A^T B
+// Weight gradients Y = H^T dP / X^T G (PAPER.md:241 Eq. 5, :298 Eq. 13): the
+// reduction runs over the n rows, so both operands are MN-major for the MMA
+// (D[k1 x n] += A'[k1 x 8 rows] B'[8 rows x n]).  Each CTA reduces a contiguous
+// slab of rows: TMA brings 32-row chunks of A and B (128B-swizzled, MN-major
+// atoms of 8 rows x 32 columns), threads split them 3xTF32, thread 0 issues
+// the MMAs; every TN_GROUP chunks the TMEM accumulator is drained into fp32
+// registers (one dW row per thread) so the tensor core's per-MMA rounding
+// never compounds over more than TN_GROUP * 12 accumulations.
+constexpr int TN_ROWS = 32;   // input rows per chunk
+constexpr int TN_GROUP = 2;   // chunks per TMEM drain
+
+// MN-major tf32 operands use the 128B swizzle with 32-byte atomicity (the only MN-major
+// smem layout for 32-bit types): atoms of 4 rows x 128 B; LBO = stride between
+// 32-element MN blocks, SBO = stride between 4-row K groups; layout type 1.
+__device__ __forceinline__ uint64_t sw128_mn_desc(uint32_t saddr, uint32_t lbo_bytes,
+                                                  uint32_t sbo_bytes) {
+  return (uint64_t)((saddr & 0x3FFFF) >> 4) | ((uint64_t)(lbo_bytes >> 4) << 16) |
+         ((uint64_t)(sbo_bytes >> 4) << 32) | ((uint64_t)1 << 46) | ((uint64_t)1 << 61);
+}
+
+template <int K1, int N>
+__global__ void __launch_bounds__(TC_THREADS, 1)
+gemm_tn_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+                  int64_t M, int64_t rows_per_cta, float* __restrict__ part) {
+  constexpr uint32_t LBO = TN_ROWS * 128;  // 32-column MN blocks (one TMA box each)
+  constexpr uint32_t SBO = 512;            // 4-row K groups
+  static_assert(K1 == 128, "the MMA M is the K1 = 128 rows of dW");
+  static_assert(N % 32 == 0 && N <= 256, "N in 32-column atoms");
+  constexpr int A_BYTES = TN_ROWS * K1 * 4;     // one chunk of A (hi); lo follows
+  constexpr int B_BYTES = TN_ROWS * N * 4;
+  constexpr int STAGE = 2 * A_BYTES + 2 * B_BYTES;
+  constexpr uint32_t IDESC = (1u << 4) | (2u << 7) | (2u << 10) | (1u << 15) | (1u << 16) |
+                             ((uint32_t)(N >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
+  constexpr uint32_t TMEM_COLS = N <= 32 ? 32 : N <= 64 ? 64 : N <= 128 ? 128 : 256;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
+                                             ~uintptr_t(1023));
+  __shared__ uint64_t tma_bar[2], mma_bar[2];
+  __shared__ uint32_t tmem_base_s;
+  const int tid = threadIdx.x, warp = tid >> 5;
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     s_addr(&tmem_base_s)),
+                 "r"(TMEM_COLS)
+                 : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+  }
+  if (tid == 0) {
+    mbar_init(&tma_bar[0], 1);
+    mbar_init(&tma_bar[1], 1);
+    mbar_init(&mma_bar[0], 1);
+    mbar_init(&mma_bar[1], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = tmem_base_s;
+  const int64_t r_beg = (int64_t)blockIdx.x * rows_per_cta;
+  const int64_t r_end = min(M, r_beg + rows_per_cta);
+  const int64_t nch = r_end > r_beg ? (r_end - r_beg + TN_ROWS - 1) / TN_ROWS : 0;
+  float acc[N];
+#pragma unroll
+  for (int c = 0; c < N; ++c) acc[c] = 0.f;
+  auto issue_tma = [&](int64_t g, int st) {
+    uint8_t* base = smem + st * STAGE;
+    const int r = (int)(r_beg + g * TN_ROWS);
+    mbar_expect_tx(&tma_bar[st], A_BYTES + B_BYTES);
+#pragma unroll
+    for (int b = 0; b < K1 / 32; ++b)
+      tma_load_2d(base + b * (TN_ROWS * 128), &tmA, &tma_bar[st], b * 32, r);
+#pragma unroll
+    for (int b = 0; b < N / 32; ++b)
+      tma_load_2d(base + 2 * A_BYTES + b * (TN_ROWS * 128), &tmB, &tma_bar[st], b * 32, r);
+  };
+  if (tid == 0 && nch > 0) issue_tma(0, 0);
+  for (int64_t g = 0; g < nch; ++g) {
+    const int st = (int)(g & 1);
+    if (tid == 0 && g + 1 < nch) {
+      if (g >= 1) mbar_wait(&mma_bar[st ^ 1], (uint32_t)(((g - 1) >> 1) & 1));
+      issue_tma(g + 1, st ^ 1);
+    }
+    mbar_wait(&tma_bar[st], (uint32_t)((g >> 1) & 1));
+    uint8_t* base = smem + st * STAGE;
+    // rows past r_end arrive as zeros (TMA out-of-bounds fill) or belong to the next
+    // CTA's slab: zero them before the split
+    const int64_t rem = r_end - (r_beg + g * TN_ROWS);
+    const int valid_rows = rem < TN_ROWS ? (int)rem : TN_ROWS;
+    for (int i = tid; i < (A_BYTES + B_BYTES) / 16; i += TC_THREADS) {
+      const bool isA = i < A_BYTES / 16;
+      const int li = isA ? i : i - A_BYTES / 16;
+      uint8_t* hp = isA ? base + li * 16 : base + 2 * A_BYTES + li * 16;
+      uint8_t* lp = hp + (isA ? A_BYTES : B_BYTES);
+      const int row = (li * 16 / 128) % TN_ROWS;   // 128-byte row inside a 32-row box
+      float4 x = *reinterpret_cast<const float4*>(hp);
+      if (row >= valid_rows) x = f4(0.f);
+      float4 hi, lo;
+      split4(x, hi, lo);
+      *reinterpret_cast<float4*>(hp) = hi;
+      *reinterpret_cast<float4*>(lp) = lo;
+    }
+    fence_proxy_async();
+    tc_fence_before();
+    __syncthreads();
+    const bool first_in_group = (g % TN_GROUP) == 0;
+    if (tid == 0) {
+      tc_fence_after();
+      const uint32_t ah = s_addr(base), al = ah + A_BYTES;
+      const uint32_t bh = s_addr(base + 2 * A_BYTES), bl = bh + B_BYTES;
+#pragma unroll
+      for (int ks = 0; ks < TN_ROWS / 8; ++ks) {  // 8 input rows per MMA = two 4-row atoms
+        const uint32_t o = ks * 1024;
+        const uint32_t acc0 = (!first_in_group || ks > 0) ? 1u : 0u;
+        mma_tf32(tmem, sw128_mn_desc(ah + o, LBO, SBO), sw128_mn_desc(bh + o, LBO, SBO), IDESC,
+                 acc0);
+        mma_tf32(tmem, sw128_mn_desc(ah + o, LBO, SBO), sw128_mn_desc(bl + o, LBO, SBO), IDESC, 1u);
+        mma_tf32(tmem, sw128_mn_desc(al + o, LBO, SBO), sw128_mn_desc(bh + o, LBO, SBO), IDESC, 1u);
+      }
+      mma_commit(&mma_bar[st]);
+    }
+    if ((g % TN_GROUP) == TN_GROUP - 1 || g == nch - 1) {
+      mbar_wait(&mma_bar[st], (uint32_t)((g >> 1) & 1));
+      tc_fence_after();
+      const uint32_t tbase = tmem + ((uint32_t)(warp * 32) << 16);
+#pragma unroll
+      for (int c0 = 0; c0 < N; c0 += 16) {
+        float v[16];
+        tmem_ld16(tbase + c0, v);
+#pragma unroll
+        for (int x = 0; x < 16; ++x) acc[c0 + x] += v[x];
+      }
+      tc_fence_before();
+      __syncthreads();
+    }
+  }
+  float* out = part + (int64_t)blockIdx.x * K1 * N + (int64_t)tid * N;  // dW row tid
+#pragma unroll
+  for (int c = 0; c < N; c += 4) st4(out + c, make_float4(acc[c], acc[c + 1], acc[c + 2], acc[c + 3]));
+  __syncthreads();
+  if (warp == 0)
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem),
+                 "r"(TMEM_COLS)
+                 : "memory");
+}
+
 PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
   static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
   static std::once_flag once;
@@ -336,6 +482,54 @@ agnn_status launch_tc(const float* A, int64_t M, const float* B, int n_real, con
   return AGNN_OK;
 }
 
+bool map_rows_box32(CUtensorMap* map, const float* base, int64_t rows, int cols) {
+  auto enc = encode_fn();
+  if (!enc) return false;
+  cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
+  cuuint64_t strides[1] = {(cuuint64_t)cols * 4};
+  cuuint32_t box[2] = {32, (cuuint32_t)TN_ROWS};
+  cuuint32_t es[2] = {1, 1};
+  return enc(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(base), dims, strides, box,
+             es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B,
+             CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+__global__ void tn_sum_kernel(const float* __restrict__ part, int splits, int64_t count,
+                              float* __restrict__ C) {
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= count) return;
+  float s = 0.f;
+  for (int p = 0; p < splits; ++p) s += part[(int64_t)p * count + i];
+  C[i] = s;
+}
+
+template <int K1, int N>
+agnn_status launch_tn_tc(const float* A, int64_t M, const float* B, float* C, float* ws,
+                         cudaStream_t s) {
+  CUtensorMap ma, mb;
+  if (!map_rows_box32(&ma, A, M, K1) || !map_rows_box32(&mb, B, M, N))
+    return fail(AGNN_ECUDA, "gemm_tn_tc: tensor map encode failed");
+  constexpr int smem = 2 * (2 * TN_ROWS * K1 * 4 + 2 * TN_ROWS * N * 4) + 1024;
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(gemm_tn_tc_kernel<K1, N>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         smem);
+    attr = true;
+  }
+  int sms = kNumSMs, dev = 0;
+  if (cudaGetDevice(&dev) == cudaSuccess)
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  int64_t rpc = (M + sms - 1) / sms;
+  rpc = (rpc + TN_ROWS - 1) / TN_ROWS * TN_ROWS;
+  const int grid = (int)((M + rpc - 1) / rpc);
+  gemm_tn_tc_kernel<K1, N><<<grid, TC_THREADS, smem, s>>>(ma, mb, M, rpc, ws);
+  AGNN_LAUNCH_CHECK("gemm_tn_kernel");
+  const int64_t cnt = (int64_t)K1 * N;
+  tn_sum_kernel<<<(unsigned)((cnt + 255) / 256), 256, 0, s>>>(ws, grid, cnt, C);
+  AGNN_LAUNCH_CHECK("sum_splits_kernel");
+  return AGNN_OK;
+}
+
 bool tc_disabled() {
   static int v = -1;
   if (v < 0) {
@@ -345,7 +539,23 @@ bool tc_disabled() {
   return v == 1;
 }
 
+template <int K1, int N>
+agnn_status launch_tn_tc(const float* A, int64_t M, const float* B, float* C, float* ws,
+                         cudaStream_t s);
+
 }  // namespace
+
+// C[K1 x N] = A^T B over M rows on tensor cores (K1 = 128, N in {64, 128}); ws holds
+// one K1 x N partial per SM.  AGNN_EUNSUPPORTED for other shapes.
+agnn_status gemm_tn_tc(const float* A, int64_t M, int K1, const float* B, int N, float* C,
+                       float* ws, cudaStream_t s) {
+  if (tc_disabled() || M <= 0) return AGNN_EUNSUPPORTED;
+  if ((reinterpret_cast<uintptr_t>(A) & 15) || (reinterpret_cast<uintptr_t>(B) & 15))
+    return AGNN_EUNSUPPORTED;
+  if (K1 == 128 && N == 128) return launch_tn_tc<128, 128>(A, M, B, C, ws, s);
+  if (K1 == 128 && N == 64) return launch_tn_tc<128, 64>(A, M, B, C, ws, s);
+  return AGNN_EUNSUPPORTED;
+}
 
 // C = A * B^T with B [n_real x K] K-major; columns padded to N_pad (multiple of 16).
 // Returns AGNN_EUNSUPPORTED when the shape has no tcgen05 instantiation.

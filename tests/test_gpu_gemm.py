@@ -41,3 +41,24 @@ def test_gemm_against_fp64(M, K, N):
     scale = np.abs(A.double().cpu().numpy()) @ np.abs(B.double().cpu().numpy()).T
     assert (err <= 1e-6 * scale + 1e-30).all(), float((err / scale).max())
     assert np.linalg.norm(c - ref) / np.linalg.norm(ref) < 5e-7
+
+
+@pytest.mark.parametrize("M,K1,N", [(1000, 128, 128), (65536, 128, 128), (300001, 128, 128),
+                                    (77, 128, 64), (20000, 64, 64), (12345, 128, 64)])
+def test_gemm_tn_against_fp64(M, K1, N):
+    g = torch.Generator(device="cpu").manual_seed(3 * M + K1 + N)
+    A = (torch.rand((M, K1), generator=g) * 2 - 1).cuda()
+    B = (torch.rand((M, N), generator=g) * 2 - 1).cuda()
+    ref = A.double().cpu().numpy().T @ B.double().cpu().numpy()
+    outs = []
+    for rep in range(2):
+        C = torch.full((K1, N), float("nan"), device="cuda")
+        agnn.debug_gemm_tn(A, B, C)
+        torch.cuda.synchronize()
+        outs.append(C.cpu().numpy())
+    assert np.array_equal(outs[0], outs[1]), "GEMM-TN not reproducible"
+    c = outs[0].astype(np.float64)
+    assert np.isfinite(c).all()
+    scale = np.abs(A.double().cpu().numpy()).T @ np.abs(B.double().cpu().numpy())
+    err = np.abs(c - ref)
+    assert (err <= 1e-6 * scale + 1e-30).all(), float((err / scale).max())

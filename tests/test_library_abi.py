@@ -18,7 +18,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 def declared_symbols():
     src = open(os.path.join(ROOT, "include", "agnn.h")).read()
-    return sorted(set(re.findall(r"^(?:agnn_status|void|uint64_t|const char\*)\s+(agnn_\w+)\(",
+    return sorted(set(re.findall(r"^(?:agnn_status|void|uint64_t|size_t|const char\*)\s+(agnn_\w+)\(",
                                  src, flags=re.M)))
 
 
