@@ -193,9 +193,9 @@ __global__ void sum_splits_kernel(const float* __restrict__ part, int splits, in
                                   float* __restrict__ C) {
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= count) return;
-  float s = 0.f;
-  for (int p = 0; p < splits; ++p) s += part[(int64_t)p * count + i];
-  C[i] = s;
+  double s = 0.0;  // fixed order, fp64 across the split partials
+  for (int p = 0; p < splits; ++p) s += (double)part[(int64_t)p * count + i];
+  C[i] = (float)s;
 }
 
 }  // namespace
@@ -229,7 +229,7 @@ agnn_status transpose(const float* X, int rows, int cols, float* Y, cudaStream_t
 
 size_t gemm_tn_ws_floats(int K1, int N) {
   const size_t simt = (size_t)tn_splits(K1, N) * K1 * N;
-  const size_t tc = (size_t)kNumSMs * K1 * N;  // one partial per SM (gemm_tn_tc)
+  const size_t tc = (size_t)2048 * K1 * N;  // one partial per row slab (gemm_tn_tc)
   return simt > tc ? simt : tc;
 }
 

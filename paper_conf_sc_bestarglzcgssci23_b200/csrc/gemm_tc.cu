@@ -303,6 +303,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const float* __restrict_
 // never compounds over more than TN_GROUP * 12 accumulations.
 constexpr int TN_ROWS = 32;   // input rows per chunk
 constexpr int TN_GROUP = 2;   // chunks per TMEM drain
+constexpr int64_t kTnMaxSlabs = 2048;  // fp32 partials per call (summed in fp64)
 
 // MN-major tf32 operands use the 128B swizzle with 32-byte atomicity (the only MN-major
 // smem layout for 32-bit types): atoms of 4 rows x 128 B; LBO = stride between
@@ -351,7 +352,10 @@ gemm_tn_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = tmem_base_s;
-  const int64_t r_beg = (int64_t)blockIdx.x * rows_per_cta;
+  const int64_t nslabs = (M + rows_per_cta - 1) / rows_per_cta;
+  int64_t G0 = 0;  // chunks this CTA processed in earlier slabs: stage = G & 1, parity = (G >> 1) & 1
+  for (int64_t slab = blockIdx.x; slab < nslabs; slab += gridDim.x) {
+  const int64_t r_beg = slab * rows_per_cta;
   const int64_t r_end = min(M, r_beg + rows_per_cta);
   const int64_t nch = r_end > r_beg ? (r_end - r_beg + TN_ROWS - 1) / TN_ROWS : 0;
   float acc[N];
@@ -368,14 +372,17 @@ gemm_tn_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
     for (int b = 0; b < N / 32; ++b)
       tma_load_2d(base + 2 * A_BYTES + b * (TN_ROWS * 128), &tmB, &tma_bar[st], b * 32, r);
   };
-  if (tid == 0 && nch > 0) issue_tma(0, 0);
+  if (tid == 0 && nch > 0) issue_tma(0, (int)(G0 & 1));
   for (int64_t g = 0; g < nch; ++g) {
-    const int st = (int)(g & 1);
+    const int64_t G = G0 + g;
+    const int st = (int)(G & 1);
     if (tid == 0 && g + 1 < nch) {
-      if (g >= 1) mbar_wait(&mma_bar[st ^ 1], (uint32_t)(((g - 1) >> 1) & 1));
+      // stage st^1 held chunk G-1 (its MMAs must finish before the TMA overwrites it;
+      // the previous slab's last chunk was already waited on by its epilogue)
+      if (g >= 1) mbar_wait(&mma_bar[st ^ 1], (uint32_t)(((G - 1) >> 1) & 1));
       issue_tma(g + 1, st ^ 1);
     }
-    mbar_wait(&tma_bar[st], (uint32_t)((g >> 1) & 1));
+    mbar_wait(&tma_bar[st], (uint32_t)((G >> 1) & 1));
     uint8_t* base = smem + st * STAGE;
     // rows past r_end arrive as zeros (TMA out-of-bounds fill) or belong to the next
     // CTA's slab: zero them before the split
@@ -414,7 +421,7 @@ gemm_tn_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       mma_commit(&mma_bar[st]);
     }
     if ((g % TN_GROUP) == TN_GROUP - 1 || g == nch - 1) {
-      mbar_wait(&mma_bar[st], (uint32_t)((g >> 1) & 1));
+      mbar_wait(&mma_bar[st], (uint32_t)((G >> 1) & 1));
       tc_fence_after();
       const uint32_t tbase = tmem + ((uint32_t)(warp * 32) << 16);
 #pragma unroll
@@ -428,9 +435,11 @@ gemm_tn_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       __syncthreads();
     }
   }
-  float* out = part + (int64_t)blockIdx.x * K1 * N + (int64_t)tid * N;  // dW row tid
+  float* out = part + slab * K1 * N + (int64_t)tid * N;  // dW row tid of this slab's partial
 #pragma unroll
   for (int c = 0; c < N; c += 4) st4(out + c, make_float4(acc[c], acc[c + 1], acc[c + 2], acc[c + 3]));
+  G0 += nch;
+  }  // slab
   __syncthreads();
   if (warp == 0)
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem),
@@ -498,9 +507,9 @@ __global__ void tn_sum_kernel(const float* __restrict__ part, int splits, int64_
                               float* __restrict__ C) {
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= count) return;
-  float s = 0.f;
-  for (int p = 0; p < splits; ++p) s += part[(int64_t)p * count + i];
-  C[i] = s;
+  double s = 0.0;  // fixed order, fp64 across the slab partials
+  for (int p = 0; p < splits; ++p) s += (double)part[(int64_t)p * count + i];
+  C[i] = (float)s;
 }
 
 template <int K1, int N>
@@ -519,13 +528,16 @@ agnn_status launch_tn_tc(const float* A, int64_t M, const float* B, float* C, fl
   int sms = kNumSMs, dev = 0;
   if (cudaGetDevice(&dev) == cudaSuccess)
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  int64_t rpc = (M + sms - 1) / sms;
-  rpc = (rpc + TN_ROWS - 1) / TN_ROWS * TN_ROWS;
-  const int grid = (int)((M + rpc - 1) / rpc);
-  gemm_tn_tc_kernel<K1, N><<<grid, TC_THREADS, smem, s>>>(ma, mb, M, rpc, ws);
+  // slabs of >= 8192 rows, at most kTnMaxSlabs of them; each slab leaves one fp32 partial
+  int64_t rps = (M + kTnMaxSlabs - 1) / kTnMaxSlabs;
+  rps = std::max<int64_t>(rps, 8192);
+  rps = (rps + TN_ROWS - 1) / TN_ROWS * TN_ROWS;
+  const int64_t nslabs = (M + rps - 1) / rps;
+  const int grid = (int)std::min<int64_t>(nslabs, sms);
+  gemm_tn_tc_kernel<K1, N><<<grid, TC_THREADS, smem, s>>>(ma, mb, M, rps, ws);
   AGNN_LAUNCH_CHECK("gemm_tn_kernel");
   const int64_t cnt = (int64_t)K1 * N;
-  tn_sum_kernel<<<(unsigned)((cnt + 255) / 256), 256, 0, s>>>(ws, grid, cnt, C);
+  tn_sum_kernel<<<(unsigned)((cnt + 255) / 256), 256, 0, s>>>(ws, (int)nslabs, cnt, C);
   AGNN_LAUNCH_CHECK("sum_splits_kernel");
   return AGNN_OK;
 }
