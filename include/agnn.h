@@ -25,9 +25,12 @@
  *    (N^(i)), by GLOBAL column id, strictly ascending.
  *    The library computes on exactly this pattern: it never adds self-loops
  *    or symmetrises (use agnn_csr_build for the paper's preprocessing).
- *    The backward's single-pass kernel requires a symmetric pattern
- *    (AGNN_CSR_SYMMETRIC, "for undirected graphs A = A^T");
- *    unsymmetric patterns are rejected with AGNN_EUNSUPPORTED by agnn_backward.
+ *    With AGNN_CSR_SYMMETRIC ("for undirected graphs A = A^T")
+ *    the backward visits every stored entry once for both of its roles.
+ *    Without it (a directed pattern, reading A4) the plan builds the
+ *    transposed pattern (CSC) once and the backward runs a row pass over the
+ *    CSR and a column pass over the CSC; this needs world == 1 and the plan
+ *    holding every row (agnn_backward returns AGNN_EUNSUPPORTED otherwise).
  *
  * Ownership
  *  - The caller owns every feature, weight, gradient, `saved` and
@@ -126,6 +129,14 @@ agnn_status agnn_plan_destroy(agnn_plan_t plan);
 /* host-side statistics: [0]=n_local [1]=nnz_local [2]=light rows [3]=heavy rows
  * [4]=heavy chunks [5]=chunk size [6]=max degree [7]=n (global)            */
 agnn_status agnn_plan_info(agnn_plan_t plan, int64_t* info8);
+
+/* The transposed pattern of the plan's CSR (test/utility; synchronises):
+ * col_ptr [n+1] (device, int64), row_idx [nnz] (device, int32) list, for
+ * every column j, the rows i with a stored entry (i,j) in ascending i, and
+ * perm [nnz] (device, int64, nullable) the CSR position of each CSC entry.
+ * Requires world == 1 and the plan holding all rows (else AGNN_EUNSUPPORTED). */
+agnn_status agnn_plan_csc(agnn_plan_t plan, int64_t* col_ptr, int32_t* row_idx, int64_t* perm,
+                          cudaStream_t stream);
 
 agnn_status agnn_model_create(agnn_plan_t plan, int n_layers, const agnn_layer_desc* descs,
                               agnn_model_t* out);

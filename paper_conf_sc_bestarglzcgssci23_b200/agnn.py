@@ -26,6 +26,7 @@ STATUS = {0: "AGNN_OK", 1: "AGNN_EINVAL", 2: "AGNN_ECUDA", 3: "AGNN_ENCCL", 4: "
 
 # every symbol include/agnn.h declares (tests check the .so exports all of them)
 EXPORTS = ("agnn_partition", "agnn_plan_create", "agnn_plan_destroy", "agnn_plan_info",
+           "agnn_plan_csc",
            "agnn_model_create", "agnn_model_destroy", "agnn_saved_bytes", "agnn_workspace_bytes",
            "agnn_forward", "agnn_backward", "agnn_debug_attention", "agnn_debug_gemm",
            "agnn_debug_gemm_tn", "agnn_debug_gemm_tn_ws_bytes",
@@ -215,6 +216,18 @@ class Plan:
         keys = ("n_local", "nnz", "light_rows", "heavy_rows", "heavy_chunks", "chunk", "max_degree",
                 "n")
         return dict(zip(keys, list(a)))
+
+    def csc(self, perm=True, stream=None):
+        """agnn_plan_csc: (col_ptr int64 [n+1], row_idx int32 [nnz], perm int64 [nnz] | None)."""
+        import torch
+        dev = self.row_ptr.device
+        nnz = int(self.col_idx.numel())
+        cp = torch.empty(self.n + 1, dtype=torch.int64, device=dev)
+        ri = torch.empty(max(nnz, 1), dtype=torch.int32, device=dev)
+        pm = torch.empty(max(nnz, 1), dtype=torch.int64, device=dev) if perm else None
+        _check(lib().agnn_plan_csc(self.handle, _ptr(cp), _ptr(ri),
+                                   _ptr(pm) if pm is not None else None, _stream(stream)))
+        return cp, ri[:nnz], (pm[:nnz] if pm is not None else None)
 
     def __del__(self):
         if getattr(self, "handle", None) and _lib is not None:

@@ -189,6 +189,7 @@ struct AvBwd {
   float beta, eps;
   float* dH;           // [n_local x K]
   float* pacc;         // [n_chunks x 2K]
+  float* dhp;          // [n_local x K] directed patterns: row-pass partial of dH (VA) / dH^ (AGNN)
 };
 
 template <int K, int MODEL>
@@ -226,8 +227,12 @@ __device__ __forceinline__ void bwd_store(const AvBwd& A, int64_t row, int64_t g
   }
 }
 
-template <int K, int MODEL, int U>
+// ROLE: 0 = both roles over the symmetric CSR; 1 = row role only over the CSR of a
+// directed pattern (partial -> A.dhp); 2 = column role only over its CSC (items are
+// columns j, it.col the rows i with stored (i,j)), adding A.dhp before the epilogue
+template <int K, int MODEL, int U, int ROLE = 0>
 __global__ void __launch_bounds__(kSparseThreads) av_bwd_kernel(Items it, AvBwd A) {
+  constexpr bool RR = ROLE != 2, CR = ROLE != 1;
   using L = RowLayout<K, 1>;
   const int lane = threadIdx.x & 31, g = lane / L::LANES, q = lane % L::LANES;
   const int64_t nitems = it.n_chunks + it.n_light;
@@ -260,7 +265,7 @@ __global__ void __launch_bounds__(kSparseThreads) av_bwd_kernel(Items it, AvBwd 
 #pragma unroll
           for (int v = 0; v < L::VPL; ++v) {
             Hi[u][v] = val[u] ? ldg4(A.H + i * K + L::col(v, q)) : f4(0.f);
-            Mi[u][v] = val[u] ? ldg4(A.M + i * K + L::col(v, q)) : f4(0.f);
+            Mi[u][v] = (CR && val[u]) ? ldg4(A.M + i * K + L::col(v, q)) : f4(0.f);
           }
           ri[u] = (MODEL == AG && val[u]) ? __ldg(A.rec + i) : f4(1.f);
         }
@@ -273,27 +278,34 @@ __global__ void __launch_bounds__(kSparseThreads) av_bwd_kernel(Items it, AvBwd 
             d1[v] = dot4(Mj[v], Hi[u][v]);   // M_j . H_i  (row role)
             d2[v] = dot4(Mi[u][v], Hj[v]);   // M_i . H_j  (column role)
           }
-          L::head_reduce(s);
-          L::head_reduce(d1);
-          L::head_reduce(d2);
+          if (MODEL == AG || CR) L::head_reduce(s);
+          if (RR) L::head_reduce(d1);
+          if (CR) L::head_reduce(d2);
           if (!val[u]) continue;
           if (MODEL == VA) {
-            const float c1 = d1[0] + d2[0];
+            const float c1 = (RR ? d1[0] : 0.f) + (CR ? d2[0] : 0.f);
 #pragma unroll
             for (int v = 0; v < L::VPL; ++v) {
               dh[v] = fma4(c1, Hi[u][v], dh[v]);
-              dh[v] = fma4(s[0], Mi[u][v], dh[v]);
+              if (CR) dh[v] = fma4(s[0], Mi[u][v], dh[v]);
             }
           } else {
             const float inv_nui = 1.f / ri[u].x;
             const float c = sj * s[0] * inv_nui;                        // beta cos(H_j, H_i)
-            const float aji = ex2((c - rj.y) * kLog2e) * rj.z;          // alpha_ji (row j)
-            const float aij = ex2((c - ri[u].y) * kLog2e) * ri[u].z;    // alpha_ij (row i)
-            const float dc = beta * (aji * (d1[0] - rj.w) + aij * (d2[0] - ri[u].w));
+            float dc = 0.f, aij = 0.f;
+            if (RR) {
+              const float aji = ex2((c - rj.y) * kLog2e) * rj.z;        // alpha_ji (row j)
+              dc = aji * (d1[0] - rj.w);
+            }
+            if (CR) {
+              aij = ex2((c - ri[u].y) * kLog2e) * ri[u].z;              // alpha_ij (row i)
+              dc += aij * (d2[0] - ri[u].w);
+            }
+            dc *= beta;
 #pragma unroll
             for (int v = 0; v < L::VPL; ++v) {
               dh[v] = fma4(dc * inv_nui, Hi[u][v], dh[v]);   // dH^_j += dc H^_i
-              acc[v] = fma4(aij, Mi[u][v], acc[v]);
+              if (CR) acc[v] = fma4(aij, Mi[u][v], acc[v]);
             }
           }
         }
@@ -307,7 +319,7 @@ __global__ void __launch_bounds__(kSparseThreads) av_bwd_kernel(Items it, AvBwd 
         dh[v].y += __shfl_xor_sync(FULL, dh[v].y, off);
         dh[v].z += __shfl_xor_sync(FULL, dh[v].z, off);
         dh[v].w += __shfl_xor_sync(FULL, dh[v].w, off);
-        if (MODEL == AG) {
+        if (MODEL == AG && CR) {
           acc[v].x += __shfl_xor_sync(FULL, acc[v].x, off);
           acc[v].y += __shfl_xor_sync(FULL, acc[v].y, off);
           acc[v].z += __shfl_xor_sync(FULL, acc[v].z, off);
@@ -320,16 +332,25 @@ __global__ void __launch_bounds__(kSparseThreads) av_bwd_kernel(Items it, AvBwd 
 #pragma unroll
         for (int v = 0; v < L::VPL; ++v) {
           st4(A.pacc + slot * 2 * K + L::col(v, q), dh[v]);
-          if (MODEL == AG) st4(A.pacc + slot * 2 * K + K + L::col(v, q), acc[v]);
+          if (MODEL == AG && CR) st4(A.pacc + slot * 2 * K + K + L::col(v, q), acc[v]);
         }
       }
+    } else if (ROLE == 1) {
+      if (g == 0) {
+#pragma unroll
+        for (int v = 0; v < L::VPL; ++v) st4(A.dhp + row * K + L::col(v, q), dh[v]);
+      }
     } else {
+      if (ROLE == 2) {
+#pragma unroll
+        for (int v = 0; v < L::VPL; ++v) dh[v] = add4(ldg4(A.dhp + row * K + L::col(v, q)), dh[v]);
+      }
       bwd_store<K, MODEL>(A, row, grow, q, dh, acc, g == 0);
     }
   }
 }
 
-template <int K, int MODEL>
+template <int K, int MODEL, int ROLE = 0>
 __global__ void __launch_bounds__(kSparseThreads) av_bwd_merge_kernel(Items it, AvBwd A) {
   using L = RowLayout<K, 1>;
   const int lane = threadIdx.x & 31, g = lane / L::LANES, q = lane % L::LANES;
@@ -343,8 +364,19 @@ __global__ void __launch_bounds__(kSparseThreads) av_bwd_merge_kernel(Items it, 
 #pragma unroll
       for (int v = 0; v < L::VPL; ++v) {
         dh[v] = add4(dh[v], ldg4(A.pacc + s * 2 * K + L::col(v, q)));
-        if (MODEL == AG) acc[v] = add4(acc[v], ldg4(A.pacc + s * 2 * K + K + L::col(v, q)));
+        if (MODEL == AG && ROLE != 1) acc[v] = add4(acc[v], ldg4(A.pacc + s * 2 * K + K + L::col(v, q)));
       }
+    }
+    if (ROLE == 1) {
+      if (g == 0) {
+#pragma unroll
+        for (int v = 0; v < L::VPL; ++v) st4(A.dhp + row * K + L::col(v, q), dh[v]);
+      }
+      continue;
+    }
+    if (ROLE == 2) {
+#pragma unroll
+      for (int v = 0; v < L::VPL; ++v) dh[v] = add4(ldg4(A.dhp + row * K + L::col(v, q)), dh[v]);
     }
     bwd_store<K, MODEL>(A, row, grow, q, dh, acc, g == 0);
   }
@@ -427,7 +459,7 @@ SavedAv carve_saved(const Plan& p, const agnn_layer_desc& d, void* base, size_t*
 }
 
 struct WsAv {
-  float *pacc, *pl, *G, *M, *gemm, *WT;
+  float *pacc, *pl, *G, *M, *gemm, *WT, *dhp;
   float4* rec;
   void* saved_inf;
 };
@@ -436,8 +468,9 @@ WsAv carve_ws(const Plan& p, const agnn_layer_desc& d, void* base, size_t* total
   WsAv w;
   size_t sv = 0;
   carve_saved(p, d, nullptr, &sv);
-  w.pacc = c.take<float>((size_t)p.n_chunks * 2 * d.k_in);
-  w.pl = c.take<float>((size_t)p.n_chunks);
+  w.pacc = c.take<float>((size_t)p.max_chunks() * 2 * d.k_in);
+  w.pl = c.take<float>((size_t)p.max_chunks());
+  w.dhp = c.take<float>(p.csc_ptr ? (size_t)p.n_local * d.k_in : 0);
   w.G = c.take<float>((size_t)p.n_local * d.k_out);
   w.M = c.take<float>((size_t)p.n * d.k_in);
   w.rec = c.take<float4>(d.kind == AGNN_AGNN ? (size_t)p.n : 0);
@@ -521,8 +554,10 @@ agnn_status av_forward(const Plan& p, const agnn_layer_desc& d, const float* W, 
 agnn_status av_backward(const Plan& p, const agnn_layer_desc& d, const float* W,
                         const float* H_in, const void* saved, const float* dH_out, float* dH_in,
                         float* dW, void* ws, cudaStream_t s) {
-  if (!(p.flags & AGNN_CSR_SYMMETRIC))
-    return fail(AGNN_EUNSUPPORTED, "agnn_backward: the single-pass backward needs a symmetric CSR");
+  const bool directed = p.directed();
+  if (directed && !p.csc_ptr)
+    return fail(AGNN_EUNSUPPORTED,
+                "agnn_backward: a directed pattern needs world == 1 and every row in the plan");
   WsAv w = carve_ws(p, d, ws, nullptr);
   SavedAv sv = carve_saved(p, d, const_cast<void*>(saved), nullptr);
   const int K_ = d.k_in;
@@ -552,7 +587,33 @@ agnn_status av_backward(const Plan& p, const agnn_layer_desc& d, const float* W,
   }
   const float* Hf = p.world > 1 ? sv.Hfull : H_in;
   Items it = items_of(p);
-  AvBwd A{Hf, w.M, w.rec, d.beta, d.eps, dH_in, w.pacc};
+  AvBwd A{Hf, w.M, w.rec, d.beta, d.eps, dH_in, w.pacc, w.dhp};
+  if (directed) {
+#define AV_PASS(ROLE_, ITEMS)                                                                      \
+    do {                                                                                           \
+      const Items itr = (ITEMS);                                                                   \
+      if (itr.n_chunks + itr.n_light > 0) {                                                        \
+        if (ag) AGNN_AV_DISPATCH(K_, (av_bwd_kernel<K, AG, av_bwd_unroll<K>(), ROLE_>               \
+                                      <<<grid_of(av_bwd_kernel<K, AG, av_bwd_unroll<K>(), ROLE_>),   \
+                                         kSparseThreads, 0, s>>>(itr, A)));                        \
+        else AGNN_AV_DISPATCH(K_, (av_bwd_kernel<K, VA, av_bwd_unroll<K>(), ROLE_>                  \
+                                   <<<grid_of(av_bwd_kernel<K, VA, av_bwd_unroll<K>(), ROLE_>),      \
+                                      kSparseThreads, 0, s>>>(itr, A)));                           \
+        AGNN_LAUNCH_CHECK("av_bwd_kernel");                                                        \
+      }                                                                                            \
+      if (itr.n_heavy > 0) {                                                                       \
+        if (ag) AGNN_AV_DISPATCH(K_, (av_bwd_merge_kernel<K, AG, ROLE_>                             \
+                                      <<<kNumSMs * 2, kSparseThreads, 0, s>>>(itr, A)));           \
+        else AGNN_AV_DISPATCH(K_, (av_bwd_merge_kernel<K, VA, ROLE_>                                \
+                                   <<<kNumSMs * 2, kSparseThreads, 0, s>>>(itr, A)));              \
+        AGNN_LAUNCH_CHECK("av_bwd_merge_kernel");                                                  \
+      }                                                                                            \
+    } while (0)
+    AV_PASS(1, it);                  // row role over the CSR  -> dhp
+    AV_PASS(2, items_of_csc(p));     // column role over the CSC (+ dhp) -> dH
+#undef AV_PASS
+    return AGNN_OK;
+  }
   if (it.n_chunks + it.n_light > 0) {
     if (ag) AGNN_AV_DISPATCH(K_, (av_bwd_kernel<K, AG, av_bwd_unroll<K>()>
                                   <<<grid_of(av_bwd_kernel<K, AG, av_bwd_unroll<K>()>),

@@ -238,6 +238,8 @@ agnn_status agnn_plan_create(const agnn_csr* csr, const agnn_dist* dist, cudaStr
     if (st == AGNN_OK && p.world > 1) st = comm_init(p, dist->nccl_unique_id);
     if (st != AGNN_OK) {
       if (p.meta_block) cudaFree(p.meta_block);
+      if (p.csc_block) cudaFree(p.csc_block);
+      if (p.c_meta_block) cudaFree(p.c_meta_block);
       delete[] p.bounds;
       delete h;
       return st;
@@ -253,6 +255,8 @@ agnn_status agnn_plan_destroy(agnn_plan_t h) {
   if (!h) return AGNN_OK;
   comm_destroy(h->p);
   if (h->p.meta_block) cudaFree(h->p.meta_block);
+  if (h->p.csc_block) cudaFree(h->p.csc_block);
+  if (h->p.c_meta_block) cudaFree(h->p.c_meta_block);
   delete[] h->p.bounds;
   delete h;
   return AGNN_OK;
@@ -270,6 +274,19 @@ agnn_status agnn_plan_info(agnn_plan_t h, int64_t* info) {
   info[6] = p.max_deg;
   info[7] = p.n;
   return AGNN_OK;
+}
+
+agnn_status agnn_plan_csc(agnn_plan_t h, int64_t* col_ptr, int32_t* row_idx, int64_t* perm,
+                          cudaStream_t s) {
+  if (!h || !col_ptr || !row_idx) return fail(AGNN_EINVAL, "agnn_plan_csc: NULL argument");
+  const Plan& p = h->p;
+  if (p.world != 1 || p.row_begin != 0 || p.n_local != p.n)
+    return fail(AGNN_EUNSUPPORTED, "agnn_plan_csc: needs world == 1 and every row in the plan");
+  try {
+    return build_csc(p.row_ptr, p.col_idx, p.n_local, p.n, p.nnz, col_ptr, row_idx, perm, s);
+  } catch (const std::exception& e) {
+    return fail(AGNN_ENOMEM, std::string("agnn_plan_csc: ") + e.what());
+  }
 }
 
 agnn_status agnn_model_create(agnn_plan_t plan, int n_layers, const agnn_layer_desc* descs,

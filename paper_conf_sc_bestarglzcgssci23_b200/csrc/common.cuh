@@ -142,6 +142,21 @@ struct Plan {
   void* meta_block = nullptr;         // single allocation backing the lists
   int32_t* empty_rows = nullptr;      // [n_empty] local rows without stored entries
   int64_t n_empty = 0;
+  // directed patterns (world == 1): the transposed pattern (CSC of the local
+  // matrix) and its work lists, for the column role of the backward
+  // (PAPER.md:252 Psi^T; reading A4).  Plan-owned; null for symmetric plans.
+  int64_t* csc_ptr = nullptr;         // [n+1] column j lists rows i with stored (i,j)
+  int32_t* csc_idx = nullptr;         // [nnz]
+  int64_t c_light = 0, c_heavy = 0, c_chunks = 0;
+  int32_t* c_light_rows = nullptr;
+  int32_t* c_chunk_row = nullptr;
+  int32_t* c_chunk_idx = nullptr;
+  int32_t* c_heavy_rows = nullptr;
+  int32_t* c_heavy_off = nullptr;
+  void* csc_block = nullptr;          // backs csc_ptr / csc_idx
+  void* c_meta_block = nullptr;       // backs the column work lists
+  bool directed() const { return !(flags & 1u); }
+  int64_t max_chunks() const { return n_chunks > c_chunks ? n_chunks : c_chunks; }
   // distribution
   int rank = 0, world = 1;
   int64_t* bounds = nullptr;          // host [world+1]

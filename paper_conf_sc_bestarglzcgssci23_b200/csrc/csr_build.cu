@@ -76,6 +76,80 @@ int bits_for(int64_t n) {
   return b;
 }
 
+// CSC keys (col << 32 | row) and CSR positions of every stored entry (warp per row)
+__global__ void csc_keys_kernel(const int64_t* __restrict__ rp, const int32_t* __restrict__ col,
+                                int64_t n_rows, uint64_t* __restrict__ keys,
+                                int64_t* __restrict__ pos) {
+  const int lane = threadIdx.x & 31;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < n_rows; i += nw) {
+    for (int64_t e = rp[i] + lane; e < rp[i + 1]; e += 32) {
+      keys[e] = ((uint64_t)(uint32_t)col[e] << 32) | (uint64_t)i;
+      if (pos) pos[e] = e;
+    }
+  }
+}
+
+}  // namespace
+
+// CSC of a local CSR (rows [0, n_rows), global columns < n): entries sorted by
+// (column, row); csc_ptr[j] = first entry of column j; perm[e_csc] = CSR position.
+// Plan-time utility (radix sort on the device; synchronises).
+agnn_status build_csc(const int64_t* row_ptr, const int32_t* col, int64_t n_rows, int64_t n,
+                      int64_t nnz, int64_t* csc_ptr, int32_t* csc_idx, int64_t* perm,
+                      cudaStream_t s) {
+  const int grid = kNumSMs * 8;
+  if (nnz == 0) {
+    AGNN_CUDA_TRY(cudaMemsetAsync(csc_ptr, 0, sizeof(int64_t) * (size_t)(n + 1), s));
+    AGNN_CUDA_TRY(cudaStreamSynchronize(s));
+    return AGNN_OK;
+  }
+  uint64_t *ka = nullptr, *kb = nullptr;
+  int64_t *va = nullptr, *vb = nullptr;
+  void* tmp = nullptr;
+  agnn_status st = AGNN_OK;
+  auto cleanup = [&]() {
+    if (ka) cudaFreeAsync(ka, s);
+    if (kb) cudaFreeAsync(kb, s);
+    if (va) cudaFreeAsync(va, s);
+    if (vb) cudaFreeAsync(vb, s);
+    if (tmp) cudaFreeAsync(tmp, s);
+    cudaStreamSynchronize(s);
+  };
+  do {
+    if ((st = cuda_status(cudaMallocAsync(&ka, sizeof(uint64_t) * nnz, s), "csc malloc")) != AGNN_OK) break;
+    if ((st = cuda_status(cudaMallocAsync(&kb, sizeof(uint64_t) * nnz, s), "csc malloc")) != AGNN_OK) break;
+    if (perm) {
+      if ((st = cuda_status(cudaMallocAsync(&va, sizeof(int64_t) * nnz, s), "csc malloc")) != AGNN_OK) break;
+      if ((st = cuda_status(cudaMallocAsync(&vb, sizeof(int64_t) * nnz, s), "csc malloc")) != AGNN_OK) break;
+    }
+    csc_keys_kernel<<<grid, 256, 0, s>>>(row_ptr, col, n_rows, ka, va);
+    count_launch();
+    const int end_bit = 32 + bits_for(n);
+    size_t need = 0;
+    cub::DoubleBuffer<uint64_t> dk(ka, kb);
+    cub::DoubleBuffer<int64_t> dv(va, vb);
+    if (perm) st = cuda_status(cub::DeviceRadixSort::SortPairs(nullptr, need, dk, dv, nnz, 0, end_bit, s), "csc sort");
+    else st = cuda_status(cub::DeviceRadixSort::SortKeys(nullptr, need, dk, nnz, 0, end_bit, s), "csc sort");
+    if (st != AGNN_OK) break;
+    if ((st = cuda_status(cudaMallocAsync(&tmp, need, s), "csc malloc")) != AGNN_OK) break;
+    if (perm) st = cuda_status(cub::DeviceRadixSort::SortPairs(tmp, need, dk, dv, nnz, 0, end_bit, s), "csc sort");
+    else st = cuda_status(cub::DeviceRadixSort::SortKeys(tmp, need, dk, nnz, 0, end_bit, s), "csc sort");
+    if (st != AGNN_OK) break;
+    count_launch(4);
+    row_ptr_kernel<<<grid, 256, 0, s>>>(dk.Current(), nnz, n, csc_ptr);
+    low_bits_kernel<<<grid, 256, 0, s>>>(dk.Current(), nnz, csc_idx);
+    count_launch(2);
+    if (perm)
+      st = cuda_status(cudaMemcpyAsync(perm, dv.Current(), sizeof(int64_t) * nnz,
+                                       cudaMemcpyDeviceToDevice, s), "csc perm copy");
+    if (st == AGNN_OK) st = cuda_status(cudaGetLastError(), "csc kernels");
+  } while (0);
+  cleanup();
+  return st;
+}
+
+namespace {
 }  // namespace
 }  // namespace agnn
 

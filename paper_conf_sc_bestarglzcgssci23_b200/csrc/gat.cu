@@ -249,9 +249,13 @@ __device__ __forceinline__ void bwd_finish(const BwdArgs& A, int64_t row, int64_
   }
 }
 
-template <int K, int NH, int U>
+// ROLE: 0 = both roles over the symmetric CSR; 1 = row role only (CSR pass of a
+// directed pattern, ds -> A.ds_dir); 2 = column role only (CSC pass: items are
+// columns j, it.col lists the rows i with stored (i,j); ds comes from A.ds_dir)
+template <int K, int NH, int U, int ROLE = 0>
 __global__ void __launch_bounds__(kSparseThreads)
 gat_bwd_kernel(Items it, BwdArgs A) {
+  constexpr bool RR = ROLE != 2, CR = ROLE != 1;
   using L = RowLayout<K, NH>;
   const int lane = threadIdx.x & 31, g = lane / L::LANES, q = lane % L::LANES;
   const int64_t nitems = it.n_chunks + it.n_light;
@@ -294,10 +298,10 @@ gat_bwd_kernel(Items it, BwdArgs A) {
           for (int v = 0; v < L::VPL; ++v) {
             const int c = L::col(v, q), h = c / L::D;
             if (val[u]) {
-              Pi[u][v] = ldg4(A.P + i * K + c);
-              Gi[u][v] = ldg4(A.G + i * K + c);
-              ri[u][v] = __ldg(A.rec + i * NH + h);
-              ti[u][v] = __ldg(A.st + i * (2 * NH) + NH + h);
+              Pi[u][v] = RR ? ldg4(A.P + i * K + c) : f4(0.f);
+              Gi[u][v] = CR ? ldg4(A.G + i * K + c) : f4(0.f);
+              ri[u][v] = CR ? __ldg(A.rec + i * NH + h) : f4(0.f);
+              ti[u][v] = RR ? __ldg(A.st + i * (2 * NH) + NH + h) : 0.f;
             } else {
               Pi[u][v] = Gi[u][v] = ri[u][v] = f4(0.f);
               ti[u][v] = 0.f;
@@ -312,22 +316,24 @@ gat_bwd_kernel(Items it, BwdArgs A) {
             d1[v] = dot4(Gj[v], Pi[u][v]);   // G_j . P_i  (row role, dalpha_ji)
             d2[v] = dot4(Gi[u][v], Pj[v]);   // G_i . P_j  (column role, dalpha_ij)
           }
-          L::head_reduce(d1);
-          L::head_reduce(d2);
+          if (RR) L::head_reduce(d1);
+          if (CR) L::head_reduce(d2);
           if (val[u]) {
 #pragma unroll
             for (int v = 0; v < L::VPL; ++v) {
-              // row role: entry (j,i) of row j, centre j
-              const float pre = rj[v].x + ti[u][v];
-              const float e = pre > 0.f ? pre : slope * pre;
-              const float aji = ex2(e - rj[v].y) * rj[v].z;
-              ds[v] = fmaf(aji * (pre > 0.f ? 1.f : slope), d1[v] - rj[v].w, ds[v]);
-              // column role: entry (i,j) of row i, centre i
-              const float pre2 = ri[u][v].x + tj[v];
-              const float e2 = pre2 > 0.f ? pre2 : slope * pre2;
-              const float aij = ex2(e2 - ri[u][v].y) * ri[u][v].z;
-              dt[v] = fmaf(aij * (pre2 > 0.f ? 1.f : slope), d2[v] - ri[u][v].w, dt[v]);
-              acc[v] = fma4(aij, Gi[u][v], acc[v]);
+              if (RR) {  // row role: entry (j,i) of row j, centre j
+                const float pre = rj[v].x + ti[u][v];
+                const float e = pre > 0.f ? pre : slope * pre;
+                const float aji = ex2(e - rj[v].y) * rj[v].z;
+                ds[v] = fmaf(aji * (pre > 0.f ? 1.f : slope), d1[v] - rj[v].w, ds[v]);
+              }
+              if (CR) {  // column role: entry (i,j) of row i, centre i
+                const float pre2 = ri[u][v].x + tj[v];
+                const float e2 = pre2 > 0.f ? pre2 : slope * pre2;
+                const float aij = ex2(e2 - ri[u][v].y) * ri[u][v].z;
+                dt[v] = fmaf(aij * (pre2 > 0.f ? 1.f : slope), d2[v] - ri[u][v].w, dt[v]);
+                acc[v] = fma4(aij, Gi[u][v], acc[v]);
+              }
             }
           }
         }
@@ -350,17 +356,27 @@ gat_bwd_kernel(Items it, BwdArgs A) {
 #pragma unroll
       for (int v = 0; v < L::VPL; ++v) {
         const int c = L::col(v, q);
-        st4(A.pacc + slot * K + c, acc[v]);
+        if (CR) st4(A.pacc + slot * K + c, acc[v]);
         if ((c % L::D) == 0) {
-          A.pds[slot * NH + c / L::D] = ds[v];
-          A.pdt[slot * NH + c / L::D] = dt[v];
+          if (RR) A.pds[slot * NH + c / L::D] = ds[v];
+          if (CR) A.pdt[slot * NH + c / L::D] = dt[v];
         }
       }
+    } else if (ROLE == 1) {
+#pragma unroll
+      for (int v = 0; v < L::VPL; ++v) {
+        const int c = L::col(v, q);
+        if ((c % L::D) == 0) A.ds_dir[row * NH + c / L::D] = ds[v];
+      }
     } else {
+      if (ROLE == 2) {
+#pragma unroll
+        for (int v = 0; v < L::VPL; ++v) ds[v] = A.ds_dir[row * NH + L::col(v, q) / L::D];
+      }
       bwd_finish<K, NH>(A, row, grow, q, ds, dt, acc, da1, da2);
     }
   }
-  if (g == 0) {
+  if (g == 0 && ROLE != 1) {
 #pragma unroll
     for (int v = 0; v < L::VPL; ++v) {
       const int c = L::col(v, q);
@@ -370,7 +386,7 @@ gat_bwd_kernel(Items it, BwdArgs A) {
   }
 }
 
-template <int K, int NH>
+template <int K, int NH, int ROLE = 0>
 __global__ void __launch_bounds__(kSparseThreads)
 gat_bwd_merge_kernel(Items it, BwdArgs A, int64_t da_row0) {
   using L = RowLayout<K, NH>;
@@ -394,15 +410,27 @@ gat_bwd_merge_kernel(Items it, BwdArgs A, int64_t da_row0) {
 #pragma unroll
         for (int v = 0; v < L::VPL; ++v) {
           const int c = L::col(v, q), hh = c / L::D;
-          acc[v] = add4(acc[v], ldg4(A.pacc + s * K + c));
-          ds[v] += A.pds[s * NH + hh];
-          dt[v] += A.pdt[s * NH + hh];
+          if (ROLE != 1) acc[v] = add4(acc[v], ldg4(A.pacc + s * K + c));
+          if (ROLE != 2) ds[v] += A.pds[s * NH + hh];
+          if (ROLE != 1) dt[v] += A.pdt[s * NH + hh];
         }
+      }
+      if (ROLE == 1) {
+#pragma unroll
+        for (int v = 0; v < L::VPL; ++v) {
+          const int c = L::col(v, q);
+          if ((c % L::D) == 0) A.ds_dir[row * NH + c / L::D] = ds[v];
+        }
+        continue;
+      }
+      if (ROLE == 2) {
+#pragma unroll
+        for (int v = 0; v < L::VPL; ++v) ds[v] = A.ds_dir[row * NH + L::col(v, q) / L::D];
       }
       bwd_finish<K, NH>(A, row, grow, q, ds, dt, acc, da1, da2);
     }
 #pragma unroll
-    for (int v = 0; v < L::VPL; ++v) {
+    for (int v = 0; v < L::VPL && ROLE != 1; ++v) {
       const int c = L::col(v, q);
       st4(A.da_part + (da_row0 + gw) * 2 * K + c, da1[v]);
       st4(A.da_part + (da_row0 + gw) * 2 * K + K + c, da2[v]);
@@ -551,7 +579,7 @@ size_t saved_size(const Plan& p, const GatShape& g) {
 }
 
 struct WsGat {
-  float *Wext, *pacc, *pm, *pl, *G, *dP, *da_part, *gemm;
+  float *Wext, *pacc, *pm, *pl, *G, *dP, *da_part, *gemm, *ds_dir;
   float4* rec;
   void* saved_inf;  // saved-layout scratch for inference
 };
@@ -562,9 +590,10 @@ WsGat carve_ws(const Plan& p, const GatShape& g, void* base, size_t* total) {
   WsGat w;
   const int NE = (g.k_out + 2 * g.heads + 3) / 4 * 4;
   w.Wext = c.take<float>((size_t)g.k_in * NE);
-  w.pacc = c.take<float>((size_t)p.n_chunks * 3 * g.k_out);
-  w.pm = c.take<float>((size_t)p.n_chunks * g.heads);
-  w.pl = c.take<float>((size_t)p.n_chunks * g.heads);
+  w.pacc = c.take<float>((size_t)p.max_chunks() * 3 * g.k_out);
+  w.pm = c.take<float>((size_t)p.max_chunks() * g.heads);
+  w.pl = c.take<float>((size_t)p.max_chunks() * g.heads);
+  w.ds_dir = c.take<float>(p.csc_ptr ? (size_t)p.n_local * g.heads : 0);
   w.G = c.take<float>((size_t)p.n * g.k_out);
   w.rec = c.take<float4>((size_t)p.n * g.heads);
   w.dP = c.take<float>((size_t)p.n_local * g.k_out);
@@ -648,8 +677,10 @@ agnn_status gat_backward(const Plan& p, const GatShape& g, const float* W, const
                          const float* H_in, const void* saved, const float* dH_out,
                          float* dH_in, float* dW, float* da, void* ws, cudaStream_t s) {
   if (!saved) return fail(AGNN_EINVAL, "agnn_backward: saved == NULL");
-  if (!(p.flags & AGNN_CSR_SYMMETRIC))
-    return fail(AGNN_EUNSUPPORTED, "agnn_backward: the single-pass backward needs a symmetric CSR");
+  const bool directed = p.directed();
+  if (directed && !p.csc_ptr)
+    return fail(AGNN_EUNSUPPORTED,
+                "agnn_backward: a directed pattern needs world == 1 and every row in the plan");
   WsGat w = carve_ws(p, g, ws, nullptr);
   SavedGat sv = carve_saved(p, g, const_cast<void*>(saved));
   const int K_ = g.k_out, NH_ = g.heads;
@@ -666,9 +697,33 @@ agnn_status gat_backward(const Plan& p, const GatShape& g, const float* W, const
       return st;
   }
   BwdArgs A{sv.P, sv.st, w.G, w.rec, a, g.slope, w.dP, w.pacc, w.pm, w.pl, w.da_part,
-            nullptr, nullptr};
+            nullptr, nullptr, w.ds_dir};
   int64_t main_warps = 0, merge_warps = 0;
-  if (gat_k128_supported(g.k_out, g.heads)) {
+  if (directed) {
+    // row role over the CSR (ds_j), then the column role over the CSC (dt_j, acc_j, dP_j)
+    Items itc = items_of_csc(p);
+    AGNN_GAT_DISPATCH(K_, NH_, (gat_bwd_kernel<K, NH, bwd_unroll<K>(), 1>
+                                <<<grid_of(gat_bwd_kernel<K, NH, bwd_unroll<K>(), 1>),
+                                   kSparseThreads, 0, s>>>(it, A)));
+    AGNN_LAUNCH_CHECK("gat_bwd_row_kernel");
+    if (it.n_heavy > 0) {
+      AGNN_GAT_DISPATCH(K_, NH_, (gat_bwd_merge_kernel<K, NH, 1>
+                                  <<<kNumSMs * 2, kSparseThreads, 0, s>>>(it, A, 0)));
+      AGNN_LAUNCH_CHECK("gat_bwd_merge_kernel");
+    }
+    it = itc;
+    AGNN_GAT_DISPATCH(K_, NH_, (main_warps = (int64_t)grid_of(gat_bwd_kernel<K, NH, bwd_unroll<K>(), 2>) *
+                                             (kSparseThreads / 32)));
+    AGNN_GAT_DISPATCH(K_, NH_, (gat_bwd_kernel<K, NH, bwd_unroll<K>(), 2>
+                                <<<(unsigned)(main_warps / 8), kSparseThreads, 0, s>>>(it, A)));
+    AGNN_LAUNCH_CHECK("gat_bwd_col_kernel");
+    AGNN_GAT_DISPATCH(K_, NH_, (merge_warps = (int64_t)grid_of(gat_bwd_merge_kernel<K, NH, 2>) *
+                                              (kSparseThreads / 32)));
+    AGNN_GAT_DISPATCH(K_, NH_, (gat_bwd_merge_kernel<K, NH, 2>
+                                <<<(unsigned)(merge_warps / 8), kSparseThreads, 0, s>>>(
+                                    it, A, main_warps)));
+    AGNN_LAUNCH_CHECK("gat_bwd_merge_kernel");
+  } else if (gat_k128_supported(g.k_out, g.heads)) {
     if ((st = gat_bwd_k128(it, g.heads, A, &main_warps, s)) != AGNN_OK) return st;
   } else {
     AGNN_GAT_DISPATCH(K_, NH_, (main_warps = (int64_t)grid_of(gat_bwd_kernel<K, NH, bwd_unroll<K>()>) *
@@ -677,12 +732,14 @@ agnn_status gat_backward(const Plan& p, const GatShape& g, const float* W, const
                                 <<<(unsigned)(main_warps / 8), kSparseThreads, 0, s>>>(it, A)));
     AGNN_LAUNCH_CHECK("gat_bwd_kernel");
   }
-  AGNN_GAT_DISPATCH(K_, NH_, (merge_warps = (int64_t)grid_of(gat_bwd_merge_kernel<K, NH>) *
-                                            (kSparseThreads / 32)));
-  AGNN_GAT_DISPATCH(K_, NH_, (gat_bwd_merge_kernel<K, NH>
-                              <<<(unsigned)(merge_warps / 8), kSparseThreads, 0, s>>>(it, A,
-                                                                                     main_warps)));
-  AGNN_LAUNCH_CHECK("gat_bwd_merge_kernel");
+  if (!directed) {
+    AGNN_GAT_DISPATCH(K_, NH_, (merge_warps = (int64_t)grid_of(gat_bwd_merge_kernel<K, NH>) *
+                                              (kSparseThreads / 32)));
+    AGNN_GAT_DISPATCH(K_, NH_, (gat_bwd_merge_kernel<K, NH>
+                                <<<(unsigned)(merge_warps / 8), kSparseThreads, 0, s>>>(
+                                    it, A, main_warps)));
+    AGNN_LAUNCH_CHECK("gat_bwd_merge_kernel");
+  }
   const int64_t da_rows_used = main_warps + merge_warps;
   if (da) {
     gat_da_reduce_kernel<<<(2 * g.k_out + 31) / 32, 1024, 0, s>>>(

@@ -28,6 +28,7 @@ struct GatBwdArgs {
   float* da_part;      // [warps x 2K]
   float* ds_out;       // [n_local x NH] nullable
   float* dt_out;       // [n_local x NH] nullable
+  float* ds_dir;       // [n_local x NH] directed patterns: row-pass ds for the column pass
 };
 
 // k' = 128 kernels (gat_k128.cu): lane-parallel scalar work, warp-parallel rows

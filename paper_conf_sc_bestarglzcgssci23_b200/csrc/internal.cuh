@@ -21,6 +21,13 @@ struct Items {
   int64_t n_local;
 };
 Items items_of(const Plan& p);
+// the transposed pattern's items (directed plans): "rows" are columns j, col = rows i
+Items items_of_csc(const Plan& p);
+// CSC (+ optional CSR position of every CSC entry) of a local CSR with n_rows rows
+// starting at global row 0; device radix sort, synchronises (plan time only)
+agnn_status build_csc(const int64_t* row_ptr, const int32_t* col, int64_t n_rows, int64_t n,
+                      int64_t nnz, int64_t* csc_ptr, int32_t* csc_idx, int64_t* perm,
+                      cudaStream_t s);
 
 
 // persistent sparse-kernel grid: 256-thread blocks, SMs x resident blocks of `func`

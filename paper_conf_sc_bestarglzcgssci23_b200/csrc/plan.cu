@@ -83,6 +83,82 @@ Items items_of(const Plan& p) {
   return it;
 }
 
+namespace {
+
+// static work list of one pattern (rows of the CSR, or columns of the CSC)
+struct Lists {
+  int64_t n_light = 0, n_heavy = 0, n_chunks = 0, n_empty = 0, max_deg = 0;
+  int32_t *light = nullptr, *chunk_row = nullptr, *chunk_idx = nullptr, *heavy = nullptr,
+          *heavy_off = nullptr, *empty = nullptr;
+  void* block = nullptr;
+};
+
+agnn_status build_lists(const std::vector<int64_t>& rp, int64_t n_rows, int chunk, bool with_empty,
+                        Lists& out, cudaStream_t s) {
+  std::vector<int32_t> light, chunk_row, chunk_idx, heavy, heavy_off{0}, empty;
+  light.reserve((size_t)n_rows);
+  int64_t maxdeg = 0;
+  for (int64_t i = 0; i < n_rows; ++i) {
+    const int64_t d = rp[(size_t)i + 1] - rp[(size_t)i];
+    maxdeg = std::max(maxdeg, d);
+    if (d == 0 && with_empty) empty.push_back((int32_t)i);
+    if (d > chunk) {
+      const int64_t c = (d + chunk - 1) / chunk;
+      heavy.push_back((int32_t)i);
+      for (int64_t q = 0; q < c; ++q) {
+        chunk_row.push_back((int32_t)i);
+        chunk_idx.push_back((int32_t)q);
+      }
+      heavy_off.push_back((int32_t)chunk_row.size());
+    } else {
+      light.push_back((int32_t)i);
+    }
+  }
+  out.max_deg = maxdeg;
+  out.n_light = (int64_t)light.size();
+  out.n_heavy = (int64_t)heavy.size();
+  out.n_chunks = (int64_t)chunk_row.size();
+  out.n_empty = (int64_t)empty.size();
+  const size_t total = light.size() + 2 * chunk_row.size() + heavy.size() + heavy_off.size() +
+                       empty.size() + 160;
+  AGNN_CUDA_TRY(cudaMalloc(&out.block, sizeof(int32_t) * total));
+  int32_t* b = static_cast<int32_t*>(out.block);
+  auto put = [&](std::vector<int32_t>& v, int32_t*& dst) -> cudaError_t {
+    dst = b;
+    b += v.size() + 16 - (v.size() % 16);
+    if (v.empty()) return cudaSuccess;
+    return cudaMemcpyAsync(dst, v.data(), sizeof(int32_t) * v.size(), cudaMemcpyHostToDevice, s);
+  };
+  AGNN_CUDA_TRY(put(light, out.light));
+  AGNN_CUDA_TRY(put(chunk_row, out.chunk_row));
+  AGNN_CUDA_TRY(put(chunk_idx, out.chunk_idx));
+  AGNN_CUDA_TRY(put(heavy, out.heavy));
+  AGNN_CUDA_TRY(put(heavy_off, out.heavy_off));
+  AGNN_CUDA_TRY(put(empty, out.empty));
+  AGNN_CUDA_TRY(cudaStreamSynchronize(s));  // the host vectors die here
+  return AGNN_OK;
+}
+
+}  // namespace
+
+Items items_of_csc(const Plan& p) {
+  Items it;
+  it.row_ptr = p.csc_ptr;
+  it.col = p.csc_idx;
+  it.light_rows = p.c_light_rows;
+  it.n_light = p.c_light;
+  it.chunk_row = p.c_chunk_row;
+  it.chunk_idx = p.c_chunk_idx;
+  it.n_chunks = p.c_chunks;
+  it.chunk = p.chunk;
+  it.heavy_rows = p.c_heavy_rows;
+  it.heavy_off = p.c_heavy_off;
+  it.n_heavy = p.c_heavy;
+  it.row_begin = 0;
+  it.n_local = p.n;
+  return it;
+}
+
 agnn_status plan_build(Plan& p, cudaStream_t s) {
   // heavy-row chunk size (edges); AGNN_CHUNK_EDGES overrides it (tests use small
   // chunks to exercise the split/merge path on small graphs)
@@ -115,47 +191,47 @@ agnn_status plan_build(Plan& p, cudaStream_t s) {
     return fail(AGNN_EINVAL, m);
   }
   p.nnz = rp[(size_t)p.n_local];
-  // 3. work lists
-  std::vector<int32_t> light, chunk_row, chunk_idx, heavy, heavy_off{0}, empty;
-  light.reserve((size_t)p.n_local);
-  int64_t maxdeg = 0;
-  for (int64_t i = 0; i < p.n_local; ++i) {
-    const int64_t d = rp[(size_t)i + 1] - rp[(size_t)i];
-    maxdeg = std::max(maxdeg, d);
-    if (d == 0) empty.push_back((int32_t)i);
-    if (d > p.chunk) {
-      const int64_t c = (d + p.chunk - 1) / p.chunk;
-      heavy.push_back((int32_t)i);
-      for (int64_t q = 0; q < c; ++q) {
-        chunk_row.push_back((int32_t)i);
-        chunk_idx.push_back((int32_t)q);
-      }
-      heavy_off.push_back((int32_t)chunk_row.size());
-    } else {
-      light.push_back((int32_t)i);
-    }
+  // 3. work lists of the rows
+  Lists L;
+  agnn_status st = build_lists(rp, p.n_local, p.chunk, true, L, s);
+  if (st != AGNN_OK) return st;
+  p.max_deg = L.max_deg;
+  p.n_light = L.n_light;
+  p.n_heavy = L.n_heavy;
+  p.n_chunks = L.n_chunks;
+  p.n_empty = L.n_empty;
+  p.light_rows = L.light;
+  p.chunk_row = L.chunk_row;
+  p.chunk_idx = L.chunk_idx;
+  p.heavy_rows = L.heavy;
+  p.heavy_off = L.heavy_off;
+  p.empty_rows = L.empty;
+  p.meta_block = L.block;
+  // 4. directed pattern on one GPU: the CSC and its work lists (column role of the backward)
+  if (p.directed() && p.world == 1 && p.n_local == p.n) {
+    const size_t ptr_bytes = ((sizeof(int64_t) * (size_t)(p.n + 1)) + 255) & ~size_t(255);
+    AGNN_CUDA_TRY(cudaMalloc(&p.csc_block, ptr_bytes + sizeof(int32_t) * (size_t)(p.nnz + 1)));
+    p.csc_ptr = static_cast<int64_t*>(p.csc_block);
+    p.csc_idx = reinterpret_cast<int32_t*>(static_cast<char*>(p.csc_block) + ptr_bytes);
+    if ((st = build_csc(p.row_ptr, p.col_idx, p.n_local, p.n, p.nnz, p.csc_ptr, p.csc_idx, nullptr,
+                        s)) != AGNN_OK)
+      return st;
+    std::vector<int64_t> cp((size_t)p.n + 1);
+    AGNN_CUDA_TRY(cudaMemcpyAsync(cp.data(), p.csc_ptr, sizeof(int64_t) * cp.size(),
+                                  cudaMemcpyDeviceToHost, s));
+    AGNN_CUDA_TRY(cudaStreamSynchronize(s));
+    Lists C;
+    if ((st = build_lists(cp, p.n, p.chunk, false, C, s)) != AGNN_OK) return st;
+    p.c_light = C.n_light;
+    p.c_heavy = C.n_heavy;
+    p.c_chunks = C.n_chunks;
+    p.c_light_rows = C.light;
+    p.c_chunk_row = C.chunk_row;
+    p.c_chunk_idx = C.chunk_idx;
+    p.c_heavy_rows = C.heavy;
+    p.c_heavy_off = C.heavy_off;
+    p.c_meta_block = C.block;
   }
-  p.max_deg = maxdeg;
-  p.n_light = (int64_t)light.size();
-  p.n_heavy = (int64_t)heavy.size();
-  p.n_chunks = (int64_t)chunk_row.size();
-  p.n_empty = (int64_t)empty.size();
-  const size_t total = light.size() + 2 * chunk_row.size() + heavy.size() + heavy_off.size() +
-                       empty.size() + 160;
-  AGNN_CUDA_TRY(cudaMalloc(&p.meta_block, sizeof(int32_t) * total));
-  int32_t* b = static_cast<int32_t*>(p.meta_block);
-  auto put = [&](std::vector<int32_t>& v, int32_t*& dst) -> cudaError_t {
-    dst = b;
-    b += v.size() + 16 - (v.size() % 16);
-    if (v.empty()) return cudaSuccess;
-    return cudaMemcpyAsync(dst, v.data(), sizeof(int32_t) * v.size(), cudaMemcpyHostToDevice, s);
-  };
-  AGNN_CUDA_TRY(put(light, p.light_rows));
-  AGNN_CUDA_TRY(put(chunk_row, p.chunk_row));
-  AGNN_CUDA_TRY(put(chunk_idx, p.chunk_idx));
-  AGNN_CUDA_TRY(put(heavy, p.heavy_rows));
-  AGNN_CUDA_TRY(put(heavy_off, p.heavy_off));
-  AGNN_CUDA_TRY(put(empty, p.empty_rows));
   AGNN_CUDA_TRY(cudaStreamSynchronize(s));
   return AGNN_OK;
 }

@@ -54,7 +54,8 @@ class Stack:
     """Buffers + plan + model for one workload on this rank."""
 
     def __init__(self, w: gen.Workload, device="cuda", rank=0, world=1, nccl_uid=None,
-                 c_v: int = 4, graph: Graph | None = None, inputs_on_device=True):
+                 c_v: int = 4, graph: Graph | None = None, inputs_on_device=True,
+                 symmetric: bool = True):
         self.w, self.device, self.rank, self.world = w, torch.device(device), rank, world
         self.stream = torch.cuda.current_stream(self.device)
         g = graph or build_graph(w, self.device)
@@ -69,7 +70,8 @@ class Stack:
             self.row_ptr, self.col_idx = g.row_ptr, g.col_idx
         self.row_begin, self.row_end, self.n_local = b0, b1, b1 - b0
         self.nnz_local = int(self.col_idx.numel())
-        self.plan = agnn.Plan(self.row_ptr, self.col_idx, w.n, b0, b1, symmetric=True, rank=rank,
+        # symmetric=False: a directed pattern (reading A4); the plan builds its CSC
+        self.plan = agnn.Plan(self.row_ptr, self.col_idx, w.n, b0, b1, symmetric=symmetric, rank=rank,
                               world=world, nccl_unique_id=nccl_uid, bounds=self.bounds)
         descs = [agnn.layer_desc(w.model, w.k, w.k, w.heads, w.act, negative_slope=w.slope,
                                  beta=w.beta, eps=w.eps) for _ in range(w.layers)]

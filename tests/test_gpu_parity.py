@@ -173,3 +173,84 @@ def test_launch_count_increases():
     c0 = agnn.launch_count()
     st.step()
     assert agnn.launch_count() > c0
+
+
+# ------------------------------------------------------------------ directed patterns (A4)
+DIRECTED_FLAGS = agnn.BUILD_SELF_LOOPS | agnn.BUILD_CONNECT_ISOLATED
+
+
+def _directed_graph(w):
+    src, dst = w.host_edges()
+    rp, ci = oracle.csr_build(w.n, src, dst, flags=DIRECTED_FLAGS)
+    s = torch.from_numpy(src.view(np.int32)).cuda()
+    d = torch.from_numpy(dst.view(np.int32)).cuda()
+    drp, dci = agnn.csr_build(w.n, s, d, DIRECTED_FLAGS)
+    np.testing.assert_array_equal(drp.cpu().numpy(), rp)
+    np.testing.assert_array_equal(dci.cpu().numpy(), ci)
+    return rp, ci, runner.Graph(w.n, drp, dci, int(dci.numel()))
+
+
+def test_plan_csc_bit_exact():
+    """agnn_plan_csc: the transposed pattern + CSR positions, against a host sort."""
+    w = W("gat", "kron", 14, 8, 16)
+    rp, ci, g = _directed_graph(w)
+    plan = agnn.Plan(g.row_ptr, g.col_idx, w.n, symmetric=False)
+    cp, ri, perm = plan.csc()
+    rows = np.repeat(np.arange(w.n, dtype=np.int64), np.diff(rp))
+    order = np.lexsort((rows, ci))  # by column, then row
+    np.testing.assert_array_equal(perm.cpu().numpy(), order)
+    np.testing.assert_array_equal(ri.cpu().numpy(), rows[order].astype(np.int32))
+    np.testing.assert_array_equal(cp.cpu().numpy(),
+                                  np.concatenate([[0], np.cumsum(np.bincount(ci, minlength=w.n))]))
+
+
+DIRECTED_CASES = [
+    W("gat", "kron", 15, 8, 16, heads=1, act="none"),
+    W("gat", "kron", 16, 8, 128, heads=4),
+    W("gat", "rmat", 14, 16, 64, heads=2, act="elu"),
+    W("agnn", "kron", 15, 8, 64),
+    W("agnn", "rmat", 14, 16, 128, act="elu"),
+    W("va", "kron", 14, 8, 32),
+    W("va", "er", 0, 0, 128, n=5000, samples=60000, act="none"),
+]
+
+
+@pytest.mark.parametrize("w", DIRECTED_CASES, ids=lambda w: w.name)
+def test_directed_layer_parity(w):
+    """Directed pattern: row pass over the CSR + column pass over the plan's CSC."""
+    rp, ci, g = _directed_graph(w)
+    # the pattern really is unsymmetric (in-degrees differ from out-degrees)
+    cols = np.bincount(ci, minlength=w.n)
+    assert not np.array_equal(cols, np.diff(rp))
+    H, Ws, As, R = w.host_inputs()
+    if w.act == "relu":
+        f0 = pu.oracle_step(w, rp, ci, H, Ws, As, R)["fwd"][-1]
+        R = pu.relu_kink_mask(w, f0["Z"], R)
+    st = pu.gpu_step(w, graph=g, R=R, symmetric=False)
+    ref = pu.oracle_step(w, rp, ci, H, Ws, As, R)
+    pu.compare(w, st, ref)
+    pu.compare_attention(w, st, ref)
+
+
+def test_directed_heavy_chunks(monkeypatch):
+    """Small chunks force heavy rows AND heavy columns through the split/merge path."""
+    monkeypatch.setenv("AGNN_CHUNK_EDGES", "64")
+    for model, heads in (("gat", 4), ("agnn", 1), ("va", 1)):
+        w = W(model, "kron", 12, 8, 64, heads=heads, act="none")
+        rp, ci, g = _directed_graph(w)
+        st = pu.gpu_step(w, graph=g, symmetric=False)
+        assert st.plan.info()["heavy_rows"] > 0
+        H, Ws, As, R = w.host_inputs()
+        pu.compare(w, st, pu.oracle_step(w, rp, ci, H, Ws, As, R))
+
+
+def test_symmetric_flag_on_directed_pattern_is_not_silently_wrong():
+    """The same directed pattern through a plan WITHOUT the flag must match the oracle;
+    a symmetric plan over a symmetric pattern gives the same result as a directed plan."""
+    w = W("gat", "kron", 13, 8, 64, heads=2, act="none")
+    src, dst, rp, ci = pu.host_graph(w)   # symmetric pattern
+    g = pu.device_graph(w, src, dst)
+    a = pu.gpu_step(w, graph=g)
+    b = pu.gpu_step(w, graph=g, symmetric=False)
+    for x, y in ((a.dH[0], b.dH[0]), (a.dW[0], b.dW[0]), (a.da[0], b.da[0])):
+        assert pu.rel(x.cpu().numpy(), y.cpu().numpy()) <= 1e-6
