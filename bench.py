@@ -109,8 +109,9 @@ def oracle_sample(w, scale):
     from paper_conf_sc_bestarglzcgssci23_b200 import gen
     ef = max(1, w.n_samples // w.n)
     n = 1 << scale if w.graph != "er" else min(w.n, 1 << scale)
-    return gen.Workload(f"{w.name}-sample-2^{scale}", w.model, w.graph, scale, n, ef * n, w.k,
-                        w.heads, w.layers, w.seed, w.act, w.slope, w.beta, w.eps)
+    import dataclasses
+    return dataclasses.replace(w, name=f"{w.name}-sample-2^{scale}", scale=scale, n=n,
+                               n_samples=ef * n)
 
 
 def time_oracle(w, scale, reps=1):
@@ -125,7 +126,7 @@ def time_oracle(w, scale, reps=1):
     times = []
     for _ in range(reps):
         t0 = time.perf_counter()
-        pu.oracle_step(ws, rp, ci, H, Ws, As, R)
+        oracle_train_step(pu, ws, rp, ci, H, Ws, As, R)
         times.append(time.perf_counter() - t0)
     cores = len(os.sched_getaffinity(0))
     return ws, len(ci), times, cores
@@ -146,10 +147,27 @@ def workload(args):
     w = gen.CONFIGS[args.config]
     if args.scale is not None and w.graph != "er":
         ef = w.n_samples // w.n
-        w = gen.Workload(f"{w.name}@2^{args.scale}", w.model, w.graph, args.scale, 1 << args.scale,
-                         ef << args.scale, w.k, w.heads, w.layers, w.seed, w.act, w.slope, w.beta,
-                         w.eps)
+        import dataclasses
+        w = dataclasses.replace(w, name=f"{w.name}@2^{args.scale}", scale=args.scale,
+                                n=1 << args.scale, n_samples=ef << args.scale)
     return w
+
+
+def metric_name(w):
+    if w.train:
+        return f"{w.model.upper()} training step (fwd+bwd+SGD) edges/s"
+    return METRIC if w.model == "gat" else f"{w.model.upper()} layer fwd+bwd edges/s"
+
+
+def oracle_train_step(pu, w, rp, ci, H, Ws, As, R):
+    """One oracle step; for training workloads also the SGD update (numpy, fp64)."""
+    ref = pu.oracle_step(w, rp, ci, H, Ws, As, R)
+    if w.train:
+        for l in range(w.layers):
+            Ws[l] = Ws[l] - w.lr * ref["dW"][l]
+            if As[l] is not None:
+                As[l] = As[l] - w.lr * ref["da"][l]
+    return ref
 
 
 def run_reference(args):
@@ -168,17 +186,17 @@ def run_reference(args):
     rp, ci = oracle.csr_build(ws.n, src, dst)
     H, Ws, As, R = ws.host_inputs()
     for _ in range(args.warmup):
-        pu.oracle_step(ws, rp, ci, H, Ws, As, R)
+        oracle_train_step(pu, ws, rp, ci, H, Ws, As, R)
     t0 = time.perf_counter()
     for _ in range(args.steps):
-        pu.oracle_step(ws, rp, ci, H, Ws, As, R)
+        oracle_train_step(pu, ws, rp, ci, H, Ws, As, R)
     T = (time.perf_counter() - t0) / args.steps
     m = len(ci)
     val = ws.layers * m / T
     cores = len(os.sched_getaffinity(0))
     sample = (f"oracle (C, FP64, OpenMP) on {gen.describe(ws)}, m={m} — a bounded sample of "
               f"{args.config} ({gen.describe(w)})")
-    line = {"impl": "reference", "metric": METRIC, "value": val, "unit": UNIT, "n_gpus": args.gpus,
+    line = {"impl": "reference", "metric": metric_name(w), "value": val, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": T * 1e3,
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
             "data": "synthetic",
@@ -312,17 +330,19 @@ def run_ours(args):
     kernels = {k: {"launches": v[0], "ms_per_step": v[1] / args.steps} for k, v in prof.items()}
 
     # ---- end-to-end through the C ABI with host buffers -------------------------
-    # Every step copies its inputs (H, dL/dH_out = R) from pinned host memory and
-    # reads its results (dH, dW, da) back.  Inputs are double-buffered on the
-    # device: step s+1's H2D runs on a copy stream while step s computes, and
-    # step s's D2H on a second stream while step s+1 computes (input prefetch as
-    # a training loop would do it); the timed region spans all K steps' copies.
+    # Every step copies its inputs (H^0 and the upstream gradient R = dL/dH^L)
+    # from pinned host memory, runs the step through agnn_forward/agnn_backward,
+    # evaluates the loss L = <R, H^L> (agnn_loss_inner, reading A13) and reads the
+    # step's results back: the loss and the parameter gradients dW (and da).
+    # Inputs are double-buffered on the device: step s+1's H2D runs on a copy
+    # stream while step s computes (input prefetch as a training loop does it);
+    # the timed region spans all K steps' copies.
     e2e = None
     if not args.no_e2e:
         nl, k, L = st.n_local, w.k, w.layers
         h_H = torch.empty((nl, k), dtype=torch.float32, pin_memory=True)
         h_R = torch.empty((nl, k), dtype=torch.float32, pin_memory=True)
-        h_dH = torch.empty((nl, k), dtype=torch.float32, pin_memory=True)
+        h_loss = torch.empty(1, dtype=torch.float64, pin_memory=True)
         h_dW = [torch.empty(tuple(x.shape), dtype=torch.float32, pin_memory=True) for x in st.dW]
         das = [x for x in st.da if x is not None]
         h_da = [torch.empty(tuple(x.shape), dtype=torch.float32, pin_memory=True) for x in das]
@@ -330,11 +350,10 @@ def run_ours(args):
         h_R.copy_(st.dH[L].cpu())
         Hb = [st.H[0], torch.empty_like(st.H[0])]
         Rb = [st.dH[L], torch.empty_like(st.dH[L])]
-        Db = [st.dH[0], torch.empty_like(st.dH[0])]
         up, down = torch.cuda.Stream(dev), torch.cuda.Stream(dev)
         ev_in = [torch.cuda.Event(), torch.cuda.Event()]
         ev_done = [torch.cuda.Event(), torch.cuda.Event()]
-        ev_out = [torch.cuda.Event(), torch.cuda.Event()]
+        st.loss()  # allocate the loss buffers outside the timed region
         barrier()
         e2, e3 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e2.record(stream)
@@ -353,24 +372,22 @@ def run_ours(args):
                     Rb[b ^ 1].copy_(h_R, non_blocking=True)
                     ev_in[b ^ 1].record(up)
             stream.wait_event(ev_in[b])
-            if s_ >= 2:
-                stream.wait_event(ev_out[b])  # dH buffer b was read back by step s-2's D2H
-            st.H[0], st.dH[L], st.dH[0] = Hb[b], Rb[b], Db[b]
+            st.H[0], st.dH[L] = Hb[b], Rb[b]
             st.step()
+            loss_d = st.loss()
             ev_done[b].record(stream)
             with torch.cuda.stream(down):
                 down.wait_event(ev_done[b])
-                h_dH.copy_(Db[b], non_blocking=True)
+                h_loss.copy_(loss_d, non_blocking=True)
                 for hw_, dw_ in zip(h_dW, st.dW):
                     hw_.copy_(dw_, non_blocking=True)
                 for ha_, da_ in zip(h_da, das):
                     ha_.copy_(da_, non_blocking=True)
-                ev_out[b].record(down)
-        stream.wait_stream(down)
+            stream.wait_stream(down)  # the next step overwrites dW / da / loss
         stream.wait_stream(up)
         e3.record(stream)
         barrier()
-        st.H[0], st.dH[L], st.dH[0] = Hb[0], Rb[0], Db[0]
+        st.H[0], st.dH[L] = Hb[0], Rb[0]
         ms2 = e2.elapsed_time(e3)
         if world > 1:
             t = torch.tensor([ms2], device=dev)
@@ -378,11 +395,14 @@ def run_ours(args):
             ms2 = float(t.item())
         T2 = ms2 / 1e3 / args.steps
         h2d = 2 * nl * k * 4
-        d2h = nl * k * 4 + sum(x.numel() * 4 for x in h_dW) + sum(x.numel() * 4 for x in h_da)
+        d2h = 8 + sum(x.numel() * 4 for x in h_dW) + sum(x.numel() * 4 for x in h_da)
         e2e = {"value": w.layers * m / T2, "unit": UNIT, "h2d_bytes_per_step": h2d * world,
                "d2h_bytes_per_step": d2h * world, "ms_per_step": T2 * 1e3,
-               "api": "agnn_forward/agnn_backward via paper_conf_sc_bestarglzcgssci23_b200.runner",
-               "overlap": "double-buffered inputs: H2D of step s+1 and D2H of step s overlap compute"}
+               "api": "agnn_forward/agnn_backward/agnn_loss_inner via "
+                      "paper_conf_sc_bestarglzcgssci23_b200.runner",
+               "result_read_back": "loss <R, H^L> (fp64) + dW + da per step",
+               "overlap": "double-buffered inputs: H2D of step s+1 overlaps step s",
+               "loss": float(h_loss.item())}
 
     # ---- CPU oracle baseline (rank 0, N = 1 only) ------------------------------
     cpu = None
@@ -395,7 +415,7 @@ def run_ours(args):
                          f"{t_med:.1f} s", "cpu": cpu_model()}
 
     if rank == 0:
-        line = {"metric": METRIC if w.model == "gat" else f"{w.model.upper()} layer fwd+bwd edges/s",
+        line = {"metric": metric_name(w),
                 "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": T * 1e3, "higher_is_better": True,
                 "scaling": "weak" if world == 1 else "strong", "vs_baseline": None,

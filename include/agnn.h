@@ -163,6 +163,19 @@ agnn_status agnn_backward(agnn_model_t model, int layer, const float* W, const f
                           float* dH_in, float* dW, float* da, void* workspace,
                           cudaStream_t stream);
 
+/* ---- the steps either side of the layer path in a training loop --------- */
+/* Loss of reading A13, L = <R, H> = sum_e R[e] * H[e] over `count` fp32
+ * elements (R = dL/dH^L, the Eq. 4 bootstrap).  scratch: device,
+ * AGNN_LOSS_SCRATCH doubles; *loss: device double (this rank's rows only: with
+ * world > 1 the caller adds the ranks' values).  Deterministic fixed-order
+ * fp64 reduction.  R, H 16-byte aligned.                                     */
+#define AGNN_LOSS_SCRATCH 1024
+agnn_status agnn_loss_inner(const float* R, const float* H, int64_t count, double* scratch,
+                            double* loss, cudaStream_t stream);
+/* SGD update of PAPER.md:244: W[e] -= lr * dW[e] for e < count (device).    */
+agnn_status agnn_sgd_step(float* W, const float* dW, int64_t count, float lr,
+                          cudaStream_t stream);
+
 /* Test-only export (excluded from timing): recompute the attention
  * coefficients alpha of `count` stored entries (positions into the LOCAL
  * col_idx) from the saved row statistics.  alpha_out: [count x heads].

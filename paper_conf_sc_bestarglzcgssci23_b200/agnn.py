@@ -26,7 +26,7 @@ STATUS = {0: "AGNN_OK", 1: "AGNN_EINVAL", 2: "AGNN_ECUDA", 3: "AGNN_ENCCL", 4: "
 
 # every symbol include/agnn.h declares (tests check the .so exports all of them)
 EXPORTS = ("agnn_partition", "agnn_plan_create", "agnn_plan_destroy", "agnn_plan_info",
-           "agnn_plan_csc",
+           "agnn_plan_csc", "agnn_loss_inner", "agnn_sgd_step",
            "agnn_model_create", "agnn_model_destroy", "agnn_saved_bytes", "agnn_workspace_bytes",
            "agnn_forward", "agnn_backward", "agnn_debug_attention", "agnn_debug_gemm",
            "agnn_debug_gemm_tn", "agnn_debug_gemm_tn_ws_bytes",
@@ -121,6 +121,23 @@ def profile_report() -> dict:
         name, cnt, ms = line.rsplit(" ", 2)
         out[name] = (int(cnt), float(ms))
     return out
+
+
+LOSS_SCRATCH = 1024  # AGNN_LOSS_SCRATCH
+
+
+def loss_inner(R, H, scratch, loss, stream=None):
+    """agnn_loss_inner: loss[0] = <R, H> in fp64 (device); scratch: >= LOSS_SCRATCH doubles."""
+    assert R.numel() == H.numel() and scratch.numel() >= LOSS_SCRATCH
+    _check(lib().agnn_loss_inner(_ptr(R), _ptr(H), ctypes.c_int64(R.numel()), _ptr(scratch),
+                                 _ptr(loss), _stream(stream)))
+
+
+def sgd_step(W, dW, lr, stream=None):
+    """agnn_sgd_step: W -= lr * dW on the device."""
+    assert W.numel() == dW.numel()
+    _check(lib().agnn_sgd_step(_ptr(W), _ptr(dW), ctypes.c_int64(W.numel()), ctypes.c_float(lr),
+                               _stream(stream)))
 
 
 def debug_gemm(A, B, C, stream=None):

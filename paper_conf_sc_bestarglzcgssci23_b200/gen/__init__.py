@@ -104,6 +104,8 @@ class Workload:
     slope: float = 0.2
     beta: float = 1.0
     eps: float = 1e-12
+    train: bool = False   # step = fwd + bwd + SGD update (C4) instead of fwd + bwd
+    lr: float = 1e-3
 
     @property
     def kind(self) -> int:
@@ -129,8 +131,8 @@ class Workload:
         return edges(self.kind, self.seed, self.scale, self.n, self.n_samples)
 
 
-def _kron(name, model, scale, ef, k, heads, layers, graph="kron"):
-    return Workload(name, model, graph, scale, 1 << scale, ef << scale, k, heads, layers)
+def _kron(name, model, scale, ef, k, heads, layers, graph="kron", **kw):
+    return Workload(name, model, graph, scale, 1 << scale, ef << scale, k, heads, layers, **kw)
 
 
 # BASELINE.json configs[0..4]
@@ -138,7 +140,7 @@ CONFIGS = {
     "C1": Workload("C1", "gat", "er", 10, 1024, 7680, 16, 1, 1),
     "C2": _kron("C2", "gat", 16, 8, 64, 1, 2),
     "C3": _kron("C3", "agnn", 20, 16, 128, 1, 3, graph="rmat"),
-    "C4": _kron("C4", "va", 22, 32, 256, 1, 1),
+    "C4": _kron("C4", "va", 22, 32, 256, 1, 1, train=True),   # "training step (fwd+bwd+SGD)"
     "C5": _kron("C5", "gat", 24, 32, 128, 4, 1),
 }
 

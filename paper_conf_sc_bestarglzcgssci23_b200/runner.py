@@ -119,10 +119,30 @@ class Stack:
             self.model.backward(l, self.W[l], self.a[l], self.H[l], self.saved[l], self.dH[l + 1],
                                 self.dH[l], self.dW[l], self.da[l], self.ws, self.stream)
 
+    def sgd(self, lr=None):
+        """W^l -= lr dW^l (and a^l for GAT) on the device."""
+        lr = self.w.lr if lr is None else lr
+        for l in range(self.w.layers):
+            agnn.sgd_step(self.W[l], self.dW[l], lr, self.stream)
+            if self.a[l] is not None:
+                agnn.sgd_step(self.a[l], self.da[l], lr, self.stream)
+
+    def loss(self):
+        """L = <R, H^L> (reading A13) into a device fp64 scalar (this rank's rows)."""
+        if not hasattr(self, "_loss"):
+            self._loss = torch.zeros(1, dtype=torch.float64, device=self.device)
+            self._loss_ws = torch.empty(agnn.LOSS_SCRATCH, dtype=torch.float64, device=self.device)
+        agnn.loss_inner(self.dH[self.w.layers], self.H[self.w.layers], self._loss_ws, self._loss,
+                        self.stream)
+        return self._loss
+
     def step(self):
-        """One fwd+bwd training pass over all L layers (the bench 'step')."""
+        """One pass over all L layers (the bench 'step'): forward + backward, plus
+        the SGD update for training workloads (C4: "training step (fwd+bwd+SGD)")."""
         self.forward()
         self.backward()
+        if self.w.train:
+            self.sgd()
 
     def edges_total(self) -> int:
         return self.graph.nnz
