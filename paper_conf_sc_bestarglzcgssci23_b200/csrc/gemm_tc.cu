@@ -59,6 +59,15 @@ __device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, u
       "l"(map), "r"(s_addr(bar)), "r"(c0), "r"(c1)
       : "memory");
 }
+// L2 prefetch of a TMA box (no shared memory): the ring holds only 1-2 chunks in
+// flight, so chunks further ahead are pulled into L2 to hide the DRAM latency
+__device__ __forceinline__ void tma_prefetch_2d(const CUtensorMap* map, int c0, int c1) {
+  asm volatile("cp.async.bulk.prefetch.tensor.2d.L2.global.tile [%0, {%1, %2}];" ::"l"(map),
+               "r"(c0), "r"(c1)
+               : "memory");
+}
+constexpr int TC_PF = 6;  // chunks prefetched ahead into L2
+
 __device__ __forceinline__ void fence_proxy_async() {
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
@@ -81,6 +90,26 @@ __device__ __forceinline__ void mma_tf32(uint32_t tmem_d, uint64_t adesc, uint64
       "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate)
       : "memory");
 }
+// A operand from tensor memory (lane = row of A, one tf32 per 32-bit column)
+__device__ __forceinline__ void mma_tf32_ta(uint32_t tmem_d, uint32_t tmem_a, uint64_t bdesc,
+                                            uint32_t idesc, uint32_t accumulate) {
+  asm volatile(
+      "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
+      "tcgen05.mma.cta_group::1.kind::tf32 [%0], [%1], %2, %3, p;\n}\n" ::"r"(tmem_d),
+      "r"(tmem_a), "l"(bdesc), "r"(idesc), "r"(accumulate)
+      : "memory");
+}
+__device__ __forceinline__ void tmem_st32(uint32_t taddr, const float (&v)[32]) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,"
+      "%14,%15,%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};" ::"r"(taddr),
+      "f"(v[0]), "f"(v[1]), "f"(v[2]), "f"(v[3]), "f"(v[4]), "f"(v[5]), "f"(v[6]), "f"(v[7]),
+      "f"(v[8]), "f"(v[9]), "f"(v[10]), "f"(v[11]), "f"(v[12]), "f"(v[13]), "f"(v[14]), "f"(v[15]),
+      "f"(v[16]), "f"(v[17]), "f"(v[18]), "f"(v[19]), "f"(v[20]), "f"(v[21]), "f"(v[22]), "f"(v[23]),
+      "f"(v[24]), "f"(v[25]), "f"(v[26]), "f"(v[27]), "f"(v[28]), "f"(v[29]), "f"(v[30]), "f"(v[31])
+      : "memory");
+  asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+}
 __device__ __forceinline__ void mma_commit(uint64_t* bar) {
   asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
                    s_addr(bar))
@@ -99,19 +128,34 @@ __device__ __forceinline__ void tmem_ld16(uint32_t taddr, float (&v)[16]) {
 #pragma unroll
   for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(r[i]);
 }
-// tf32 split with round-to-nearest (cvt.rna): hi = tf32(x), lo = tf32(x - hi).
-// |x - hi - lo| <= 2^-22 |x| and the rounding errors are unbiased, so the
-// 3-term product matches an fp32 FFMA dot (truncating splits are biased and
-// lose ~2^-21 per element, which the ill-conditioned da1 = P^T ds amplifies).
-__device__ __forceinline__ float tf32_rna(float x) {
-  uint32_t r;
-  asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(r) : "f"(x));
-  return __uint_as_float(r);
+// tf32 split with round-to-nearest: hi = tf32(x), lo = tf32(x - hi), so
+// |x - hi - lo| <= 2^-22 |x| with unbiased rounding errors and the 3-term
+// product matches an fp32 FFMA dot (truncating splits are biased and lose
+// ~2^-21 per element, which the ill-conditioned da1 = P^T ds amplifies).
+// cvt.rna.tf32.f32 issues on the XU pipe at a quarter of the FMA rate and
+// capped the k = 256 GEMM (ncu: XU > 100% of peak), so the rounding runs on the
+// FMA and integer pipes instead:
+//   hi: Veltkamp splitting with sigma = 2^13 + 1 (fp32 p = 24 -> 11 significant
+//       bits = tf32's 10 + 1), round-to-nearest; __fmul_rn/__fsub_rn keep the
+//       compiler from contracting p - x into an FMA (which would break it);
+//   lo: x - hi is exact; rounded to 11 bits by adding half an ulp of tf32 to the
+//       magnitude bits and clearing the 13 dropped bits (round half away).
+__device__ __forceinline__ float tf32_hi(float x) {
+  const float p = __fmul_rn(x, 8193.0f);
+  return __fsub_rn(p, __fsub_rn(p, x));
+}
+__device__ __forceinline__ float tf32_rna_int(float x) {
+  return __uint_as_float((__float_as_uint(x) + 0x1000u) & 0xFFFFE000u);
+}
+__device__ __forceinline__ void split1(float x, float& hi, float& lo) {
+  hi = tf32_hi(x);
+  lo = tf32_rna_int(__fsub_rn(x, hi));
 }
 __device__ __forceinline__ void split4(float4 x, float4& hi, float4& lo) {
-  hi = make_float4(tf32_rna(x.x), tf32_rna(x.y), tf32_rna(x.z), tf32_rna(x.w));
-  lo = make_float4(tf32_rna(x.x - hi.x), tf32_rna(x.y - hi.y), tf32_rna(x.z - hi.z),
-                   tf32_rna(x.w - hi.w));
+  split1(x.x, hi.x, lo.x);
+  split1(x.y, hi.y, lo.y);
+  split1(x.z, hi.z, lo.z);
+  split1(x.w, hi.w, lo.w);
 }
 
 struct TcOut {
@@ -121,20 +165,103 @@ struct TcOut {
   int n_split, n_store, act;
 };
 
-template <int N, int K>
-__global__ void __launch_bounds__(TC_THREADS, 1)
-gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const float* __restrict__ B, int n_real,
-               int64_t M, TcOut out) {
+// 16 consecutive columns c0.. of output row `row` (C0 | C1 split, optional sigma copy)
+__device__ __forceinline__ void store_row16(const TcOut& out, int64_t row, int c0,
+                                            const float (&v)[16]) {
+#pragma unroll
+  for (int j = 0; j < 16; j += 4) {
+    const int c = c0 + j;
+    const float4 q = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
+    if (c + 3 < out.n_split && (out.n_split & 3) == 0) {
+      if (out.C0) st4(out.C0 + row * out.n_split + c, q);
+      if (out.Cact) st4(out.Cact + row * out.n_split + c, act_fwd4(out.act, q));
+    } else if (c < out.n_split) {
+#pragma unroll
+      for (int x = 0; x < 4; ++x) {
+        if (c + x < out.n_split) {
+          if (out.C0) out.C0[row * out.n_split + c + x] = v[j + x];
+          if (out.Cact) out.Cact[row * out.n_split + c + x] = act_fwd(out.act, v[j + x]);
+        } else if (c + x < out.n_store) {
+          out.C1[row * (out.n_store - out.n_split) + (c + x - out.n_split)] = v[j + x];
+        }
+      }
+    } else if (c < out.n_store) {
+      const int w1 = out.n_store - out.n_split;
+#pragma unroll
+      for (int x = 0; x < 4; ++x)
+        if (c + x < out.n_store) out.C1[row * w1 + (c + x - out.n_split)] = v[j + x];
+    }
+  }
+}
+
+// 32 columns [c0, c0+32) of the warp's 32 rows [row0, row0+32) through a per-warp
+// shared-memory transpose, so every store instruction writes 4 full 128-byte rows
+// (a thread-per-row store touches 32 lines per instruction, 8x the L2 write requests)
+__device__ __forceinline__ void store_block32(const TcOut& out, int64_t row0, int64_t M, int c0,
+                                              const float (&v)[32], float* stg, int lane) {
+  // stg: [32 rows][36 floats] (16-byte aligned rows, 4-float pad against bank conflicts)
+#pragma unroll
+  for (int j = 0; j < 32; j += 4)
+    *reinterpret_cast<float4*>(stg + lane * 36 + j) = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
+  __syncwarp();
+  const int rr = lane >> 3, cc = (lane & 7) * 4;
+#pragma unroll
+  for (int k = 0; k < 8; ++k) {
+    const int r = 4 * k + rr;
+    const int64_t row = row0 + r;
+    const float4 q = *reinterpret_cast<const float4*>(stg + r * 36 + cc);
+    if (row < M) {
+      if (out.C0) st4(out.C0 + row * out.n_split + c0 + cc, q);
+      if (out.Cact) st4(out.Cact + row * out.n_split + c0 + cc, act_fwd4(out.act, q));
+    }
+  }
+  __syncwarp();
+}
+
+// Warp-specialised CTA (one per SM, persistent over 128-row tiles), 8 warps:
+//   warps 0-3 ("math"): thread 0 keeps the TMA ring S - 1 chunks ahead (plus L2
+//     prefetches further out); all 128 threads split each landed chunk in place;
+//     thread 0 issues the tcgen05.mma chain and commits to the stage's barrier
+//     (stage free) and, after a tile's last chunk, to acc_full;
+//   warps 4-7 ("epilogue"): wait acc_full, drain the NG TMEM accumulators into
+//     registers (summed with round-to-nearest FADDs), release TMEM (acc_empty)
+//     and only then write the rows to global memory — the stores of tile t
+//     overlap the loads, splits and MMAs of tile t+1.
+// SB = false: B (hi/lo) resident in shared memory, split once per CTA;
+// SB = true:  B streamed through the ring with A (wide operands, k = 256).
+constexpr int TC_WS_THREADS = 256;
+
+__device__ __forceinline__ void mbar_arrive(uint64_t* b) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(s_addr(b)) : "memory");
+}
+__device__ __forceinline__ void math_barrier() {  // the 128 math threads only
+  asm volatile("bar.sync 1, 128;" ::: "memory");
+}
+
+template <int N, int K, int S, bool SB>
+__global__ void __launch_bounds__(TC_WS_THREADS, 1)
+gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+               const float* __restrict__ B, int n_real, int64_t M, TcOut out) {
   static_assert(N % 16 == 0 && N >= 16 && N <= 256, "UMMA N for M = 128");
   static_assert(K % TC_KC == 0, "K must be a multiple of 32");
   constexpr int KCH = K / TC_KC;                    // 128-byte chunks along K
-  constexpr int B_BYTES = KCH * N * 128;            // one of hi / lo
-  constexpr int A_STAGE = TC_BM * 128;              // 16 KB raw / hi
-  // Accumulation groups: the tensor core rounds the fp32 accumulator once per MMA
-  // (biased), so the K loop is spread over NG TMEM accumulators (one per 32-wide
-  // K chunk where they fit) that the epilogue adds with round-to-nearest FADDs.
-  constexpr int NG = (KCH < (N <= 128 ? 4 : N <= 160 ? 3 : 2)) ? KCH : (N <= 128 ? 4 : N <= 160 ? 3 : 2);
-  constexpr uint32_t TMEM_NEED = (uint32_t)(NG * N);
+  constexpr int A_BYTES = TC_BM * 128;              // one of A hi / lo per stage
+  constexpr int BC_BYTES = N * 128;                 // one of B hi / lo per chunk
+  constexpr int BRES = SB ? 0 : KCH * BC_BYTES;     // resident B (one of hi / lo)
+  constexpr int STAGE = SB ? 2 * A_BYTES + 2 * BC_BYTES : A_BYTES;
+  // Accumulation groups: the tensor core rounds the fp32 accumulator once per MMA, so
+  // the K loop is spread over NG TMEM accumulators (one per 32-wide K chunk where they
+  // fit) that the epilogue adds with round-to-nearest FADDs.
+  // LOT (resident B): the A lo part goes to TMEM (2 slots of 32 columns) instead of
+  // shared memory, so a stage is 16 KB and the ring holds S - 1 chunks in flight
+  constexpr bool LOT = !SB;
+  constexpr int LO_COLS = LOT ? 64 : 0;
+  constexpr int NG0 = N <= 128 ? 4 : N <= 160 ? 3 : 2;
+  constexpr int NGT = (NG0 * N + LO_COLS <= 512) ? NG0 : (NG0 - 1) * N + LO_COLS <= 512 ? NG0 - 1 : 2;
+  constexpr int NG = KCH < NGT ? KCH : NGT;
+  constexpr uint32_t LO_COL = (uint32_t)(NG * N);  // first TMEM column of the lo slots
+  constexpr uint32_t TMEM_NEED = (uint32_t)(NG * N + LO_COLS);
+  static_assert(TMEM_NEED <= 512, "TMEM columns");
   constexpr uint32_t TMEM_COLS = TMEM_NEED <= 32 ? 32 : TMEM_NEED <= 64 ? 64 : TMEM_NEED <= 128 ? 128
                                  : TMEM_NEED <= 256 ? 256 : 512;
   constexpr uint32_t IDESC = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(N >> 3) << 17) |
@@ -142,12 +269,14 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const float* __restrict_
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
                                              ~uintptr_t(1023));
-  uint8_t* Bh = smem;
-  uint8_t* Bl = smem + B_BYTES;
-  uint8_t* As = smem + 2 * B_BYTES;                 // [2 stages][hi 16KB | lo 16KB]
-  __shared__ uint64_t tma_bar[2], mma_bar[2];
+  uint8_t* Bh = smem;                  // resident B (SB = false)
+  uint8_t* Bl = smem + BRES;
+  uint8_t* ring = smem + 2 * BRES;     // S stages
+  float* stg = reinterpret_cast<float*>(ring + S * STAGE);  // epilogue transpose, 4 x 32 x 36
+  __shared__ uint64_t tma_bar[S], mma_bar[S], acc_full, acc_empty;
   __shared__ uint32_t tmem_base_s;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const bool math = warp < 4;
 
   if (warp == 0) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
@@ -157,25 +286,31 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const float* __restrict_
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
   }
   if (tid == 0) {
-    mbar_init(&tma_bar[0], 1);
-    mbar_init(&tma_bar[1], 1);
-    mbar_init(&mma_bar[0], 1);
-    mbar_init(&mma_bar[1], 1);
+#pragma unroll
+    for (int i = 0; i < S; ++i) {
+      mbar_init(&tma_bar[i], 1);
+      mbar_init(&mma_bar[i], 1);
+    }
+    mbar_init(&acc_full, 1);
+    mbar_init(&acc_empty, 128);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(&tmA) : "memory");
+    if (SB) asm volatile("prefetch.tensormap [%0];" ::"l"(&tmB) : "memory");
   }
-  // B -> hi/lo tiles in the swizzled K-major layout (rows >= n_real are zero)
-  for (int idx = tid; idx < N * (K / 4); idx += TC_THREADS) {
-    const int n = idx / (K / 4), c16 = idx % (K / 4), kc = c16 / 8, cc = c16 % 8;
-    float4 v = f4(0.f);
-    if (n < n_real) v = ldg4(B + (int64_t)n * K + c16 * 4);
-    float4 hi, lo;
-    split4(v, hi, lo);
-    const int off = kc * N * 128 + (n >> 3) * 1024 + (n & 7) * 128 + ((cc ^ (n & 7)) << 4);
-    *reinterpret_cast<float4*>(Bh + off) = hi;
-    *reinterpret_cast<float4*>(Bl + off) = lo;
+  if (!SB) {
+    // B -> hi/lo tiles in the swizzled K-major layout (rows >= n_real are zero)
+    for (int idx = tid; idx < N * (K / 4); idx += TC_WS_THREADS) {
+      const int n = idx / (K / 4), c16 = idx % (K / 4), kc = c16 / 8, cc = c16 % 8;
+      float4 v = f4(0.f);
+      if (n < n_real) v = ldg4(B + (int64_t)n * K + c16 * 4);
+      float4 hi, lo;
+      split4(v, hi, lo);
+      const int off = kc * N * 128 + (n >> 3) * 1024 + (n & 7) * 128 + ((cc ^ (n & 7)) << 4);
+      *reinterpret_cast<float4*>(Bh + off) = hi;
+      *reinterpret_cast<float4*>(Bl + off) = lo;
+    }
+    fence_proxy_async();
   }
-  fence_proxy_async();
   tc_fence_before();
   __syncthreads();
   tc_fence_after();
@@ -184,105 +319,150 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const float* __restrict_
   const int64_t ntiles = (M + TC_BM - 1) / TC_BM;
   const int64_t first = blockIdx.x;
   const int64_t my_tiles = first < ntiles ? (ntiles - 1 - first) / gridDim.x + 1 : 0;
-  const int64_t nchunks = my_tiles * KCH;
-  auto chunk_coords = [&](int64_t g, int& kcol, int& mrow) {
-    const int64_t t = first + (g / KCH) * gridDim.x;
-    kcol = (int)(g % KCH) * TC_KC;
-    mrow = (int)(t * TC_BM);
-  };
-  if (tid == 0 && nchunks > 0) {
-    int kcol, mrow;
-    chunk_coords(0, kcol, mrow);
-    mbar_expect_tx(&tma_bar[0], A_STAGE);
-    tma_load_2d(As, &tmA, &tma_bar[0], kcol, mrow);
-  }
-  for (int64_t g = 0; g < nchunks; ++g) {
-    const int s = (int)(g & 1);
-    const int kc = (int)(g % KCH);
-    if (tid == 0 && g + 1 < nchunks) {
-      // stage s^1 held chunk g-1: its MMAs must be done before it is overwritten
-      if (g >= 1) mbar_wait(&mma_bar[s ^ 1], (uint32_t)(((g - 1) >> 1) & 1));
-      int kcol, mrow;
-      chunk_coords(g + 1, kcol, mrow);
-      mbar_expect_tx(&tma_bar[s ^ 1], A_STAGE);
-      tma_load_2d(As + (s ^ 1) * 2 * A_STAGE, &tmA, &tma_bar[s ^ 1], kcol, mrow);
-    }
-    mbar_wait(&tma_bar[s], (uint32_t)((g >> 1) & 1));
-    uint8_t* Ahi = As + s * 2 * A_STAGE;
-    uint8_t* Alo = Ahi + A_STAGE;
-#pragma unroll 4
-    for (int i = tid; i < A_STAGE / 16; i += TC_THREADS) {
-      float4 hi, lo;
-      split4(*reinterpret_cast<const float4*>(Ahi + i * 16), hi, lo);
-      *reinterpret_cast<float4*>(Ahi + i * 16) = hi;
-      *reinterpret_cast<float4*>(Alo + i * 16) = lo;
-    }
-    fence_proxy_async();
-    tc_fence_before();
-    __syncthreads();
-    if (tid == 0) {
-      tc_fence_after();
-      const uint32_t ah = s_addr(Ahi), al = s_addr(Alo);
-      const uint32_t bh = s_addr(Bh + kc * N * 128), bl = s_addr(Bl + kc * N * 128);
-      const int grp = kc < NG ? kc : NG - 1;
-      const uint32_t tacc = tmem + (uint32_t)(grp * N);
-#pragma unroll
-      for (int ks = 0; ks < TC_KC / 8; ++ks) {  // K = 8 tf32 (32 bytes) per MMA
-        const uint32_t o = ks * 32;
-        const uint32_t acc0 = (kc > grp || ks > 0) ? 1u : 0u;  // first MMA of the group
-        mma_tf32(tacc, sw128_desc(ah + o), sw128_desc(bh + o), IDESC, acc0);
-        mma_tf32(tacc, sw128_desc(ah + o), sw128_desc(bl + o), IDESC, 1u);
-        mma_tf32(tacc, sw128_desc(al + o), sw128_desc(bh + o), IDESC, 1u);
-      }
-      mma_commit(&mma_bar[s]);
-    }
-    if (kc == KCH - 1) {
-      // tile complete: epilogue from TMEM (all MMAs of the tile precede this commit)
-      mbar_wait(&mma_bar[s], (uint32_t)((g >> 1) & 1));
-      tc_fence_after();
+
+  if (math) {
+    const int64_t nchunks = my_tiles * KCH;
+    auto issue = [&](int64_t g) {
+      const int st = (int)(g % S);
       const int64_t t = first + (g / KCH) * gridDim.x;
-      const int64_t row = t * TC_BM + warp * 32 + lane;
-      const uint32_t tbase = tmem + ((uint32_t)(warp * 32) << 16);
-#pragma unroll 1
-      for (int c0 = 0; c0 < N; c0 += 16) {
-        float v[16];
-        tmem_ld16(tbase + c0, v);
-#pragma unroll
-        for (int gi = 1; gi < NG; ++gi) {
-          float w2[16];
-          tmem_ld16(tbase + (uint32_t)(gi * N) + c0, w2);
-#pragma unroll
-          for (int x = 0; x < 16; ++x) v[x] += w2[x];
+      const int kcol = (int)(g % KCH) * TC_KC;
+      uint8_t* base = ring + st * STAGE;
+      mbar_expect_tx(&tma_bar[st], A_BYTES + (SB ? BC_BYTES : 0));
+      tma_load_2d(base, &tmA, &tma_bar[st], kcol, (int)(t * TC_BM));
+      if (SB) tma_load_2d(base + 2 * A_BYTES, &tmB, &tma_bar[st], kcol, 0);
+    };
+    if (tid == 0)
+      for (int64_t g = 0; g < S - 1 && g < nchunks; ++g) issue(g);
+    for (int64_t g = 0; g < nchunks; ++g) {
+      const int st = (int)(g % S);
+      const uint32_t par = (uint32_t)((g / S) & 1);
+      const int kc = (int)(g % KCH);
+      const int64_t tl = g / KCH;  // this CTA's tile ordinal
+      if (tid == 0) {
+        if (g + S - 1 + TC_PF < nchunks) {
+          const int64_t gp = g + S - 1 + TC_PF;
+          tma_prefetch_2d(&tmA, (int)(gp % KCH) * TC_KC,
+                          (int)((first + (gp / KCH) * gridDim.x) * TC_BM));
         }
-        if (row < M) {
+        if (g + S - 1 < nchunks) {
+          // the stage of chunk g+S-1 held chunk g-1: its MMAs must be done
+          if (g >= 1) mbar_wait(&mma_bar[(g - 1) % S], (uint32_t)(((g - 1) / S) & 1));
+          issue(g + S - 1);
+        }
+      }
+      mbar_wait(&tma_bar[st], par);
+      uint8_t* Ahi = ring + st * STAGE;
+      uint8_t* Alo = Ahi + A_BYTES;  // SB only
+      const uint32_t lo_slot = LO_COL + (uint32_t)((g & 1) * 32);
+      if (LOT) {
+        // thread r splits row r of the tile: hi in place (swizzled 128-byte row),
+        // lo into TMEM lane r.  The slot was last read by chunk g-2's MMAs.
+        if (g >= 2) mbar_wait(&mma_bar[(g - 2) % S], (uint32_t)(((g - 2) / S) & 1));
+        uint8_t* rowp = Ahi + tid * 128;
+        float lo[32];
 #pragma unroll
-          for (int j = 0; j < 16; j += 4) {
-            const int c = c0 + j;
-            const float4 q = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
-            if (c + 3 < out.n_split && (out.n_split & 3) == 0) {
-              if (out.C0) st4(out.C0 + row * out.n_split + c, q);
-              if (out.Cact) st4(out.Cact + row * out.n_split + c, act_fwd4(out.act, q));
-            } else if (c < out.n_split) {
+        for (int c = 0; c < 8; ++c) {
+          float4* q = reinterpret_cast<float4*>(rowp + ((c ^ (tid & 7)) << 4));
+          float4 hi, l4;
+          split4(*q, hi, l4);
+          *q = hi;
+          lo[4 * c] = l4.x;
+          lo[4 * c + 1] = l4.y;
+          lo[4 * c + 2] = l4.z;
+          lo[4 * c + 3] = l4.w;
+        }
+        tc_fence_after();
+        tmem_st32(tmem + ((uint32_t)(warp * 32) << 16) + lo_slot, lo);
+      } else {
+        constexpr int SPLIT16 = (A_BYTES + (SB ? BC_BYTES : 0)) / 16;
+#pragma unroll 4
+        for (int i = tid; i < SPLIT16; i += 128) {
+          const bool isA = !SB || i < A_BYTES / 16;
+          uint8_t* hp = isA ? Ahi + i * 16 : Ahi + 2 * A_BYTES + (i - A_BYTES / 16) * 16;
+          uint8_t* lp = hp + (isA ? A_BYTES : BC_BYTES);
+          float4 hi, lo;
+          split4(*reinterpret_cast<const float4*>(hp), hi, lo);
+          *reinterpret_cast<float4*>(hp) = hi;
+          *reinterpret_cast<float4*>(lp) = lo;
+        }
+      }
+      fence_proxy_async();
+      tc_fence_before();
+      math_barrier();
+      if (tid == 0) {
+        // the first MMA of a tile overwrites the accumulators: the epilogue must have
+        // drained the previous tile
+        if (kc == 0 && tl >= 1) mbar_wait(&acc_empty, (uint32_t)((tl - 1) & 1));
+        tc_fence_after();
+        const uint32_t ah = s_addr(Ahi), al = s_addr(Alo);
+        const uint32_t bh = SB ? s_addr(Ahi + 2 * A_BYTES) : s_addr(Bh + kc * BC_BYTES);
+        const uint32_t bl = SB ? bh + BC_BYTES : s_addr(Bl + kc * BC_BYTES);
+        const int grp = kc % NG;
+        const uint32_t tacc = tmem + (uint32_t)(grp * N);
 #pragma unroll
-              for (int x = 0; x < 4; ++x) {
-                if (c + x < out.n_split) {
-                  if (out.C0) out.C0[row * out.n_split + c + x] = v[j + x];
-                  if (out.Cact) out.Cact[row * out.n_split + c + x] = act_fwd(out.act, v[j + x]);
-                } else if (c + x < out.n_store) {
-                  out.C1[row * (out.n_store - out.n_split) + (c + x - out.n_split)] = v[j + x];
-                }
-              }
-            } else if (c < out.n_store) {
-              const int w1 = out.n_store - out.n_split;
+        for (int ks = 0; ks < TC_KC / 8; ++ks) {  // K = 8 tf32 (32 bytes) per MMA
+          const uint32_t o = ks * 32;
+          const uint32_t acc0 = (kc >= NG || ks > 0) ? 1u : 0u;  // first MMA of the group
+          mma_tf32(tacc, sw128_desc(ah + o), sw128_desc(bh + o), IDESC, acc0);
+          mma_tf32(tacc, sw128_desc(ah + o), sw128_desc(bl + o), IDESC, 1u);
+          if (LOT) mma_tf32_ta(tacc, tmem + lo_slot + (uint32_t)(ks * 8), sw128_desc(bh + o), IDESC, 1u);
+          else mma_tf32(tacc, sw128_desc(al + o), sw128_desc(bh + o), IDESC, 1u);
+        }
+        mma_commit(&mma_bar[st]);
+        if (kc == KCH - 1) mma_commit(&acc_full);
+      }
+    }
+  } else {
+    const int ew = warp - 4;  // TMEM lanes 32 ew .. 32 ew + 31
+    for (int64_t tl = 0; tl < my_tiles; ++tl) {
+      mbar_wait(&acc_full, (uint32_t)(tl & 1));
+      tc_fence_after();
+      const uint32_t tbase = tmem + ((uint32_t)(ew * 32) << 16);
+      const int64_t t = first + tl * gridDim.x;
+      const int64_t row0 = t * TC_BM + ew * 32;
+      const int64_t row = row0 + lane;
+      // wide tiles drain in two halves (registers); TMEM is released after the last
+      constexpr int NP = N > 160 ? N / 2 : N;
+#pragma unroll 1
+      for (int h0 = 0; h0 < N; h0 += NP) {
+        float v[NP];
 #pragma unroll
-              for (int x = 0; x < 4; ++x)
-                if (c + x < out.n_store) out.C1[row * w1 + (c + x - out.n_split)] = v[j + x];
+        for (int c0 = 0; c0 < NP; c0 += 16) {
+          float a16[16];
+          tmem_ld16(tbase + h0 + c0, a16);
+#pragma unroll
+          for (int gi = 1; gi < NG; ++gi) {
+            float w2[16];
+            tmem_ld16(tbase + (uint32_t)(gi * N) + h0 + c0, w2);
+#pragma unroll
+            for (int x = 0; x < 16; ++x) a16[x] += w2[x];
+          }
+#pragma unroll
+          for (int x = 0; x < 16; ++x) v[c0 + x] = a16[x];
+        }
+        if (h0 + NP >= N) {
+          tc_fence_before();
+          mbar_arrive(&acc_empty);
+        }
+        const bool coal = (out.n_split & 3) == 0;
+#pragma unroll
+        for (int c0 = 0; c0 < NP; c0 += 32) {
+          if (c0 + 32 <= NP && coal && h0 + c0 + 32 <= out.n_split) {
+            float q[32];
+#pragma unroll
+            for (int x = 0; x < 32; ++x) q[x] = v[c0 + x];
+            store_block32(out, row0, M, h0 + c0, q, stg + ew * 32 * 36, lane);
+          } else if (row < M) {
+#pragma unroll
+            for (int c1 = c0; c1 < c0 + 32 && c1 < NP; c1 += 16) {
+              float q[16];
+#pragma unroll
+              for (int x = 0; x < 16; ++x) q[x] = v[c1 + x];
+              store_row16(out, row, h0 + c1, q);
             }
           }
         }
       }
-      tc_fence_before();
-      __syncthreads();  // TMEM reads done before the next tile's first MMA
     }
   }
   __syncthreads();
@@ -376,6 +556,13 @@ gemm_tn_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
   for (int64_t g = 0; g < nch; ++g) {
     const int64_t G = G0 + g;
     const int st = (int)(G & 1);
+    if (tid == 0 && g + 1 + TC_PF / 2 < nch) {
+      const int r = (int)(r_beg + (g + 1 + TC_PF / 2) * TN_ROWS);
+#pragma unroll
+      for (int b = 0; b < K1 / 32; ++b) tma_prefetch_2d(&tmA, b * 32, r);
+#pragma unroll
+      for (int b = 0; b < N / 32; ++b) tma_prefetch_2d(&tmB, b * 32, r);
+    }
     if (tid == 0 && g + 1 < nch) {
       // stage st^1 held chunk G-1 (its MMAs must finish before the TMA overwrites it;
       // the previous slab's last chunk was already waited on by its epilogue)
@@ -461,24 +648,36 @@ PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
   return fn;
 }
 
-template <int N, int K>
+template <int N, int K, int S, bool SB>
 agnn_status launch_tc(const float* A, int64_t M, const float* B, int n_real, const TcOut& o,
                       cudaStream_t s) {
   auto enc = encode_fn();
   if (!enc) return fail(AGNN_ECUDA, "gemm_tc: cuTensorMapEncodeTiled unavailable");
-  CUtensorMap map;
-  cuuint64_t dims[2] = {(cuuint64_t)K, (cuuint64_t)M};
+  CUtensorMap ma, mb;
+  cuuint64_t da[2] = {(cuuint64_t)K, (cuuint64_t)M};
+  cuuint64_t db[2] = {(cuuint64_t)K, (cuuint64_t)n_real};
   cuuint64_t strides[1] = {(cuuint64_t)K * 4};
-  cuuint32_t box[2] = {(cuuint32_t)TC_KC, (cuuint32_t)TC_BM};
+  cuuint32_t boxa[2] = {(cuuint32_t)TC_KC, (cuuint32_t)TC_BM};
+  cuuint32_t boxb[2] = {(cuuint32_t)TC_KC, (cuuint32_t)N};  // rows >= n_real arrive as zeros
   cuuint32_t es[2] = {1, 1};
-  CUresult r = enc(&map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(A), dims, strides,
-                   box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
-                   CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-  if (r != CUDA_SUCCESS) return fail(AGNN_ECUDA, "gemm_tc: tensor map encode failed");
-  constexpr int smem = 2 * (K / TC_KC) * N * 128 + 2 * 2 * TC_BM * 128 + 1024;
+  if (enc(&ma, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(A), da, strides, boxa, es,
+          CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+          CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+    return fail(AGNN_ECUDA, "gemm_tc: tensor map encode failed");
+  if (SB && enc(&mb, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(B), db, strides, boxb,
+                es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+    return fail(AGNN_ECUDA, "gemm_tc: tensor map encode failed");
+  if (!SB) mb = ma;  // unused
+  constexpr int smem = (SB ? 0 : 2 * (K / TC_KC) * N * 128) +
+                       S * (SB ? 2 * TC_BM * 128 + 2 * N * 128 : TC_BM * 128) + 4 * 32 * 36 * 4 +
+                       1024;
+  static_assert(smem <= 232448 - 1024, "shared memory");
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(gemm_tc_kernel<N, K>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    cudaFuncSetAttribute(gemm_tc_kernel<N, K, S, SB>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         smem);
     attr = true;
   }
   int sms = kNumSMs, dev = 0;
@@ -486,16 +685,16 @@ agnn_status launch_tc(const float* A, int64_t M, const float* B, int n_real, con
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   const int64_t ntiles = (M + TC_BM - 1) / TC_BM;
   const int grid = (int)std::min<int64_t>(ntiles, sms);
-  gemm_tc_kernel<N, K><<<grid, TC_THREADS, smem, s>>>(map, B, n_real, M, o);
+  gemm_tc_kernel<N, K, S, SB><<<grid, TC_WS_THREADS, smem, s>>>(ma, mb, B, n_real, M, o);
   AGNN_LAUNCH_CHECK("gemm_tc_kernel");
   return AGNN_OK;
 }
 
-bool map_rows_box32(CUtensorMap* map, const float* base, int64_t rows, int cols) {
+bool map_rows_box32(CUtensorMap* map, const float* base, int64_t rows, int cols, int ld) {
   auto enc = encode_fn();
   if (!enc) return false;
   cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
-  cuuint64_t strides[1] = {(cuuint64_t)cols * 4};
+  cuuint64_t strides[1] = {(cuuint64_t)ld * 4};
   cuuint32_t box[2] = {32, (cuuint32_t)TN_ROWS};
   cuuint32_t es[2] = {1, 1};
   return enc(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(base), dims, strides, box,
@@ -503,20 +702,24 @@ bool map_rows_box32(CUtensorMap* map, const float* base, int64_t rows, int cols)
              CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
-__global__ void tn_sum_kernel(const float* __restrict__ part, int splits, int64_t count,
-                              float* __restrict__ C) {
+// C[r][c] (row stride ldc) = sum over the slab partials of part[p][r][c] (r < K1, c < N)
+__global__ void tn_sum_kernel(const float* __restrict__ part, int splits, int K1, int N,
+                              float* __restrict__ C, int ldc) {
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const int64_t count = (int64_t)K1 * N;
   if (i >= count) return;
   double s = 0.0;  // fixed order, fp64 across the slab partials
   for (int p = 0; p < splits; ++p) s += (double)part[(int64_t)p * count + i];
-  C[i] = (float)s;
+  C[(i / N) * ldc + (i % N)] = (float)s;
 }
 
+// C block [K1 x N] (row stride ldc) = A^T B over M rows; A, B column blocks of row
+// strides lda, ldb
 template <int K1, int N>
-agnn_status launch_tn_tc(const float* A, int64_t M, const float* B, float* C, float* ws,
-                         cudaStream_t s) {
+agnn_status launch_tn_tc(const float* A, int lda, int64_t M, const float* B, int ldb, float* C,
+                         int ldc, float* ws, cudaStream_t s) {
   CUtensorMap ma, mb;
-  if (!map_rows_box32(&ma, A, M, K1) || !map_rows_box32(&mb, B, M, N))
+  if (!map_rows_box32(&ma, A, M, K1, lda) || !map_rows_box32(&mb, B, M, N, ldb))
     return fail(AGNN_ECUDA, "gemm_tn_tc: tensor map encode failed");
   constexpr int smem = 2 * (2 * TN_ROWS * K1 * 4 + 2 * TN_ROWS * N * 4) + 1024;
   static bool attr = false;
@@ -537,7 +740,7 @@ agnn_status launch_tn_tc(const float* A, int64_t M, const float* B, float* C, fl
   gemm_tn_tc_kernel<K1, N><<<grid, TC_THREADS, smem, s>>>(ma, mb, M, rps, ws);
   AGNN_LAUNCH_CHECK("gemm_tn_kernel");
   const int64_t cnt = (int64_t)K1 * N;
-  tn_sum_kernel<<<(unsigned)((cnt + 255) / 256), 256, 0, s>>>(ws, (int)nslabs, cnt, C);
+  tn_sum_kernel<<<(unsigned)((cnt + 255) / 256), 256, 0, s>>>(ws, (int)nslabs, K1, N, C, ldc);
   AGNN_LAUNCH_CHECK("sum_splits_kernel");
   return AGNN_OK;
 }
@@ -551,21 +754,29 @@ bool tc_disabled() {
   return v == 1;
 }
 
-template <int K1, int N>
-agnn_status launch_tn_tc(const float* A, int64_t M, const float* B, float* C, float* ws,
-                         cudaStream_t s);
 
 }  // namespace
 
-// C[K1 x N] = A^T B over M rows on tensor cores (K1 = 128, N in {64, 128}); ws holds
-// one K1 x N partial per SM.  AGNN_EUNSUPPORTED for other shapes.
+// C[K1 x N] = A^T B over M rows on tensor cores (K1 = 128 with N in {64, 128}; K1 = 256
+// with N in {128, 256} as 128 x 128 blocks); ws holds the slab partials of one block.
+// AGNN_EUNSUPPORTED for other shapes.
 agnn_status gemm_tn_tc(const float* A, int64_t M, int K1, const float* B, int N, float* C,
                        float* ws, cudaStream_t s) {
   if (tc_disabled() || M <= 0) return AGNN_EUNSUPPORTED;
   if ((reinterpret_cast<uintptr_t>(A) & 15) || (reinterpret_cast<uintptr_t>(B) & 15))
     return AGNN_EUNSUPPORTED;
-  if (K1 == 128 && N == 128) return launch_tn_tc<128, 128>(A, M, B, C, ws, s);
-  if (K1 == 128 && N == 64) return launch_tn_tc<128, 64>(A, M, B, C, ws, s);
+  if (K1 == 128 && N == 128) return launch_tn_tc<128, 128>(A, K1, M, B, N, C, N, ws, s);
+  if (K1 == 128 && N == 64) return launch_tn_tc<128, 64>(A, K1, M, B, N, C, N, ws, s);
+  if (K1 == 256 && (N == 256 || N == 128)) {
+    // 128 x 128 blocks of C, one pass each over the matching column blocks of A and B
+    for (int qa = 0; qa < K1 / 128; ++qa)
+      for (int qb = 0; qb < N / 128; ++qb) {
+        const agnn_status st = launch_tn_tc<128, 128>(A + qa * 128, K1, M, B + qb * 128, N,
+                                                      C + (int64_t)qa * 128 * N + qb * 128, N, ws, s);
+        if (st != AGNN_OK) return st;
+      }
+    return AGNN_OK;
+  }
   return AGNN_EUNSUPPORTED;
 }
 
@@ -578,13 +789,16 @@ agnn_status gemm_tc(const float* A, int64_t M, int K, const float* B, int n_real
   if ((reinterpret_cast<uintptr_t>(A) & 15) || (K % 32)) return AGNN_EUNSUPPORTED;
   TcOut o{C0, C1, Cact, n_split, n_store, act};
   const int npad = (n_real + 15) / 16 * 16;
-  if (K == 128 && npad == 128) return launch_tc<128, 128>(A, M, B, n_real, o, s);
-  if (K == 128 && npad == 144) return launch_tc<144, 128>(A, M, B, n_real, o, s);
-  if (K == 128 && npad == 160) return launch_tc<160, 128>(A, M, B, n_real, o, s);
-  if (K == 64 && npad == 64) return launch_tc<64, 64>(A, M, B, n_real, o, s);
-  if (K == 64 && npad == 80) return launch_tc<80, 64>(A, M, B, n_real, o, s);
-  if (K == 64 && npad == 128) return launch_tc<128, 64>(A, M, B, n_real, o, s);
-  if (K == 128 && npad == 64) return launch_tc<64, 128>(A, M, B, n_real, o, s);
+  // resident B: S = the 16 KB stages that fit next to B (2 x K x N x 4 bytes), <= 8
+  if (K == 128 && npad == 128) return launch_tc<128, 128, 4, false>(A, M, B, n_real, o, s);
+  if (K == 128 && npad == 144) return launch_tc<144, 128, 3, false>(A, M, B, n_real, o, s);
+  if (K == 128 && npad == 160) return launch_tc<160, 128, 2, false>(A, M, B, n_real, o, s);
+  if (K == 128 && npad == 64) return launch_tc<64, 128, 8, false>(A, M, B, n_real, o, s);
+  if (K == 64 && npad == 64) return launch_tc<64, 64, 8, false>(A, M, B, n_real, o, s);
+  if (K == 64 && npad == 80) return launch_tc<80, 64, 8, false>(A, M, B, n_real, o, s);
+  if (K == 64 && npad == 128) return launch_tc<128, 64, 8, false>(A, M, B, n_real, o, s);
+  if (K == 256 && npad == 256) return launch_tc<256, 256, 2, true>(A, M, B, n_real, o, s);
+  if (K == 256 && npad == 128) return launch_tc<128, 256, 3, true>(A, M, B, n_real, o, s);
   return AGNN_EUNSUPPORTED;
 }
 

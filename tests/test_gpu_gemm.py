@@ -18,7 +18,8 @@ from paper_conf_sc_bestarglzcgssci23_b200 import agnn  # noqa: E402
 
 @pytest.mark.parametrize("M,K,N", [(128, 128, 128), (1000, 128, 144), (65536, 64, 66),
                                    (300001, 128, 136), (4097, 64, 64), (77, 128, 128),
-                                   (20000, 128, 130)])
+                                   (20000, 128, 130), (4096, 256, 256), (100003, 256, 256),
+                                   (5000, 256, 128), (129, 256, 256)])
 def test_gemm_against_fp64(M, K, N):
     g = torch.Generator(device="cpu").manual_seed(M + K + N)
     A = (torch.rand((M, K), generator=g) * 2 - 1).cuda()
@@ -40,11 +41,15 @@ def test_gemm_against_fp64(M, K, N):
     # dot is ~1e-7), normwise <= 5e-7 -- far inside the layers' 1e-5 parity bar
     scale = np.abs(A.double().cpu().numpy()) @ np.abs(B.double().cpu().numpy()).T
     assert (err <= 1e-6 * scale + 1e-30).all(), float((err / scale).max())
-    assert np.linalg.norm(c - ref) / np.linalg.norm(ref) < 5e-7
+    # k = 256 with N = 256: two TMEM accumulation groups (TMEM holds 2 x 256 fp32
+    # columns) of 4 K-chunks each -> ~1e-6 normwise, the level of an fp32 FFMA dot of
+    # length 256 (gamma bound ~ K u); the layers' bar stays 1e-5
+    assert np.linalg.norm(c - ref) / np.linalg.norm(ref) < (5e-7 if K <= 128 else 1.5e-6)
 
 
 @pytest.mark.parametrize("M,K1,N", [(1000, 128, 128), (65536, 128, 128), (300001, 128, 128),
-                                    (77, 128, 64), (20000, 64, 64), (12345, 128, 64)])
+                                    (77, 128, 64), (20000, 64, 64), (12345, 128, 64),
+                                    (100003, 256, 256), (3000, 256, 128)])
 def test_gemm_tn_against_fp64(M, K1, N):
     g = torch.Generator(device="cpu").manual_seed(3 * M + K1 + N)
     A = (torch.rand((M, K1), generator=g) * 2 - 1).cuda()

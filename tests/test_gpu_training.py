@@ -49,7 +49,7 @@ def test_training_loop_matches_oracle(model, heads):
     track the oracle-driven loop (same inputs, same lr)."""
     w = dataclasses.replace(gen.Workload(f"train-{model}", model, "kron", 12, 1 << 12, 8 << 12,
                                          32, heads, 2, act="elu", beta=1.3 if model == "agnn" else 1.0),
-                            train=True, lr=0.05)
+                            train=True, lr=1e-3)
     src, dst, rp, ci = pu.host_graph(w)
     g = pu.device_graph(w, src, dst)
     st = runner.Stack(w, "cuda", graph=g)
