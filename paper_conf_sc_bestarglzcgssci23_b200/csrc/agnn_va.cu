@@ -15,24 +15,16 @@
 //   AGNN dc_ji = beta alpha_ji (M_j.H_i - delta_j), dc_ij = beta alpha_ij (M_i.H_j - delta_i)
 //        dH^_j += (dc_ji + dc_ij) H^_i ; acc_j += alpha_ij M_i
 //        dH_j = acc_j + (dH^_j - (dH^_j.H^_j) H^_j) / nu_j
-#include "internal.cuh"
+#include "av_args.cuh"
 
 namespace agnn {
 
 namespace {
 
 constexpr unsigned FULL = 0xffffffffu;
-enum { VA = 0, AG = 1 };
+enum { VA = AV_VA, AG = AV_AG };
 
-struct AvFwd {
-  const float* H;     // [n_tot x K]  (replicated when world > 1)
-  const float* nu;    // [n_tot]      AGNN
-  float beta, bound;  // bound = |beta|
-  float* X;           // [n_local x K]
-  float* l;           // [n_local]    AGNN
-  float* pacc;        // [n_chunks x K]
-  float* pl;          // [n_chunks]
-};
+
 
 template <int K>
 __device__ __forceinline__ void item_range(const Items& it, int64_t w, int64_t& row, int64_t& beg,
@@ -182,15 +174,7 @@ nu_kernel(const float* __restrict__ H, int64_t n_local, float eps, float* __rest
 }
 
 // ---------------------------------------------------------------- backward
-struct AvBwd {
-  const float* H;      // [n_tot x K]
-  const float* M;      // [n_tot x K]
-  const float4* rec;   // [n_tot] {nu, m, 1/l, delta}   AGNN
-  float beta, eps;
-  float* dH;           // [n_local x K]
-  float* pacc;         // [n_chunks x 2K]
-  float* dhp;          // [n_local x K] directed patterns: row-pass partial of dH (VA) / dH^ (AGNN)
-};
+
 
 template <int K, int MODEL>
 __device__ __forceinline__ void bwd_store(const AvBwd& A, int64_t row, int64_t grow, int q,
@@ -502,6 +486,16 @@ agnn_status av_workspace_bytes(const Plan& p, const agnn_layer_desc& d, size_t* 
     else return fail(AGNN_EUNSUPPORTED, "AGNN/VA: k_in must be 16/32/64/128/256"); \
   } while (0)
 
+// AGNN_AV_K128=0 selects the generic kernels at k = 128 (A/B comparisons)
+bool k128_disabled() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("AGNN_AV_K128");
+    v = (e && e[0] == '0') ? 1 : 0;
+  }
+  return v == 1;
+}
+
 template <int K>
 constexpr int av_fwd_unroll() { return K >= 256 ? 2 : 4; }
 template <int K>
@@ -529,7 +523,9 @@ agnn_status av_forward(const Plan& p, const agnn_layer_desc& d, const float* W, 
   }
   Items it = items_of(p);
   AvFwd A{Hf, sv.nu, d.beta, fabsf(d.beta), sv.X, sv.l, w.pacc, w.pl};
-  if (it.n_chunks + it.n_light > 0) {
+  if (K_ == 128 && !k128_disabled()) {
+    if ((st = av_fwd_k128(it, ag, A, s)) != AGNN_OK) return st;
+  } else if (it.n_chunks + it.n_light > 0) {
     if (ag) AGNN_AV_DISPATCH(K_, (av_fwd_kernel<K, AG, av_fwd_unroll<K>()>
                                   <<<grid_of(av_fwd_kernel<K, AG, av_fwd_unroll<K>()>),
                                      kSparseThreads, 0, s>>>(it, A)));
@@ -614,7 +610,9 @@ agnn_status av_backward(const Plan& p, const agnn_layer_desc& d, const float* W,
 #undef AV_PASS
     return AGNN_OK;
   }
-  if (it.n_chunks + it.n_light > 0) {
+  if (K_ == 128 && !k128_disabled()) {
+    if ((st = av_bwd_k128(it, ag, A, s)) != AGNN_OK) return st;
+  } else if (it.n_chunks + it.n_light > 0) {
     if (ag) AGNN_AV_DISPATCH(K_, (av_bwd_kernel<K, AG, av_bwd_unroll<K>()>
                                   <<<grid_of(av_bwd_kernel<K, AG, av_bwd_unroll<K>()>),
                                      kSparseThreads, 0, s>>>(it, A)));

@@ -1,0 +1,34 @@
+// av_args.cuh — argument blocks shared by the AGNN / VA sparse kernels
+// (agnn_va.cu generic widths, av_k128.cu for k = 128)
+#pragma once
+#include "internal.cuh"
+
+namespace agnn {
+
+struct AvFwd {
+  const float* H;     // [n_tot x K]  (replicated when world > 1)
+  const float* nu;    // [n_tot]      AGNN
+  float beta, bound;  // bound = |beta|
+  float* X;           // [n_local x K]
+  float* l;           // [n_local]    AGNN
+  float* pacc;        // [n_chunks x K]
+  float* pl;          // [n_chunks]
+};
+
+struct AvBwd {
+  const float* H;      // [n_tot x K]
+  const float* M;      // [n_tot x K]
+  const float4* rec;   // [n_tot] {nu, m, 1/l, delta}   AGNN
+  float beta, eps;
+  float* dH;           // [n_local x K]
+  float* pacc;         // [n_chunks x 2K]
+  float* dhp;          // [n_local x K] directed patterns: row-pass partial of dH (VA) / dH^ (AGNN)
+};
+
+enum { AV_VA = 0, AV_AG = 1 };
+
+// k = 128 lane-parallel kernels (av_k128.cu); symmetric patterns (ROLE 0) only
+agnn_status av_fwd_k128(const Items& it, bool agnn, const AvFwd& A, cudaStream_t s);
+agnn_status av_bwd_k128(const Items& it, bool agnn, const AvBwd& A, cudaStream_t s);
+
+}  // namespace agnn

@@ -22,9 +22,13 @@
 #include <mutex>
 
 #include "gat_args.cuh"
+#include "warp_batch.cuh"
 
 namespace agnn {
 namespace {
+
+using wb::item_of;
+using wb::Transpose;
 
 constexpr unsigned FULL = 0xffffffffu;
 constexpr int K = 128;
@@ -47,21 +51,6 @@ __device__ __forceinline__ void load_n(const float* p, float (&x)[N]) {
   } else {
 #pragma unroll
     for (int i = 0; i < N; ++i) x[i] = __ldg(p + i);
-  }
-}
-
-__device__ __forceinline__ void item_of(const Items& it, int64_t w, int64_t& row, int64_t& beg,
-                                        int64_t& end, int64_t& slot) {
-  if (w < it.n_chunks) {
-    row = it.chunk_row[w];
-    beg = it.row_ptr[row] + (int64_t)it.chunk_idx[w] * it.chunk;
-    end = min(beg + (int64_t)it.chunk, it.row_ptr[row + 1]);
-    slot = w;
-  } else {
-    row = it.light_rows[w - it.n_chunks];
-    beg = it.row_ptr[row];
-    end = it.row_ptr[row + 1];
-    slot = -1;
   }
 }
 
@@ -370,47 +359,6 @@ gat_fwd_tma_kernel(const __grid_constant__ CUtensorMap mapP, Items it, const flo
 }
 
 // ---------------------------------------------------------------- backward
-template <int B>
-struct Transpose {
-  static constexpr int T = (B >= 8) ? 3 : (B >= 4) ? 2 : (B >= 2) ? 1 : 0;
-  // edge index held by lane-in-group ql after the transposed reduction
-  __device__ static __forceinline__ int edge_of(int ql) {
-    int b = 0;
-#pragma unroll
-    for (int s = 0; s < T; ++s) b |= ((ql >> s) & 1) * (B >> (s + 1));
-    return b;
-  }
-  // lane-in-group that holds edge b
-  __device__ static __forceinline__ int lane_of(int b) {
-    int q = 0;
-#pragma unroll
-    for (int s = 0; s < T; ++s) q |= ((b / (B >> (s + 1))) & 1) << s;
-    return q;
-  }
-  // x[0..B) partial sums over the HL lanes of a head group -> x[0] = full sum of
-  // element edge_of(lane % HL), every lane
-  template <int HL>
-  __device__ static __forceinline__ void reduce(float (&x)[B], int lane) {
-    int len = B;
-#pragma unroll
-    for (int s = 0; s < T; ++s) {
-      const int o = 1 << s;
-      const bool upper = (lane & o) != 0;
-      len >>= 1;
-#pragma unroll
-      for (int k = 0; k < B / 2; ++k) {
-        if (k < len) {
-          const float keep = upper ? x[k + len] : x[k];
-          const float send = upper ? x[k] : x[k + len];
-          x[k] = keep + __shfl_xor_sync(FULL, send, o);
-        }
-      }
-    }
-#pragma unroll
-    for (int o = B; o < HL; o <<= 1) x[0] += __shfl_xor_sync(FULL, x[0], o);
-  }
-};
-
 template <int B>
 struct BwdBatch {  // operands of one batch of B edges held by one lane
   float4 Pi[B], Gi[B];

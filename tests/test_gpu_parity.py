@@ -82,6 +82,7 @@ CASES = [
     W("gat", "kron", 14, 8, 64, heads=2, layers=2, act="none"),
     W("agnn", "rmat", 14, 16, 128, layers=2, act="elu"),  # C3 shape (R-MAT, k=128)
     W("agnn", "kron", 13, 8, 64, act="elu"),
+    W("agnn", "kron", 16, 8, 128, act="none", beta=0.7),  # k=128 kernels, heavy rows, beta != 1
     W("agnn", "er", 0, 0, 256, n=1500, samples=9000, act="none", beta=1.5),
     W("agnn", "er", 0, 0, 16, n=1024, samples=7680),
     W("va", "kron", 13, 8, 256, act="none"),              # C4 shape (VA, k=256)
