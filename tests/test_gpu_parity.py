@@ -2,7 +2,7 @@
 
 Inputs are the seeded synthetic workloads (paper_conf_sc_bestarglzcgssci23_b200.gen)
 at sizes the oracle finishes in seconds that still span many tiles, heavy-row
-chunks (degree > 2048) and ragged tails.  Bars (north_star / SURVEY §8(c)):
+chunks (degree > the plan's chunk size) and ragged tails.  Bars (north_star / SURVEY §8(c)):
   * CSR metadata bit-exact with the oracle's host builder;
   * every float output normwise <= 1e-5 relative (FP32);
   * attention alpha elementwise |a - a_ref| <= 1e-5 a_ref + 1e-9.
