@@ -490,6 +490,87 @@ int oracle_va_backward(int64_t n, const int64_t* rp, const int32_t* ci, int k, i
 }
 
 /* ================================================================== */
+/* C-GNN layer over a semiring ("C-GNNs ... sigma(A H W) ... the
+ * adjacency matrix A (potentially normalized)"; §4.3 the
+ * aggregation (+) as a matrix product over a semiring; readings C1-C4 in
+ * DESIGN.md §2):
+ *   agg 0 SUM   real semiring (R, +, *, 0, 1):      X_i = sum_{j in N(i)} H_j
+ *   agg 1 MEAN  averaging semiring (tuples, :201):  X_i = (1/|N(i)|) sum_j H_j
+ *   agg 2 GCN   symmetric normalisation of A:       X_i = sum_j H_j / sqrt(d_i d_j)
+ *   agg 3 MAX   tropical (R u {-inf}, max, +):      X_ic = max_j H_jc
+ *   agg 4 MIN   tropical (R u {+inf}, min, +):      X_ic = min_j H_jc
+ * d_i = |N(i)| (stored entries of row i).  Z = X W, Hout = sigma(Z).  An empty
+ * row gives X_i = 0 (reading C3).  MAX/MIN record the arg index (the first,
+ * i.e. smallest, column j among ties; reading C4) in arg[n x k].          */
+static double cg_coef(int agg, const int64_t* rp, int64_t i, int64_t j) {
+  const double di = (double)(rp[i + 1] - rp[i]), dj = (double)(rp[j + 1] - rp[j]);
+  if (agg == 1) return 1.0 / di;
+  if (agg == 2) return 1.0 / sqrt(di * dj);
+  return 1.0;
+}
+int oracle_cgnn_forward(int64_t n, const int64_t* rp, const int32_t* ci, int k, int kout,
+                        const double* H, const double* W, int agg, int act, double* X,
+                        int32_t* arg, double* Z, double* Hout) {
+  if (agg < 0 || agg > 4) return 1;
+#pragma omp parallel for schedule(dynamic, 64)
+  for (int64_t i = 0; i < n; ++i)
+    for (int c = 0; c < k; ++c) {
+      if (agg <= 2) {
+        double x = 0.0;
+        for (int64_t p = rp[i]; p < rp[i + 1]; ++p)
+          x += cg_coef(agg, rp, i, ci[p]) * H[(int64_t)ci[p] * k + c];
+        X[i * k + c] = x;
+      } else {
+        int64_t best = -1;
+        for (int64_t p = rp[i]; p < rp[i + 1]; ++p) {
+          const double v = H[(int64_t)ci[p] * k + c];
+          if (best < 0 || (agg == 3 ? v > H[best * k + c] : v < H[best * k + c])) best = ci[p];
+        }
+        X[i * k + c] = best < 0 ? 0.0 : H[best * k + c];
+        arg[i * k + c] = (int32_t)best;
+      }
+    }
+  mm(n, k, kout, X, W, Z);
+#pragma omp parallel for schedule(static)
+  for (int64_t x = 0; x < n * kout; ++x) Hout[x] = act_f(act, Z[x]);
+  return 0;
+}
+
+/* Backward: G = dHout (.) sigma'(Z); dW = X^T G; M = G W^T = dL/dX;
+ *   SUM/MEAN/GCN: dH_j = sum_{(i,j) stored} coef_ij M_i     (= A'^T M)
+ *   MAX/MIN:      dH_jc = sum_{(i,j) stored, arg_ic = j} M_ic              */
+int oracle_cgnn_backward(int64_t n, const int64_t* rp, const int32_t* ci, int k, int kout,
+                         const double* H, const double* W, int agg, int act, const double* X,
+                         const int32_t* arg, const double* Z, const double* dHout, double* dH,
+                         double* dW) {
+  const int64_t nnz = rp[n];
+  (void)H;
+  double* G = (double*)malloc(sizeof(double) * (size_t)(n * kout + 1));
+  double* M = (double*)malloc(sizeof(double) * (size_t)(n * k + 1));
+  int64_t* cp = (int64_t*)malloc(sizeof(int64_t) * (size_t)(n + 1));
+  int64_t* pos = (int64_t*)malloc(sizeof(int64_t) * (size_t)(nnz + 1));
+  int64_t* erow = row_of_edge(n, rp);
+  build_csc(n, rp, ci, cp, pos);
+#pragma omp parallel for schedule(static)
+  for (int64_t x = 0; x < n * kout; ++x) G[x] = dHout[x] * act_df(act, Z[x]);
+  mm_tn(n, k, kout, X, G, dW);
+  mm_nt(n, kout, k, G, W, M);
+#pragma omp parallel for schedule(dynamic, 64)
+  for (int64_t j = 0; j < n; ++j)
+    for (int c = 0; c < k; ++c) {
+      double acc = 0.0;
+      for (int64_t q = cp[j]; q < cp[j + 1]; ++q) {
+        const int64_t i = erow[pos[q]];
+        if (agg <= 2) acc += cg_coef(agg, rp, i, j) * M[i * k + c];
+        else if (arg[i * k + c] == (int32_t)j) acc += M[i * k + c];
+      }
+      dH[j * k + c] = acc;
+    }
+  free(G); free(M); free(cp); free(pos); free(erow);
+  return 0;
+}
+
+/* ================================================================== */
 /* 1D row-block partition bounds (reading A20; the paper's own scheme is 2D,
  * PAPER.md:321): w(r) = row_ptr[r] + c_v r ; bounds[0] = 0, bounds[P] = n,
  * bounds[p] = min{ r : w(r) >= ceil(p w(n) / P) }.                       */

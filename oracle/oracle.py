@@ -175,8 +175,40 @@ def va_backward(rp, ci, H, W, fwd, dHout, act="relu"):
     return out
 
 
+AGG = {"sum": 0, "mean": 1, "gcn": 2, "max": 3, "min": 4}
+
+
+def cgnn_forward(rp, ci, H, W, agg="sum", act="relu"):
+    rp, ci, n, nnz = _csr(rp, ci)
+    H, W = _d(H), _d(W)
+    k, kout = W.shape
+    out = {"X": np.zeros((n, k)), "arg": np.full((n, k), -1, np.int32), "Z": np.zeros((n, kout)),
+           "Hout": np.zeros((n, kout))}
+    rc = lib().oracle_cgnn_forward(
+        _i64(n), _p(rp), _p(ci), ctypes.c_int(k), ctypes.c_int(kout), _p(H), _p(W),
+        ctypes.c_int(AGG[agg]), ctypes.c_int(ACT[act]), _p(out["X"]), _p(out["arg"]),
+        _p(out["Z"]), _p(out["Hout"]))
+    if rc:
+        raise ValueError("oracle_cgnn_forward failed")
+    return out
+
+
+def cgnn_backward(rp, ci, H, W, fwd, dHout, agg="sum", act="relu"):
+    rp, ci, n, nnz = _csr(rp, ci)
+    H, W, dHout = _d(H), _d(W), _d(dHout)
+    k, kout = W.shape
+    out = {"dH": np.zeros((n, k)), "dW": np.zeros((k, kout))}
+    rc = lib().oracle_cgnn_backward(
+        _i64(n), _p(rp), _p(ci), ctypes.c_int(k), ctypes.c_int(kout), _p(H), _p(W),
+        ctypes.c_int(AGG[agg]), ctypes.c_int(ACT[act]), _p(fwd["X"]), _p(fwd["arg"]),
+        _p(fwd["Z"]), _p(dHout), _p(out["dH"]), _p(out["dW"]))
+    if rc:
+        raise ValueError("oracle_cgnn_backward failed")
+    return out
+
+
 def layer(model, rp, ci, H, W, a=None, heads=1, dHout=None, act="relu", slope=0.2, beta=1.0,
-          eps=1e-12):
+          eps=1e-12, agg="sum"):
     """Forward (+ backward when dHout is given) of one layer of `model`."""
     if model == "gat":
         f = gat_forward(rp, ci, H, W, a, heads, slope, act)
@@ -187,6 +219,9 @@ def layer(model, rp, ci, H, W, a=None, heads=1, dHout=None, act="relu", slope=0.
     elif model == "va":
         f = va_forward(rp, ci, H, W, act)
         b = va_backward(rp, ci, H, W, f, dHout, act) if dHout is not None else None
+    elif model == "cgnn":
+        f = cgnn_forward(rp, ci, H, W, agg, act)
+        b = cgnn_backward(rp, ci, H, W, f, dHout, agg, act) if dHout is not None else None
     else:
         raise ValueError(model)
     return f, b

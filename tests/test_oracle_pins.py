@@ -391,3 +391,107 @@ def test_partition_bruteforce(world, c_v):
         b = oracle.partition(rp, world, c_v)
         np.testing.assert_array_equal(b, brute_bounds(rp, world, c_v))
         assert (np.diff(b) >= 0).all()
+
+
+# ------------------------------------------------ C-GNN over semirings (f3)
+def _dense_adj(rp, ci, n):
+    A = np.zeros((n, n))
+    for i in range(n):
+        A[i, ci[rp[i]:rp[i + 1]]] = 1.0
+    return A
+
+
+def _cgnn_dense_torch(A, H, W, R, agg, kind):
+    """sigma(A' H W) (PAPER.md:213) with A' the (normalised) adjacency, or the
+    tropical max/min product, in torch fp64 with autograd."""
+    import torch
+    At = torch.tensor(A)
+    Ht = torch.tensor(H, requires_grad=True)
+    Wt = torch.tensor(W, requires_grad=True)
+    d = At.sum(1)
+    if agg == "sum":
+        X = At @ Ht
+    elif agg == "mean":
+        X = (At / d[:, None]) @ Ht
+    elif agg == "gcn":
+        X = (At / torch.sqrt(d[:, None] * d[None, :])) @ Ht
+    else:
+        big = torch.where(At[:, :, None] > 0, Ht[None, :, :],
+                          torch.tensor(-np.inf if agg == "max" else np.inf, dtype=torch.float64))
+        X = big.amax(1) if agg == "max" else big.amin(1)
+    Z = X @ Wt
+    Hout = {"none": Z, "relu": torch.relu(Z), "elu": torch.nn.functional.elu(Z)}[kind]
+    (Hout * torch.tensor(R)).sum().backward()
+    return X.detach().numpy(), Z.detach().numpy(), Ht.grad.numpy(), Wt.grad.numpy()
+
+
+@pytest.mark.parametrize("agg", ["sum", "mean", "gcn", "max", "min"])
+@pytest.mark.parametrize("kind", ["none", "elu"])
+@pytest.mark.parametrize("symmetric", [True, False])
+def test_cgnn_local_equals_dense_semiring(agg, kind, symmetric):
+    """Local edge loops == the dense matrix product over the semiring + autograd.
+    Features are distinct per column (no ties), so amax/amin autograd is exact."""
+    rng = np.random.default_rng(60)
+    n, k, kout = 14, 5, 6
+    rp, ci = rand_graph(n, 0.3, rng, symmetric=symmetric)
+    H = rng.permutation(n * k).reshape(n, k) / (n * k) - 0.5   # distinct values
+    W = rng.uniform(-1, 1, (k, kout)) / np.sqrt(k)
+    R = rng.uniform(-1, 1, (n, kout))
+    f, b = oracle.layer("cgnn", rp, ci, H, W, dHout=R, act=kind, agg=agg)
+    X, Z, dH, dW = _cgnn_dense_torch(_dense_adj(rp, ci, n), H, W, R, agg, kind)
+    assert rel(f["X"], X) < 1e-14
+    assert rel(f["Z"], Z) < 1e-13
+    assert rel(b["dH"], dH) < 1e-12
+    assert rel(b["dW"], dW) < 1e-12
+
+
+def test_cgnn_mean_equals_paper_tuple_semiring():
+    """the averaging aggregation as a product over R^2 with
+    a op1 b = (a1 b1, a1) and a op2 b = ((a1 a2 + b1 b2)/(a2 + b2), a2 + b2),
+    every stored entry x of A mapped to (x, x) — evaluated literally."""
+    rng = np.random.default_rng(61)
+    n, k = 12, 4
+    rp, ci = rand_graph(n, 0.3, rng, symmetric=False)
+    H = rng.uniform(-1, 1, (n, k))
+    W = np.eye(k)
+    f = oracle.cgnn_forward(rp, ci, H, W, "mean", "none")
+    for i in range(n):
+        for c in range(k):
+            acc = None
+            for p in range(rp[i], rp[i + 1]):
+                a = (1.0, 1.0)                          # entry x = 1 -> (x, x)
+                prod = (a[0] * H[ci[p], c], a[0])       # op1 with (h, .)
+                acc = prod if acc is None else (
+                    (acc[0] * acc[1] + prod[0] * prod[1]) / (acc[1] + prod[1]), acc[1] + prod[1])
+            assert abs(f["X"][i, c] - acc[0]) < 1e-14
+
+
+def test_cgnn_tropical_ties_and_empty_rows():
+    """Readings C3/C4: an empty row aggregates to 0 with zero gradient; among tied
+    maxima the smallest column index receives the whole gradient."""
+    n, k = 4, 1
+    rp = np.array([0, 3, 3, 4, 5], np.int64)        # row 1 empty
+    ci = np.array([0, 2, 3, 2, 3], np.int32)
+    H = np.array([[0.5], [9.0], [0.5], [0.5]])      # row 0: H_0 = H_2 = H_3 (tie)
+    W = np.eye(1)
+    R = np.array([[1.0], [1.0], [1.0], [1.0]])
+    for agg in ("max", "min"):
+        f = oracle.cgnn_forward(rp, ci, H, W, agg, "none")
+        b = oracle.cgnn_backward(rp, ci, H, W, f, R, agg, "none")
+        assert f["X"][1, 0] == 0.0 and f["arg"][0, 0] == 0
+        # dH_0 gets row 0's gradient (first of the tie); rows 2, 3 get their own rows'
+        np.testing.assert_array_equal(b["dH"][:, 0], [1.0, 0.0, 1.0, 1.0])
+
+
+@pytest.mark.parametrize("agg", ["sum", "gcn", "max"])
+def test_cgnn_finite_differences(agg):
+    rng = np.random.default_rng(62)
+    n, k, kout = 9, 3, 4
+    rp, ci = rand_graph(n, 0.35, rng, symmetric=True)
+    H = rng.permutation(n * k).reshape(n, k) / (n * k) - 0.5
+    W = rng.uniform(-1, 1, (k, kout))
+    R = rng.uniform(-1, 1, (n, kout))
+    f, b = oracle.layer("cgnn", rp, ci, H, W, dHout=R, act="elu", agg=agg)
+    loss = lambda: float((oracle.cgnn_forward(rp, ci, H, W, agg, "elu")["Hout"] * R).sum())
+    assert rel(_fd(loss, H, 1e-7), b["dH"]) < 1e-6
+    assert rel(_fd(loss, W, 1e-7), b["dW"]) < 1e-6
