@@ -21,6 +21,7 @@
  *    a1 = a[h][0:d] (centre vertex = row i), a2 = a[h][d:2d] (neighbour =
  *    column j), d = k_out/heads; H_out, dH_out: [n_local x k_out];
  *    dH_in: [n_local x k_in]; dW: [k_in x k_out]; da: [heads][2d].
+ *    AGNN_CGNN: heads == 1, a and da NULL, k_in in 16..256 (multiple of 16).
  *  - The CSR lists, for every local row i, the vertices i aggregates from
  *    (N^(i)), by GLOBAL column id, strictly ascending.
  *    The library computes on exactly this pattern: it never adds self-loops
@@ -73,7 +74,23 @@ typedef enum {
   AGNN_ESTATE = 6
 } agnn_status;
 
-typedef enum { AGNN_VA = 0, AGNN_AGNN = 1, AGNN_GAT = 2 } agnn_kind;
+/* AGNN_CGNN: a C-GNN layer sigma((A (x) H) W), the aggregation a
+ * matrix product over the semiring `agg` (S§8(f) f3)        */
+typedef enum { AGNN_VA = 0, AGNN_AGNN = 1, AGNN_GAT = 2, AGNN_CGNN = 3 } agnn_kind;
+
+/* C-GNN aggregation (readings C1-C4), d_i = stored entries of row i:
+ *   SUM  X_i = sum_{j in N(i)} H_j               (real semiring)
+ *   MEAN X_i = sum_j H_j / d_i                   (averaging semiring)
+ *   GCN  X_i = sum_j H_j / sqrt(d_i d_j)         (normalised A)
+ *   MAX / MIN  X_ic = max / min_j H_jc           (tropical semirings);
+ *        an empty row gives 0; the gradient goes to the smallest j among ties */
+typedef enum {
+  AGNN_AGG_SUM = 0,
+  AGNN_AGG_MEAN = 1,
+  AGNN_AGG_GCN = 2,
+  AGNN_AGG_MAX = 3,
+  AGNN_AGG_MIN = 4
+} agnn_agg;
 
 /* sigma; reading A6: ReLU with sigma'(0) = 0, ELU(alpha = 1) */
 typedef enum { AGNN_ACT_NONE = 0, AGNN_ACT_RELU = 1, AGNN_ACT_ELU = 2 } agnn_act;
@@ -109,6 +126,7 @@ typedef struct {
   float negative_slope;    /* GAT LeakyReLU slope lambda (reading A5), 0.2          */
   float beta;              /* AGNN temperature (reading A8), 1.0, not trained        */
   float eps;               /* AGNN norm floor nu_i = max(||h_i||, eps), 1e-12        */
+  agnn_agg agg;            /* C-GNN aggregation semiring (ignored by the A-GNNs)     */
 } agnn_layer_desc;
 
 typedef struct agnn_plan_s* agnn_plan_t;

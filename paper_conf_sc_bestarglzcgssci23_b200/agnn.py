@@ -14,7 +14,8 @@ import os
 from . import _build
 
 VA, AGNN, GAT = 0, 1, 2
-KIND = {"va": VA, "agnn": AGNN, "gat": GAT}
+KIND = {"va": VA, "agnn": AGNN, "gat": GAT, "cgnn": 3}
+AGG = {"sum": 0, "mean": 1, "gcn": 2, "max": 3, "min": 4}
 ACT = {"none": 0, "relu": 1, "elu": 2}
 PREC_FP32, PREC_TF32X3 = 0, 1
 CSR_SYMMETRIC = 1
@@ -57,7 +58,7 @@ class LayerDesc(ctypes.Structure):
     _fields_ = [("kind", ctypes.c_int), ("k_in", ctypes.c_int), ("k_out", ctypes.c_int),
                 ("heads", ctypes.c_int), ("act", ctypes.c_int), ("prec", ctypes.c_int),
                 ("negative_slope", ctypes.c_float), ("beta", ctypes.c_float),
-                ("eps", ctypes.c_float)]
+                ("eps", ctypes.c_float), ("agg", ctypes.c_int)]
 
 
 _lib = None
@@ -253,9 +254,10 @@ class Plan:
 
 
 def layer_desc(kind, k_in, k_out, heads=1, act="relu", prec=PREC_FP32, negative_slope=0.2,
-               beta=1.0, eps=1e-12) -> LayerDesc:
+               beta=1.0, eps=1e-12, agg="sum") -> LayerDesc:
     return LayerDesc(KIND[kind] if isinstance(kind, str) else kind, k_in, k_out, heads,
-                     ACT[act] if isinstance(act, str) else act, prec, negative_slope, beta, eps)
+                     ACT[act] if isinstance(act, str) else act, prec, negative_slope, beta, eps,
+                     AGG[agg] if isinstance(agg, str) else agg)
 
 
 class Model:

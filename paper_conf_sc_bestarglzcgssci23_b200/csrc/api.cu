@@ -100,6 +100,11 @@ static agnn_status check_desc(const agnn_layer_desc& d) {
     if (d.heads != 1) return fail(AGNN_EINVAL, "AGNN/VA: heads must be 1");
     if (d.k_in > 256 || d.k_in % 16)
       return fail(AGNN_EUNSUPPORTED, "AGNN/VA: k_in must be one of 16..256, multiple of 16");
+  } else if (d.kind == AGNN_CGNN) {
+    if (d.heads != 1) return fail(AGNN_EINVAL, "C-GNN: heads must be 1");
+    if (d.agg < AGNN_AGG_SUM || d.agg > AGNN_AGG_MIN) return fail(AGNN_EINVAL, "C-GNN: agg");
+    if (d.k_in > 256 || d.k_in % 16)
+      return fail(AGNN_EUNSUPPORTED, "C-GNN: k_in must be one of 16..256, multiple of 16");
   } else {
     return fail(AGNN_EINVAL, "layer desc: kind");
   }
@@ -109,6 +114,15 @@ static agnn_status check_desc(const agnn_layer_desc& d) {
 static GatShape gat_shape(const agnn_layer_desc& d) {
   return GatShape{d.k_in, d.k_out, d.heads, d.negative_slope, (int)d.act};
 }
+
+// C-GNN entry points live in cgnn.cu
+agnn_status cg_saved_bytes(const Plan& p, const agnn_layer_desc& d, size_t* b);
+agnn_status cg_workspace_bytes(const Plan& p, const agnn_layer_desc& d, size_t* b);
+agnn_status cg_forward(const Plan& p, const agnn_layer_desc& d, const float* W, const float* H_in,
+                       float* H_out, void* saved, void* ws, cudaStream_t s);
+agnn_status cg_backward(const Plan& p, const agnn_layer_desc& d, const float* W,
+                        const float* H_in, const void* saved, const float* dH_out, float* dH_in,
+                        float* dW, void* ws, cudaStream_t s);
 
 // AGNN / VA entry points live in agnn_va.cu
 agnn_status av_saved_bytes(const Plan& p, const agnn_layer_desc& d, size_t* b);
@@ -332,6 +346,7 @@ agnn_status agnn_saved_bytes(agnn_model_t h, int layer, size_t* bytes) {
     *bytes = gat_saved_bytes(*h->m.plan, gat_shape(*d));
     return AGNN_OK;
   }
+  if (d->kind == AGNN_CGNN) return cg_saved_bytes(*h->m.plan, *d, bytes);
   return av_saved_bytes(*h->m.plan, *d, bytes);
 }
 
@@ -344,6 +359,7 @@ agnn_status agnn_workspace_bytes(agnn_model_t h, int layer, size_t* bytes) {
     *bytes = gat_workspace_bytes(*h->m.plan, gat_shape(*d));
     return AGNN_OK;
   }
+  if (d->kind == AGNN_CGNN) return cg_workspace_bytes(*h->m.plan, *d, bytes);
   return av_workspace_bytes(*h->m.plan, *d, bytes);
 }
 
@@ -363,6 +379,7 @@ agnn_status agnn_forward(agnn_model_t h, int layer, const float* W, const float*
     if (!a || !aligned16(a)) return fail(AGNN_EINVAL, "agnn_forward: GAT needs an aligned `a`");
     return gat_forward(p, gat_shape(*d), W, a, H_in, H_out, saved, ws, s);
   }
+  if (d->kind == AGNN_CGNN) return cg_forward(p, *d, W, H_in, H_out, saved, ws, s);
   return av_forward(p, *d, W, H_in, H_out, saved, ws, s);
 }
 
@@ -383,6 +400,7 @@ agnn_status agnn_backward(agnn_model_t h, int layer, const float* W, const float
     if (!a || !aligned16(a)) return fail(AGNN_EINVAL, "agnn_backward: GAT needs an aligned `a`");
     return gat_backward(p, gat_shape(*d), W, a, H_in, saved, dH_out, dH_in, dW, da, ws, s);
   }
+  if (d->kind == AGNN_CGNN) return cg_backward(p, *d, W, H_in, saved, dH_out, dH_in, dW, ws, s);
   return av_backward(p, *d, W, H_in, saved, dH_out, dH_in, dW, ws, s);
 }
 
@@ -395,6 +413,8 @@ agnn_status agnn_debug_attention(agnn_model_t h, int layer, const void* saved,
   if (count > 0 && (!edge_pos || !out)) return fail(AGNN_EINVAL, "agnn_debug_attention: NULL");
   if (d->kind == AGNN_GAT)
     return gat_debug_alpha(*h->m.plan, gat_shape(*d), saved, edge_pos, count, out, s);
+  if (d->kind == AGNN_CGNN)
+    return fail(AGNN_EUNSUPPORTED, "debug_attention: a C-GNN layer has no attention");
   return av_debug_attention(*h->m.plan, *d, saved, H_in, edge_pos, count, out, s);
 }
 

@@ -91,7 +91,7 @@ def fill_device(seed, stream_id, count, scale, out_ptr: int, stream: int = 0, of
 class Workload:
     """One BASELINE.json config as a concrete synthetic input recipe."""
     name: str
-    model: str            # "gat" | "agnn" | "va"
+    model: str            # "gat" | "agnn" | "va" | "cgnn"
     graph: str            # "er" | "kron" | "rmat"
     scale: int            # log2 n (ER: n need not be a power of two)
     n: int
@@ -105,6 +105,7 @@ class Workload:
     beta: float = 1.0
     eps: float = 1e-12
     train: bool = False   # step = fwd + bwd + SGD update (C4) instead of fwd + bwd
+    agg: str = "sum"      # C-GNN aggregation semiring (model "cgnn")
     lr: float = 1e-3
 
     @property

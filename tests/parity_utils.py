@@ -54,7 +54,7 @@ def oracle_step(w: gen.Workload, rp, ci, H, Ws, As, R):
     Hs, fwd = [np.asarray(H, np.float64)], []
     for l in range(w.layers):
         f, _ = oracle.layer(w.model, rp, ci, Hs[-1], Ws[l], As[l], w.heads, act=w.act,
-                            slope=w.slope, beta=w.beta, eps=w.eps)
+                            slope=w.slope, beta=w.beta, eps=w.eps, agg=w.agg)
         fwd.append(f)
         Hs.append(f["Hout"])
     dHs = [None] * (w.layers + 1)
@@ -67,6 +67,8 @@ def oracle_step(w: gen.Workload, rp, ci, H, Ws, As, R):
             das[l] = b["da"]
         elif w.model == "agnn":
             b = oracle.agnn_backward(rp, ci, Hs[l], Ws[l], fwd[l], dHs[l + 1], w.beta, w.eps, w.act)
+        elif w.model == "cgnn":
+            b = oracle.cgnn_backward(rp, ci, Hs[l], Ws[l], fwd[l], dHs[l + 1], w.agg, w.act)
         else:
             b = oracle.va_backward(rp, ci, Hs[l], Ws[l], fwd[l], dHs[l + 1], w.act)
         dHs[l], dWs[l] = b["dH"], b["dW"]

@@ -255,3 +255,44 @@ def test_symmetric_flag_on_directed_pattern_is_not_silently_wrong():
     b = pu.gpu_step(w, graph=g, symmetric=False)
     for x, y in ((a.dH[0], b.dH[0]), (a.dW[0], b.dW[0]), (a.da[0], b.da[0])):
         assert pu.rel(x.cpu().numpy(), y.cpu().numpy()) <= 1e-6
+
+
+# ------------------------------------------------------------------ C-GNN over semirings (f3)
+CGNN_CASES = [
+    W("cgnn", "kron", 14, 8, 64, act="elu", agg="sum"),
+    W("cgnn", "kron", 14, 8, 128, act="none", agg="mean"),
+    W("cgnn", "rmat", 13, 16, 32, act="elu", agg="gcn"),
+    W("cgnn", "kron", 15, 8, 16, act="relu", agg="max"),
+    W("cgnn", "er", 0, 0, 256, n=3000, samples=30000, act="none", agg="min"),
+    W("cgnn", "kron", 13, 8, 64, layers=2, act="elu", agg="gcn"),
+    W("cgnn", "kron", 13, 8, 128, layers=2, act="elu", agg="max"),
+]
+
+
+def _cgnn_check(w, rp, ci, g, symmetric=True):
+    H, Ws, As, R = w.host_inputs()
+    if w.act == "relu":
+        f0 = pu.oracle_step(w, rp, ci, H, Ws, As, R)["fwd"][-1]
+        R = pu.relu_kink_mask(w, f0["Z"], R)
+    st = pu.gpu_step(w, graph=g, R=R, symmetric=symmetric)
+    ref = pu.oracle_step(w, rp, ci, H, Ws, As, R)
+    pu.compare(w, st, ref)
+    return st, ref
+
+
+@pytest.mark.parametrize("w", CGNN_CASES, ids=lambda w: f"{w.name}-{w.agg}")
+def test_cgnn_layer_parity(w):
+    src, dst, rp, ci = pu.host_graph(w)
+    g = pu.device_graph(w, src, dst)
+    _cgnn_check(w, rp, ci, g)
+
+
+@pytest.mark.parametrize("agg", ["sum", "mean", "gcn", "max", "min"])
+def test_cgnn_directed_and_heavy_chunks(agg, monkeypatch):
+    """Directed pattern (backward gathers over the CSC) with heavy rows and columns
+    split into 64-edge chunks."""
+    monkeypatch.setenv("AGNN_CHUNK_EDGES", "64")
+    w = W("cgnn", "kron", 12, 8, 64, act="none", agg=agg)
+    rp, ci, g = _directed_graph(w)
+    st, _ = _cgnn_check(w, rp, ci, g, symmetric=False)
+    assert st.plan.info()["heavy_rows"] > 0
