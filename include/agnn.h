@@ -114,7 +114,8 @@ typedef struct {
 
 typedef struct {
   int rank, world;
-  const void* nccl_unique_id; /* host, 128 bytes (ncclUniqueId); NULL iff world == 1 */
+  const void* nccl_unique_id; /* host, 128 bytes (ncclUniqueId): NCCL exchange; NULL:
+                                 peer-memory exchange (world <= 8, see agnn_plan_connect) */
   const int64_t* bounds;      /* host, [world + 1] row bounds (agnn_partition)      */
 } agnn_dist;
 
@@ -227,6 +228,23 @@ uint64_t agnn_launch_count(void);
 agnn_status agnn_profile_enable(int on);
 agnn_status agnn_profile_report(char* buf, size_t len);
 agnn_status agnn_profile_reset(void);
+/* ---- peer-memory exchange (world > 1, agnn_dist.nccl_unique_id == NULL) ----
+ * The ranks' replicated buffers are mapped into each other with CUDA IPC
+ * (loads / stores over NVLink / NVSwitch; S§8(e)).  Setup, once per plan (host,
+ * synchronising; the caller moves the 64-byte handles between ranks, e.g. with
+ * torch.distributed all_gather_object):
+ *   1. agnn_plan_ctl_export on every rank, all-gather, agnn_plan_connect;
+ *   2. for every `saved` and `workspace` buffer passed to forward/backward:
+ *      agnn_ipc_export on every rank, all-gather, agnn_plan_register.
+ * Every rank must register its buffers in the same order with the same sizes.
+ * handles: [world][64 B] in rank order; offsets: [world] byte offsets of the
+ * buffer inside each rank's allocation (both host).                          */
+agnn_status agnn_ipc_export(const void* device_ptr, void* handle64, int64_t* offset);
+agnn_status agnn_plan_ctl_export(agnn_plan_t plan, void* handle64, int64_t* offset);
+agnn_status agnn_plan_connect(agnn_plan_t plan, const void* handles, const int64_t* offsets);
+agnn_status agnn_plan_register(agnn_plan_t plan, void* local, size_t bytes, const void* handles,
+                               const int64_t* offsets);
+
 /* ncclGetUniqueId for the multi-GPU plan (host, 128 bytes).                 */
 agnn_status agnn_nccl_unique_id(void* out128);
 

@@ -28,6 +28,7 @@ STATUS = {0: "AGNN_OK", 1: "AGNN_EINVAL", 2: "AGNN_ECUDA", 3: "AGNN_ENCCL", 4: "
 # every symbol include/agnn.h declares (tests check the .so exports all of them)
 EXPORTS = ("agnn_partition", "agnn_plan_create", "agnn_plan_destroy", "agnn_plan_info",
            "agnn_plan_csc", "agnn_loss_inner", "agnn_sgd_step",
+           "agnn_ipc_export", "agnn_plan_ctl_export", "agnn_plan_connect", "agnn_plan_register",
            "agnn_model_create", "agnn_model_destroy", "agnn_saved_bytes", "agnn_workspace_bytes",
            "agnn_forward", "agnn_backward", "agnn_debug_attention", "agnn_debug_gemm",
            "agnn_debug_gemm_tn", "agnn_debug_gemm_tn_ws_bytes",
@@ -124,6 +125,14 @@ def profile_report() -> dict:
     return out
 
 
+def ipc_export(tensor):
+    """(64-byte CUDA IPC handle of the allocation holding `tensor`, byte offset)."""
+    h = ctypes.create_string_buffer(64)
+    off = ctypes.c_int64()
+    _check(lib().agnn_ipc_export(ctypes.c_void_p(tensor.data_ptr()), h, ctypes.byref(off)))
+    return h.raw, off.value
+
+
 LOSS_SCRATCH = 1024  # AGNN_LOSS_SCRATCH
 
 
@@ -217,9 +226,11 @@ class Plan:
         if world > 1:
             import numpy as np
             self._bounds = np.ascontiguousarray(bounds, dtype=np.int64)
-            self._uid = ctypes.create_string_buffer(bytes(nccl_unique_id), 128)
-            dist = Dist(rank, world, ctypes.cast(self._uid, ctypes.c_void_p),
-                        self._bounds.ctypes.data_as(ctypes.c_void_p))
+            uid = None
+            if nccl_unique_id is not None:  # NCCL exchange; None: peer-memory exchange
+                self._uid = ctypes.create_string_buffer(bytes(nccl_unique_id), 128)
+                uid = ctypes.cast(self._uid, ctypes.c_void_p)
+            dist = Dist(rank, world, uid, self._bounds.ctypes.data_as(ctypes.c_void_p))
         h = ctypes.c_void_p()
         _check(lib().agnn_plan_create(ctypes.byref(self._csr),
                                       ctypes.byref(dist) if dist is not None else None,
@@ -234,6 +245,28 @@ class Plan:
         keys = ("n_local", "nnz", "light_rows", "heavy_rows", "heavy_chunks", "chunk", "max_degree",
                 "n")
         return dict(zip(keys, list(a)))
+
+    # ---- peer-memory exchange setup (world > 1 without an NCCL id) -------------
+    def ctl_export(self):
+        """(handle bytes, offset) of this rank's control block."""
+        h = ctypes.create_string_buffer(64)
+        off = ctypes.c_int64()
+        _check(lib().agnn_plan_ctl_export(self.handle, h, ctypes.byref(off)))
+        return h.raw, off.value
+
+    def connect(self, exports):
+        """exports: [(handle, offset)] of every rank's control block, rank order."""
+        hs = b"".join(h for h, _ in exports)
+        offs = (ctypes.c_int64 * len(exports))(*[o for _, o in exports])
+        _check(lib().agnn_plan_connect(self.handle, hs, offs))
+
+    def register(self, tensor, exports):
+        """Map every rank's copy of `tensor` (its replicated prefix sits at the same offsets)."""
+        hs = b"".join(h for h, _ in exports)
+        offs = (ctypes.c_int64 * len(exports))(*[o for _, o in exports])
+        _check(lib().agnn_plan_register(self.handle, ctypes.c_void_p(tensor.data_ptr()),
+                                        ctypes.c_size_t(tensor.numel() * tensor.element_size()),
+                                        hs, offs))
 
     def csc(self, perm=True, stream=None):
         """agnn_plan_csc: (col_ptr int64 [n+1], row_idx int32 [nnz], perm int64 [nnz] | None)."""

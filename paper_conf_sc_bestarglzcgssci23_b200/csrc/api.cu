@@ -233,7 +233,8 @@ agnn_status agnn_plan_create(const agnn_csr* csr, const agnn_dist* dist, cudaStr
     p.col_idx = csr->col_idx;
     p.flags = csr->flags;
     if (dist && dist->world > 1) {
-      if (!dist->nccl_unique_id || !dist->bounds || dist->rank < 0 || dist->rank >= dist->world) {
+      if (!dist->bounds || dist->rank < 0 || dist->rank >= dist->world ||
+          (!dist->nccl_unique_id && dist->world > kMaxPeers)) {
         delete h;
         return fail(AGNN_EINVAL, "agnn_plan_create: bad dist (unique id / bounds / rank)");
       }
@@ -251,6 +252,7 @@ agnn_status agnn_plan_create(const agnn_csr* csr, const agnn_dist* dist, cudaStr
     agnn_status st = plan_build(p, s);
     if (st == AGNN_OK && p.world > 1) st = comm_init(p, dist->nccl_unique_id);
     if (st != AGNN_OK) {
+      comm_destroy(p);
       if (p.meta_block) cudaFree(p.meta_block);
       if (p.csc_block) cudaFree(p.csc_block);
       if (p.c_meta_block) cudaFree(p.c_meta_block);
@@ -287,6 +289,38 @@ agnn_status agnn_plan_info(agnn_plan_t h, int64_t* info) {
   info[5] = p.chunk;
   info[6] = p.max_deg;
   info[7] = p.n;
+  return AGNN_OK;
+}
+
+agnn_status agnn_plan_ctl_export(agnn_plan_t h, void* handle, int64_t* offset) {
+  if (!h || !handle || !offset) return fail(AGNN_EINVAL, "agnn_plan_ctl_export: NULL argument");
+  if (!h->p.peer) return fail(AGNN_ESTATE, "agnn_plan_ctl_export: plan does not use peer exchange");
+  return agnn_ipc_export(h->p.ctl, handle, offset);
+}
+
+agnn_status agnn_plan_connect(agnn_plan_t h, const void* handles, const int64_t* offsets) {
+  if (!h || !handles || !offsets) return fail(AGNN_EINVAL, "agnn_plan_connect: NULL argument");
+  Plan& p = h->p;
+  if (!p.peer) return fail(AGNN_ESTATE, "agnn_plan_connect: plan does not use peer exchange");
+  char* out[kMaxPeers] = {};
+  agnn_status st = peer_open(p, handles, offsets, p.ctl, out);
+  if (st != AGNN_OK) return st;
+  for (int r = 0; r < p.world; ++r) p.peer_ctl[r] = out[r];
+  p.peer_ready = true;
+  return AGNN_OK;
+}
+
+agnn_status agnn_plan_register(agnn_plan_t h, void* local, size_t bytes, const void* handles,
+                               const int64_t* offsets) {
+  if (!h || !local || !handles || !offsets) return fail(AGNN_EINVAL, "agnn_plan_register: NULL argument");
+  Plan& p = h->p;
+  if (!p.peer) return fail(AGNN_ESTATE, "agnn_plan_register: plan does not use peer exchange");
+  Plan::Reg g;
+  g.local = static_cast<char*>(local);
+  g.bytes = bytes;
+  agnn_status st = peer_open(p, handles, offsets, local, g.peer);
+  if (st != AGNN_OK) return st;
+  p.regs->push_back(g);
   return AGNN_OK;
 }
 

@@ -277,11 +277,12 @@ struct SavedCg {
 SavedCg carve_saved(const Plan& p, const agnn_layer_desc& d, void* base, size_t* total) {
   Carver c(base);
   SavedCg s;
+  // replicated (n-row) arrays first (same offsets on every rank; peer exchange)
   s.Hfull = c.take<float>(p.world > 1 ? (size_t)p.n * d.k_in : 0);
-  s.X = c.take<float>((size_t)p.n_local * d.k_in);
-  s.Z = c.take<float>((size_t)p.n_local * d.k_out);
   s.rdeg = c.take<float>((size_t)p.n);
   s.arg = c.take<int32_t>(trop(d) ? (size_t)p.n * d.k_in : 0);
+  s.X = c.take<float>((size_t)p.n_local * d.k_in);
+  s.Z = c.take<float>((size_t)p.n_local * d.k_out);
   if (total) *total = c.off + 256;
   return s;
 }
@@ -295,10 +296,10 @@ WsCg carve_ws(const Plan& p, const agnn_layer_desc& d, void* base, size_t* total
   WsCg w;
   size_t sv = 0;
   carve_saved(p, d, nullptr, &sv);
+  w.M = c.take<float>((size_t)p.n * d.k_in);  // replicated first (peer exchange)
   w.pacc = c.take<float>((size_t)p.max_chunks() * d.k_in);
   w.pidx = c.take<int32_t>(trop(d) ? (size_t)p.max_chunks() * d.k_in : 0);
   w.G = c.take<float>((size_t)p.n_local * d.k_out);
-  w.M = c.take<float>((size_t)p.n * d.k_in);
   w.gemm = c.take<float>(gemm_tn_ws_floats(d.k_in, d.k_out));
   w.WT = c.take<float>((size_t)d.k_in * d.k_out);
   w.saved_inf = c.take<char>(sv);

@@ -1,5 +1,6 @@
 // common.cuh — shared device helpers and internal structures of libagnn.so.
 #pragma once
+#include <vector>
 #include <cuda_runtime.h>
 #include <stdint.h>
 #include <string>
@@ -125,6 +126,8 @@ struct RowLayout {
 };
 
 // ---- plan / model (host structures) ------------------------------------------
+constexpr int kMaxPeers = 8;
+
 struct Plan {
   int64_t n = 0, row_begin = 0, row_end = 0, n_local = 0, nnz = 0;
   const int64_t* row_ptr = nullptr;   // caller-owned, local rows
@@ -160,7 +163,23 @@ struct Plan {
   // distribution
   int rank = 0, world = 1;
   int64_t* bounds = nullptr;          // host [world+1]
-  void* nccl = nullptr;               // ncclComm_t
+  void* nccl = nullptr;               // ncclComm_t (NCCL exchange)
+  // peer-memory exchange (world > 1 without an NCCL id): every rank's replicated
+  // buffers and control block are mapped into every other rank (CUDA IPC over
+  // NVLink / NVSwitch); see comm.cu
+  bool peer = false;
+  bool peer_ready = false;
+  void* ctl = nullptr;                // plan-owned: barrier flags + reduce slots
+  void* peer_ctl[kMaxPeers] = {};     // every rank's control block ([rank] = ctl)
+  struct Reg {                        // registered (symmetric) buffer
+    char* local;
+    size_t bytes;
+    char* peer[kMaxPeers];
+  };
+  std::vector<Reg>* regs = nullptr;
+  std::vector<void*>* opened = nullptr;  // IPC mappings to close at destroy
+  mutable int64_t epoch = 0;          // barrier generation (host, in stream order)
+  mutable int64_t red_calls = 0;      // all-reduce slot-set parity
 };
 
 struct Model {

@@ -589,13 +589,15 @@ WsGat carve_ws(const Plan& p, const GatShape& g, void* base, size_t* total) {
   Carver c(base);
   WsGat w;
   const int NE = (g.k_out + 2 * g.heads + 3) / 4 * 4;
+  // replicated (n-row) arrays first: their offsets are the same on every rank, which
+  // the peer-memory exchange relies on (agnn_plan_register maps whole buffers)
+  w.G = c.take<float>((size_t)p.n * g.k_out);
+  w.rec = c.take<float4>((size_t)p.n * g.heads);
   w.Wext = c.take<float>((size_t)g.k_in * NE);
   w.pacc = c.take<float>((size_t)p.max_chunks() * 3 * g.k_out);
   w.pm = c.take<float>((size_t)p.max_chunks() * g.heads);
   w.pl = c.take<float>((size_t)p.max_chunks() * g.heads);
   w.ds_dir = c.take<float>(p.csc_ptr ? (size_t)p.n_local * g.heads : 0);
-  w.G = c.take<float>((size_t)p.n * g.k_out);
-  w.rec = c.take<float4>((size_t)p.n * g.heads);
   w.dP = c.take<float>((size_t)p.n_local * g.k_out);
   w.da_part = c.take<float>((size_t)da_rows() * 2 * g.k_out);
   w.gemm = c.take<float>(gemm_tn_ws_floats(g.k_in, g.k_out));

@@ -75,7 +75,14 @@ agnn_status gat_debug_alpha(const Plan& p, const GatShape& g, const void* saved,
 // `width` floats) are broadcast from rank r; in place.
 agnn_status allgather_rows(const Plan& p, float* full, int64_t width, cudaStream_t s);
 agnn_status allreduce_sum(const Plan& p, float* buf, int64_t count, cudaStream_t s);
-agnn_status comm_init(Plan& p, const void* unique_id);
+agnn_status comm_init(Plan& p, const void* unique_id);  // unique_id NULL: peer-memory exchange
+// peer-memory exchange helpers (comm.cu)
+agnn_status peer_barrier(const Plan& p, cudaStream_t s);
+// map every rank's IPC handle (rank order, 64 B each) + byte offset; own rank -> local
+agnn_status peer_open(Plan& p, const void* handles, const int64_t* offsets, void* local,
+                      char* out[kMaxPeers]);
+// the addresses of `local` (inside a registered buffer) in every rank's copy
+agnn_status peer_targets(const Plan& p, const void* local, void* out[kMaxPeers]);
 void comm_destroy(Plan& p);
 
 }  // namespace agnn

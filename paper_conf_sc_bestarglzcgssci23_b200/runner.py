@@ -51,11 +51,15 @@ def row_block(row_ptr_host, world: int, rank: int, c_v: int = 4):
 
 
 class Stack:
-    """Buffers + plan + model for one workload on this rank."""
+    """Buffers + plan + model for one workload on this rank.
+
+    world > 1: `nccl_uid` selects the NCCL exchange; without it the ranks exchange
+    through peer memory, and `allgather_obj` (list <- object, every rank; e.g.
+    torch.distributed.all_gather_object) moves the IPC handles at setup."""
 
     def __init__(self, w: gen.Workload, device="cuda", rank=0, world=1, nccl_uid=None,
                  c_v: int = 4, graph: Graph | None = None, inputs_on_device=True,
-                 symmetric: bool = True):
+                 symmetric: bool = True, allgather_obj=None):
         self.w, self.device, self.rank, self.world = w, torch.device(device), rank, world
         self.stream = torch.cuda.current_stream(self.device)
         g = graph or build_graph(w, self.device)
@@ -77,6 +81,17 @@ class Stack:
                                  beta=w.beta, eps=w.eps, agg=w.agg) for _ in range(w.layers)]
         self.model = agnn.Model(self.plan, descs)
         self._alloc(inputs_on_device)
+        if world > 1 and nccl_uid is None:
+            if allgather_obj is None:
+                import torch.distributed as dist
+
+                def allgather_obj(obj):
+                    out = [None] * world
+                    dist.all_gather_object(out, obj)
+                    return out
+            self.plan.connect(allgather_obj(self.plan.ctl_export()))
+            for t in self.saved + [self.ws]:   # same order and sizes on every rank
+                self.plan.register(t, allgather_obj(agnn.ipc_export(t)))
 
     def _alloc(self, inputs_on_device):
         w, dev, nl = self.w, self.device, self.n_local

@@ -1,0 +1,95 @@
+"""World-size-2 runs of the peer-memory exchange on ONE GPU (two processes).
+
+The gpurun pool gives one B200, and NCCL refuses two ranks on one device, but
+CUDA IPC maps memory between two processes on the same device exactly as
+between two GPUs on an NVSwitch.  So the peer transport — IPC setup, the
+row-pushing all-gather, the flag barrier, the slot all-reduce — runs here for
+real, and every output must match the single-process run: H_out and dH bitwise
+for the row-local outputs (the chunk order does not depend on the number of
+ranks), dW / da within fp32 rounding of the different partial-sum grouping.
+"""
+from __future__ import annotations
+
+import os
+import socket
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = [pytest.mark.gpu,
+              pytest.mark.skipif(not torch.cuda.is_available(), reason="needs a CUDA device")]
+
+from paper_conf_sc_bestarglzcgssci23_b200 import gen  # noqa: E402
+
+CASES = {
+    "gat-k64h2": gen.Workload("mr-gat", "gat", "kron", 13, 1 << 13, 8 << 13, 64, 2, 1, act="elu"),
+    "gat-k128h4": gen.Workload("mr-gat128", "gat", "kron", 14, 1 << 14, 8 << 14, 128, 4, 1,
+                               act="none"),
+    "agnn-k128-L2": gen.Workload("mr-agnn", "agnn", "rmat", 13, 1 << 13, 8 << 13, 128, 1, 2,
+                                 act="elu"),
+    "va-k64": gen.Workload("mr-va", "va", "kron", 13, 1 << 13, 8 << 13, 64, 1, 1, act="none"),
+    "cgnn-max": gen.Workload("mr-cg", "cgnn", "kron", 13, 1 << 13, 8 << 13, 64, 1, 1, act="elu",
+                             agg="max"),
+}
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    return port
+
+
+def _outputs(st):
+    L = st.w.layers
+    out = {"H": st.H[L].cpu().numpy(), "dH": st.dH[0].cpu().numpy(),
+           "dW": [x.cpu().numpy() for x in st.dW]}
+    out["da"] = [x.cpu().numpy() for x in st.da if x is not None]
+    return out
+
+
+def _worker(rank, world, port, name):
+    import torch.distributed as dist
+    from paper_conf_sc_bestarglzcgssci23_b200 import runner
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    torch.cuda.set_device(0)
+    w = CASES[name]
+    st = runner.Stack(w, "cuda", rank=rank, world=world, nccl_uid=None)
+    for _ in range(2):  # two steps: the second reuses every replica buffer
+        st.step()
+    torch.cuda.synchronize()
+    mine = _outputs(st)
+    mine["rows"] = (st.row_begin, st.row_end)
+    allout = [None] * world
+    dist.all_gather_object(allout, mine)
+    if rank == 0:
+        ref = runner.Stack(w, "cuda")
+        for _ in range(2):
+            ref.step()
+        torch.cuda.synchronize()
+        r = _outputs(ref)
+        for o in allout:
+            b0, b1 = o["rows"]
+            assert b1 > b0
+            np.testing.assert_array_equal(o["H"], r["H"][b0:b1])
+            np.testing.assert_array_equal(o["dH"], r["dH"][b0:b1])
+            for x, y in zip(o["dW"], r["dW"]):
+                assert np.linalg.norm(x - y) <= 1e-6 * np.linalg.norm(y)
+            for x, y in zip(o["da"], r["da"]):
+                assert np.linalg.norm(x - y) <= 1e-6 * np.linalg.norm(y)
+        # every rank ends with the same (all-reduced) weight gradient, bit for bit
+        for o in allout[1:]:
+            for x, y in zip(o["dW"], allout[0]["dW"]):
+                np.testing.assert_array_equal(x, y)
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("name", list(CASES))
+def test_peer_exchange_two_ranks_one_gpu(name):
+    import torch.multiprocessing as mp
+    mp.spawn(_worker, args=(2, _free_port(), name), nprocs=2, join=True)
