@@ -42,6 +42,9 @@ def parse():
     p.add_argument("--config", default="C5")
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
     p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--comm", default="peer", choices=["peer", "nccl"],
+                   help="multi-GPU exchange: peer memory (fused GEMM -> all-gather stores over "
+                        "NVLink, flag barriers) or NCCL collectives")
     p.add_argument("--graph", default="auto", choices=["auto", "on", "off"],
                    help="time the step as one CUDA-graph replay (auto: small, launch-bound "
                         "workloads on one GPU)")
@@ -256,7 +259,7 @@ def run_ours(args):
     w = workload(args)
     agnn.lib()
     uid = None
-    if world > 1:
+    if world > 1 and args.comm == "nccl":
         obj = [agnn.nccl_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
         uid = obj[0]
@@ -485,6 +488,7 @@ def run_ours(args):
                 "config": {"workload": args.config, "model": w.model, "graph": w.graph,
                            "n": n, "edges": m, "k": w.k, "heads": w.heads, "layers": w.layers,
                            "parallelism": f"1d-rowblock{world}",
+                           "comm": (args.comm if world > 1 else None),
                            "l2_flush": "inputs > L2 (126 MB)" if not small else
                                        "256 MB buffer written between timed steps (per-step "
                                        "event pairs)",

@@ -455,13 +455,13 @@ WsAv carve_ws(const Plan& p, const agnn_layer_desc& d, void* base, size_t* total
   // replicated (n-row) arrays first (same offsets on every rank; peer exchange)
   w.M = c.take<float>((size_t)p.n * d.k_in);
   w.rec = c.take<float4>(d.kind == AGNN_AGNN ? (size_t)p.n : 0);
+  w.saved_inf = c.take<char>(sv);  // its replicated prefix (H_full, nu) too
   w.pacc = c.take<float>((size_t)p.max_chunks() * 2 * d.k_in);
   w.pl = c.take<float>((size_t)p.max_chunks());
   w.dhp = c.take<float>(p.csc_ptr ? (size_t)p.n_local * d.k_in : 0);
   w.G = c.take<float>((size_t)p.n_local * d.k_out);
   w.gemm = c.take<float>(gemm_tn_ws_floats(d.k_in, d.k_out));
   w.WT = c.take<float>((size_t)d.k_in * d.k_out);
-  w.saved_inf = c.take<char>(sv);
   if (total) *total = c.off + 256;
   return w;
 }

@@ -297,12 +297,12 @@ WsCg carve_ws(const Plan& p, const agnn_layer_desc& d, void* base, size_t* total
   size_t sv = 0;
   carve_saved(p, d, nullptr, &sv);
   w.M = c.take<float>((size_t)p.n * d.k_in);  // replicated first (peer exchange)
+  w.saved_inf = c.take<char>(sv);             // its replicated prefix too
   w.pacc = c.take<float>((size_t)p.max_chunks() * d.k_in);
   w.pidx = c.take<int32_t>(trop(d) ? (size_t)p.max_chunks() * d.k_in : 0);
   w.G = c.take<float>((size_t)p.n_local * d.k_out);
   w.gemm = c.take<float>(gemm_tn_ws_floats(d.k_in, d.k_out));
   w.WT = c.take<float>((size_t)d.k_in * d.k_out);
-  w.saved_inf = c.take<char>(sv);
   if (total) *total = c.off + 256;
   return w;
 }

@@ -593,6 +593,7 @@ WsGat carve_ws(const Plan& p, const GatShape& g, void* base, size_t* total) {
   // the peer-memory exchange relies on (agnn_plan_register maps whole buffers)
   w.G = c.take<float>((size_t)p.n * g.k_out);
   w.rec = c.take<float4>((size_t)p.n * g.heads);
+  w.saved_inf = c.take<char>(saved_size(p, g));  // its replicated prefix (P, st) too
   w.Wext = c.take<float>((size_t)g.k_in * NE);
   w.pacc = c.take<float>((size_t)p.max_chunks() * 3 * g.k_out);
   w.pm = c.take<float>((size_t)p.max_chunks() * g.heads);
@@ -601,7 +602,6 @@ WsGat carve_ws(const Plan& p, const GatShape& g, void* base, size_t* total) {
   w.dP = c.take<float>((size_t)p.n_local * g.k_out);
   w.da_part = c.take<float>((size_t)da_rows() * 2 * g.k_out);
   w.gemm = c.take<float>(gemm_tn_ws_floats(g.k_in, g.k_out));
-  w.saved_inf = c.take<char>(saved_size(p, g));
   if (total) *total = c.off + 256;
   return w;
 }
@@ -648,13 +648,44 @@ agnn_status gat_forward(const Plan& p, const GatShape& g, const float* W, const 
   gat_wext_kernel<<<64, 256, 0, s>>>(W, a, g.k_in, g.k_out, g.heads, NE, w.Wext);
   AGNN_LAUNCH_CHECK("gat_wext_kernel");
   // P (and s, t) for the local rows, written at their global offsets
-  agnn_status st = gemm_rows(H_in, p.n_local, g.k_in, w.Wext, true, NE,
-                             sv.P + p.row_begin * g.k_out, g.k_out,
-                             sv.st + p.row_begin * 2 * g.heads, s, nullptr, 0, NEs);
-  if (st != AGNN_OK) return st;
-  if (p.world > 1) {
-    if ((st = allgather_rows(p, sv.P, g.k_out, s)) != AGNN_OK) return st;
-    if ((st = allgather_rows(p, sv.st, 2 * g.heads, s)) != AGNN_OK) return st;
+  float* Ploc = sv.P + p.row_begin * g.k_out;
+  float* stloc = sv.st + p.row_begin * 2 * g.heads;
+  agnn_status st;
+  if (p.world > 1 && p.peer) {
+    // fused GEMM -> all-gather over peer memory: the GEMM epilogue stores every
+    // output tile into the local P | st and into every peer's replica (NVLink
+    // stores overlap the next tiles' MMAs); entry / exit barriers order it with
+    // the peers' reads of the previous contents and of these rows
+    void* tp[kMaxPeers];
+    void* ts[kMaxPeers];
+    if ((st = peer_targets(p, Ploc, tp)) != AGNN_OK) return st;
+    if ((st = peer_targets(p, stloc, ts)) != AGNN_OK) return st;
+    PeerOut po;
+    for (int r = 0; r < p.world; ++r) {
+      if (r == p.rank) continue;
+      po.C0[po.n] = static_cast<float*>(tp[r]);
+      po.C1[po.n] = static_cast<float*>(ts[r]);
+      ++po.n;
+    }
+    if ((st = peer_barrier(p, s)) != AGNN_OK) return st;
+    bool fused = false;
+    if ((st = gemm_rows(H_in, p.n_local, g.k_in, w.Wext, true, NE, Ploc, g.k_out, stloc, s,
+                        nullptr, 0, NEs, &po, &fused)) != AGNN_OK)
+      return st;
+    if (fused) {
+      if ((st = peer_barrier(p, s)) != AGNN_OK) return st;
+    } else {
+      if ((st = allgather_rows(p, sv.P, g.k_out, s)) != AGNN_OK) return st;
+      if ((st = allgather_rows(p, sv.st, 2 * g.heads, s)) != AGNN_OK) return st;
+    }
+  } else {
+    if ((st = gemm_rows(H_in, p.n_local, g.k_in, w.Wext, true, NE, Ploc, g.k_out, stloc, s,
+                        nullptr, 0, NEs)) != AGNN_OK)
+      return st;
+    if (p.world > 1) {
+      if ((st = allgather_rows(p, sv.P, g.k_out, s)) != AGNN_OK) return st;
+      if ((st = allgather_rows(p, sv.st, 2 * g.heads, s)) != AGNN_OK) return st;
+    }
   }
   Items it = items_of(p);
   FwdOut o{saved ? sv.Z : nullptr, H_out, saved ? sv.m : nullptr, saved ? sv.l : nullptr,

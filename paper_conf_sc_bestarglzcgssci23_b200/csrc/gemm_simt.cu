@@ -201,16 +201,24 @@ __global__ void sum_splits_kernel(const float* __restrict__ part, int splits, in
 }  // namespace
 
 agnn_status gemm_tc(const float* A, int64_t M, int K, const float* B, int n_real, float* C0,
-                    int n_split, float* C1, int n_store, float* Cact, int act, cudaStream_t s);
+                    int n_split, float* C1, int n_store, float* Cact, int act, cudaStream_t s,
+                    const PeerOut* peers);
 
 agnn_status gemm_rows(const float* A, int64_t M, int K, const float* B, bool b_trans, int N,
                       float* C0, int n_split, float* C1, cudaStream_t s, float* Cact, int act,
-                      int n_store) {
-  if (M <= 0) return AGNN_OK;
+                      int n_store, const PeerOut* peers, bool* peers_done) {
+  if (peers_done) *peers_done = false;
+  if (M <= 0) {
+    if (peers_done) *peers_done = true;
+    return AGNN_OK;
+  }
   if (b_trans) {  // tcgen05 3xTF32 path when the shape has an instantiation
     const int ns = (n_store <= 0 || n_store > N) ? N : n_store;
-    const agnn_status st = gemm_tc(A, M, K, B, ns, C0, n_split, C1, ns, Cact, act, s);
-    if (st != AGNN_EUNSUPPORTED) return st;
+    const agnn_status st = gemm_tc(A, M, K, B, ns, C0, n_split, C1, ns, Cact, act, s, peers);
+    if (st != AGNN_EUNSUPPORTED) {
+      if (peers_done) *peers_done = st == AGNN_OK;
+      return st;
+    }
   }
   if (K % 4 || N % 4) return fail(AGNN_EINVAL, "gemm_rows: K and N must be multiples of 4");
   dim3 grid((unsigned)((M + BM - 1) / BM), (N + BN - 1) / BN);

@@ -163,33 +163,41 @@ struct TcOut {
   float* C1;    // columns [n_split, n_store), row stride n_store - n_split
   float* Cact;  // sigma(C) for columns < n_split (nullable)
   int n_split, n_store, act;
+  int npeer;                       // peer replicas also written (peer-memory exchange)
+  float* pC0[kMaxPeers - 1];
+  float* pC1[kMaxPeers - 1];
 };
 
 // 16 consecutive columns c0.. of output row `row` (C0 | C1 split, optional sigma copy)
 __device__ __forceinline__ void store_row16(const TcOut& out, int64_t row, int c0,
                                             const float (&v)[16]) {
+  for (int pi = -1; pi < out.npeer; ++pi) {  // own copy, then the peers' replicas
+    float* C0 = pi < 0 ? out.C0 : out.pC0[pi];
+    float* C1 = pi < 0 ? out.C1 : out.pC1[pi];
+    float* Ca = pi < 0 ? out.Cact : nullptr;
 #pragma unroll
-  for (int j = 0; j < 16; j += 4) {
-    const int c = c0 + j;
-    const float4 q = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
-    if (c + 3 < out.n_split && (out.n_split & 3) == 0) {
-      if (out.C0) st4(out.C0 + row * out.n_split + c, q);
-      if (out.Cact) st4(out.Cact + row * out.n_split + c, act_fwd4(out.act, q));
-    } else if (c < out.n_split) {
+    for (int j = 0; j < 16; j += 4) {
+      const int c = c0 + j;
+      const float4 q = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
+      if (c + 3 < out.n_split && (out.n_split & 3) == 0) {
+        if (C0) st4(C0 + row * out.n_split + c, q);
+        if (Ca) st4(Ca + row * out.n_split + c, act_fwd4(out.act, q));
+      } else if (c < out.n_split) {
 #pragma unroll
-      for (int x = 0; x < 4; ++x) {
-        if (c + x < out.n_split) {
-          if (out.C0) out.C0[row * out.n_split + c + x] = v[j + x];
-          if (out.Cact) out.Cact[row * out.n_split + c + x] = act_fwd(out.act, v[j + x]);
-        } else if (c + x < out.n_store) {
-          out.C1[row * (out.n_store - out.n_split) + (c + x - out.n_split)] = v[j + x];
+        for (int x = 0; x < 4; ++x) {
+          if (c + x < out.n_split) {
+            if (C0) C0[row * out.n_split + c + x] = v[j + x];
+            if (Ca) Ca[row * out.n_split + c + x] = act_fwd(out.act, v[j + x]);
+          } else if (c + x < out.n_store) {
+            C1[row * (out.n_store - out.n_split) + (c + x - out.n_split)] = v[j + x];
+          }
         }
-      }
-    } else if (c < out.n_store) {
-      const int w1 = out.n_store - out.n_split;
+      } else if (c < out.n_store) {
+        const int w1 = out.n_store - out.n_split;
 #pragma unroll
-      for (int x = 0; x < 4; ++x)
-        if (c + x < out.n_store) out.C1[row * w1 + (c + x - out.n_split)] = v[j + x];
+        for (int x = 0; x < 4; ++x)
+          if (c + x < out.n_store) C1[row * w1 + (c + x - out.n_split)] = v[j + x];
+      }
     }
   }
 }
@@ -213,6 +221,8 @@ __device__ __forceinline__ void store_block32(const TcOut& out, int64_t row0, in
     if (row < M) {
       if (out.C0) st4(out.C0 + row * out.n_split + c0 + cc, q);
       if (out.Cact) st4(out.Cact + row * out.n_split + c0 + cc, act_fwd4(out.act, q));
+      for (int pi = 0; pi < out.npeer; ++pi)  // peers' replicas (NVLink stores)
+        st4(out.pC0[pi] + row * out.n_split + c0 + cc, q);
     }
   }
   __syncwarp();
@@ -783,11 +793,20 @@ agnn_status gemm_tn_tc(const float* A, int64_t M, int K1, const float* B, int N,
 // C = A * B^T with B [n_real x K] K-major; columns padded to N_pad (multiple of 16).
 // Returns AGNN_EUNSUPPORTED when the shape has no tcgen05 instantiation.
 agnn_status gemm_tc(const float* A, int64_t M, int K, const float* B, int n_real, float* C0,
-                    int n_split, float* C1, int n_store, float* Cact, int act, cudaStream_t s) {
+                    int n_split, float* C1, int n_store, float* Cact, int act, cudaStream_t s,
+                    const PeerOut* peers) {
   if (tc_disabled()) return AGNN_EUNSUPPORTED;
   if (M <= 0) return AGNN_OK;
   if ((reinterpret_cast<uintptr_t>(A) & 15) || (K % 32)) return AGNN_EUNSUPPORTED;
-  TcOut o{C0, C1, Cact, n_split, n_store, act};
+  TcOut o{C0, C1, Cact, n_split, n_store, act, 0, {}, {}};
+  if (peers) {
+    if (peers->n > kMaxPeers - 1 || (!C0 && peers->n > 0)) return AGNN_EUNSUPPORTED;
+    o.npeer = peers->n;
+    for (int i = 0; i < peers->n; ++i) {
+      o.pC0[i] = peers->C0[i];
+      o.pC1[i] = peers->C1[i];
+    }
+  }
   const int npad = (n_real + 15) / 16 * 16;
   // resident B: S = the 16 KB stages that fit next to B (2 x K x N x 4 bytes), <= 8
   if (K == 128 && npad == 128) return launch_tc<128, 128, 4, false>(A, M, B, n_real, o, s);

@@ -42,9 +42,18 @@ inline int grid_of(F* func) { return persistent_blocks(reinterpret_cast<const vo
 // Columns [0, n_split) go to C0 (ld = n_split), [n_split, N) to C1 (ld = N - n_split).
 // If Cact != NULL, sigma(C) (act) is also written to Cact (layout of C0); C0 may be NULL.
 // Columns >= n_store (padding) are computed but not stored (n_store <= 0: N).
+// peers (peer-memory exchange): the tcgen05 epilogue also stores C0 / C1 at the same
+// offsets into every peer's replica (the fused GEMM -> all-gather); *peers_done
+// tells whether it did (shapes on the SIMT fallback leave it to the caller).
+struct PeerOut {
+  int n = 0;
+  float* C0[kMaxPeers] = {};
+  float* C1[kMaxPeers] = {};
+};
 agnn_status gemm_rows(const float* A, int64_t M, int K, const float* B, bool b_trans, int N,
                       float* C0, int n_split, float* C1, cudaStream_t s, float* Cact = nullptr,
-                      int act = 0, int n_store = 0);
+                      int act = 0, int n_store = 0, const PeerOut* peers = nullptr,
+                      bool* peers_done = nullptr);
 // C[K1 x N] = A^T B over M rows (A [M x K1], B [M x N]); deterministic split-M with
 // partials in `ws` (gemm_tn_ws_floats) and an ordered reduction.  If accumulate,
 // C += result.

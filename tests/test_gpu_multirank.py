@@ -64,6 +64,11 @@ def _worker(rank, world, port, name):
     torch.cuda.synchronize()
     mine = _outputs(st)
     mine["rows"] = (st.row_begin, st.row_end)
+    # inference mode (nothing saved; the replicas live in the workspace)
+    st.H[w.layers].zero_()
+    st.forward(inference=True)
+    torch.cuda.synchronize()
+    mine["Hinf"] = st.H[w.layers].cpu().numpy()
     allout = [None] * world
     dist.all_gather_object(allout, mine)
     if rank == 0:
@@ -77,6 +82,7 @@ def _worker(rank, world, port, name):
             assert b1 > b0
             np.testing.assert_array_equal(o["H"], r["H"][b0:b1])
             np.testing.assert_array_equal(o["dH"], r["dH"][b0:b1])
+            np.testing.assert_array_equal(o["Hinf"], r["H"][b0:b1])
             for x, y in zip(o["dW"], r["dW"]):
                 assert np.linalg.norm(x - y) <= 1e-6 * np.linalg.norm(y)
             for x, y in zip(o["da"], r["da"]):
