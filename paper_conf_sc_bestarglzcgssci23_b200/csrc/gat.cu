@@ -444,7 +444,7 @@ __global__ void __launch_bounds__(kSparseThreads)
 gat_bwd_prologue_kernel(int64_t n_local, int64_t row_begin, const float* __restrict__ dHout,
                         const float* __restrict__ Z, const float* __restrict__ st,
                         const float* __restrict__ mrow, const float* __restrict__ lrow, int act,
-                        float* __restrict__ G, float4* __restrict__ rec) {
+                        float* __restrict__ G, float4* __restrict__ rec, PeerRows peers) {
   using L = RowLayout<K, NH>;
   const int lane = threadIdx.x & 31, g = lane / L::LANES, q = lane % L::LANES;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
@@ -473,10 +473,15 @@ gat_bwd_prologue_kernel(int64_t n_local, int64_t row_begin, const float* __restr
     for (int v = 0; v < L::VPL; ++v) {
       const int c = L::col(v, q), h = c / L::D;
       st4(G + grow * K + c, gv[v]);
+      for (int pi = 0; pi < peers.n; ++pi)  // peers' replicas (fused all-gather)
+        st4(peers.a[pi] + grow * K + c, gv[v]);
       if ((c % L::D) == 0) {
         const float lv = lrow[row * NH + h];
-        rec[grow * NH + h] = make_float4(st[grow * 2 * NH + h], mrow[row * NH + h],
-                                         lv > 0.f ? 1.f / lv : 0.f, dl[v]);
+        const float4 r4 = make_float4(st[grow * 2 * NH + h], mrow[row * NH + h],
+                                      lv > 0.f ? 1.f / lv : 0.f, dl[v]);
+        rec[grow * NH + h] = r4;
+        for (int pi = 0; pi < peers.n; ++pi)
+          reinterpret_cast<float4*>(peers.b[pi])[grow * NH + h] = r4;
       }
     }
   }
@@ -719,15 +724,34 @@ agnn_status gat_backward(const Plan& p, const GatShape& g, const float* W, const
   const int K_ = g.k_out, NH_ = g.heads;
   Items it = items_of(p);
   agnn_status st;
+  PeerRows pr;  // peer mode: G and rec rows also go straight to every peer's replica
+  if (p.world > 1 && p.peer) {
+    void* tg[kMaxPeers];
+    void* tr[kMaxPeers];
+    if ((st = peer_targets(p, w.G, tg)) != AGNN_OK) return st;
+    if ((st = peer_targets(p, w.rec, tr)) != AGNN_OK) return st;
+    for (int r = 0; r < p.world; ++r) {
+      if (r == p.rank) continue;
+      pr.a[pr.n] = static_cast<float*>(tg[r]);
+      pr.b[pr.n] = static_cast<float*>(tr[r]);
+      ++pr.n;
+    }
+    // entry barrier: every peer has finished reading its G / rec (previous layer)
+    if ((st = peer_barrier(p, s)) != AGNN_OK) return st;
+  }
   AGNN_GAT_DISPATCH(K_, NH_, (gat_bwd_prologue_kernel<K, NH>
                               <<<grid_of(gat_bwd_prologue_kernel<K, NH>), kSparseThreads, 0, s>>>(
                                   p.n_local, p.row_begin, dH_out, sv.Z, sv.st, sv.m, sv.l, g.act,
-                                  w.G, w.rec)));
+                                  w.G, w.rec, pr)));
   AGNN_LAUNCH_CHECK("gat_bwd_prologue_kernel");
   if (p.world > 1) {
-    if ((st = allgather_rows(p, w.G, g.k_out, s)) != AGNN_OK) return st;
-    if ((st = allgather_rows(p, reinterpret_cast<float*>(w.rec), 4 * g.heads, s)) != AGNN_OK)
-      return st;
+    if (p.peer) {  // the prologue stored G | rec into the peers' replicas: exit barrier
+      if ((st = peer_barrier(p, s)) != AGNN_OK) return st;
+    } else {
+      if ((st = allgather_rows(p, w.G, g.k_out, s)) != AGNN_OK) return st;
+      if ((st = allgather_rows(p, reinterpret_cast<float*>(w.rec), 4 * g.heads, s)) != AGNN_OK)
+        return st;
+    }
   }
   BwdArgs A{sv.P, sv.st, w.G, w.rec, a, g.slope, w.dP, w.pacc, w.pm, w.pl, w.da_part,
             nullptr, nullptr, w.ds_dir};

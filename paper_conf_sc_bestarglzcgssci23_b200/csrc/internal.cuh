@@ -45,6 +45,12 @@ inline int grid_of(F* func) { return persistent_blocks(reinterpret_cast<const vo
 // peers (peer-memory exchange): the tcgen05 epilogue also stores C0 / C1 at the same
 // offsets into every peer's replica (the fused GEMM -> all-gather); *peers_done
 // tells whether it did (shapes on the SIMT fallback leave it to the caller).
+// replicas of up to two row arrays in the other ranks (kernel argument)
+struct PeerRows {
+  int n = 0;
+  float* a[kMaxPeers - 1] = {};
+  float* b[kMaxPeers - 1] = {};
+};
 struct PeerOut {
   int n = 0;
   float* C0[kMaxPeers] = {};

@@ -1,4 +1,4 @@
-"""World-size-2 runs of the peer-memory exchange on ONE GPU (two processes).
+"""World-size-2 and -3 runs of the peer-memory exchange on ONE GPU (one process per rank).
 
 The gpurun pool gives one B200, and NCCL refuses two ranks on one device, but
 CUDA IPC maps memory between two processes on the same device exactly as
@@ -99,3 +99,10 @@ def _worker(rank, world, port, name):
 def test_peer_exchange_two_ranks_one_gpu(name):
     import torch.multiprocessing as mp
     mp.spawn(_worker, args=(2, _free_port(), name), nprocs=2, join=True)
+
+
+@pytest.mark.parametrize("name", ["gat-k128h4", "agnn-k128-L2"])
+def test_peer_exchange_three_ranks_one_gpu(name):
+    """Three ranks: uneven row blocks and two peers per rank in every exchange."""
+    import torch.multiprocessing as mp
+    mp.spawn(_worker, args=(3, _free_port(), name), nprocs=3, join=True)
