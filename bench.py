@@ -251,11 +251,20 @@ def run_ours(args):
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if not torch.cuda.is_available():
         raise RuntimeError("bench.py needs CUDA GPUs (no CPU fallback)")
+    # AGNN_BENCH_SAME_GPU=1 (test only): every rank on cuda:0 with a gloo process group,
+    # so the multi-rank bench path runs on a one-GPU box (peer exchange between processes
+    # on one device; numbers from such a run are not scaling measurements)
+    same_gpu = os.environ.get("AGNN_BENCH_SAME_GPU") == "1"
+    if same_gpu:
+        local = 0
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
-        dist.init_process_group("nccl", device_id=dev)
+        if same_gpu:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=dev)
     w = workload(args)
     agnn.lib()
     uid = None
@@ -359,7 +368,7 @@ def run_ours(args):
         keep_busy(graph.replay, 0.25)
         ck = clocks.stop()
     if world > 1:
-        t = torch.tensor([ms], device=dev)
+        t = torch.tensor([ms], device="cpu" if same_gpu else dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms = float(t.item())
     T = ms / 1e3 / args.steps
@@ -455,7 +464,7 @@ def run_ours(args):
         st.H[0], st.dH[L] = Hb[0], Rb[0]
         ms2 = e2.elapsed_time(e3)
         if world > 1:
-            t = torch.tensor([ms2], device=dev)
+            t = torch.tensor([ms2], device="cpu" if same_gpu else dev)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             ms2 = float(t.item())
         T2 = ms2 / 1e3 / args.steps
