@@ -487,7 +487,7 @@ agnn_status av_workspace_bytes(const Plan& p, const agnn_layer_desc& d, size_t* 
     else return fail(AGNN_EUNSUPPORTED, "AGNN/VA: k_in must be 16/32/64/128/256"); \
   } while (0)
 
-// AGNN_AV_K128=0 selects the generic kernels at k = 128 (A/B comparisons)
+// AGNN_AV_K128=0 selects the generic kernels at k = 128 / 256 (A/B comparisons)
 bool k128_disabled() {
   static int v = -1;
   if (v < 0) {
@@ -524,8 +524,8 @@ agnn_status av_forward(const Plan& p, const agnn_layer_desc& d, const float* W, 
   }
   Items it = items_of(p);
   AvFwd A{Hf, sv.nu, d.beta, fabsf(d.beta), sv.X, sv.l, w.pacc, w.pl};
-  if (K_ == 128 && !k128_disabled()) {
-    if ((st = av_fwd_k128(it, ag, A, s)) != AGNN_OK) return st;
+  if ((K_ == 128 || K_ == 256) && !k128_disabled()) {
+    if ((st = av_fwd_batched(it, K_, ag, A, s)) != AGNN_OK) return st;
   } else if (it.n_chunks + it.n_light > 0) {
     if (ag) AGNN_AV_DISPATCH(K_, (av_fwd_kernel<K, AG, av_fwd_unroll<K>()>
                                   <<<grid_of(av_fwd_kernel<K, AG, av_fwd_unroll<K>()>),
@@ -626,8 +626,8 @@ agnn_status av_backward(const Plan& p, const agnn_layer_desc& d, const float* W,
 #undef AV_PASS
     return AGNN_OK;
   }
-  if (K_ == 128 && !k128_disabled()) {
-    if ((st = av_bwd_k128(it, ag, A, s)) != AGNN_OK) return st;
+  if ((K_ == 128 || K_ == 256) && !k128_disabled()) {
+    if ((st = av_bwd_batched(it, K_, ag, A, s)) != AGNN_OK) return st;
   } else if (it.n_chunks + it.n_light > 0) {
     if (ag) AGNN_AV_DISPATCH(K_, (av_bwd_kernel<K, AG, av_bwd_unroll<K>()>
                                   <<<grid_of(av_bwd_kernel<K, AG, av_bwd_unroll<K>()>),

@@ -1,5 +1,5 @@
 // av_args.cuh — argument blocks shared by the AGNN / VA sparse kernels
-// (agnn_va.cu generic widths, av_k128.cu for k = 128)
+// (agnn_va.cu generic widths, av_batched.cu for k = 128 / 256)
 #pragma once
 #include "internal.cuh"
 
@@ -27,8 +27,9 @@ struct AvBwd {
 
 enum { AV_VA = 0, AV_AG = 1 };
 
-// k = 128 lane-parallel kernels (av_k128.cu); symmetric patterns (ROLE 0) only
-agnn_status av_fwd_k128(const Items& it, bool agnn, const AvFwd& A, cudaStream_t s);
-agnn_status av_bwd_k128(const Items& it, bool agnn, const AvBwd& A, cudaStream_t s);
+// k = 128 / 256 batched lane-parallel kernels (av_batched.cu); symmetric patterns
+// (ROLE 0) only; AGNN_EUNSUPPORTED for other widths
+agnn_status av_fwd_batched(const Items& it, int k, bool agnn, const AvFwd& A, cudaStream_t s);
+agnn_status av_bwd_batched(const Items& it, int k, bool agnn, const AvBwd& A, cudaStream_t s);
 
 }  // namespace agnn

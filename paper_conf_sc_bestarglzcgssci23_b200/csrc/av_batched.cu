@@ -1,6 +1,7 @@
-// av_k128.cu — AGNN / VA sparse kernels for k = 128 (the C3 shape), organised
-// like gat_k128.cu: feature-row work warp-parallel (lane q owns columns
-// 4q..4q+3), scalar per-edge work lane-parallel.
+// av_batched.cu — AGNN / VA sparse kernels for k = 128 and 256 (the C3 and C4
+// shapes), organised like gat_k128.cu: feature-row work warp-parallel (lane q
+// owns columns 4q..4q+3 of every 128-column block), scalar per-edge work
+// lane-parallel.
 //
 // Arithmetic is exactly that of agnn_va.cu (PAPER.md:173/:175 scores, Eq. 7;
 // PAPER.md:250-254 backward, VA Eq. 11-13; reading A8: softmax with the fixed
@@ -21,18 +22,25 @@ using wb::FULL;
 using wb::item_of;
 using wb::Transpose;
 
-constexpr int K = 128;
-
-template <int B>
+template <int B, int V>
 struct FwdBatch {
-  float4 Hj[B];
+  float4 Hj[B][V];
   float nuj;  // nu of the edge this lane owns after the reduction (AGNN)
 };
 
+template <int V>
+__device__ __forceinline__ float dotv(const float4 (&a)[V], const float4 (&b)[V]) {
+  float d = dot4(a[0], b[0]);
+#pragma unroll
+  for (int v = 1; v < V; ++v) d += dot4(a[v], b[v]);
+  return d;
+}
+
 // X_i = sum_j w_ij H_j, w = exp(beta cos(H_i, H_j) - |beta|) (AGNN, l_i = sum w) or
 // w = H_i . H_j (VA)
-template <int MODEL, int B, int MINB>
-__global__ void __launch_bounds__(256, MINB) av_fwd_k128_kernel(Items it, AvFwd A) {
+template <int K, int MODEL, int B, int MINB>
+__global__ void __launch_bounds__(256, MINB) av_fwd_batched_kernel(Items it, AvFwd A) {
+  constexpr int V = K / 128;
   using TR = Transpose<B>;
   const int lane = threadIdx.x & 31, cq = lane * 4;
   const int my_b = TR::edge_of(lane);
@@ -45,25 +53,31 @@ __global__ void __launch_bounds__(256, MINB) av_fwd_k128_kernel(Items it, AvFwd 
     int64_t row, beg, end, slot;
     item_of(it, w, row, beg, end, slot);
     const int64_t grow = it.row_begin + row;
-    const float4 Hi = ldg4(A.H + grow * K + cq);
+    float4 Hi[V], acc[V];
+#pragma unroll
+    for (int v = 0; v < V; ++v) {
+      Hi[v] = ldg4(A.H + grow * K + v * 128 + cq);
+      acc[v] = f4(0.f);
+    }
     const float scale_i = (MODEL == AV_AG) ? beta / __ldg(A.nu + grow) : 1.f;
-    float4 acc = f4(0.f);
     float lp = 0.f;
-    auto load = [&](FwdBatch<B>& q, int cidx, int off, int cnt) {
+    auto load = [&](FwdBatch<B, V>& q, int cidx, int off, int cnt) {
 #pragma unroll
       for (int b = 0; b < B; ++b) {
         const uint32_t j = (uint32_t)__shfl_sync(FULL, cidx, off + b);
-        q.Hj[b] = b < cnt ? ldg4(Hl + (int64_t)j * K) : f4(0.f);
+#pragma unroll
+        for (int v = 0; v < V; ++v)
+          q.Hj[b][v] = b < cnt ? ldg4(Hl + (int64_t)j * K + v * 128) : f4(0.f);
       }
       if (MODEL == AV_AG) {
         const uint32_t jm = (uint32_t)__shfl_sync(FULL, cidx, off + my_b);
         q.nuj = my_b < cnt ? __ldg(A.nu + jm) : 1.f;
       }
     };
-    auto body = [&](const FwdBatch<B>& q, int cnt) {
+    auto body = [&](const FwdBatch<B, V>& q, int cnt) {
       float x[B];
 #pragma unroll
-      for (int b = 0; b < B; ++b) x[b] = dot4(Hi, q.Hj[b]);
+      for (int b = 0; b < B; ++b) x[b] = dotv<V>(Hi, q.Hj[b]);
       TR::template reduce<32>(x, lane);
       float wgt;
       if (MODEL == AV_AG) wgt = ex2((scale_i * x[0] / q.nuj - bound) * kLog2e);  // exp(c_ij - |beta|)
@@ -73,14 +87,15 @@ __global__ void __launch_bounds__(256, MINB) av_fwd_k128_kernel(Items it, AvFwd 
 #pragma unroll
       for (int b = 0; b < B; ++b) {
         const float wbv = __shfl_sync(FULL, wgt, TR::lane_of(b));
-        acc = fma4(wbv, q.Hj[b], acc);
+#pragma unroll
+        for (int v = 0; v < V; ++v) acc[v] = fma4(wbv, q.Hj[b][v], acc[v]);
       }
     };
     for (int64_t w0 = beg; w0 < end; w0 += 32) {
       const int wcnt = (int)(end - w0 < 32 ? end - w0 : 32);
       const int cidx = lane < wcnt ? __ldg(it.col + w0 + lane) : 0;
       if (wcnt == 32) {
-        FwdBatch<B> qa, qb;
+        FwdBatch<B, V> qa, qb;
         load(qa, cidx, 0, B);
 #pragma unroll
         for (int bb = 0; bb < 32 / B; bb += 2) {
@@ -91,7 +106,7 @@ __global__ void __launch_bounds__(256, MINB) av_fwd_k128_kernel(Items it, AvFwd 
         }
       } else {
         for (int off = 0; off < wcnt; off += B) {
-          FwdBatch<B> q;
+          FwdBatch<B, V> q;
           const int cnt = wcnt - off < B ? wcnt - off : B;
           load(q, cidx, off, cnt);
           body(q, cnt);
@@ -105,19 +120,21 @@ __global__ void __launch_bounds__(256, MINB) av_fwd_k128_kernel(Items it, AvFwd 
       for (int o = 1; o < 32; o <<= 1) l += __shfl_xor_sync(FULL, l, o);
     }
     if (slot >= 0) {
-      st4(A.pacc + slot * K + cq, acc);
+#pragma unroll
+      for (int v = 0; v < V; ++v) st4(A.pacc + slot * K + v * 128 + cq, acc[v]);
       if (MODEL == AV_AG && lane == 0) A.pl[slot] = l;
     } else {
       const float inv = (MODEL == AV_AG) ? (l > 0.f ? 1.f / l : 0.f) : 1.f;
-      st4(A.X + row * K + cq, mul4(inv, acc));
+#pragma unroll
+      for (int v = 0; v < V; ++v) st4(A.X + row * K + v * 128 + cq, mul4(inv, acc[v]));
       if (MODEL == AV_AG && lane == 0) A.l[row] = l;
     }
   }
 }
 
-template <int B>
+template <int B, int V>
 struct BwdBatchAV {
-  float4 Hi[B], Mi[B];
+  float4 Hi[B][V], Mi[B][V];
   float4 ri;  // record {nu, m, 1/l, delta} of the owned edge's vertex (AGNN)
 };
 
@@ -125,8 +142,9 @@ struct BwdBatchAV {
 //   VA   dH_j += (M_j.H_i + M_i.H_j) H_i + (H_i.H_j) M_i
 //   AGNN dH^_j += beta (a_ji (M_j.H_i - d_j) + a_ij (M_i.H_j - d_i)) H^_i,
 //        acc_j += a_ij M_i ;  dH_j = acc_j + (dH^_j - (dH^_j.H^_j) H^_j) / nu_j
-template <int MODEL, int B, int MINB>
-__global__ void __launch_bounds__(256, MINB) av_bwd_k128_kernel(Items it, AvBwd A) {
+template <int K, int MODEL, int B, int MINB>
+__global__ void __launch_bounds__(256, MINB) av_bwd_batched_kernel(Items it, AvBwd A) {
+  constexpr int V = K / 128;
   using TR = Transpose<B>;
   const int lane = threadIdx.x & 31, cq = lane * 4;
   const int my_b = TR::edge_of(lane);
@@ -139,20 +157,27 @@ __global__ void __launch_bounds__(256, MINB) av_bwd_k128_kernel(Items it, AvBwd 
     int64_t row, beg, end, slot;
     item_of(it, w, row, beg, end, slot);
     const int64_t grow = it.row_begin + row;
-    const float4 Hj = ldg4(A.H + grow * K + cq);
-    const float4 Mj = ldg4(A.M + grow * K + cq);
+    float4 Hj[V], Mj[V], dh[V], acc[V];
+#pragma unroll
+    for (int v = 0; v < V; ++v) {
+      Hj[v] = ldg4(A.H + grow * K + v * 128 + cq);
+      Mj[v] = ldg4(A.M + grow * K + v * 128 + cq);
+      dh[v] = acc[v] = f4(0.f);
+    }
     const float4 rj = (MODEL == AV_AG) ? __ldg(A.rec + grow) : f4(1.f);
     const float sj = (MODEL == AV_AG) ? beta / rj.x : 0.f;
-    float4 dh = f4(0.f), acc = f4(0.f);
-    auto load = [&](BwdBatchAV<B>& q, int cidx, int off, int cnt) {
+    auto load = [&](BwdBatchAV<B, V>& q, int cidx, int off, int cnt) {
 #pragma unroll
       for (int b = 0; b < B; ++b) {
         const uint32_t i = (uint32_t)__shfl_sync(FULL, cidx, off + b);
-        if (b < cnt) {
-          q.Hi[b] = ldg4(Hl + (int64_t)i * K);
-          q.Mi[b] = ldg4(Ml + (int64_t)i * K);
-        } else {
-          q.Hi[b] = q.Mi[b] = f4(0.f);
+#pragma unroll
+        for (int v = 0; v < V; ++v) {
+          if (b < cnt) {
+            q.Hi[b][v] = ldg4(Hl + (int64_t)i * K + v * 128);
+            q.Mi[b][v] = ldg4(Ml + (int64_t)i * K + v * 128);
+          } else {
+            q.Hi[b][v] = q.Mi[b][v] = f4(0.f);
+          }
         }
       }
       if (MODEL == AV_AG) {
@@ -160,13 +185,13 @@ __global__ void __launch_bounds__(256, MINB) av_bwd_k128_kernel(Items it, AvBwd 
         q.ri = my_b < cnt ? __ldg(A.rec + im) : f4(1.f);
       }
     };
-    auto body = [&](const BwdBatchAV<B>& q, int cnt) {
+    auto body = [&](const BwdBatchAV<B, V>& q, int cnt) {
       float xs[B], x1[B], x2[B];
 #pragma unroll
       for (int b = 0; b < B; ++b) {
-        xs[b] = dot4(Hj, q.Hi[b]);   // H_j . H_i
-        x1[b] = dot4(Mj, q.Hi[b]);   // M_j . H_i  (row role)
-        x2[b] = dot4(q.Mi[b], Hj);   // M_i . H_j  (column role)
+        xs[b] = dotv<V>(Hj, q.Hi[b]);   // H_j . H_i
+        x1[b] = dotv<V>(Mj, q.Hi[b]);   // M_j . H_i  (row role)
+        x2[b] = dotv<V>(q.Mi[b], Hj);   // M_i . H_j  (column role)
       }
       TR::template reduce<32>(xs, lane);
       TR::template reduce<32>(x1, lane);
@@ -189,16 +214,19 @@ __global__ void __launch_bounds__(256, MINB) av_bwd_k128_kernel(Items it, AvBwd 
       for (int b = 0; b < B; ++b) {
         const float chb = __shfl_sync(FULL, ch, TR::lane_of(b));
         const float cmb = __shfl_sync(FULL, cm, TR::lane_of(b));
-        dh = fma4(chb, q.Hi[b], dh);
-        if (MODEL == AV_VA) dh = fma4(cmb, q.Mi[b], dh);
-        else acc = fma4(cmb, q.Mi[b], acc);
+#pragma unroll
+        for (int v = 0; v < V; ++v) {
+          dh[v] = fma4(chb, q.Hi[b][v], dh[v]);
+          if (MODEL == AV_VA) dh[v] = fma4(cmb, q.Mi[b][v], dh[v]);
+          else acc[v] = fma4(cmb, q.Mi[b][v], acc[v]);
+        }
       }
     };
     for (int64_t w0 = beg; w0 < end; w0 += 32) {
       const int wcnt = (int)(end - w0 < 32 ? end - w0 : 32);
       const int cidx = lane < wcnt ? __ldg(it.col + w0 + lane) : 0;
       if (wcnt == 32) {
-        BwdBatchAV<B> qa, qb;
+        BwdBatchAV<B, V> qa, qb;
         load(qa, cidx, 0, B);
 #pragma unroll
         for (int bb = 0; bb < 32 / B; bb += 2) {
@@ -209,7 +237,7 @@ __global__ void __launch_bounds__(256, MINB) av_bwd_k128_kernel(Items it, AvBwd 
         }
       } else {
         for (int off = 0; off < wcnt; off += B) {
-          BwdBatchAV<B> q;
+          BwdBatchAV<B, V> q;
           const int cnt = wcnt - off < B ? wcnt - off : B;
           load(q, cidx, off, cnt);
           body(q, cnt);
@@ -217,24 +245,31 @@ __global__ void __launch_bounds__(256, MINB) av_bwd_k128_kernel(Items it, AvBwd 
       }
     }
     if (slot >= 0) {
-      st4(A.pacc + slot * 2 * K + cq, dh);
-      if (MODEL == AV_AG) st4(A.pacc + slot * 2 * K + K + cq, acc);
+#pragma unroll
+      for (int v = 0; v < V; ++v) {
+        st4(A.pacc + slot * 2 * K + v * 128 + cq, dh[v]);
+        if (MODEL == AV_AG) st4(A.pacc + slot * 2 * K + K + v * 128 + cq, acc[v]);
+      }
       continue;
     }
     if (MODEL == AV_VA) {
-      st4(A.dH + row * K + cq, dh);
+#pragma unroll
+      for (int v = 0; v < V; ++v) st4(A.dH + row * K + v * 128 + cq, dh[v]);
     } else {
       // dH_j = acc_j + (dH^_j - (dH^_j . H^_j) H^_j) / nu_j   (nu const on the eps branch)
-      float pr = dot4(dh, Hj);
+      float pr = dotv<V>(dh, Hj);
 #pragma unroll
       for (int o = 1; o < 32; o <<= 1) pr += __shfl_xor_sync(FULL, pr, o);
       const float nuj = rj.x;
       const bool on_eps = !(nuj > A.eps);
       const float inv = 1.f / nuj;
       const float proj = on_eps ? 0.f : pr * inv * inv;
-      float4 gv = fma4(-proj, Hj, dh);
-      gv = fma4(inv, gv, acc);
-      st4(A.dH + row * K + cq, gv);
+#pragma unroll
+      for (int v = 0; v < V; ++v) {
+        float4 gv = fma4(-proj, Hj[v], dh[v]);
+        gv = fma4(inv, gv, acc[v]);
+        st4(A.dH + row * K + v * 128 + cq, gv);
+      }
     }
   }
 }
@@ -246,32 +281,47 @@ int grid_for(F* f) {
 
 // batch sizes / residency measured at C3 (AGNN, R-MAT 2^20, k = 128): forward B = 8,
 // backward B = 4 (two batches of H_i, M_i in flight), 2 CTAs of 256 per SM; larger
-// batches or 3 CTAs per SM spill and lose 10-40 %
-template <int MODEL>
+// batches or 3 CTAs per SM spill and lose 10-40 %.  k = 256 halves the batches
+// (same registers per batch).
+template <int K, int MODEL>
 void launch_fwd(const Items& it, const AvFwd& A, cudaStream_t s) {
-  auto k = av_fwd_k128_kernel<MODEL, 8, 2>;
+  auto k = av_fwd_batched_kernel<K, MODEL, K == 128 ? 8 : 4, 2>;
   k<<<grid_for(k), 256, 0, s>>>(it, A);
 }
-template <int MODEL>
+template <int K, int MODEL>
 void launch_bwd(const Items& it, const AvBwd& A, cudaStream_t s) {
-  auto k = av_bwd_k128_kernel<MODEL, 4, 2>;
+  auto k = av_bwd_batched_kernel<K, MODEL, K == 128 ? 4 : 2, 2>;
   k<<<grid_for(k), 256, 0, s>>>(it, A);
 }
 
 }  // namespace
 
-agnn_status av_fwd_k128(const Items& it, bool agnn, const AvFwd& A, cudaStream_t s) {
+agnn_status av_fwd_batched(const Items& it, int k, bool agnn, const AvFwd& A, cudaStream_t s) {
   if (it.n_chunks + it.n_light == 0) return AGNN_OK;
-  if (agnn) launch_fwd<AV_AG>(it, A, s);
-  else launch_fwd<AV_VA>(it, A, s);
+  if (k == 128) {
+    if (agnn) launch_fwd<128, AV_AG>(it, A, s);
+    else launch_fwd<128, AV_VA>(it, A, s);
+  } else if (k == 256) {
+    if (agnn) launch_fwd<256, AV_AG>(it, A, s);
+    else launch_fwd<256, AV_VA>(it, A, s);
+  } else {
+    return AGNN_EUNSUPPORTED;
+  }
   AGNN_LAUNCH_CHECK("av_fwd_kernel");
   return AGNN_OK;
 }
 
-agnn_status av_bwd_k128(const Items& it, bool agnn, const AvBwd& A, cudaStream_t s) {
+agnn_status av_bwd_batched(const Items& it, int k, bool agnn, const AvBwd& A, cudaStream_t s) {
   if (it.n_chunks + it.n_light == 0) return AGNN_OK;
-  if (agnn) launch_bwd<AV_AG>(it, A, s);
-  else launch_bwd<AV_VA>(it, A, s);
+  if (k == 128) {
+    if (agnn) launch_bwd<128, AV_AG>(it, A, s);
+    else launch_bwd<128, AV_VA>(it, A, s);
+  } else if (k == 256) {
+    if (agnn) launch_bwd<256, AV_AG>(it, A, s);
+    else launch_bwd<256, AV_VA>(it, A, s);
+  } else {
+    return AGNN_EUNSUPPORTED;
+  }
   AGNN_LAUNCH_CHECK("av_bwd_kernel");
   return AGNN_OK;
 }

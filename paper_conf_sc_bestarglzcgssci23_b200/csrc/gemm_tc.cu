@@ -168,43 +168,51 @@ struct TcOut {
   float* pC1[kMaxPeers - 1];
 };
 
-// 16 consecutive columns c0.. of output row `row` (C0 | C1 split, optional sigma copy)
+// 16 consecutive columns c0.. of output row `row` (C0 | C1 split, optional sigma copy).
+// PEER: the same values also go to every peer's replica (peer-memory all-gather);
+// a compile-time flag, so the single-GPU epilogue carries no peer code at all.
+__device__ __forceinline__ void store_row16_to(const TcOut& out, float* C0, float* C1, float* Ca,
+                                               int64_t row, int c0, const float (&v)[16]) {
+#pragma unroll
+  for (int j = 0; j < 16; j += 4) {
+    const int c = c0 + j;
+    const float4 q = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
+    if (c + 3 < out.n_split && (out.n_split & 3) == 0) {
+      if (C0) st4(C0 + row * out.n_split + c, q);
+      if (Ca) st4(Ca + row * out.n_split + c, act_fwd4(out.act, q));
+    } else if (c < out.n_split) {
+#pragma unroll
+      for (int x = 0; x < 4; ++x) {
+        if (c + x < out.n_split) {
+          if (C0) C0[row * out.n_split + c + x] = v[j + x];
+          if (Ca) Ca[row * out.n_split + c + x] = act_fwd(out.act, v[j + x]);
+        } else if (c + x < out.n_store) {
+          C1[row * (out.n_store - out.n_split) + (c + x - out.n_split)] = v[j + x];
+        }
+      }
+    } else if (c < out.n_store) {
+      const int w1 = out.n_store - out.n_split;
+#pragma unroll
+      for (int x = 0; x < 4; ++x)
+        if (c + x < out.n_store) C1[row * w1 + (c + x - out.n_split)] = v[j + x];
+    }
+  }
+}
+template <bool PEER>
 __device__ __forceinline__ void store_row16(const TcOut& out, int64_t row, int c0,
                                             const float (&v)[16]) {
-  for (int pi = -1; pi < out.npeer; ++pi) {  // own copy, then the peers' replicas
-    float* C0 = pi < 0 ? out.C0 : out.pC0[pi];
-    float* C1 = pi < 0 ? out.C1 : out.pC1[pi];
-    float* Ca = pi < 0 ? out.Cact : nullptr;
-#pragma unroll
-    for (int j = 0; j < 16; j += 4) {
-      const int c = c0 + j;
-      const float4 q = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
-      if (c + 3 < out.n_split && (out.n_split & 3) == 0) {
-        if (C0) st4(C0 + row * out.n_split + c, q);
-        if (Ca) st4(Ca + row * out.n_split + c, act_fwd4(out.act, q));
-      } else if (c < out.n_split) {
-#pragma unroll
-        for (int x = 0; x < 4; ++x) {
-          if (c + x < out.n_split) {
-            if (C0) C0[row * out.n_split + c + x] = v[j + x];
-            if (Ca) Ca[row * out.n_split + c + x] = act_fwd(out.act, v[j + x]);
-          } else if (c + x < out.n_store) {
-            C1[row * (out.n_store - out.n_split) + (c + x - out.n_split)] = v[j + x];
-          }
-        }
-      } else if (c < out.n_store) {
-        const int w1 = out.n_store - out.n_split;
-#pragma unroll
-        for (int x = 0; x < 4; ++x)
-          if (c + x < out.n_store) C1[row * w1 + (c + x - out.n_split)] = v[j + x];
-      }
-    }
+  store_row16_to(out, out.C0, out.C1, out.Cact, row, c0, v);
+  if constexpr (PEER) {
+#pragma unroll 1
+    for (int pi = 0; pi < out.npeer; ++pi)
+      store_row16_to(out, out.pC0[pi], out.pC1[pi], nullptr, row, c0, v);
   }
 }
 
 // 32 columns [c0, c0+32) of the warp's 32 rows [row0, row0+32) through a per-warp
 // shared-memory transpose, so every store instruction writes 4 full 128-byte rows
 // (a thread-per-row store touches 32 lines per instruction, 8x the L2 write requests)
+template <bool PEER>
 __device__ __forceinline__ void store_block32(const TcOut& out, int64_t row0, int64_t M, int c0,
                                               const float (&v)[32], float* stg, int lane) {
   // stg: [32 rows][36 floats] (16-byte aligned rows, 4-float pad against bank conflicts)
@@ -221,8 +229,11 @@ __device__ __forceinline__ void store_block32(const TcOut& out, int64_t row0, in
     if (row < M) {
       if (out.C0) st4(out.C0 + row * out.n_split + c0 + cc, q);
       if (out.Cact) st4(out.Cact + row * out.n_split + c0 + cc, act_fwd4(out.act, q));
-      for (int pi = 0; pi < out.npeer; ++pi)  // peers' replicas (NVLink stores)
-        st4(out.pC0[pi] + row * out.n_split + c0 + cc, q);
+      if constexpr (PEER) {
+#pragma unroll 1
+        for (int pi = 0; pi < out.npeer; ++pi)  // peers' replicas (NVLink stores)
+          st4(out.pC0[pi] + row * out.n_split + c0 + cc, q);
+      }
     }
   }
   __syncwarp();
@@ -248,7 +259,7 @@ __device__ __forceinline__ void math_barrier() {  // the 128 math threads only
   asm volatile("bar.sync 1, 128;" ::: "memory");
 }
 
-template <int N, int K, int S, bool SB>
+template <int N, int K, int S, bool SB, bool PEER>
 __global__ void __launch_bounds__(TC_WS_THREADS, 1)
 gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                const float* __restrict__ B, int n_real, int64_t M, TcOut out) {
@@ -461,14 +472,14 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
             float q[32];
 #pragma unroll
             for (int x = 0; x < 32; ++x) q[x] = v[c0 + x];
-            store_block32(out, row0, M, h0 + c0, q, stg + ew * 32 * 36, lane);
+            store_block32<PEER>(out, row0, M, h0 + c0, q, stg + ew * 32 * 36, lane);
           } else if (row < M) {
 #pragma unroll
             for (int c1 = c0; c1 < c0 + 32 && c1 < NP; c1 += 16) {
               float q[16];
 #pragma unroll
               for (int x = 0; x < 16; ++x) q[x] = v[c1 + x];
-              store_row16(out, row, h0 + c1, q);
+              store_row16<PEER>(out, row, h0 + c1, q);
             }
           }
         }
@@ -686,8 +697,10 @@ agnn_status launch_tc(const float* A, int64_t M, const float* B, int n_real, con
   static_assert(smem <= 232448 - 1024, "shared memory");
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(gemm_tc_kernel<N, K, S, SB>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                         smem);
+    cudaFuncSetAttribute(gemm_tc_kernel<N, K, S, SB, false>,
+                         cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    cudaFuncSetAttribute(gemm_tc_kernel<N, K, S, SB, true>,
+                         cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     attr = true;
   }
   int sms = kNumSMs, dev = 0;
@@ -695,7 +708,10 @@ agnn_status launch_tc(const float* A, int64_t M, const float* B, int n_real, con
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   const int64_t ntiles = (M + TC_BM - 1) / TC_BM;
   const int grid = (int)std::min<int64_t>(ntiles, sms);
-  gemm_tc_kernel<N, K, S, SB><<<grid, TC_WS_THREADS, smem, s>>>(ma, mb, B, n_real, M, o);
+  if (o.npeer > 0)
+    gemm_tc_kernel<N, K, S, SB, true><<<grid, TC_WS_THREADS, smem, s>>>(ma, mb, B, n_real, M, o);
+  else
+    gemm_tc_kernel<N, K, S, SB, false><<<grid, TC_WS_THREADS, smem, s>>>(ma, mb, B, n_real, M, o);
   AGNN_LAUNCH_CHECK("gemm_tc_kernel");
   return AGNN_OK;
 }
