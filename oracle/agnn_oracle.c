@@ -172,10 +172,26 @@ static void mm_nt(int64_t n, int c, int b, const double* A, const double* B, dou
  *   s,t[n x heads]: s_i^h = P_i^h . a1^h, t_j^h = P_j^h . a2^h
  *   alpha[nnz x heads], m,l[n x heads] (row max / row sum of exp)
  *   Z[n x kout] = sum_j alpha_ij P_j ; Hout = sigma(Z)                   */
-int oracle_gat_forward(int64_t n, const int64_t* rp, const int32_t* ci, int k, int kout, int heads,
-                       const double* H, const double* W, const double* a, double slope, int act,
-                       double* P, double* s, double* t, double* alpha, double* m, double* l,
-                       double* Z, double* Hout) {
+/* BF16 storage mode (north_star "1e-2 with BF16 projection"; DESIGN.md reading
+ * B1): the projected rows P and the backward's G are STORED in bfloat16 — the
+ * value the kernels gather is round(fp32(x)) to the nearest bf16 (ties to even),
+ * exactly what an fp32 result converted with __float2bfloat16_rn holds.        */
+static double bf16_round(double x) {
+  float f = (float)x;
+  uint32_t u;
+  memcpy(&u, &f, 4);
+  if ((u & 0x7f800000u) != 0x7f800000u) {  /* finite: round to nearest even */
+    u += 0x7fffu + ((u >> 16) & 1u);
+    u &= 0xffff0000u;
+  }
+  memcpy(&f, &u, 4);
+  return (double)f;
+}
+
+static int gat_forward_impl(int64_t n, const int64_t* rp, const int32_t* ci, int k, int kout,
+                            int heads, const double* H, const double* W, const double* a,
+                            double slope, int act, double* P, double* s, double* t, double* alpha,
+                            double* m, double* l, double* Z, double* Hout, int bf16) {
   if (heads <= 0 || kout % heads) return 1;
   const int d = kout / heads;
   mm(n, k, kout, H, W, P);
@@ -190,6 +206,12 @@ int oracle_gat_forward(int64_t n, const int64_t* rp, const int32_t* ci, int k, i
       s[i * heads + h] = si;
       t[i * heads + h] = ti;
     }
+  /* BF16 mode: the scores above come from the unrounded projection (a' = W a,
+   * PAPER.md:141, is its own GEMM column); what is stored and gathered is P~ */
+  if (bf16) {
+#pragma omp parallel for schedule(static)
+    for (int64_t x = 0; x < n * kout; ++x) P[x] = bf16_round(P[x]);
+  }
 #pragma omp parallel for schedule(dynamic, 64)
   for (int64_t i = 0; i < n; ++i) {
     for (int h = 0; h < heads; ++h) {
@@ -224,6 +246,21 @@ int oracle_gat_forward(int64_t n, const int64_t* rp, const int32_t* ci, int k, i
   }
   return 0;
 }
+int oracle_gat_forward(int64_t n, const int64_t* rp, const int32_t* ci, int k, int kout, int heads,
+                       const double* H, const double* W, const double* a, double slope, int act,
+                       double* P, double* s, double* t, double* alpha, double* m, double* l,
+                       double* Z, double* Hout) {
+  return gat_forward_impl(n, rp, ci, k, kout, heads, H, W, a, slope, act, P, s, t, alpha, m, l, Z,
+                          Hout, 0);
+}
+/* BF16 storage mode: P (output) holds the stored P~ */
+int oracle_gat_forward_bf16(int64_t n, const int64_t* rp, const int32_t* ci, int k, int kout,
+                            int heads, const double* H, const double* W, const double* a,
+                            double slope, int act, double* P, double* s, double* t, double* alpha,
+                            double* m, double* l, double* Z, double* Hout) {
+  return gat_forward_impl(n, rp, ci, k, kout, heads, H, W, a, slope, act, P, s, t, alpha, m, l, Z,
+                          Hout, 1);
+}
 
 /* GAT backward (Eq. 3-6; derivation in DESIGN.md §2,
  * readings A11 Psi^T, A12 da):
@@ -235,11 +272,12 @@ int oracle_gat_forward(int64_t n, const int64_t* rp, const int32_t* ci, int k, i
  *   da1^h = sum_i ds_i P_i^h ; da2^h = sum_j dt_j P_j^h
  *   dW = H^T dP ; dH = dP W^T
  * Outputs: dH[n x k], dW[k x kout], da[heads x 2d]; G, dP optional (NULL). */
-int oracle_gat_backward(int64_t n, const int64_t* rp, const int32_t* ci, int k, int kout, int heads,
-                        const double* H, const double* W, const double* a, double slope, int act,
-                        const double* P, const double* s, const double* t, const double* alpha,
-                        const double* Z, const double* dHout, double* dH, double* dW, double* da,
-                        double* G_out, double* dP_out) {
+static int gat_backward_impl(int64_t n, const int64_t* rp, const int32_t* ci, int k, int kout,
+                             int heads, const double* H, const double* W, const double* a,
+                             double slope, int act, const double* P, const double* s,
+                             const double* t, const double* alpha, const double* Z,
+                             const double* dHout, double* dH, double* dW, double* da,
+                             double* G_out, double* dP_out, int bf16) {
   if (heads <= 0 || kout % heads) return 1;
   const int d = kout / heads;
   const int64_t nnz = rp[n];
@@ -255,7 +293,10 @@ int oracle_gat_backward(int64_t n, const int64_t* rp, const int32_t* ci, int k, 
   build_csc(n, rp, ci, cp, pos);
 
 #pragma omp parallel for schedule(static)
-  for (int64_t x = 0; x < n * kout; ++x) G[x] = dHout[x] * act_df(act, Z[x]);
+  for (int64_t x = 0; x < n * kout; ++x) {
+    G[x] = dHout[x] * act_df(act, Z[x]);
+    if (bf16) G[x] = bf16_round(G[x]);  /* BF16 mode: G~ is stored and used throughout */
+  }
 
 #pragma omp parallel for schedule(dynamic, 64)
   for (int64_t i = 0; i < n; ++i)
@@ -310,6 +351,24 @@ int oracle_gat_backward(int64_t n, const int64_t* rp, const int32_t* ci, int k, 
   if (dP_out) memcpy(dP_out, dP, sizeof(double) * (size_t)(n * kout));
   free(G); free(delta); free(dc); free(ds); free(dt); free(dP); free(cp); free(pos); free(erow);
   return 0;
+}
+int oracle_gat_backward(int64_t n, const int64_t* rp, const int32_t* ci, int k, int kout, int heads,
+                        const double* H, const double* W, const double* a, double slope, int act,
+                        const double* P, const double* s, const double* t, const double* alpha,
+                        const double* Z, const double* dHout, double* dH, double* dW, double* da,
+                        double* G_out, double* dP_out) {
+  return gat_backward_impl(n, rp, ci, k, kout, heads, H, W, a, slope, act, P, s, t, alpha, Z,
+                           dHout, dH, dW, da, G_out, dP_out, 0);
+}
+/* BF16 storage mode: P is the forward's stored P~; G is rounded to G~ */
+int oracle_gat_backward_bf16(int64_t n, const int64_t* rp, const int32_t* ci, int k, int kout,
+                             int heads, const double* H, const double* W, const double* a,
+                             double slope, int act, const double* P, const double* s,
+                             const double* t, const double* alpha, const double* Z,
+                             const double* dHout, double* dH, double* dW, double* da,
+                             double* G_out, double* dP_out) {
+  return gat_backward_impl(n, rp, ci, k, kout, heads, H, W, a, slope, act, P, s, t, alpha, Z,
+                           dHout, dH, dW, da, G_out, dP_out, 1);
 }
 
 /* ================================================================== */

@@ -82,14 +82,16 @@ def _csr(rp, ci):
             len(rp) - 1, int(rp[-1]))
 
 
-def gat_forward(rp, ci, H, W, a, heads, slope=0.2, act="relu"):
+def gat_forward(rp, ci, H, W, a, heads, slope=0.2, act="relu", bf16=False):
+    """bf16: BF16 storage mode (P stored as bf16; out["P"] is the stored P~)."""
     rp, ci, n, nnz = _csr(rp, ci)
     H, W, a = _d(H), _d(W), _d(a)
     k, kout = W.shape
     out = {x: np.zeros((n, kout)) for x in ("P", "Z", "Hout")}
     out.update({x: np.zeros((n, heads)) for x in ("s", "t", "m", "l")})
     out["alpha"] = np.zeros((nnz, heads))
-    rc = lib().oracle_gat_forward(
+    fn = lib().oracle_gat_forward_bf16 if bf16 else lib().oracle_gat_forward
+    rc = fn(
         _i64(n), _p(rp), _p(ci), ctypes.c_int(k), ctypes.c_int(kout), ctypes.c_int(heads),
         _p(H), _p(W), _p(a), ctypes.c_double(slope), ctypes.c_int(ACT[act]),
         _p(out["P"]), _p(out["s"]), _p(out["t"]), _p(out["alpha"]), _p(out["m"]), _p(out["l"]),
@@ -99,14 +101,16 @@ def gat_forward(rp, ci, H, W, a, heads, slope=0.2, act="relu"):
     return out
 
 
-def gat_backward(rp, ci, H, W, a, heads, fwd, dHout, slope=0.2, act="relu"):
+def gat_backward(rp, ci, H, W, a, heads, fwd, dHout, slope=0.2, act="relu", bf16=False):
+    """bf16: BF16 storage mode (G stored as bf16; fwd from gat_forward(bf16=True))."""
     rp, ci, n, nnz = _csr(rp, ci)
     H, W, a, dHout = _d(H), _d(W), _d(a), _d(dHout)
     k, kout = W.shape
     d = kout // heads
     out = {"dH": np.zeros((n, k)), "dW": np.zeros((k, kout)), "da": np.zeros((heads, 2 * d)),
            "G": np.zeros((n, kout)), "dP": np.zeros((n, kout))}
-    rc = lib().oracle_gat_backward(
+    fn = lib().oracle_gat_backward_bf16 if bf16 else lib().oracle_gat_backward
+    rc = fn(
         _i64(n), _p(rp), _p(ci), ctypes.c_int(k), ctypes.c_int(kout), ctypes.c_int(heads),
         _p(H), _p(W), _p(a), ctypes.c_double(slope), ctypes.c_int(ACT[act]),
         _p(fwd["P"]), _p(fwd["s"]), _p(fwd["t"]), _p(fwd["alpha"]), _p(fwd["Z"]), _p(dHout),
@@ -208,11 +212,12 @@ def cgnn_backward(rp, ci, H, W, fwd, dHout, agg="sum", act="relu"):
 
 
 def layer(model, rp, ci, H, W, a=None, heads=1, dHout=None, act="relu", slope=0.2, beta=1.0,
-          eps=1e-12, agg="sum"):
+          eps=1e-12, agg="sum", bf16=False):
     """Forward (+ backward when dHout is given) of one layer of `model`."""
     if model == "gat":
-        f = gat_forward(rp, ci, H, W, a, heads, slope, act)
-        b = gat_backward(rp, ci, H, W, a, heads, f, dHout, slope, act) if dHout is not None else None
+        f = gat_forward(rp, ci, H, W, a, heads, slope, act, bf16)
+        b = (gat_backward(rp, ci, H, W, a, heads, f, dHout, slope, act, bf16)
+             if dHout is not None else None)
     elif model == "agnn":
         f = agnn_forward(rp, ci, H, W, beta, eps, act)
         b = agnn_backward(rp, ci, H, W, f, dHout, beta, eps, act) if dHout is not None else None

@@ -495,3 +495,51 @@ def test_cgnn_finite_differences(agg):
     loss = lambda: float((oracle.cgnn_forward(rp, ci, H, W, agg, "elu")["Hout"] * R).sum())
     assert rel(_fd(loss, H, 1e-7), b["dH"]) < 1e-6
     assert rel(_fd(loss, W, 1e-7), b["dW"]) < 1e-6
+
+
+# ------------------------------------------------ BF16 storage mode (reading B1)
+def test_bf16_round_matches_torch():
+    """The oracle's bf16 rounding == torch's fp32 -> bfloat16 conversion (RNE)."""
+    import torch
+    rng = np.random.default_rng(70)
+    x = np.concatenate([rng.standard_normal(10000) * 10.0 ** rng.integers(-30, 30, 10000),
+                        [0.0, -0.0, 1.0, 1.00390625, 1.0 + 2 ** -9, 3.0e38]])
+    rp = np.arange(len(x) + 1, dtype=np.int64)
+    ci = np.arange(len(x), dtype=np.int32)
+    # P = H W with W = 1 (k = kout = 1): the stored P~ is round_bf16(fp32(x))
+    f = oracle.gat_forward(rp, ci, x[:, None], np.ones((1, 1)), np.zeros((1, 2)), 1,
+                           act="none", bf16=True)
+    ref = torch.tensor(x, dtype=torch.float64).float().bfloat16().double().numpy()
+    np.testing.assert_array_equal(f["P"][:, 0], ref)
+
+
+@pytest.mark.parametrize("heads", [1, 2])
+def test_bf16_mode_exact_when_representable(heads):
+    """When P and G are bf16-representable the BF16 mode IS the fp64 oracle (the
+    rounding is the only difference): small-integer H, W, R and sigma = identity."""
+    rng = np.random.default_rng(71)
+    n, k, kout = 10, 3, 4
+    rp, ci = rand_graph(n, 0.4, rng)
+    H = rng.integers(-2, 3, (n, k)).astype(float)
+    W = rng.integers(-2, 3, (k, kout)).astype(float)
+    a = rng.uniform(-0.5, 0.5, (heads, 2 * (kout // heads)))
+    R = rng.integers(-2, 3, (n, kout)).astype(float)
+    f0, b0 = oracle.layer("gat", rp, ci, H, W, a, heads, R, act="none")
+    f1, b1 = oracle.layer("gat", rp, ci, H, W, a, heads, R, act="none", bf16=True)
+    for key in ("P", "Z", "alpha"):
+        np.testing.assert_array_equal(f0[key], f1[key])
+    for key in ("dH", "dW", "da"):
+        np.testing.assert_array_equal(b0[key], b1[key])
+
+
+def test_bf16_mode_within_the_north_star_bound():
+    """Against the fp64 oracle the BF16 mode stays within the 1e-2 (north_star)."""
+    rng = np.random.default_rng(72)
+    n, k, kout, heads = 30, 8, 8, 2
+    rp, ci = rand_graph(n, 0.3, rng)
+    H, W, a, R = rand_inputs(n, k, kout, heads, rng)
+    f0, b0 = oracle.layer("gat", rp, ci, H, W, a, heads, R, act="elu")
+    f1, b1 = oracle.layer("gat", rp, ci, H, W, a, heads, R, act="elu", bf16=True)
+    assert 0 < rel(f1["Z"], f0["Z"]) < 1e-2
+    for key in ("dH", "dW"):
+        assert 0 < rel(b1[key], b0[key]) < 1e-2
