@@ -49,6 +49,9 @@ def parse():
                    help="time the step as one CUDA-graph replay (auto: small, launch-bound "
                         "workloads on one GPU)")
     p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--prec", default="fp32", choices=["fp32", "bf16"],
+                   help="GAT feature storage: fp32, or bf16 (P and G stored as bfloat16, "
+                        "fp32 arithmetic; include/agnn.h AGNN_PREC_BF16, reading B1)")
     p.add_argument("--scale", type=int, default=None,
                    help="override log2 n of the workload (same recipe and edge factor)")
     p.add_argument("--cpu-sample-scale", type=int, default=17,
@@ -151,6 +154,9 @@ def cpu_model():
 def workload(args):
     from paper_conf_sc_bestarglzcgssci23_b200 import gen
     w = gen.CONFIGS[args.config]
+    if getattr(args, "prec", "fp32") != "fp32":
+        import dataclasses
+        w = dataclasses.replace(w, prec=args.prec)
     if args.scale is not None and w.graph != "er":
         ef = w.n_samples // w.n
         import dataclasses
@@ -227,8 +233,9 @@ def algorithmic_bytes(w, m, n):
     """
     f = 4
     if w.model == "gat":
-        per_edge = 4 + 2 * w.k * f + 20 * w.heads
-        per_row = 3 * w.k * f + 20 * w.heads + 8
+        fs = 2 if w.prec == "bf16" else 4   # stored P, G (reading B1); dP stays fp32
+        per_edge = 4 + 2 * w.k * fs + 20 * w.heads
+        per_row = 2 * w.k * fs + w.k * f + 20 * w.heads + 8
     else:
         rec = 16 if w.model == "agnn" else 0
         per_edge = 4 + 2 * w.k * f + rec
@@ -391,7 +398,8 @@ def run_ours(args):
     try:  # ncu DRAM bytes per launch of the same kernel on the same workload (committed)
         tr = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))
         if args.scale is None and world == 1:
-            traffic = tr.get(args.config, {}).get(dom)
+            key = args.config + ("" if w.prec == "fp32" else "-" + w.prec)
+            traffic = tr.get(key, {}).get(dom)
     except Exception:
         traffic = None
     roof = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": hbm, "unit": "GB/s",
@@ -496,6 +504,8 @@ def run_ours(args):
                 "dtype": "f32", "data": "synthetic",
                 "config": {"workload": args.config, "model": w.model, "graph": w.graph,
                            "n": n, "edges": m, "k": w.k, "heads": w.heads, "layers": w.layers,
+                           "storage": ("bf16 P, G (fp32 arithmetic; AGNN_PREC_BF16, tol 1e-2)"
+                                       if w.prec == "bf16" else "fp32"),
                            "parallelism": f"1d-rowblock{world}",
                            "comm": (args.comm if world > 1 else None),
                            "l2_flush": "inputs > L2 (126 MB)" if not small else

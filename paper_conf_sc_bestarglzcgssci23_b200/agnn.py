@@ -17,7 +17,8 @@ VA, AGNN, GAT = 0, 1, 2
 KIND = {"va": VA, "agnn": AGNN, "gat": GAT, "cgnn": 3}
 AGG = {"sum": 0, "mean": 1, "gcn": 2, "max": 3, "min": 4}
 ACT = {"none": 0, "relu": 1, "elu": 2}
-PREC_FP32, PREC_TF32X3 = 0, 1
+PREC_FP32, PREC_TF32X3, PREC_BF16 = 0, 1, 2
+PREC = {"fp32": PREC_FP32, "tf32x3": PREC_TF32X3, "bf16": PREC_BF16}
 CSR_SYMMETRIC = 1
 BUILD_SYMMETRIZE, BUILD_SELF_LOOPS, BUILD_CONNECT_ISOLATED = 1, 2, 4
 BUILD_PAPER = BUILD_SYMMETRIZE | BUILD_SELF_LOOPS | BUILD_CONNECT_ISOLATED

@@ -91,6 +91,11 @@ static agnn_status check_desc(const agnn_layer_desc& d) {
   if (d.k_in <= 0 || d.k_out <= 0 || d.k_in % 4 || d.k_out % 4)
     return fail(AGNN_EINVAL, "layer desc: k_in/k_out must be positive multiples of 4");
   if (d.act < AGNN_ACT_NONE || d.act > AGNN_ACT_ELU) return fail(AGNN_EINVAL, "layer desc: act");
+  if (d.prec < AGNN_PREC_FP32 || d.prec > AGNN_PREC_BF16) return fail(AGNN_EINVAL, "layer desc: prec");
+  if (d.prec == AGNN_PREC_BF16 &&
+      !(d.kind == AGNN_GAT && d.k_out == 128 &&
+        (d.heads == 1 || d.heads == 2 || d.heads == 4 || d.heads == 8)))
+    return fail(AGNN_EUNSUPPORTED, "AGNN_PREC_BF16: GAT with k_out = 128 and 1/2/4/8 heads only");
   if (d.kind == AGNN_GAT) {
     if (d.heads <= 0 || d.k_out % d.heads || (d.k_out / d.heads) % 4)
       return fail(AGNN_EINVAL, "GAT: k_out must split into heads of a multiple of 4 features");
@@ -112,7 +117,8 @@ static agnn_status check_desc(const agnn_layer_desc& d) {
 }
 
 static GatShape gat_shape(const agnn_layer_desc& d) {
-  return GatShape{d.k_in, d.k_out, d.heads, d.negative_slope, (int)d.act};
+  return GatShape{d.k_in, d.k_out, d.heads, d.negative_slope, (int)d.act,
+                  d.prec == AGNN_PREC_BF16};
 }
 
 // C-GNN entry points live in cgnn.cu

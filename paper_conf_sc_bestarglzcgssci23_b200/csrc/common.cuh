@@ -2,6 +2,7 @@
 #pragma once
 #include <vector>
 #include <cuda_runtime.h>
+#include <cuda_bf16.h>
 #include <stdint.h>
 #include <string>
 
@@ -56,6 +57,31 @@ __device__ __forceinline__ float4 ld_stream4(const float* p) {
   return r;
 }
 __device__ __forceinline__ void st4(float* p, float4 v) { *reinterpret_cast<float4*>(p) = v; }
+
+// ---- bfloat16 feature storage (GAT BF16 mode, reading B1) ---------------------
+// 4 consecutive bf16 features = 8 bytes; widened to fp32 exactly (bf16 is the high
+// half of an fp32), narrowed with round-to-nearest-even (cvt.rn.bf16x2.f32).
+typedef __nv_bfloat16 bf16;
+__device__ __forceinline__ float4 bf4_to_f4(uint2 u) {
+  return make_float4(__uint_as_float(u.x << 16), __uint_as_float(u.x & 0xffff0000u),
+                     __uint_as_float(u.y << 16), __uint_as_float(u.y & 0xffff0000u));
+}
+__device__ __forceinline__ float4 ldg4(const bf16* p) {
+  return bf4_to_f4(__ldg(reinterpret_cast<const uint2*>(p)));
+}
+__device__ __forceinline__ uint32_t pack_bf2(float lo, float hi) {
+  uint32_t r;
+  asm("cvt.rn.bf16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(hi), "f"(lo));
+  return r;
+}
+__device__ __forceinline__ uint2 f4_to_bf4(float4 v) {
+  return make_uint2(pack_bf2(v.x, v.y), pack_bf2(v.z, v.w));
+}
+__device__ __forceinline__ void st4(bf16* p, float4 v) {
+  *reinterpret_cast<uint2*>(p) = f4_to_bf4(v);
+}
+// the value a bf16 store of v holds, widened back (G~ of reading B1)
+__device__ __forceinline__ float4 round_bf4(float4 v) { return bf4_to_f4(f4_to_bf4(v)); }
 
 __device__ __forceinline__ float dot4(float4 a, float4 b) {
   return fmaf(a.x, b.x, fmaf(a.y, b.y, fmaf(a.z, b.z, a.w * b.w)));

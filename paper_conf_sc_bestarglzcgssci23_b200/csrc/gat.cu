@@ -239,7 +239,7 @@ __device__ __forceinline__ void bwd_finish(const BwdArgs& A, int64_t row, int64_
     float4 dp = fma4(ds[v], a1, acc[v]);
     dp = fma4(dt[v], a2, dp);
     st4(A.dP + row * K + c, dp);
-    const float4 pj = ldg4(A.P + grow * K + c);
+    const float4 pj = A.P16 ? ldg4(A.P16 + grow * K + c) : ldg4(A.P + grow * K + c);
     da1[v] = fma4(ds[v], pj, da1[v]);
     da2[v] = fma4(dt[v], pj, da2[v]);
     if (A.ds_out && cc == 0) {
@@ -438,13 +438,15 @@ gat_bwd_merge_kernel(Items it, BwdArgs A, int64_t da_row0) {
   }
 }
 
-// G = dH_out (.) sigma'(Z) ; rec = {s, m, 1/l, delta = G^h . Z^h} (per head)
-template <int K, int NH>
+// G = dH_out (.) sigma'(Z) ; rec = {s, m, 1/l, delta = G^h . Z^h} (per head).
+// TG = bf16 (BF16 mode, reading B1): G is rounded to bfloat16 first and the rounded
+// G~ is what delta uses and what is stored.
+template <int K, int NH, typename TG = float>
 __global__ void __launch_bounds__(kSparseThreads)
 gat_bwd_prologue_kernel(int64_t n_local, int64_t row_begin, const float* __restrict__ dHout,
                         const float* __restrict__ Z, const float* __restrict__ st,
                         const float* __restrict__ mrow, const float* __restrict__ lrow, int act,
-                        float* __restrict__ G, float4* __restrict__ rec, PeerRows peers) {
+                        TG* __restrict__ G, float4* __restrict__ rec, PeerRows peers) {
   using L = RowLayout<K, NH>;
   const int lane = threadIdx.x & 31, g = lane / L::LANES, q = lane % L::LANES;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
@@ -464,6 +466,7 @@ gat_bwd_prologue_kernel(int64_t n_local, int64_t row_begin, const float* __restr
       }
       gv[v] = make_float4(dh.x * act_grad(act, z.x), dh.y * act_grad(act, z.y),
                           dh.z * act_grad(act, z.z), dh.w * act_grad(act, z.w));
+      if constexpr (sizeof(TG) == 2) gv[v] = round_bf4(gv[v]);
       dl[v] = dot4(gv[v], z);
     }
     L::head_reduce(dl);
@@ -474,7 +477,7 @@ gat_bwd_prologue_kernel(int64_t n_local, int64_t row_begin, const float* __restr
       const int c = L::col(v, q), h = c / L::D;
       st4(G + grow * K + c, gv[v]);
       for (int pi = 0; pi < peers.n; ++pi)  // peers' replicas (fused all-gather)
-        st4(peers.a[pi] + grow * K + c, gv[v]);
+        st4(reinterpret_cast<TG*>(peers.a[pi]) + grow * K + c, gv[v]);
       if ((c % L::D) == 0) {
         const float lv = lrow[row * NH + h];
         const float4 r4 = make_float4(st[grow * 2 * NH + h], mrow[row * NH + h],
@@ -562,11 +565,17 @@ __global__ void gat_debug_alpha_kernel(const int64_t* __restrict__ rp, int64_t n
 // ---------------------------------------------------------------- layout
 struct SavedGat {
   float *P, *st, *Z, *m, *l;
+  bf16* P16;  // BF16 mode: P stored as bfloat16 (P == NULL)
 };
 SavedGat carve_saved(const Plan& p, const GatShape& g, void* base) {
   Carver c(base);
   SavedGat s;
-  s.P = c.take<float>((size_t)p.n * g.k_out);
+  s.P = nullptr;
+  s.P16 = nullptr;
+  if (g.bf16)
+    s.P16 = c.take<bf16>((size_t)p.n * g.k_out);
+  else
+    s.P = c.take<float>((size_t)p.n * g.k_out);
   s.st = c.take<float>((size_t)p.n * 2 * g.heads);
   s.Z = c.take<float>((size_t)p.n_local * g.k_out);
   s.m = c.take<float>((size_t)p.n_local * g.heads);
@@ -575,7 +584,10 @@ SavedGat carve_saved(const Plan& p, const GatShape& g, void* base) {
 }
 size_t saved_size(const Plan& p, const GatShape& g) {
   Carver c(nullptr);
-  c.take<float>((size_t)p.n * g.k_out);
+  if (g.bf16)
+    c.take<bf16>((size_t)p.n * g.k_out);
+  else
+    c.take<float>((size_t)p.n * g.k_out);
   c.take<float>((size_t)p.n * 2 * g.heads);
   c.take<float>((size_t)p.n_local * g.k_out);
   c.take<float>((size_t)p.n_local * g.heads);
@@ -585,6 +597,7 @@ size_t saved_size(const Plan& p, const GatShape& g) {
 
 struct WsGat {
   float *Wext, *pacc, *pm, *pl, *G, *dP, *da_part, *gemm, *ds_dir;
+  bf16* G16;  // BF16 mode: G stored as bfloat16 (G == NULL)
   float4* rec;
   void* saved_inf;  // saved-layout scratch for inference
 };
@@ -596,7 +609,12 @@ WsGat carve_ws(const Plan& p, const GatShape& g, void* base, size_t* total) {
   const int NE = (g.k_out + 2 * g.heads + 3) / 4 * 4;
   // replicated (n-row) arrays first: their offsets are the same on every rank, which
   // the peer-memory exchange relies on (agnn_plan_register maps whole buffers)
-  w.G = c.take<float>((size_t)p.n * g.k_out);
+  w.G = nullptr;
+  w.G16 = nullptr;
+  if (g.bf16)
+    w.G16 = c.take<bf16>((size_t)p.n * g.k_out);
+  else
+    w.G = c.take<float>((size_t)p.n * g.k_out);
   w.rec = c.take<float4>((size_t)p.n * g.heads);
   w.saved_inf = c.take<char>(saved_size(p, g));  // its replicated prefix (P, st) too
   w.Wext = c.take<float>((size_t)g.k_in * NE);
@@ -653,9 +671,32 @@ agnn_status gat_forward(const Plan& p, const GatShape& g, const float* W, const 
   gat_wext_kernel<<<64, 256, 0, s>>>(W, a, g.k_in, g.k_out, g.heads, NE, w.Wext);
   AGNN_LAUNCH_CHECK("gat_wext_kernel");
   // P (and s, t) for the local rows, written at their global offsets
-  float* Ploc = sv.P + p.row_begin * g.k_out;
   float* stloc = sv.st + p.row_begin * 2 * g.heads;
   agnn_status st;
+  if (g.bf16) {
+    // BF16 mode (reading B1): the tcgen05 epilogue rounds P to bfloat16; s, t come
+    // from the same (unrounded) accumulators; then the plain all-gather of P~ | st
+    Items it = items_of(p);
+    FwdOut o{saved ? sv.Z : nullptr, H_out, saved ? sv.m : nullptr, saved ? sv.l : nullptr,
+             w.pacc, w.pm, w.pl};
+    if ((st = gemm_rows_bf16(H_in, p.n_local, g.k_in, w.Wext, NEs, sv.P16 + p.row_begin * g.k_out,
+                             g.k_out, stloc, w.dP, s)) != AGNN_OK)
+      return st;
+    if (p.world > 1) {
+      if ((st = allgather_rows(p, reinterpret_cast<float*>(sv.P16), g.k_out / 2, s)) != AGNN_OK)
+        return st;
+      if ((st = allgather_rows(p, sv.st, 2 * g.heads, s)) != AGNN_OK) return st;
+    }
+    if ((st = gat_fwd_k128_bf16(it, g.heads, sv.P16, sv.st, g.slope, g.act, o, s)) != AGNN_OK)
+      return st;
+    if (it.n_heavy > 0) {
+      AGNN_GAT_DISPATCH(K_, NH_, (gat_fwd_merge_kernel<K, NH>
+                                  <<<kNumSMs * 2, kSparseThreads, 0, s>>>(it, g.act, o)));
+      AGNN_LAUNCH_CHECK("gat_fwd_merge_kernel");
+    }
+    return AGNN_OK;
+  }
+  float* Ploc = sv.P + p.row_begin * g.k_out;
   if (p.world > 1 && p.peer) {
     // fused GEMM -> all-gather over peer memory: the GEMM epilogue stores every
     // output tile into the local P | st and into every peer's replica (NVLink
@@ -728,7 +769,7 @@ agnn_status gat_backward(const Plan& p, const GatShape& g, const float* W, const
   if (p.world > 1 && p.peer) {
     void* tg[kMaxPeers];
     void* tr[kMaxPeers];
-    if ((st = peer_targets(p, w.G, tg)) != AGNN_OK) return st;
+    if ((st = peer_targets(p, g.bf16 ? (void*)w.G16 : (void*)w.G, tg)) != AGNN_OK) return st;
     if ((st = peer_targets(p, w.rec, tr)) != AGNN_OK) return st;
     for (int r = 0; r < p.world; ++r) {
       if (r == p.rank) continue;
@@ -739,14 +780,28 @@ agnn_status gat_backward(const Plan& p, const GatShape& g, const float* W, const
     // entry barrier: every peer has finished reading its G / rec (previous layer)
     if ((st = peer_barrier(p, s)) != AGNN_OK) return st;
   }
-  AGNN_GAT_DISPATCH(K_, NH_, (gat_bwd_prologue_kernel<K, NH>
-                              <<<grid_of(gat_bwd_prologue_kernel<K, NH>), kSparseThreads, 0, s>>>(
-                                  p.n_local, p.row_begin, dH_out, sv.Z, sv.st, sv.m, sv.l, g.act,
-                                  w.G, w.rec, pr)));
+  if (g.bf16) {
+    if (directed)
+      return fail(AGNN_EUNSUPPORTED, "AGNN_PREC_BF16: symmetric patterns only");
+    AGNN_GAT_DISPATCH(K_, NH_, (gat_bwd_prologue_kernel<K, NH, bf16>
+                                <<<grid_of(gat_bwd_prologue_kernel<K, NH, bf16>), kSparseThreads, 0,
+                                   s>>>(p.n_local, p.row_begin, dH_out, sv.Z, sv.st, sv.m, sv.l,
+                                        g.act, w.G16, w.rec, pr)));
+  } else {
+    AGNN_GAT_DISPATCH(K_, NH_, (gat_bwd_prologue_kernel<K, NH>
+                                <<<grid_of(gat_bwd_prologue_kernel<K, NH>), kSparseThreads, 0, s>>>(
+                                    p.n_local, p.row_begin, dH_out, sv.Z, sv.st, sv.m, sv.l, g.act,
+                                    w.G, w.rec, pr)));
+  }
   AGNN_LAUNCH_CHECK("gat_bwd_prologue_kernel");
   if (p.world > 1) {
     if (p.peer) {  // the prologue stored G | rec into the peers' replicas: exit barrier
       if ((st = peer_barrier(p, s)) != AGNN_OK) return st;
+    } else if (g.bf16) {
+      if ((st = allgather_rows(p, reinterpret_cast<float*>(w.G16), g.k_out / 2, s)) != AGNN_OK)
+        return st;
+      if ((st = allgather_rows(p, reinterpret_cast<float*>(w.rec), 4 * g.heads, s)) != AGNN_OK)
+        return st;
     } else {
       if ((st = allgather_rows(p, w.G, g.k_out, s)) != AGNN_OK) return st;
       if ((st = allgather_rows(p, reinterpret_cast<float*>(w.rec), 4 * g.heads, s)) != AGNN_OK)
@@ -754,7 +809,7 @@ agnn_status gat_backward(const Plan& p, const GatShape& g, const float* W, const
     }
   }
   BwdArgs A{sv.P, sv.st, w.G, w.rec, a, g.slope, w.dP, w.pacc, w.pm, w.pl, w.da_part,
-            nullptr, nullptr, w.ds_dir};
+            nullptr, nullptr, w.ds_dir, sv.P16, w.G16};
   int64_t main_warps = 0, merge_warps = 0;
   if (directed) {
     // row role over the CSR (ds_j), then the column role over the CSC (dt_j, acc_j, dP_j)

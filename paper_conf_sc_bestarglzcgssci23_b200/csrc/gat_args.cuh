@@ -29,13 +29,18 @@ struct GatBwdArgs {
   float* ds_out;       // [n_local x NH] nullable
   float* dt_out;       // [n_local x NH] nullable
   float* ds_dir;       // [n_local x NH] directed patterns: row-pass ds for the column pass
+  const bf16* P16;     // BF16 mode (reading B1): P and G stored as bfloat16 (P, G unused)
+  const bf16* G16;
 };
 
 // k' = 128 kernels (gat_k128.cu): lane-parallel scalar work, warp-parallel rows
 bool gat_k128_supported(int k_out, int heads);
 agnn_status gat_fwd_k128(const Items& it, int heads, const float* P, const float* st, float slope,
                          int act, const GatFwdOut& o, int64_t n_rows, cudaStream_t s);
+// BF16 mode: P stored as bfloat16
+agnn_status gat_fwd_k128_bf16(const Items& it, int heads, const bf16* P, const float* st,
+                              float slope, int act, const GatFwdOut& o, cudaStream_t s);
 agnn_status gat_bwd_k128(const Items& it, int heads, const GatBwdArgs& A, int64_t* warps,
-                         cudaStream_t s);
+                         cudaStream_t s);  // A.P16 != NULL: BF16 mode
 
 }  // namespace agnn

@@ -54,10 +54,46 @@ __device__ __forceinline__ void load_n(const float* p, float (&x)[N]) {
   }
 }
 
+// fp32 rows, or bfloat16 rows (BF16 mode, reading B1): same code, the gathers
+// widen 4 bf16 (8 bytes) to a float4 (common.cuh ldg4 overloads)
+template <typename TP>
+__device__ __forceinline__ const TP* pick(const float* f, const bf16* h);
+template <>
+__device__ __forceinline__ const float* pick<float>(const float* f, const bf16*) { return f; }
+template <>
+__device__ __forceinline__ const bf16* pick<bf16>(const float*, const bf16* h) { return h; }
+
+// a gathered 4-column slice of a feature row as loaded (raw) and widened to fp32:
+// bf16 slices stay packed (2 registers) until their use, so twice as many rows
+// can be in flight per lane for the same registers
+template <typename TP>
+struct Slice;
+template <>
+struct Slice<float> {
+  using raw = float4;
+  __device__ static __forceinline__ raw load(const float* p) { return ldg4(p); }
+  __device__ static __forceinline__ float4 f(raw r) { return r; }
+  __device__ static __forceinline__ raw zero() { return f4(0.f); }
+};
+template <>
+struct Slice<bf16> {
+  using raw = uint2;
+  __device__ static __forceinline__ raw load(const bf16* p) {
+    return __ldg(reinterpret_cast<const uint2*>(p));
+  }
+  __device__ static __forceinline__ float4 f(raw r) { return bf4_to_f4(r); }
+  __device__ static __forceinline__ raw zero() { return make_uint2(0u, 0u); }
+};
+
 // ---------------------------------------------------------------- forward
-template <int NH, int U, int MINB>
+// rows per gather group of the full-batch path: 4 fp32 rows (2 KB) or 8 bf16 rows
+// (2 KB) per lane-slice group, two groups in flight
+template <typename TP>
+constexpr int fwd_group() { return sizeof(TP) == 2 ? 8 : 4; }
+
+template <typename TP, int NH, int U, int MINB>
 __global__ void __launch_bounds__(256, MINB)
-gat_fwd_k128_kernel(Items it, const float* __restrict__ P, const float* __restrict__ st,
+gat_fwd_k128_kernel(Items it, const TP* __restrict__ P, const float* __restrict__ st,
                     float slope, int act, GatFwdOut o) {
   constexpr int D = K / NH, HL = D / 4;
   __shared__ float sPw[8][NH][33];  // +1: heads read different rows without bank conflicts
@@ -85,10 +121,11 @@ gat_fwd_k128_kernel(Items it, const float* __restrict__ P, const float* __restri
       sJ[wib][lane] = j;
       __syncwarp();
       // the first U neighbour rows are in flight while the scores are computed
-      float4 pv[U];
+      using SL = Slice<TP>;
+      typename SL::raw pv[U];
 #pragma unroll
       for (int u = 0; u < U; ++u)
-        pv[u] = u < cnt ? ldg4(P + (int64_t)sJ[wib][u] * K + cq) : f4(0.f);
+        pv[u] = u < cnt ? SL::load(P + (int64_t)sJ[wib][u] * K + cq) : SL::zero();
       float tj[NH];
       load_n<NH>(st + (int64_t)j * (2 * NH) + NH, tj);
       float sch = 1.f;
@@ -111,25 +148,29 @@ gat_fwd_k128_kernel(Items it, const float* __restrict__ P, const float* __restri
       acc = mul4(sch, acc);
       __syncwarp();
       if (cnt == 32) {
-        // full batch: 8 groups of 4 rows, the next group in flight during this group's FMAs
-        const float* Pl = P + cq;
-        float4 qa[4], qb[4];
+        // full batch: 32/GR groups of GR rows, the next group in flight during this
+        // group's FMAs
+        constexpr int GR = fwd_group<TP>(), NGR = 32 / GR;
+        static_assert(U >= GR, "the prefetch covers the first group");
+        const TP* Pl = P + cq;
+        typename SL::raw qa[GR], qb[GR];
 #pragma unroll
-        for (int u = 0; u < 4; ++u) qa[u] = pv[u];  // group 0 was prefetched before the scores
+        for (int u = 0; u < GR; ++u) qa[u] = pv[u];  // group 0 was prefetched before the scores
 #pragma unroll
-        for (int g = 0; g < 8; g += 2) {
+        for (int g = 0; g < NGR; g += 2) {
 #pragma unroll
-          for (int u = 0; u < 4; ++u)
-            qb[u] = ldg4(Pl + (int64_t)(uint32_t)__shfl_sync(FULL, j, 4 * g + 4 + u) * K);
+          for (int u = 0; u < GR; ++u)
+            qb[u] = SL::load(Pl + (int64_t)(uint32_t)__shfl_sync(FULL, j, GR * g + GR + u) * K);
 #pragma unroll
-          for (int u = 0; u < 4; ++u) acc = fma4(sPw[wib][hv][4 * g + u], qa[u], acc);
-          if (g + 2 < 8) {
+          for (int u = 0; u < GR; ++u) acc = fma4(sPw[wib][hv][GR * g + u], SL::f(qa[u]), acc);
+          if (g + 2 < NGR) {
 #pragma unroll
-            for (int u = 0; u < 4; ++u)
-              qa[u] = ldg4(Pl + (int64_t)(uint32_t)__shfl_sync(FULL, j, 4 * g + 8 + u) * K);
+            for (int u = 0; u < GR; ++u)
+              qa[u] = SL::load(Pl + (int64_t)(uint32_t)__shfl_sync(FULL, j, GR * g + 2 * GR + u) * K);
           }
 #pragma unroll
-          for (int u = 0; u < 4; ++u) acc = fma4(sPw[wib][hv][4 * g + 4 + u], qb[u], acc);
+          for (int u = 0; u < GR; ++u)
+            acc = fma4(sPw[wib][hv][GR * g + GR + u], SL::f(qb[u]), acc);
         }
       } else {
         for (int k = 0; k < cnt; k += U) {
@@ -137,11 +178,11 @@ gat_fwd_k128_kernel(Items it, const float* __restrict__ P, const float* __restri
 #pragma unroll
           for (int u = 0; u < U; ++u) {
             const int kk = k + u;
-            if (k > 0) pv[u] = kk < cnt ? ldg4(P + (int64_t)sJ[wib][kk] * K + cq) : f4(0.f);
+            if (k > 0) pv[u] = kk < cnt ? SL::load(P + (int64_t)sJ[wib][kk] * K + cq) : SL::zero();
             pw[u] = kk < cnt ? sPw[wib][hv][kk] : 0.f;
           }
 #pragma unroll
-          for (int u = 0; u < U; ++u) acc = fma4(pw[u], pv[u], acc);
+          for (int u = 0; u < U; ++u) acc = fma4(pw[u], SL::f(pv[u]), acc);
         }
       }
       __syncwarp();
@@ -359,14 +400,14 @@ gat_fwd_tma_kernel(const __grid_constant__ CUtensorMap mapP, Items it, const flo
 }
 
 // ---------------------------------------------------------------- backward
-template <int B>
-struct BwdBatch {  // operands of one batch of B edges held by one lane
-  float4 Pi[B], Gi[B];
+template <typename TP, int B>
+struct BwdBatch {  // operands of one batch of B edges held by one lane (raw slices)
+  typename Slice<TP>::raw Pi[B], Gi[B];
   float4 ri;
   float ti;
 };
 
-template <int NH, int B, int MINB>
+template <typename TP, int NH, int B, int MINB>
 __global__ void __launch_bounds__(256, MINB)
 gat_bwd_k128_kernel(Items it, GatBwdArgs A) {
   constexpr int D = K / NH, HL = D / 4;
@@ -380,31 +421,34 @@ gat_bwd_k128_kernel(Items it, GatBwdArgs A) {
   const int64_t nitems = it.n_chunks + it.n_light;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  const float* Pl = A.P + cq;
-  const float* Gl = A.G + cq;
+  const TP* Pb = pick<TP>(A.P, A.P16);
+  const TP* Gb = pick<TP>(A.G, A.G16);
+  const TP* Pl = Pb + cq;
+  const TP* Gl = Gb + cq;
   float4 da1 = f4(0.f), da2 = f4(0.f);
 
   for (int64_t w = gw; w < nitems; w += nw) {
     int64_t row, beg, end, slot;
     item_of(it, w, row, beg, end, slot);
     const int64_t grow = it.row_begin + row;
-    const float4 Pj = ldg4(A.P + grow * K + cq);
-    const float4 Gj = ldg4(A.G + grow * K + cq);
+    const float4 Pj = ldg4(Pb + grow * K + cq);
+    const float4 Gj = ldg4(Gb + grow * K + cq);
     const float4 rj = __ldg(A.rec + grow * NH + hv);        // {s_j, m_j, 1/l_j, delta_j}
     const float tj = __ldg(A.st + grow * (2 * NH) + NH + hv);
     float4 acc = f4(0.f);
     float dsp = 0.f, dtp = 0.f;
     // gathers of batch (window offset off, cnt valid edges): rows i of P, G and the
     // record of the edge this lane owns after the reduction
-    auto load = [&](BwdBatch<B>& q, int cidx, int off, int cnt) {
+    using SL = Slice<TP>;
+    auto load = [&](BwdBatch<TP, B>& q, int cidx, int off, int cnt) {
 #pragma unroll
       for (int b = 0; b < B; ++b) {
         const uint32_t i = (uint32_t)__shfl_sync(FULL, cidx, off + b);
         if (b < cnt) {
-          q.Pi[b] = ldg4(Pl + (int64_t)i * K);
-          q.Gi[b] = ldg4(Gl + (int64_t)i * K);
+          q.Pi[b] = SL::load(Pl + (int64_t)i * K);
+          q.Gi[b] = SL::load(Gl + (int64_t)i * K);
         } else {
-          q.Pi[b] = q.Gi[b] = f4(0.f);
+          q.Pi[b] = q.Gi[b] = SL::zero();
         }
       }
       const uint32_t im = (uint32_t)__shfl_sync(FULL, cidx, off + my_b);
@@ -412,12 +456,12 @@ gat_bwd_k128_kernel(Items it, GatBwdArgs A) {
       q.ri = vm ? __ldg(A.rec + (int64_t)im * NH + hv) : f4(0.f);
       q.ti = vm ? __ldg(A.st + (int64_t)im * (2 * NH) + NH + hv) : 0.f;
     };
-    auto body = [&](const BwdBatch<B>& q, int cnt) {
+    auto body = [&](const BwdBatch<TP, B>& q, int cnt) {
       float x1[B], x2[B];
 #pragma unroll
       for (int b = 0; b < B; ++b) {
-        x1[b] = dot4(Gj, q.Pi[b]);  // G_j . P_i  (row role)
-        x2[b] = dot4(q.Gi[b], Pj);  // G_i . P_j  (column role)
+        x1[b] = dot4(Gj, SL::f(q.Pi[b]));  // G_j . P_i  (row role)
+        x2[b] = dot4(SL::f(q.Gi[b]), Pj);  // G_i . P_j  (column role)
       }
       TR::template reduce<HL>(x1, lane);
       TR::template reduce<HL>(x2, lane);
@@ -440,7 +484,7 @@ gat_bwd_k128_kernel(Items it, GatBwdArgs A) {
 #pragma unroll
       for (int b = 0; b < B; ++b) {
         const float ab = __shfl_sync(FULL, aij, gbase + TR::lane_of(b));
-        acc = fma4(ab, q.Gi[b], acc);
+        acc = fma4(ab, SL::f(q.Gi[b]), acc);
       }
     };
     for (int64_t w0 = beg; w0 < end; w0 += 32) {
@@ -448,7 +492,7 @@ gat_bwd_k128_kernel(Items it, GatBwdArgs A) {
       const int cidx = lane < wcnt ? __ldg(it.col + w0 + lane) : 0;
       if (wcnt == 32) {
         // full window: 32/B batches, the next batch's gathers in flight during this one
-        BwdBatch<B> qa, qb;
+        BwdBatch<TP, B> qa, qb;
         load(qa, cidx, 0, B);
 #pragma unroll
         for (int bb = 0; bb < 32 / B; bb += 2) {
@@ -459,7 +503,7 @@ gat_bwd_k128_kernel(Items it, GatBwdArgs A) {
         }
       } else {
         for (int off = 0; off < wcnt; off += B) {
-          BwdBatch<B> q;
+          BwdBatch<TP, B> q;
           const int cnt = wcnt - off < B ? wcnt - off : B;
           load(q, cidx, off, cnt);
           body(q, cnt);
@@ -514,6 +558,10 @@ bool gat_k128_supported(int k_out, int heads) {
 
 template <int NH>
 constexpr int bwd_batch() { return (K / NH / 4) >= 4 ? 4 : K / NH / 4; }
+// bf16 rows are half the bytes: 8 edges per batch (one per lane of a head group
+// when HL = 8) keep as many bytes in flight per lane as 4 fp32 edges
+template <int NH>
+constexpr int bwd_batch_bf16() { return (K / NH / 4) >= 8 ? 8 : K / NH / 4; }
 
 PFN_cuTensorMapEncodeTiled_v12000 tmap_encoder() {
   static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
@@ -580,14 +628,35 @@ agnn_status gat_fwd_k128(const Items& it, int heads, const float* P, const float
   }
   AGNN_K128_DISPATCH(heads, ({
     if (minb == 4) {
-      gat_fwd_k128_kernel<NH, 4, 4><<<grid_for(gat_fwd_k128_kernel<NH, 4, 4>), 256, 0, s>>>(
-          it, P, st, slope, act, o);
+      gat_fwd_k128_kernel<float, NH, 4, 4><<<grid_for(gat_fwd_k128_kernel<float, NH, 4, 4>), 256,
+                                             0, s>>>(it, P, st, slope, act, o);
     } else if (minb == 2) {
-      gat_fwd_k128_kernel<NH, 4, 2><<<grid_for(gat_fwd_k128_kernel<NH, 4, 2>), 256, 0, s>>>(
-          it, P, st, slope, act, o);
+      gat_fwd_k128_kernel<float, NH, 4, 2><<<grid_for(gat_fwd_k128_kernel<float, NH, 4, 2>), 256,
+                                             0, s>>>(it, P, st, slope, act, o);
     } else {
-      gat_fwd_k128_kernel<NH, 4, 3><<<grid_for(gat_fwd_k128_kernel<NH, 4, 3>), 256, 0, s>>>(
-          it, P, st, slope, act, o);
+      gat_fwd_k128_kernel<float, NH, 4, 3><<<grid_for(gat_fwd_k128_kernel<float, NH, 4, 3>), 256,
+                                             0, s>>>(it, P, st, slope, act, o);
+    }
+    AGNN_LAUNCH_CHECK("gat_fwd_kernel");
+  }));
+  return AGNN_OK;
+}
+
+agnn_status gat_fwd_k128_bf16(const Items& it, int heads, const bf16* P, const float* st,
+                              float slope, int act, const GatFwdOut& o, cudaStream_t s) {
+  if (it.n_chunks + it.n_light == 0) return AGNN_OK;
+  static int minb = -1;
+  if (minb < 0) {
+    const char* e = getenv("AGNN_FWD_MINB");
+    minb = e ? atoi(e) : 3;
+  }
+  AGNN_K128_DISPATCH(heads, ({
+    if (minb == 4) {
+      gat_fwd_k128_kernel<bf16, NH, 8, 4><<<grid_for(gat_fwd_k128_kernel<bf16, NH, 8, 4>), 256, 0,
+                                            s>>>(it, P, st, slope, act, o);
+    } else {
+      gat_fwd_k128_kernel<bf16, NH, 8, 3><<<grid_for(gat_fwd_k128_kernel<bf16, NH, 8, 3>), 256, 0,
+                                            s>>>(it, P, st, slope, act, o);
     }
     AGNN_LAUNCH_CHECK("gat_fwd_kernel");
   }));
@@ -604,13 +673,22 @@ agnn_status gat_bwd_k128(const Items& it, int heads, const GatBwdArgs& A, int64_
   }
   AGNN_K128_DISPATCH(heads, ({
     constexpr int B = bwd_batch<NH>();
+    constexpr int B16 = bwd_batch_bf16<NH>();
     int grid;
-    if (minb == 3) {
-      grid = grid_for(gat_bwd_k128_kernel<NH, B, 3>);
-      gat_bwd_k128_kernel<NH, B, 3><<<grid, 256, 0, s>>>(it, A);
+    if (A.P16) {  // BF16 mode (reading B1)
+      if (minb == 3) {
+        grid = grid_for(gat_bwd_k128_kernel<bf16, NH, B16, 3>);
+        gat_bwd_k128_kernel<bf16, NH, B16, 3><<<grid, 256, 0, s>>>(it, A);
+      } else {
+        grid = grid_for(gat_bwd_k128_kernel<bf16, NH, B16, 2>);
+        gat_bwd_k128_kernel<bf16, NH, B16, 2><<<grid, 256, 0, s>>>(it, A);
+      }
+    } else if (minb == 3) {
+      grid = grid_for(gat_bwd_k128_kernel<float, NH, B, 3>);
+      gat_bwd_k128_kernel<float, NH, B, 3><<<grid, 256, 0, s>>>(it, A);
     } else {
-      grid = grid_for(gat_bwd_k128_kernel<NH, B, 2>);
-      gat_bwd_k128_kernel<NH, B, 2><<<grid, 256, 0, s>>>(it, A);
+      grid = grid_for(gat_bwd_k128_kernel<float, NH, B, 2>);
+      gat_bwd_k128_kernel<float, NH, B, 2><<<grid, 256, 0, s>>>(it, A);
     }
     AGNN_LAUNCH_CHECK("gat_bwd_kernel");
     *warps = (int64_t)grid * 8;

@@ -4,6 +4,8 @@
 // Exact fp32 arithmetic (one rounding per FMA), 128x128 block tiles, 8x8 register
 // micro-tiles, register-prefetched 8-deep K slices.  These are the fp32-accurate
 // path; the tcgen05 3xTF32 GEMM (gemm_tc.cu) replaces gemm_rows where enabled.
+#include <algorithm>
+
 #include "internal.cuh"
 
 namespace agnn {
@@ -202,7 +204,33 @@ __global__ void sum_splits_kernel(const float* __restrict__ part, int splits, in
 
 agnn_status gemm_tc(const float* A, int64_t M, int K, const float* B, int n_real, float* C0,
                     int n_split, float* C1, int n_store, float* Cact, int act, cudaStream_t s,
-                    const PeerOut* peers);
+                    const PeerOut* peers, bf16* C0h = nullptr);
+
+namespace {
+// Y[i] = bf16_rn(X[i]) over rows x cols (cols % 4 == 0)
+__global__ void to_bf16_kernel(const float* __restrict__ X, int64_t count4, bf16* __restrict__ Y) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < count4;
+       i += (int64_t)gridDim.x * blockDim.x)
+    st4(Y + 4 * i, ldg4(X + 4 * i));
+}
+}  // namespace
+
+agnn_status gemm_rows_bf16(const float* A, int64_t M, int K, const float* B, int N, bf16* C0h,
+                           int n_split, float* C1, float* scratch, cudaStream_t s) {
+  if (M <= 0) return AGNN_OK;
+  agnn_status st = gemm_tc(A, M, K, B, N, nullptr, n_split, C1, N, nullptr, 0, s, nullptr, C0h);
+  if (st != AGNN_EUNSUPPORTED) return st;
+  // no tcgen05 instantiation for this shape: fp32 product into scratch, then round
+  // (B has (N + 3) / 4 * 4 rows, the padding rows zero; columns >= N are not stored)
+  if ((st = gemm_rows(A, M, K, B, true, (N + 3) / 4 * 4, scratch, n_split, C1, s, nullptr, 0, N)) !=
+      AGNN_OK)
+    return st;
+  const int64_t c4 = M * n_split / 4;
+  to_bf16_kernel<<<(unsigned)std::min<int64_t>((c4 + 255) / 256, kNumSMs * 16), 256, 0, s>>>(
+      scratch, c4, C0h);
+  AGNN_LAUNCH_CHECK("to_bf16_kernel");
+  return AGNN_OK;
+}
 
 agnn_status gemm_rows(const float* A, int64_t M, int K, const float* B, bool b_trans, int N,
                       float* C0, int n_split, float* C1, cudaStream_t s, float* Cact, int act,

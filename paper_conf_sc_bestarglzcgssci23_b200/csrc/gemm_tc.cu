@@ -166,7 +166,13 @@ struct TcOut {
   int npeer;                       // peer replicas also written (peer-memory exchange)
   float* pC0[kMaxPeers - 1];
   float* pC1[kMaxPeers - 1];
+  bf16* C0h;    // EPI_BF16: columns [0, n_split) stored as bfloat16 here instead of C0
 };
+
+// epilogue variants (compile time, so the plain fp32 epilogue carries neither)
+constexpr int EPI_PLAIN = 0;  // C0 | C1 fp32 (+ sigma copy)
+constexpr int EPI_PEER = 1;   // also every peer's replica (peer-memory all-gather)
+constexpr int EPI_BF16 = 2;   // C0 columns rounded to bfloat16 into C0h (reading B1)
 
 // 16 consecutive columns c0.. of output row `row` (C0 | C1 split, optional sigma copy).
 // PEER: the same values also go to every peer's replica (peer-memory all-gather);
@@ -198,11 +204,20 @@ __device__ __forceinline__ void store_row16_to(const TcOut& out, float* C0, floa
     }
   }
 }
-template <bool PEER>
+template <int EPI>
 __device__ __forceinline__ void store_row16(const TcOut& out, int64_t row, int c0,
                                             const float (&v)[16]) {
+  if constexpr (EPI == EPI_BF16) {
+#pragma unroll
+    for (int x = 0; x < 16; ++x) {
+      const int c = c0 + x;
+      if (c < out.n_split) out.C0h[row * out.n_split + c] = __float2bfloat16_rn(v[x]);
+      else if (c < out.n_store) out.C1[row * (out.n_store - out.n_split) + (c - out.n_split)] = v[x];
+    }
+    return;
+  }
   store_row16_to(out, out.C0, out.C1, out.Cact, row, c0, v);
-  if constexpr (PEER) {
+  if constexpr (EPI == EPI_PEER) {
 #pragma unroll 1
     for (int pi = 0; pi < out.npeer; ++pi)
       store_row16_to(out, out.pC0[pi], out.pC1[pi], nullptr, row, c0, v);
@@ -212,7 +227,7 @@ __device__ __forceinline__ void store_row16(const TcOut& out, int64_t row, int c
 // 32 columns [c0, c0+32) of the warp's 32 rows [row0, row0+32) through a per-warp
 // shared-memory transpose, so every store instruction writes 4 full 128-byte rows
 // (a thread-per-row store touches 32 lines per instruction, 8x the L2 write requests)
-template <bool PEER>
+template <int EPI>
 __device__ __forceinline__ void store_block32(const TcOut& out, int64_t row0, int64_t M, int c0,
                                               const float (&v)[32], float* stg, int lane) {
   // stg: [32 rows][36 floats] (16-byte aligned rows, 4-float pad against bank conflicts)
@@ -227,9 +242,13 @@ __device__ __forceinline__ void store_block32(const TcOut& out, int64_t row0, in
     const int64_t row = row0 + r;
     const float4 q = *reinterpret_cast<const float4*>(stg + r * 36 + cc);
     if (row < M) {
+      if constexpr (EPI == EPI_BF16) {
+        st4(out.C0h + row * out.n_split + c0 + cc, q);  // 8 lanes x 8 B: a 64-byte run per row
+        continue;
+      }
       if (out.C0) st4(out.C0 + row * out.n_split + c0 + cc, q);
       if (out.Cact) st4(out.Cact + row * out.n_split + c0 + cc, act_fwd4(out.act, q));
-      if constexpr (PEER) {
+      if constexpr (EPI == EPI_PEER) {
 #pragma unroll 1
         for (int pi = 0; pi < out.npeer; ++pi)  // peers' replicas (NVLink stores)
           st4(out.pC0[pi] + row * out.n_split + c0 + cc, q);
@@ -259,7 +278,7 @@ __device__ __forceinline__ void math_barrier() {  // the 128 math threads only
   asm volatile("bar.sync 1, 128;" ::: "memory");
 }
 
-template <int N, int K, int S, bool SB, bool PEER>
+template <int N, int K, int S, bool SB, int EPI>
 __global__ void __launch_bounds__(TC_WS_THREADS, 1)
 gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                const float* __restrict__ B, int n_real, int64_t M, TcOut out) {
@@ -472,14 +491,14 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
             float q[32];
 #pragma unroll
             for (int x = 0; x < 32; ++x) q[x] = v[c0 + x];
-            store_block32<PEER>(out, row0, M, h0 + c0, q, stg + ew * 32 * 36, lane);
+            store_block32<EPI>(out, row0, M, h0 + c0, q, stg + ew * 32 * 36, lane);
           } else if (row < M) {
 #pragma unroll
             for (int c1 = c0; c1 < c0 + 32 && c1 < NP; c1 += 16) {
               float q[16];
 #pragma unroll
               for (int x = 0; x < 16; ++x) q[x] = v[c1 + x];
-              store_row16<PEER>(out, row, h0 + c1, q);
+              store_row16<EPI>(out, row, h0 + c1, q);
             }
           }
         }
@@ -697,9 +716,11 @@ agnn_status launch_tc(const float* A, int64_t M, const float* B, int n_real, con
   static_assert(smem <= 232448 - 1024, "shared memory");
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(gemm_tc_kernel<N, K, S, SB, false>,
+    cudaFuncSetAttribute(gemm_tc_kernel<N, K, S, SB, EPI_PLAIN>,
                          cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    cudaFuncSetAttribute(gemm_tc_kernel<N, K, S, SB, true>,
+    cudaFuncSetAttribute(gemm_tc_kernel<N, K, S, SB, EPI_PEER>,
+                         cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    cudaFuncSetAttribute(gemm_tc_kernel<N, K, S, SB, EPI_BF16>,
                          cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     attr = true;
   }
@@ -708,10 +729,12 @@ agnn_status launch_tc(const float* A, int64_t M, const float* B, int n_real, con
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   const int64_t ntiles = (M + TC_BM - 1) / TC_BM;
   const int grid = (int)std::min<int64_t>(ntiles, sms);
-  if (o.npeer > 0)
-    gemm_tc_kernel<N, K, S, SB, true><<<grid, TC_WS_THREADS, smem, s>>>(ma, mb, B, n_real, M, o);
+  if (o.C0h)
+    gemm_tc_kernel<N, K, S, SB, EPI_BF16><<<grid, TC_WS_THREADS, smem, s>>>(ma, mb, B, n_real, M, o);
+  else if (o.npeer > 0)
+    gemm_tc_kernel<N, K, S, SB, EPI_PEER><<<grid, TC_WS_THREADS, smem, s>>>(ma, mb, B, n_real, M, o);
   else
-    gemm_tc_kernel<N, K, S, SB, false><<<grid, TC_WS_THREADS, smem, s>>>(ma, mb, B, n_real, M, o);
+    gemm_tc_kernel<N, K, S, SB, EPI_PLAIN><<<grid, TC_WS_THREADS, smem, s>>>(ma, mb, B, n_real, M, o);
   AGNN_LAUNCH_CHECK("gemm_tc_kernel");
   return AGNN_OK;
 }
@@ -810,11 +833,12 @@ agnn_status gemm_tn_tc(const float* A, int64_t M, int K1, const float* B, int N,
 // Returns AGNN_EUNSUPPORTED when the shape has no tcgen05 instantiation.
 agnn_status gemm_tc(const float* A, int64_t M, int K, const float* B, int n_real, float* C0,
                     int n_split, float* C1, int n_store, float* Cact, int act, cudaStream_t s,
-                    const PeerOut* peers) {
+                    const PeerOut* peers, bf16* C0h) {
   if (tc_disabled()) return AGNN_EUNSUPPORTED;
   if (M <= 0) return AGNN_OK;
   if ((reinterpret_cast<uintptr_t>(A) & 15) || (K % 32)) return AGNN_EUNSUPPORTED;
-  TcOut o{C0, C1, Cact, n_split, n_store, act, 0, {}, {}};
+  if (C0h && (peers || Cact || (n_split & 3))) return AGNN_EUNSUPPORTED;
+  TcOut o{C0, C1, Cact, n_split, n_store, act, 0, {}, {}, C0h};
   if (peers) {
     if (peers->n > kMaxPeers - 1 || (!C0 && peers->n > 0)) return AGNN_EUNSUPPORTED;
     o.npeer = peers->n;

@@ -60,6 +60,11 @@ agnn_status gemm_rows(const float* A, int64_t M, int K, const float* B, bool b_t
                       float* C0, int n_split, float* C1, cudaStream_t s, float* Cact = nullptr,
                       int act = 0, int n_store = 0, const PeerOut* peers = nullptr,
                       bool* peers_done = nullptr);
+// BF16 storage (reading B1): C = A * B^T with columns [0, n_split) rounded to bf16
+// into C0h (ld n_split) and [n_split, N) fp32 into C1 (ld N - n_split); scratch
+// [M x n_split] fp32 is used only when the shape has no tcgen05 instantiation.
+agnn_status gemm_rows_bf16(const float* A, int64_t M, int K, const float* B, int N, bf16* C0h,
+                           int n_split, float* C1, float* scratch, cudaStream_t s);
 // C[K1 x N] = A^T B over M rows (A [M x K1], B [M x N]); deterministic split-M with
 // partials in `ws` (gemm_tn_ws_floats) and an ordered reduction.  If accumulate,
 // C += result.
@@ -74,6 +79,7 @@ struct GatShape {
   int k_in, k_out, heads;
   float slope;
   int act;
+  bool bf16;  // AGNN_PREC_BF16: P and G stored as bfloat16 (reading B1)
 };
 size_t gat_saved_bytes(const Plan& p, const GatShape& g);
 size_t gat_workspace_bytes(const Plan& p, const GatShape& g);

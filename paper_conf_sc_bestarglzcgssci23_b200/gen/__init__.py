@@ -107,6 +107,7 @@ class Workload:
     train: bool = False   # step = fwd + bwd + SGD update (C4) instead of fwd + bwd
     agg: str = "sum"      # C-GNN aggregation semiring (model "cgnn")
     lr: float = 1e-3
+    prec: str = "fp32"    # "bf16": GAT P and G stored as bfloat16 (include/agnn.h AGNN_PREC_BF16)
 
     @property
     def kind(self) -> int:

@@ -77,7 +77,8 @@ class Stack:
         # symmetric=False: a directed pattern (reading A4); the plan builds its CSC
         self.plan = agnn.Plan(self.row_ptr, self.col_idx, w.n, b0, b1, symmetric=symmetric, rank=rank,
                               world=world, nccl_unique_id=nccl_uid, bounds=self.bounds)
-        descs = [agnn.layer_desc(w.model, w.k, w.k, w.heads, w.act, negative_slope=w.slope,
+        descs = [agnn.layer_desc(w.model, w.k, w.k, w.heads, w.act, prec=agnn.PREC[w.prec],
+                                 negative_slope=w.slope,
                                  beta=w.beta, eps=w.eps, agg=w.agg) for _ in range(w.layers)]
         self.model = agnn.Model(self.plan, descs)
         self._alloc(inputs_on_device)

@@ -8,6 +8,7 @@ import oracle
 from paper_conf_sc_bestarglzcgssci23_b200 import agnn, gen, runner
 
 TOL_FP32 = 1e-5  # north_star: "within 1e-5 relative in FP32" (normwise, SURVEY §8(c) parity protocol)
+TOL_BF16 = 1e-2  # north_star: "1e-2 with BF16 projection" (reading B1: oracle on the same bf16 rounding)
 
 
 def rel(x, y):
@@ -54,7 +55,8 @@ def oracle_step(w: gen.Workload, rp, ci, H, Ws, As, R):
     Hs, fwd = [np.asarray(H, np.float64)], []
     for l in range(w.layers):
         f, _ = oracle.layer(w.model, rp, ci, Hs[-1], Ws[l], As[l], w.heads, act=w.act,
-                            slope=w.slope, beta=w.beta, eps=w.eps, agg=w.agg)
+                            slope=w.slope, beta=w.beta, eps=w.eps, agg=w.agg,
+                            bf16=w.prec == "bf16")
         fwd.append(f)
         Hs.append(f["Hout"])
     dHs = [None] * (w.layers + 1)
@@ -63,7 +65,7 @@ def oracle_step(w: gen.Workload, rp, ci, H, Ws, As, R):
     for l in reversed(range(w.layers)):
         if w.model == "gat":
             b = oracle.gat_backward(rp, ci, Hs[l], Ws[l], As[l], w.heads, fwd[l], dHs[l + 1],
-                                    w.slope, w.act)
+                                    w.slope, w.act, bf16=w.prec == "bf16")
             das[l] = b["da"]
         elif w.model == "agnn":
             b = oracle.agnn_backward(rp, ci, Hs[l], Ws[l], fwd[l], dHs[l + 1], w.beta, w.eps, w.act)

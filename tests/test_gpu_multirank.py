@@ -26,6 +26,8 @@ CASES = {
     "gat-k64h2": gen.Workload("mr-gat", "gat", "kron", 13, 1 << 13, 8 << 13, 64, 2, 1, act="elu"),
     "gat-k128h4": gen.Workload("mr-gat128", "gat", "kron", 14, 1 << 14, 8 << 14, 128, 4, 1,
                                act="none"),
+    "gat-k128h4-bf16": gen.Workload("mr-gat128b", "gat", "kron", 14, 1 << 14, 8 << 14, 128, 4, 1,
+                                    act="elu", prec="bf16"),
     "agnn-k128-L2": gen.Workload("mr-agnn", "agnn", "rmat", 13, 1 << 13, 8 << 13, 128, 1, 2,
                                  act="elu"),
     "va-k64": gen.Workload("mr-va", "va", "kron", 13, 1 << 13, 8 << 13, 64, 1, 1, act="none"),
@@ -101,7 +103,7 @@ def test_peer_exchange_two_ranks_one_gpu(name):
     mp.spawn(_worker, args=(2, _free_port(), name), nprocs=2, join=True)
 
 
-@pytest.mark.parametrize("name", ["gat-k128h4", "agnn-k128-L2"])
+@pytest.mark.parametrize("name", ["gat-k128h4", "gat-k128h4-bf16", "agnn-k128-L2"])
 def test_peer_exchange_three_ranks_one_gpu(name):
     """Three ranks: uneven row blocks and two peers per rank in every exchange."""
     import torch.multiprocessing as mp
