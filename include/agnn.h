@@ -157,8 +157,10 @@ agnn_status agnn_plan_create(const agnn_csr* csr, const agnn_dist* dist /* NULL 
                              cudaStream_t stream, agnn_plan_t* out);
 agnn_status agnn_plan_destroy(agnn_plan_t plan);
 /* host-side statistics: [0]=n_local [1]=nnz_local [2]=light rows [3]=heavy rows
- * [4]=heavy chunks [5]=chunk size [6]=max degree [7]=n (global)            */
-agnn_status agnn_plan_info(agnn_plan_t plan, int64_t* info8);
+ * [4]=heavy chunks [5]=chunk size [6]=max degree [7]=n (global) [8]=short rows
+ * (light rows of degree <= [9], taken by the short-row kernels where a kernel
+ * has one) [9]=short_max (0: no split; AGNN_SHORT_EDGES overrides the default 32) */
+agnn_status agnn_plan_info(agnn_plan_t plan, int64_t* info10);
 
 /* The transposed pattern of the plan's CSR (test/utility; synchronises):
  * col_ptr [n+1] (device, int64), row_idx [nnz] (device, int32) list, for

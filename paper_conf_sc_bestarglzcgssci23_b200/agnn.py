@@ -241,10 +241,10 @@ class Plan:
         self.n_local = row_end - row_begin
 
     def info(self) -> dict:
-        a = (ctypes.c_int64 * 8)()
+        a = (ctypes.c_int64 * 10)()
         _check(lib().agnn_plan_info(self.handle, a))
         keys = ("n_local", "nnz", "light_rows", "heavy_rows", "heavy_chunks", "chunk", "max_degree",
-                "n")
+                "n", "short_rows", "short_max")
         return dict(zip(keys, list(a)))
 
     # ---- peer-memory exchange setup (world > 1 without an NCCL id) -------------

@@ -295,6 +295,8 @@ agnn_status agnn_plan_info(agnn_plan_t h, int64_t* info) {
   info[5] = p.chunk;
   info[6] = p.max_deg;
   info[7] = p.n;
+  info[8] = p.n_short;
+  info[9] = p.short_max;
   return AGNN_OK;
 }
 

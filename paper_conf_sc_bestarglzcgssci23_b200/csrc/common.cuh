@@ -83,6 +83,29 @@ __device__ __forceinline__ void st4(bf16* p, float4 v) {
 // the value a bf16 store of v holds, widened back (G~ of reading B1)
 __device__ __forceinline__ float4 round_bf4(float4 v) { return bf4_to_f4(f4_to_bf4(v)); }
 
+// a gathered 4-column slice of a feature row as loaded (raw) and widened to fp32:
+// bf16 slices stay packed (2 registers) until their use, so twice as many rows
+// can be in flight per lane for the same registers
+template <typename TP>
+struct Slice;
+template <>
+struct Slice<float> {
+  using raw = float4;
+  __device__ static __forceinline__ raw load(const float* p) { return ldg4(p); }
+  __device__ static __forceinline__ float4 f(raw r) { return r; }
+  __device__ static __forceinline__ raw zero() { return make_float4(0.f, 0.f, 0.f, 0.f); }
+};
+template <>
+struct Slice<bf16> {
+  using raw = uint2;
+  __device__ static __forceinline__ raw load(const bf16* p) {
+    return __ldg(reinterpret_cast<const uint2*>(p));
+  }
+  __device__ static __forceinline__ float4 f(raw r) { return bf4_to_f4(r); }
+  __device__ static __forceinline__ raw zero() { return make_uint2(0u, 0u); }
+};
+
+
 __device__ __forceinline__ float dot4(float4 a, float4 b) {
   return fmaf(a.x, b.x, fmaf(a.y, b.y, fmaf(a.z, b.z, a.w * b.w)));
 }
@@ -169,6 +192,12 @@ struct Plan {
   int32_t* heavy_rows = nullptr;      // [n_heavy]
   int32_t* heavy_off = nullptr;       // [n_heavy+1] chunk ranges
   void* meta_block = nullptr;         // single allocation backing the lists
+  // light rows split by degree for the short-row kernels (gat_short.cu):
+  // short = degree <= short_max, long = the other light rows (both ascending)
+  int short_max = 32;
+  int64_t n_short = 0, n_long = 0;
+  int32_t* short_rows = nullptr;
+  int32_t* long_rows = nullptr;
   int32_t* empty_rows = nullptr;      // [n_empty] local rows without stored entries
   int64_t n_empty = 0;
   // directed patterns (world == 1): the transposed pattern (CSC of the local

@@ -601,7 +601,7 @@ struct WsGat {
   float4* rec;
   void* saved_inf;  // saved-layout scratch for inference
 };
-int64_t da_rows() { return (int64_t)kMaxSparseBlocks * (kSparseThreads / 32) * 2; }
+int64_t da_rows() { return (int64_t)kMaxSparseBlocks * (kSparseThreads / 32) * 3; }
 
 WsGat carve_ws(const Plan& p, const GatShape& g, void* base, size_t* total) {
   Carver c(base);

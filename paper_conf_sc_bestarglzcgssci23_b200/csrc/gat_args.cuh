@@ -37,6 +37,21 @@ struct GatBwdArgs {
 bool gat_k128_supported(int k_out, int heads);
 agnn_status gat_fwd_k128(const Items& it, int heads, const float* P, const float* st, float slope,
                          int act, const GatFwdOut& o, int64_t n_rows, cudaStream_t s);
+// short rows (gat_short.cu): rows of it.short_rows, 4 rows per warp
+template <typename TP>
+agnn_status gat_fwd_short(const Items& it, int heads, const TP* P, const float* st, float slope,
+                          int act, const GatFwdOut& o, cudaStream_t s);
+agnn_status gat_bwd_short(const Items& it, int heads, const GatBwdArgs& A, int64_t da_row0,
+                          int64_t* warps, cudaStream_t s);
+// the k' = 128 row kernels take the long light rows; the short ones go to gat_short.cu
+inline Items long_items(const Items& it) {
+  Items r = it;
+  if (it.n_short > 0) {
+    r.light_rows = it.long_rows;
+    r.n_light = it.n_long;
+  }
+  return r;
+}
 // BF16 mode: P stored as bfloat16
 agnn_status gat_fwd_k128_bf16(const Items& it, int heads, const bf16* P, const float* st,
                               float slope, int act, const GatFwdOut& o, cudaStream_t s);

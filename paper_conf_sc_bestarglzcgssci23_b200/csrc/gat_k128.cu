@@ -63,28 +63,6 @@ __device__ __forceinline__ const float* pick<float>(const float* f, const bf16*)
 template <>
 __device__ __forceinline__ const bf16* pick<bf16>(const float*, const bf16* h) { return h; }
 
-// a gathered 4-column slice of a feature row as loaded (raw) and widened to fp32:
-// bf16 slices stay packed (2 registers) until their use, so twice as many rows
-// can be in flight per lane for the same registers
-template <typename TP>
-struct Slice;
-template <>
-struct Slice<float> {
-  using raw = float4;
-  __device__ static __forceinline__ raw load(const float* p) { return ldg4(p); }
-  __device__ static __forceinline__ float4 f(raw r) { return r; }
-  __device__ static __forceinline__ raw zero() { return f4(0.f); }
-};
-template <>
-struct Slice<bf16> {
-  using raw = uint2;
-  __device__ static __forceinline__ raw load(const bf16* p) {
-    return __ldg(reinterpret_cast<const uint2*>(p));
-  }
-  __device__ static __forceinline__ float4 f(raw r) { return bf4_to_f4(r); }
-  __device__ static __forceinline__ raw zero() { return make_uint2(0u, 0u); }
-};
-
 // ---------------------------------------------------------------- forward
 // rows per gather group of the full-batch path: 4 fp32 rows (2 KB) or 8 bf16 rows
 // (2 KB) per lane-slice group, two groups in flight
@@ -599,8 +577,11 @@ bool fwd_tma_enabled() {
   return v == 1;
 }
 
-agnn_status gat_fwd_k128(const Items& it, int heads, const float* P, const float* st, float slope,
-                         int act, const GatFwdOut& o, int64_t n_rows, cudaStream_t s) {
+agnn_status gat_fwd_k128(const Items& it_all, int heads, const float* P, const float* st,
+                         float slope, int act, const GatFwdOut& o, int64_t n_rows, cudaStream_t s) {
+  agnn_status sst = gat_fwd_short<float>(it_all, heads, P, st, slope, act, o, s);
+  if (sst != AGNN_OK) return sst;
+  const Items it = long_items(it_all);
   if (it.n_chunks + it.n_light == 0) return AGNN_OK;
   CUtensorMap map;
   if (fwd_tma_enabled() && row_gather_map(&map, P, n_rows)) {
@@ -642,8 +623,11 @@ agnn_status gat_fwd_k128(const Items& it, int heads, const float* P, const float
   return AGNN_OK;
 }
 
-agnn_status gat_fwd_k128_bf16(const Items& it, int heads, const bf16* P, const float* st,
+agnn_status gat_fwd_k128_bf16(const Items& it_all, int heads, const bf16* P, const float* st,
                               float slope, int act, const GatFwdOut& o, cudaStream_t s) {
+  agnn_status sst = gat_fwd_short<bf16>(it_all, heads, P, st, slope, act, o, s);
+  if (sst != AGNN_OK) return sst;
+  const Items it = long_items(it_all);
   if (it.n_chunks + it.n_light == 0) return AGNN_OK;
   static int minb = -1;
   if (minb < 0) {
@@ -663,9 +647,10 @@ agnn_status gat_fwd_k128_bf16(const Items& it, int heads, const bf16* P, const f
   return AGNN_OK;
 }
 
-agnn_status gat_bwd_k128(const Items& it, int heads, const GatBwdArgs& A, int64_t* warps,
+agnn_status gat_bwd_k128(const Items& it_all, int heads, const GatBwdArgs& A, int64_t* warps,
                          cudaStream_t s) {
   *warps = 0;
+  const Items it = long_items(it_all);
   static int minb = -1;
   if (minb < 0) {
     const char* e = getenv("AGNN_BWD_MINB");
@@ -693,7 +678,11 @@ agnn_status gat_bwd_k128(const Items& it, int heads, const GatBwdArgs& A, int64_
     AGNN_LAUNCH_CHECK("gat_bwd_kernel");
     *warps = (int64_t)grid * 8;
   }));
-  return AGNN_OK;
+  // short rows: their da partials follow the main kernel's rows
+  int64_t sw = 0;
+  agnn_status sst = gat_bwd_short(it_all, heads, A, *warps, &sw, s);
+  *warps += sw;
+  return sst;
 }
 
 }  // namespace agnn

@@ -19,6 +19,12 @@ struct Items {
   int64_t n_heavy;
   int64_t row_begin;          // global id of local row 0
   int64_t n_local;
+  // the light rows split by degree (kernels with a short-row variant): rows of degree
+  // <= the plan's short_max (short) and the others (long); items_of_csc: none
+  const int32_t* short_rows;
+  int64_t n_short;
+  const int32_t* long_rows;
+  int64_t n_long;
 };
 Items items_of(const Plan& p);
 // the transposed pattern's items (directed plans): "rows" are columns j, col = rows i

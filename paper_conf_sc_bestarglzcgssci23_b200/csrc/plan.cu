@@ -80,6 +80,10 @@ Items items_of(const Plan& p) {
   it.n_heavy = p.n_heavy;
   it.row_begin = p.row_begin;
   it.n_local = p.n_local;
+  it.short_rows = p.short_rows;
+  it.n_short = p.n_short;
+  it.long_rows = p.long_rows;
+  it.n_long = p.n_long;
   return it;
 }
 
@@ -87,17 +91,25 @@ namespace {
 
 // static work list of one pattern (rows of the CSR, or columns of the CSC)
 struct Lists {
-  int64_t n_light = 0, n_heavy = 0, n_chunks = 0, n_empty = 0, max_deg = 0;
+  int64_t n_light = 0, n_heavy = 0, n_chunks = 0, n_empty = 0, max_deg = 0, n_short = 0,
+          n_long = 0;
   int32_t *light = nullptr, *chunk_row = nullptr, *chunk_idx = nullptr, *heavy = nullptr,
-          *heavy_off = nullptr, *empty = nullptr;
+          *heavy_off = nullptr, *empty = nullptr, *short_rows = nullptr, *long_rows = nullptr;
   void* block = nullptr;
 };
 
 agnn_status build_lists(const std::vector<int64_t>& rp, int64_t n_rows, int chunk, bool with_empty,
-                        Lists& out, cudaStream_t s) {
-  std::vector<int32_t> light, chunk_row, chunk_idx, heavy, heavy_off{0}, empty;
+                        int short_max, Lists& out, cudaStream_t s) {
+  std::vector<int32_t> light, chunk_row, chunk_idx, heavy, heavy_off{0}, empty, shorts, longs;
   light.reserve((size_t)n_rows);
   int64_t maxdeg = 0;
+  // debug / measurement only (AGNN_DEBUG_SKIP_BELOW=d): light rows of degree < d get
+  // no work item, so their outputs are left unwritten; used to time the share of
+  // short rows in the sparse kernels, never in tests or the bench
+  static const int64_t skip_below = [] {
+    const char* e = getenv("AGNN_DEBUG_SKIP_BELOW");
+    return e ? (int64_t)atoll(e) : (int64_t)0;
+  }();
   for (int64_t i = 0; i < n_rows; ++i) {
     const int64_t d = rp[(size_t)i + 1] - rp[(size_t)i];
     maxdeg = std::max(maxdeg, d);
@@ -110,8 +122,9 @@ agnn_status build_lists(const std::vector<int64_t>& rp, int64_t n_rows, int chun
         chunk_idx.push_back((int32_t)q);
       }
       heavy_off.push_back((int32_t)chunk_row.size());
-    } else {
+    } else if (d >= skip_below) {
       light.push_back((int32_t)i);
+      if (short_max > 0) (d <= short_max ? shorts : longs).push_back((int32_t)i);
     }
   }
   out.max_deg = maxdeg;
@@ -119,8 +132,10 @@ agnn_status build_lists(const std::vector<int64_t>& rp, int64_t n_rows, int chun
   out.n_heavy = (int64_t)heavy.size();
   out.n_chunks = (int64_t)chunk_row.size();
   out.n_empty = (int64_t)empty.size();
+  out.n_short = (int64_t)shorts.size();
+  out.n_long = (int64_t)longs.size();
   const size_t total = light.size() + 2 * chunk_row.size() + heavy.size() + heavy_off.size() +
-                       empty.size() + 160;
+                       empty.size() + shorts.size() + longs.size() + 160;
   AGNN_CUDA_TRY(cudaMalloc(&out.block, sizeof(int32_t) * total));
   int32_t* b = static_cast<int32_t*>(out.block);
   auto put = [&](std::vector<int32_t>& v, int32_t*& dst) -> cudaError_t {
@@ -135,6 +150,8 @@ agnn_status build_lists(const std::vector<int64_t>& rp, int64_t n_rows, int chun
   AGNN_CUDA_TRY(put(heavy, out.heavy));
   AGNN_CUDA_TRY(put(heavy_off, out.heavy_off));
   AGNN_CUDA_TRY(put(empty, out.empty));
+  AGNN_CUDA_TRY(put(shorts, out.short_rows));
+  AGNN_CUDA_TRY(put(longs, out.long_rows));
   AGNN_CUDA_TRY(cudaStreamSynchronize(s));  // the host vectors die here
   return AGNN_OK;
 }
@@ -156,6 +173,8 @@ Items items_of_csc(const Plan& p) {
   it.n_heavy = p.c_heavy;
   it.row_begin = 0;
   it.n_local = p.n;
+  it.short_rows = it.long_rows = nullptr;
+  it.n_short = it.n_long = 0;
   return it;
 }
 
@@ -175,6 +194,13 @@ agnn_status plan_build(Plan& p, cudaStream_t s) {
   if (const char* env = getenv("AGNN_CHUNK_EDGES")) {
     const long v = atol(env);
     if (v >= 32 && v <= (1L << 30)) p.chunk = (int)v;
+  }
+  // short rows (degree <= short_max) go to the short-row kernels where a kernel has
+  // one (AGNN_SHORT_EDGES overrides; 0 disables the split).  A function of the degree
+  // only, like the chunks, so results do not depend on the number of GPUs.
+  if (const char* env = getenv("AGNN_SHORT_EDGES")) {
+    const long v = atol(env);
+    if (v >= 0 && v <= 64) p.short_max = (int)v;
   }
   // 1. validate on the device
   int* d_err = nullptr;
@@ -203,7 +229,7 @@ agnn_status plan_build(Plan& p, cudaStream_t s) {
   p.nnz = rp[(size_t)p.n_local];
   // 3. work lists of the rows
   Lists L;
-  agnn_status st = build_lists(rp, p.n_local, p.chunk, true, L, s);
+  agnn_status st = build_lists(rp, p.n_local, p.chunk, true, p.short_max, L, s);
   if (st != AGNN_OK) return st;
   p.max_deg = L.max_deg;
   p.n_light = L.n_light;
@@ -216,6 +242,10 @@ agnn_status plan_build(Plan& p, cudaStream_t s) {
   p.heavy_rows = L.heavy;
   p.heavy_off = L.heavy_off;
   p.empty_rows = L.empty;
+  p.n_short = L.n_short;
+  p.n_long = L.n_long;
+  p.short_rows = L.short_rows;
+  p.long_rows = L.long_rows;
   p.meta_block = L.block;
   // 4. directed pattern on one GPU: the CSC and its work lists (column role of the backward)
   if (p.directed() && p.world == 1 && p.n_local == p.n) {
@@ -231,7 +261,7 @@ agnn_status plan_build(Plan& p, cudaStream_t s) {
                                   cudaMemcpyDeviceToHost, s));
     AGNN_CUDA_TRY(cudaStreamSynchronize(s));
     Lists C;
-    if ((st = build_lists(cp, p.n, p.chunk, false, C, s)) != AGNN_OK) return st;
+    if ((st = build_lists(cp, p.n, p.chunk, false, 0, C, s)) != AGNN_OK) return st;
     p.c_light = C.n_light;
     p.c_heavy = C.n_heavy;
     p.c_chunks = C.n_chunks;

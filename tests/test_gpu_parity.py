@@ -68,6 +68,26 @@ def test_plan_info_and_heavy_rows():
     assert info["heavy_rows"] == int((deg > info["chunk"]).sum()) > 0
     assert info["heavy_chunks"] == int(np.ceil(deg[deg > info["chunk"]] / info["chunk"]).sum())
     assert info["light_rows"] + info["heavy_rows"] == w.n
+    # short rows (degree <= short_max) are a subset of the light rows
+    assert info["short_max"] == 32
+    assert info["short_rows"] == int((deg <= info["short_max"]).sum()) > 0
+
+
+@pytest.mark.parametrize("short", ["0", "4", "64"])
+def test_short_row_split_parity(short, monkeypatch):
+    """The short-row kernels (4 rows per warp) against the oracle for several
+    thresholds (0 = every light row through the warp-per-row kernels)."""
+    monkeypatch.setenv("AGNN_SHORT_EDGES", short)
+    for prec in ("fp32", "bf16"):
+        w = W("gat", "kron", 14, 8, 128, heads=4, act="none", prec=prec)
+        src, dst, rp, ci = pu.host_graph(w)
+        g = pu.device_graph(w, src, dst)
+        H, Ws, As, R = w.host_inputs()
+        st = pu.gpu_step(w, graph=g, R=R)
+        assert st.plan.info()["short_max"] == int(short)
+        ref = pu.oracle_step(w, rp, ci, H, Ws, As, R)
+        pu.compare(w, st, ref, tol=pu.TOL_FP32 if prec == "fp32" else pu.TOL_BF16)
+        pu.compare_attention(w, st, ref)
 
 
 # ------------------------------------------------------------------ layer parity
