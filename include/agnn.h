@@ -159,7 +159,8 @@ agnn_status agnn_plan_destroy(agnn_plan_t plan);
 /* host-side statistics: [0]=n_local [1]=nnz_local [2]=light rows [3]=heavy rows
  * [4]=heavy chunks [5]=chunk size [6]=max degree [7]=n (global) [8]=short rows
  * (light rows of degree <= [9], taken by the short-row kernels where a kernel
- * has one) [9]=short_max (0: no split; AGNN_SHORT_EDGES overrides the default 32) */
+ * has one) [9]=short_max (0: no split; AGNN_SHORT_EDGES overrides the default and
+ * maximum 32) */
 agnn_status agnn_plan_info(agnn_plan_t plan, int64_t* info10);
 
 /* The transposed pattern of the plan's CSR (test/utility; synchronises):

@@ -262,6 +262,7 @@ agnn_status agnn_plan_create(const agnn_csr* csr, const agnn_dist* dist, cudaStr
       if (p.meta_block) cudaFree(p.meta_block);
       if (p.csc_block) cudaFree(p.csc_block);
       if (p.c_meta_block) cudaFree(p.c_meta_block);
+      if (p.short_block) cudaFree(p.short_block);
       delete[] p.bounds;
       delete h;
       return st;
@@ -279,6 +280,7 @@ agnn_status agnn_plan_destroy(agnn_plan_t h) {
   if (h->p.meta_block) cudaFree(h->p.meta_block);
   if (h->p.csc_block) cudaFree(h->p.csc_block);
   if (h->p.c_meta_block) cudaFree(h->p.c_meta_block);
+  if (h->p.short_block) cudaFree(h->p.short_block);
   delete[] h->p.bounds;
   delete h;
   return AGNN_OK;

@@ -198,6 +198,8 @@ struct Plan {
   int64_t n_short = 0, n_long = 0;
   int32_t* short_rows = nullptr;
   int32_t* long_rows = nullptr;
+  int4* short_meta = nullptr;         // [n_short] {row, degree, beg lo, beg hi}: one 16-B load
+  void* short_block = nullptr;        // backs short_meta
   int32_t* empty_rows = nullptr;      // [n_empty] local rows without stored entries
   int64_t n_empty = 0;
   // directed patterns (world == 1): the transposed pattern (CSC of the local

@@ -43,6 +43,10 @@ agnn_status gat_fwd_short(const Items& it, int heads, const TP* P, const float* 
                           int act, const GatFwdOut& o, cudaStream_t s);
 agnn_status gat_bwd_short(const Items& it, int heads, const GatBwdArgs& A, int64_t da_row0,
                           int64_t* warps, cudaStream_t s);
+// BF16 backward with cp.async staging (gat_async.cu); opt-in with AGNN_BWD_ASYNC=1
+bool gat_bwd_async_enabled();
+agnn_status gat_bwd_async(const Items& it, int heads, const GatBwdArgs& A, int64_t* warps,
+                          cudaStream_t s);
 // the k' = 128 row kernels take the long light rows; the short ones go to gat_short.cu
 inline Items long_items(const Items& it) {
   Items r = it;

@@ -92,10 +92,13 @@ gat_fwd_k128_kernel(Items it, const TP* __restrict__ P, const float* __restrict_
       lp[h] = 0.f;
     }
     float4 acc = f4(0.f);
+    // column ids one batch ahead: the next batch's ids load during this batch
+    int jpre = beg + lane < end ? __ldg(it.col + beg + lane) : 0;
     for (int64_t b0 = beg; b0 < end; b0 += 32) {
       const int cnt = (int)(end - b0 < 32 ? end - b0 : 32);
       const bool valid = lane < cnt;
-      const int j = valid ? __ldg(it.col + b0 + lane) : 0;
+      const int j = jpre;
+      jpre = b0 + 32 + lane < end ? __ldg(it.col + b0 + 32 + lane) : 0;
       sJ[wib][lane] = j;
       __syncwarp();
       // the first U neighbour rows are in flight while the scores are computed
@@ -465,9 +468,12 @@ gat_bwd_k128_kernel(Items it, GatBwdArgs A) {
         acc = fma4(ab, SL::f(q.Gi[b]), acc);
       }
     };
+    // column ids one window ahead: the next window's ids load during this window
+    int cpre = beg + lane < end ? __ldg(it.col + beg + lane) : 0;
     for (int64_t w0 = beg; w0 < end; w0 += 32) {
       const int wcnt = (int)(end - w0 < 32 ? end - w0 : 32);
-      const int cidx = lane < wcnt ? __ldg(it.col + w0 + lane) : 0;
+      const int cidx = cpre;
+      cpre = w0 + 32 + lane < end ? __ldg(it.col + w0 + 32 + lane) : 0;
       if (wcnt == 32) {
         // full window: 32/B batches, the next batch's gathers in flight during this one
         BwdBatch<TP, B> qa, qb;
@@ -651,6 +657,14 @@ agnn_status gat_bwd_k128(const Items& it_all, int heads, const GatBwdArgs& A, in
                          cudaStream_t s) {
   *warps = 0;
   const Items it = long_items(it_all);
+  if (A.P16 && gat_bwd_async_enabled()) {
+    agnn_status st = gat_bwd_async(it, heads, A, warps, s);
+    if (st != AGNN_OK) return st;
+    int64_t sw = 0;
+    st = gat_bwd_short(it_all, heads, A, *warps, &sw, s);
+    *warps += sw;
+    return st;
+  }
   static int minb = -1;
   if (minb < 0) {
     const char* e = getenv("AGNN_BWD_MINB");

@@ -65,88 +65,143 @@ struct Cols<bf16, V4> {
   }
 };
 
-template <typename TP>
-constexpr int fwd_u() { return sizeof(TP) == 2 ? 8 : 4; }
+template <typename TP, int U16>
+constexpr int fwd_u() { return sizeof(TP) == 2 ? U16 : 4; }
+
+constexpr int kMaxShort = 32;  // plan short_max <= 64 is clamped to this by the launcher
+
+// Software pipeline over a warp's rows (iteration k = RPW rows): the 16-byte record
+// {row, degree, beg} of iteration k+2 and the column ids of iteration k+1 load
+// while iteration k computes, so a short row costs one exposed latency (its
+// gathers) instead of a chain of four (row id, row_ptr, column ids, gathers).
+// Lane q of a row's SUB lanes holds the ids of edges q, q + SUB, ... (CW words).
+template <int SUB>
+struct RowPipe {
+  static constexpr int RPW = 32 / SUB, CW = kMaxShort / SUB;
+  const int4* meta;
+  const int32_t* col;
+  int64_t n;
+  int g, q;
+  __device__ __forceinline__ int4 rec(int64_t base) const {
+    const int64_t r = base + g;
+    return r < n ? __ldg(meta + r) : make_int4(0, 0, 0, 0);
+  }
+  __device__ static __forceinline__ int64_t beg_of(int4 m) {
+    return (int64_t)(((uint64_t)(uint32_t)m.w << 32) | (uint64_t)(uint32_t)m.z);
+  }
+  __device__ __forceinline__ void cols(int4 m, int (&c)[CW]) const {
+    const int64_t b = beg_of(m);
+#pragma unroll
+    for (int k = 0; k < CW; ++k) {
+      const int e = q + k * SUB;
+      c[k] = e < m.y ? __ldg(col + b + e) : -1;
+    }
+  }
+  // id of edge e of this lane's row, or -1 (e warp-uniform; register selects, no
+  // local-memory indexing)
+  __device__ __forceinline__ int id(const int (&c)[CW], int e, int lane) const {
+    const int w = e / SUB;
+    int v = c[0];
+#pragma unroll
+    for (int k = 1; k < CW; ++k) v = w == k ? c[k] : v;
+    return __shfl_sync(0xffffffffu, v, (lane & ~(SUB - 1)) + (e % SUB));
+  }
+};
 
 // ---------------------------------------------------------------- forward
-template <typename TP, int NH, int SUB, int MINB>
+template <typename TP, int NH, int SUB, int MINB, int U16>
 __global__ void __launch_bounds__(256, MINB)
-gat_fwd_short_kernel(const int64_t* __restrict__ row_ptr, const int32_t* __restrict__ col,
-                     const int32_t* __restrict__ rows, int64_t n_rows, int64_t row_begin,
-                     const TP* __restrict__ P, const float* __restrict__ st, float slope, int act,
-                     GatFwdOut o) {
+gat_fwd_short_kernel(const int4* __restrict__ meta, const int32_t* __restrict__ col,
+                     int64_t n_rows, int64_t row_begin, const TP* __restrict__ P,
+                     const float* __restrict__ st, float slope, int act, GatFwdOut o) {
   using LY = Lay<SUB>;
-  constexpr int RPW = LY::RPW, CPL = LY::CPL, V4 = LY::V4;
-  constexpr int D = K / NH, U = fwd_u<TP>();
+  using RP = RowPipe<SUB>;
+  constexpr int RPW = LY::RPW, CPL = LY::CPL, V4 = LY::V4, CW = RP::CW;
+  constexpr int D = K / NH, U = fwd_u<TP, U16>();
   static_assert(D >= CPL, "a lane's columns lie in one head");
+  static_assert(kMaxShort % U == 0, "whole batches");
   const int lane = threadIdx.x & 31, g = lane / SUB, q = lane % SUB;
   const int c0 = q * CPL, h = c0 / D;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  for (int64_t base = gw * RPW; base < n_rows; base += nw * RPW) {
-    const int64_t r = base + g;
-    const bool ok = r < n_rows;
-    int64_t row = 0, beg = 0, end = 0;
-    if (ok) {
-      row = rows[r];
-      beg = row_ptr[row];
-      end = row_ptr[row + 1];
-    }
-    const int deg = (int)(end - beg);
+  const int64_t step = nw * RPW;
+  const RP rp{meta, col, n_rows, g, q};
+  int64_t base = gw * RPW;
+  int4 m_cur = rp.rec(base), m_nxt = rp.rec(base + step);
+  int c_cur[CW];
+  rp.cols(m_cur, c_cur);
+  for (; base < n_rows; base += step) {
+    int c_nxt[CW];
+    rp.cols(m_nxt, c_nxt);
+    const int4 m_nn = rp.rec(base + 2 * step);
+    const bool ok = base + g < n_rows;
+    const int64_t row = m_cur.x;
+    const int deg = min(m_cur.y, kMaxShort);
+    const int maxdeg = __reduce_max_sync(FULL, deg);
     const int64_t grow = row_begin + row;
     const float si = ok ? __ldg(st + grow * (2 * NH) + h) : 0.f;
     float m = -INFINITY, l = 0.f;
     float4 acc[V4];
 #pragma unroll
     for (int v = 0; v < V4; ++v) acc[v] = f4(0.f);
-    for (int b0 = 0; b0 < deg; b0 += U) {
-      int j[U];
+#pragma unroll 1
+    for (int b0 = 0; b0 < maxdeg; b0 += U) {
+      {
+        int j[U];
 #pragma unroll
-      for (int u = 0; u < U; ++u) j[u] = b0 + u < deg ? __ldg(col + beg + b0 + u) : -1;
-      float tj[U];
-      Cols<TP, V4> pj[U];
+        for (int u = 0; u < U; ++u) j[u] = rp.id(c_cur, b0 + u, lane);
+        float tj[U];
+        Cols<TP, V4> pj[U];
 #pragma unroll
-      for (int u = 0; u < U; ++u) {
-        if (j[u] >= 0) {
-          tj[u] = __ldg(st + (int64_t)j[u] * (2 * NH) + NH + h);
-          pj[u].load(P + (int64_t)j[u] * K + c0);
-        } else {
-          tj[u] = 0.f;
-          pj[u].zero();
+        for (int u = 0; u < U; ++u) {
+          if (j[u] >= 0) {
+            tj[u] = __ldg(st + (int64_t)j[u] * (2 * NH) + NH + h);
+            pj[u].load(P + (int64_t)j[u] * K + c0);
+          } else {
+            tj[u] = 0.f;
+            pj[u].zero();
+          }
+        }
+        float e[U], bm = m;
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          const float pre = si + tj[u];
+          e[u] = j[u] >= 0 ? fmaxf(pre, slope * pre) : -INFINITY;  // LReLU, 0 <= slope <= 1
+          bm = fmaxf(bm, e[u]);
+        }
+        if (bm != -INFINITY) {  // this row has edges in the batch
+          const float sc = ex2(m - bm);  // 0 on the first batch (m = -inf)
+          l *= sc;
+#pragma unroll
+          for (int v = 0; v < V4; ++v) acc[v] = mul4(sc, acc[v]);
+          m = bm;
+#pragma unroll
+          for (int u = 0; u < U; ++u) {
+            const float p = ex2(e[u] - m);  // 0 for padding edges
+            l += p;
+#pragma unroll
+            for (int v = 0; v < V4; ++v) acc[v] = fma4(p, pj[u].get(v), acc[v]);
+          }
         }
       }
-      float e[U], bm = m;
+    }
+    if (ok) {
+      const float inv = l > 0.f ? 1.f / l : 0.f;
 #pragma unroll
-      for (int u = 0; u < U; ++u) {
-        const float pre = si + tj[u];
-        e[u] = j[u] >= 0 ? fmaxf(pre, slope * pre) : -INFINITY;  // LReLU, 0 <= slope <= 1
-        bm = fmaxf(bm, e[u]);
+      for (int v = 0; v < V4; ++v) {
+        const float4 z = mul4(inv, acc[v]);
+        if (o.Z) st4(o.Z + row * K + c0 + 4 * v, z);
+        st4(o.Hout + row * K + c0 + 4 * v, act_fwd4(act, z));
       }
-      const float sc = ex2(m - bm);  // 0 on the first batch (m = -inf)
-      l *= sc;
-#pragma unroll
-      for (int v = 0; v < V4; ++v) acc[v] = mul4(sc, acc[v]);
-      m = bm;
-#pragma unroll
-      for (int u = 0; u < U; ++u) {
-        const float p = ex2(e[u] - m);  // 0 for padding edges
-        l += p;
-#pragma unroll
-        for (int v = 0; v < V4; ++v) acc[v] = fma4(p, pj[u].get(v), acc[v]);
+      if (o.m && (c0 % D) == 0) {
+        o.m[row * NH + h] = l > 0.f ? m : 0.f;
+        o.l[row * NH + h] = l;
       }
     }
-    if (!ok) continue;
-    const float inv = l > 0.f ? 1.f / l : 0.f;
+    m_cur = m_nxt;
+    m_nxt = m_nn;
 #pragma unroll
-    for (int v = 0; v < V4; ++v) {
-      const float4 z = mul4(inv, acc[v]);
-      if (o.Z) st4(o.Z + row * K + c0 + 4 * v, z);
-      st4(o.Hout + row * K + c0 + 4 * v, act_fwd4(act, z));
-    }
-    if (o.m && (c0 % D) == 0) {
-      o.m[row * NH + h] = l > 0.f ? m : 0.f;
-      o.l[row * NH + h] = l;
-    }
+    for (int k = 0; k < CW; ++k) c_cur[k] = c_nxt[k];
   }
 }
 
@@ -160,33 +215,37 @@ __device__ __forceinline__ const bf16* pick_rows<bf16>(const float*, const bf16*
 
 template <typename TP, int NH, int SUB, int U, int MINB>
 __global__ void __launch_bounds__(256, MINB)
-gat_bwd_short_kernel(const int64_t* __restrict__ row_ptr, const int32_t* __restrict__ col,
-                     const int32_t* __restrict__ rows, int64_t n_rows, int64_t row_begin,
-                     GatBwdArgs A, int64_t da_row0) {
+gat_bwd_short_kernel(const int4* __restrict__ meta, const int32_t* __restrict__ col,
+                     int64_t n_rows, int64_t row_begin, GatBwdArgs A, int64_t da_row0) {
   using LY = Lay<SUB>;
-  constexpr int RPW = LY::RPW, CPL = LY::CPL, V4 = LY::V4;
+  using RP = RowPipe<SUB>;
+  constexpr int RPW = LY::RPW, CPL = LY::CPL, V4 = LY::V4, CW = RP::CW;
   constexpr int D = K / NH, HLS = D / CPL;  // HLS lanes share a head
   static_assert(D >= CPL, "a lane's columns lie in one head");
+  static_assert(kMaxShort % U == 0, "whole batches");
   const int lane = threadIdx.x & 31, g = lane / SUB, q = lane % SUB;
   const int c0 = q * CPL, h = c0 / D;
   const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const int64_t step = nw * RPW;
   const TP* Pb = pick_rows<TP>(A.P, A.P16);
   const TP* Gb = pick_rows<TP>(A.G, A.G16);
   const float slope = A.slope;
+  const RP rp{meta, col, n_rows, g, q};
   float4 da1[V4], da2[V4];
 #pragma unroll
   for (int v = 0; v < V4; ++v) da1[v] = da2[v] = f4(0.f);
-  for (int64_t base = gw * RPW; base < n_rows; base += nw * RPW) {
-    const int64_t r = base + g;
-    const bool ok = r < n_rows;
-    int64_t row = 0, beg = 0, end = 0;
-    if (ok) {
-      row = rows[r];
-      beg = row_ptr[row];
-      end = row_ptr[row + 1];
-    }
-    const int deg = (int)(end - beg);
+  int64_t base = gw * RPW;
+  int4 m_cur = rp.rec(base), m_nxt = rp.rec(base + step);
+  int c_cur[CW];
+  rp.cols(m_cur, c_cur);
+  for (; base < n_rows; base += step) {
+    int c_nxt[CW];
+    rp.cols(m_nxt, c_nxt);
+    const int4 m_nn = rp.rec(base + 2 * step);
+    const bool ok = base + g < n_rows;
+    const int64_t row = m_cur.x;
+    const int deg = min(m_cur.y, kMaxShort);
     const int maxdeg = __reduce_max_sync(FULL, deg);  // warp-uniform trip count (shuffles inside)
     const int64_t grow = row_begin + row;
     float4 Pj[V4], Gj[V4];
@@ -206,80 +265,88 @@ gat_bwd_short_kernel(const int64_t* __restrict__ row_ptr, const int32_t* __restr
 #pragma unroll
     for (int v = 0; v < V4; ++v) acc[v] = f4(0.f);
     float ds = 0.f, dt = 0.f;
+#pragma unroll 1
     for (int b0 = 0; b0 < maxdeg; b0 += U) {
-      int i[U];
+      {
+        int i[U];
 #pragma unroll
-      for (int u = 0; u < U; ++u) i[u] = b0 + u < deg ? __ldg(col + beg + b0 + u) : -1;
-      Cols<TP, V4> pi[U], gi[U];
-      float4 ri[U];
-      float ti[U];
-#pragma unroll
-      for (int u = 0; u < U; ++u) {
-        if (i[u] >= 0) {
-          pi[u].load(Pb + (int64_t)i[u] * K + c0);
-          gi[u].load(Gb + (int64_t)i[u] * K + c0);
-          ri[u] = __ldg(A.rec + (int64_t)i[u] * NH + h);
-          ti[u] = __ldg(A.st + (int64_t)i[u] * (2 * NH) + NH + h);
-        } else {
-          pi[u].zero();
-          gi[u].zero();
-          ri[u] = f4(0.f);
-          ti[u] = 0.f;
-        }
-      }
-      float x1[U], x2[U];
-#pragma unroll
-      for (int u = 0; u < U; ++u) {
-        float a = 0.f, b = 0.f;
-#pragma unroll
-        for (int v = 0; v < V4; ++v) {
-          a += dot4(Gj[v], pi[u].get(v));  // G_j . P_i  (row role)
-          b += dot4(gi[u].get(v), Pj[v]);  // G_i . P_j  (column role)
-        }
-        x1[u] = a;
-        x2[u] = b;
-      }
-#pragma unroll
-      for (int o = 1; o < HLS; o <<= 1) {
+        for (int u = 0; u < U; ++u) i[u] = rp.id(c_cur, b0 + u, lane);
+        Cols<TP, V4> pi[U], gi[U];
+        float4 ri[U];
+        float ti[U];
 #pragma unroll
         for (int u = 0; u < U; ++u) {
-          x1[u] += __shfl_xor_sync(FULL, x1[u], o);
-          x2[u] += __shfl_xor_sync(FULL, x2[u], o);
+          if (i[u] >= 0) {
+            pi[u].load(Pb + (int64_t)i[u] * K + c0);
+            gi[u].load(Gb + (int64_t)i[u] * K + c0);
+            ri[u] = __ldg(A.rec + (int64_t)i[u] * NH + h);
+            ti[u] = __ldg(A.st + (int64_t)i[u] * (2 * NH) + NH + h);
+          } else {
+            pi[u].zero();
+            gi[u].zero();
+            ri[u] = f4(0.f);
+            ti[u] = 0.f;
+          }
         }
-      }
+        float x1[U], x2[U];
 #pragma unroll
-      for (int u = 0; u < U; ++u) {
-        const bool vm = i[u] >= 0;
-        // row role: entry (j,i) of row j
-        const float pre = rj.x + ti[u];
-        const float e = fmaxf(pre, slope * pre);
-        const float aji = ex2(e - rj.y) * rj.z;
-        const float dcji = aji * (pre > 0.f ? 1.f : slope) * (x1[u] - rj.w);
-        // column role: entry (i,j) of row i
-        const float pre2 = ri[u].x + tj;
-        const float e2 = fmaxf(pre2, slope * pre2);
-        const float aij = ex2(e2 - ri[u].y) * ri[u].z;
-        const float dcij = aij * (pre2 > 0.f ? 1.f : slope) * (x2[u] - ri[u].w);
-        if (vm) {
-          ds += dcji;
-          dt += dcij;
+        for (int u = 0; u < U; ++u) {
+          float a = 0.f, b = 0.f;
 #pragma unroll
-          for (int v = 0; v < V4; ++v) acc[v] = fma4(aij, gi[u].get(v), acc[v]);
+          for (int v = 0; v < V4; ++v) {
+            a += dot4(Gj[v], pi[u].get(v));  // G_j . P_i  (row role)
+            b += dot4(gi[u].get(v), Pj[v]);  // G_i . P_j  (column role)
+          }
+          x1[u] = a;
+          x2[u] = b;
+        }
+#pragma unroll
+        for (int o = 1; o < HLS; o <<= 1) {
+#pragma unroll
+          for (int u = 0; u < U; ++u) {
+            x1[u] += __shfl_xor_sync(FULL, x1[u], o);
+            x2[u] += __shfl_xor_sync(FULL, x2[u], o);
+          }
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          const bool vm = i[u] >= 0;
+          // row role: entry (j,i) of row j
+          const float pre = rj.x + ti[u];
+          const float e = fmaxf(pre, slope * pre);
+          const float aji = ex2(e - rj.y) * rj.z;
+          const float dcji = aji * (pre > 0.f ? 1.f : slope) * (x1[u] - rj.w);
+          // column role: entry (i,j) of row i
+          const float pre2 = ri[u].x + tj;
+          const float e2 = fmaxf(pre2, slope * pre2);
+          const float aij = ex2(e2 - ri[u].y) * ri[u].z;
+          const float dcij = aij * (pre2 > 0.f ? 1.f : slope) * (x2[u] - ri[u].w);
+          if (vm) {
+            ds += dcji;
+            dt += dcij;
+#pragma unroll
+            for (int v = 0; v < V4; ++v) acc[v] = fma4(aij, gi[u].get(v), acc[v]);
+          }
         }
       }
     }
-    if (!ok) continue;
+    if (ok) {
 #pragma unroll
-    for (int v = 0; v < V4; ++v) {
-      const int cc = (c0 % D) + 4 * v;
-      const float4 a1v = ldg4(A.a + h * 2 * D + cc);
-      const float4 a2v = ldg4(A.a + h * 2 * D + D + cc);
-      float4 dp = fma4(ds, a1v, acc[v]);
-      dp = fma4(dt, a2v, dp);
-      st4(A.dP + row * K + c0 + 4 * v, dp);
-      da1[v] = fma4(ds, Pj[v], da1[v]);
-      da2[v] = fma4(dt, Pj[v], da2[v]);
+      for (int v = 0; v < V4; ++v) {
+        const int cc = (c0 % D) + 4 * v;
+        const float4 a1v = ldg4(A.a + h * 2 * D + cc);
+        const float4 a2v = ldg4(A.a + h * 2 * D + D + cc);
+        float4 dp = fma4(ds, a1v, acc[v]);
+        dp = fma4(dt, a2v, dp);
+        st4(A.dP + row * K + c0 + 4 * v, dp);
+        da1[v] = fma4(ds, Pj[v], da1[v]);
+        da2[v] = fma4(dt, Pj[v], da2[v]);
+      }
     }
+    m_cur = m_nxt;
+    m_nxt = m_nn;
+#pragma unroll
+    for (int k = 0; k < CW; ++k) c_cur[k] = c_nxt[k];
   }
   // the RPW row slots of the warp hold the same columns: fold them (fixed order), then
   // the first slot writes the warp's da partial row
@@ -327,9 +394,17 @@ agnn_status gat_fwd_short(const Items& it, int heads, const TP* P, const float* 
                           int act, const GatFwdOut& o, cudaStream_t s) {
   if (it.n_short == 0) return AGNN_OK;
   AGNN_SHORT_DISPATCH(heads, ({
-    auto* kern = gat_fwd_short_kernel<TP, NH, 8, 3>;
-    kern<<<grid_for(kern), 256, 0, s>>>(it.row_ptr, it.col, it.short_rows, it.n_short,
-                                         it.row_begin, P, st, slope, act, o);
+    static int minb = -1;  // AGNN_FWD_SHORT_MINB (measurement): resident 256-thread blocks
+    if (minb < 0) {
+      const char* e = getenv("AGNN_FWD_SHORT_MINB");
+      minb = e ? atoi(e) : 2;
+    }
+    // 3 blocks / SM with 4 bf16 rows per batch, or 2 blocks / SM with 8
+    // (fp32: 2 blocks / SM, 4 rows per batch; the 3-block variant spills)
+    auto* kern = (sizeof(TP) == 4 || minb == 2) ? gat_fwd_short_kernel<TP, NH, 8, 2, 8>
+                                                : gat_fwd_short_kernel<TP, NH, 8, 3, 4>;
+    kern<<<grid_for(kern), 256, 0, s>>>(it.short_meta, it.col, it.n_short, it.row_begin, P, st,
+                                         slope, act, o);
     AGNN_LAUNCH_CHECK("gat_fwd_short_kernel");
   }));
   return AGNN_OK;
@@ -355,8 +430,7 @@ agnn_status gat_bwd_short(const Items& it, int heads, const GatBwdArgs& A, int64
     if (A.P16) {
       auto launch = [&](auto* kern) {
         grid = grid_for(kern);
-        kern<<<grid, 256, 0, s>>>(it.row_ptr, it.col, it.short_rows, it.n_short, it.row_begin, A,
-                                  da_row0);
+        kern<<<grid, 256, 0, s>>>(it.short_meta, it.col, it.n_short, it.row_begin, A, da_row0);
       };
       if (variant == 1)
         launch(gat_bwd_short_kernel<bf16, NH, 8, 4, 1>);
@@ -367,8 +441,7 @@ agnn_status gat_bwd_short(const Items& it, int heads, const GatBwdArgs& A, int64
     } else {
       auto* kern = gat_bwd_short_kernel<float, NH, 16, 2, 2>;
       grid = grid_for(kern);
-      kern<<<grid, 256, 0, s>>>(it.row_ptr, it.col, it.short_rows, it.n_short, it.row_begin, A,
-                                da_row0);
+      kern<<<grid, 256, 0, s>>>(it.short_meta, it.col, it.n_short, it.row_begin, A, da_row0);
     }
     AGNN_LAUNCH_CHECK("gat_bwd_short_kernel");
     *warps = (int64_t)grid * 8;

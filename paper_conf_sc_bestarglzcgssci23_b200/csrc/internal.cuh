@@ -22,6 +22,7 @@ struct Items {
   // the light rows split by degree (kernels with a short-row variant): rows of degree
   // <= the plan's short_max (short) and the others (long); items_of_csc: none
   const int32_t* short_rows;
+  const int4* short_meta;     // per short row {row, degree, beg lo, beg hi}
   int64_t n_short;
   const int32_t* long_rows;
   int64_t n_long;

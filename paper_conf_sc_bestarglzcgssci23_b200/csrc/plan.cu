@@ -81,6 +81,7 @@ Items items_of(const Plan& p) {
   it.row_begin = p.row_begin;
   it.n_local = p.n_local;
   it.short_rows = p.short_rows;
+  it.short_meta = p.short_meta;
   it.n_short = p.n_short;
   it.long_rows = p.long_rows;
   it.n_long = p.n_long;
@@ -174,6 +175,7 @@ Items items_of_csc(const Plan& p) {
   it.row_begin = 0;
   it.n_local = p.n;
   it.short_rows = it.long_rows = nullptr;
+  it.short_meta = nullptr;
   it.n_short = it.n_long = 0;
   return it;
 }
@@ -199,8 +201,8 @@ agnn_status plan_build(Plan& p, cudaStream_t s) {
   // one (AGNN_SHORT_EDGES overrides; 0 disables the split).  A function of the degree
   // only, like the chunks, so results do not depend on the number of GPUs.
   if (const char* env = getenv("AGNN_SHORT_EDGES")) {
-    const long v = atol(env);
-    if (v >= 0 && v <= 64) p.short_max = (int)v;
+    const long v = atol(env);  // the short-row kernels take up to 32 edges per row
+    if (v >= 0) p.short_max = (int)(v < 32 ? v : 32);
   }
   // 1. validate on the device
   int* d_err = nullptr;
@@ -246,6 +248,25 @@ agnn_status plan_build(Plan& p, cudaStream_t s) {
   p.n_long = L.n_long;
   p.short_rows = L.short_rows;
   p.long_rows = L.long_rows;
+  if (p.n_short > 0) {
+    // {row, degree, beg} of every short row in one 16-byte record (the short-row
+    // kernels prefetch the next rows' records and column ids a step ahead)
+    std::vector<int4> meta((size_t)p.n_short);
+    std::vector<int32_t> srows((size_t)p.n_short);
+    AGNN_CUDA_TRY(cudaMemcpyAsync(srows.data(), p.short_rows, sizeof(int32_t) * srows.size(),
+                                  cudaMemcpyDeviceToHost, s));
+    AGNN_CUDA_TRY(cudaStreamSynchronize(s));
+    for (size_t x = 0; x < srows.size(); ++x) {
+      const int64_t r = srows[x], b = rp[(size_t)r];
+      meta[x] = make_int4(srows[x], (int)(rp[(size_t)r + 1] - b), (int)(uint32_t)(uint64_t)b,
+                          (int)(uint32_t)((uint64_t)b >> 32));
+    }
+    AGNN_CUDA_TRY(cudaMalloc(&p.short_block, sizeof(int4) * meta.size()));
+    p.short_meta = static_cast<int4*>(p.short_block);
+    AGNN_CUDA_TRY(cudaMemcpyAsync(p.short_meta, meta.data(), sizeof(int4) * meta.size(),
+                                  cudaMemcpyHostToDevice, s));
+    AGNN_CUDA_TRY(cudaStreamSynchronize(s));
+  }
   p.meta_block = L.block;
   // 4. directed pattern on one GPU: the CSC and its work lists (column role of the backward)
   if (p.directed() && p.world == 1 && p.n_local == p.n) {

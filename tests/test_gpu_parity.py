@@ -73,7 +73,7 @@ def test_plan_info_and_heavy_rows():
     assert info["short_rows"] == int((deg <= info["short_max"]).sum()) > 0
 
 
-@pytest.mark.parametrize("short", ["0", "4", "64"])
+@pytest.mark.parametrize("short", ["0", "4", "32"])
 def test_short_row_split_parity(short, monkeypatch):
     """The short-row kernels (4 rows per warp) against the oracle for several
     thresholds (0 = every light row through the warp-per-row kernels)."""
