@@ -5,9 +5,10 @@ names, which bench.py uses for roofline.traffic)."""
 import csv, json, re, sys, collections
 
 ALIAS = {"gat_bwd_k128_kernel": "gat_bwd_kernel", "gat_fwd_k128_kernel": "gat_fwd_kernel",
+         "gat_bwd_async_kernel": "gat_bwd_kernel",
          "av_bwd_k128_kernel": "av_bwd_kernel", "av_fwd_k128_kernel": "av_fwd_kernel",
          "gemm_tn_tc_kernel": "gemm_tn_kernel", "tn_sum_kernel": "sum_splits_kernel"}
-STEP = re.compile(r"(gat_|av_|gemm_|agnn_rec|nu_kernel|grad_act|sum_splits|tn_sum|sgd|transpose)")
+STEP = re.compile(r"(gat_|av_|gemm_|agnn_rec|nu_kernel|grad_act|sum_splits|tn_sum|sgd|transpose|to_bf16|cg_)")
 
 
 def short(name):
