@@ -224,64 +224,94 @@ def run_reference(args):
 
 
 # ----------------------------------------------------------------------------- ours
-def algorithmic_bytes(w, m, n):
-    """Bytes the dominant kernel must move per launch.
+def gat_factored(w):
+    """The factored GAT backward runs for k' = 128 on symmetric patterns (gat_args.cuh)."""
+    return (w.model == "gat" and w.k == 128 and w.heads in (1, 2, 4, 8)
+            and os.environ.get("AGNN_GAT_FACTORED", "1") != "0")
 
-    GAT backward sparse kernel, per stored edge: 4 B column index + the gathered
-    rows P_i and G_i (2 k' f) + the neighbour record {s,m,1/l,delta} (16 h) and
-    t_i (4 h); per row: P_j, G_j read, dP_j written (3 k' f) + own record/t
-    (20 h) + row_ptr (8 B).  AGNN/VA backward: per edge 4 + 2 k f (+16 AGNN
-    record); per row H_j, M_j read, dH_j written (3 k f) (+16) + 8.
+
+def pass_bytes(w, m, n):
+    """Algorithmic bytes of each sparse pass per launch:
+    {pass: (bytes, per stored edge, per row)}.  f = stored feature bytes (bf16 P, G
+    in BF16 mode, reading B1); outputs and dP are fp32.
+
+    GAT forward, per edge: 4 B column index + the gathered P_j row + t_j (4 h);
+      per row: s_i (4 h), Z_i and H_out_i written (2 k' 4), Q_i written when the
+      backward is factored (k' 4), m, l (8 h), row_ptr (8).
+    GAT backward, factored: per edge 4 + the gathered G_i row + rec_i (16 h); per
+      row P_j read, dP_j written, ds_j and t_j (8 h), row_ptr.
+    GAT backward, unfactored: per edge 4 + P_i and G_i rows + rec_i and t_i
+      (20 h); per row P_j, G_j read, dP_j written, record + t (20 h), row_ptr.
+    AGNN/VA backward: per edge 4 + 2 k f (+16 AGNN record); per row H_j, M_j read,
+      dH_j written (3 k f) (+16) + 8.
     """
     f = 4
+    out = {}
     if w.model == "gat":
-        fs = 2 if w.prec == "bf16" else 4   # stored P, G (reading B1); dP stays fp32
-        per_edge = 4 + 2 * w.k * fs + 20 * w.heads
-        per_row = 2 * w.k * fs + w.k * f + 20 * w.heads + 8
+        fs = 2 if w.prec == "bf16" else 4
+        fac = gat_factored(w)
+        pe = 4 + w.k * fs + 4 * w.heads
+        pr = 4 * w.heads + (3 if fac else 2) * w.k * f + 8 * w.heads + 8
+        out["fwd"] = (pe * m + pr * n, pe, pr)
+        if fac:
+            pe, pr = 4 + w.k * fs + 16 * w.heads, w.k * fs + w.k * f + 8 * w.heads + 8
+        else:
+            pe, pr = 4 + 2 * w.k * fs + 20 * w.heads, 2 * w.k * fs + w.k * f + 20 * w.heads + 8
+        out["bwd"] = (pe * m + pr * n, pe, pr)
     else:
         rec = 16 if w.model == "agnn" else 0
-        per_edge = 4 + 2 * w.k * f + rec
-        per_row = 3 * w.k * f + rec + 8
-    return per_edge * m + per_row * n, per_edge, per_row
+        pe, pr = 4 + 2 * w.k * f + rec, 3 * w.k * f + rec + 8
+        out["bwd"] = (pe * m + pr * n, pe, pr)
+    return out
 
 
-DOMINANT = {"gat": "gat_bwd_kernel", "agnn": "av_bwd_kernel", "va": "av_bwd_kernel"}
-# the launches of the dominant pass: the row kernel plus, where the plan splits rows by
-# degree, the short-row kernel (both cover the edges of algorithmic_bytes together)
-PASS = {"gat": ("gat_bwd_kernel", "gat_bwd_short_kernel")}
+# the launches of each sparse pass: the row kernel plus, where the plan splits rows by
+# degree, the short-row kernel (both cover the edges of pass_bytes together)
+PASSES = {"gat": {"bwd": ("gat_bwd_kernel", "gat_bwd_short_kernel"),
+                  "fwd": ("gat_fwd_kernel", "gat_fwd_short_kernel")},
+          "agnn": {"bwd": ("av_bwd_kernel",)}, "va": {"bwd": ("av_bwd_kernel",)}}
 
 
 def roofline(args, w, st, prof, world):
-    """Roofline object of the dominant kernel from the live per-kernel event profile."""
+    """Roofline object of the dominant sparse pass (largest share of the step) from the
+    live per-kernel event profile; every sparse pass is listed under "passes"."""
     peaks = measured_peaks()
     hbm = peaks.get("hbm_gbs")
     peak_src = "measured (MEASURED_PEAKS.json hbm_gbs)" if hbm else "fallback (B200_PROFILING.md)"
     hbm = hbm or 6650.0
-    dom = DOMINANT[w.model]
-    names = [k for k in PASS.get(w.model, (dom,)) if k in prof]
-    cnt = prof.get(dom, (0, 0.0))[0]
-    tot = sum(prof[k][1] for k in names)
-    alg, per_edge, per_row = algorithmic_bytes(w, st.nnz_local, st.n_local)
-    dom_ms = tot / cnt if cnt else None  # the pass per layer (its launches back to back)
-    # one launch per layer per step: alg bytes per launch over the mean launch time
-    achieved = (alg / (dom_ms / 1e3) / 1e9) if dom_ms else None
     step_ms_prof = sum(v[1] for v in prof.values()) / args.steps
-    traffic = None
-    try:  # ncu DRAM bytes per launch of the same kernel on the same workload (committed)
+    try:  # ncu DRAM bytes per launch of the same kernels on the same workload (committed)
         tr = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))
-        if args.scale is None and world == 1:
-            key = args.config + ("" if w.prec == "fp32" else "-" + w.prec)
-            per = tr.get(key, {})
-            traffic = sum(per[k] for k in names) if all(k in per for k in names) else None
+        key = args.config + ("" if w.prec == "fp32" else "-" + w.prec)
+        per = tr.get(key, {}) if (args.scale is None and world == 1) else {}
     except Exception:
-        traffic = None
-    return {"bound": "hbm", "kernel": "+".join(names) if names else dom, "achieved": achieved, "peak": hbm, "unit": "GB/s",
-            "frac": (achieved / hbm) if achieved else None, "traffic": traffic,
-            "dram_frac": (traffic / (dom_ms / 1e3) / 1e9 / hbm) if (traffic and dom_ms) else None,
+        per = {}
+    passes = {}
+    pb = pass_bytes(w, st.nnz_local, st.n_local)
+    for pname, kernels in PASSES.get(w.model, {}).items():
+        names = [k for k in kernels if k in prof]
+        if not names or pname not in pb:
+            continue
+        cnt = prof[names[0]][0]
+        tot = sum(prof[k][1] for k in names)
+        alg, per_edge, per_row = pb[pname]
+        ms = tot / cnt if cnt else None  # the pass per layer (its launches back to back)
+        achieved = (alg / (ms / 1e3) / 1e9) if ms else None
+        traffic = sum(per[k] for k in names) if names and all(k in per for k in names) else None
+        passes[pname] = {
+            "bound": "hbm", "kernel": "+".join(names), "achieved": achieved, "peak": hbm,
+            "unit": "GB/s", "frac": (achieved / hbm) if achieved else None, "traffic": traffic,
+            "dram_frac": (traffic / (ms / 1e3) / 1e9 / hbm) if (traffic and ms) else None,
             "peak_source": peak_src, "algorithmic_bytes_per_launch": alg,
-            "bytes_per_edge": per_edge, "bytes_per_row": per_row,
-            "launch_ms": dom_ms, "share_of_step": (tot / args.steps / step_ms_prof)
-            if step_ms_prof else None}
+            "bytes_per_edge": per_edge, "bytes_per_row": per_row, "launch_ms": ms,
+            "share_of_step": (tot / args.steps / step_ms_prof) if step_ms_prof else None}
+    if not passes:
+        return None
+    dom = max(passes, key=lambda k: passes[k]["share_of_step"] or 0)
+    r = dict(passes[dom])
+    r["pass"] = dom
+    r["passes"] = passes
+    return r
 
 
 def run_ours(args):

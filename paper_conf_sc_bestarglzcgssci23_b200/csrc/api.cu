@@ -263,6 +263,7 @@ agnn_status agnn_plan_create(const agnn_csr* csr, const agnn_dist* dist, cudaStr
       if (p.csc_block) cudaFree(p.csc_block);
       if (p.c_meta_block) cudaFree(p.c_meta_block);
       if (p.short_block) cudaFree(p.short_block);
+      if (p.col_hint) cudaFree(p.col_hint);
       delete[] p.bounds;
       delete h;
       return st;
@@ -281,6 +282,7 @@ agnn_status agnn_plan_destroy(agnn_plan_t h) {
   if (h->p.csc_block) cudaFree(h->p.csc_block);
   if (h->p.c_meta_block) cudaFree(h->p.c_meta_block);
   if (h->p.short_block) cudaFree(h->p.short_block);
+  if (h->p.col_hint) cudaFree(h->p.col_hint);
   delete[] h->p.bounds;
   delete h;
   return AGNN_OK;

@@ -58,6 +58,49 @@ __device__ __forceinline__ float4 ld_stream4(const float* p) {
 }
 __device__ __forceinline__ void st4(float* p, float4 v) { *reinterpret_cast<float4*>(p) = v; }
 
+// ---- L2 residency of gathered rows (plan column classes, see plan.cu) ----------
+// A gathered neighbour row is loaded with an explicit L2 eviction policy: rows of
+// the most-gathered vertices (the hubs of a skewed graph) with evict_last, so they
+// stay in the 126 MB L2 across the pass, the rest with evict_first (or normal).
+struct L2Pol {
+  uint64_t hot, cold;
+};
+__device__ __forceinline__ L2Pol make_l2pol(int cold_first) {
+  L2Pol p;
+  asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p.hot));
+  if (cold_first)
+    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p.cold));
+  else
+    asm("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(p.cold));
+  return p;
+}
+__device__ __forceinline__ float4 ldg4_pol(const float* p, uint64_t pol) {
+  float4 r;
+  asm("ld.global.nc.L2::cache_hint.v4.f32 {%0,%1,%2,%3}, [%4], %5;"
+               : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w)
+               : "l"(p), "l"(pol));
+  return r;
+}
+__device__ __forceinline__ uint2 ldg8_pol(const void* p, uint64_t pol) {
+  uint2 r;
+  asm("ld.global.nc.L2::cache_hint.v2.u32 {%0,%1}, [%2], %3;"
+               : "=r"(r.x), "=r"(r.y)
+               : "l"(p), "l"(pol));
+  return r;
+}
+__device__ __forceinline__ uint4 ldg16_pol(const void* p, uint64_t pol) {
+  uint4 r;
+  asm("ld.global.nc.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+               : "l"(p), "l"(pol));
+  return r;
+}
+__device__ __forceinline__ float ldg1_pol(const float* p, uint64_t pol) {
+  float r;
+  asm("ld.global.nc.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(r) : "l"(p), "l"(pol));
+  return r;
+}
+
 // ---- bfloat16 feature storage (GAT BF16 mode, reading B1) ---------------------
 // 4 consecutive bf16 features = 8 bytes; widened to fp32 exactly (bf16 is the high
 // half of an fp32), narrowed with round-to-nearest-even (cvt.rn.bf16x2.f32).
@@ -92,6 +135,9 @@ template <>
 struct Slice<float> {
   using raw = float4;
   __device__ static __forceinline__ raw load(const float* p) { return ldg4(p); }
+  __device__ static __forceinline__ raw load(const float* p, uint64_t pol) {
+    return ldg4_pol(p, pol);
+  }
   __device__ static __forceinline__ float4 f(raw r) { return r; }
   __device__ static __forceinline__ raw zero() { return make_float4(0.f, 0.f, 0.f, 0.f); }
 };
@@ -101,6 +147,7 @@ struct Slice<bf16> {
   __device__ static __forceinline__ raw load(const bf16* p) {
     return __ldg(reinterpret_cast<const uint2*>(p));
   }
+  __device__ static __forceinline__ raw load(const bf16* p, uint64_t pol) { return ldg8_pol(p, pol); }
   __device__ static __forceinline__ float4 f(raw r) { return bf4_to_f4(r); }
   __device__ static __forceinline__ raw zero() { return make_uint2(0u, 0u); }
 };
@@ -202,6 +249,12 @@ struct Plan {
   void* short_block = nullptr;        // backs short_meta
   int32_t* empty_rows = nullptr;      // [n_empty] local rows without stored entries
   int64_t n_empty = 0;
+  // L2 residency classes of the gathered rows (plan.cu "column classes"): a
+  // plan-owned copy of col_idx whose bits [28, 31) hold the class c in 0..7 of
+  // the column (c >= q: among the 2^(21-q) most-gathered vertices of this rank);
+  // null when n > 2^28 or disabled (AGNN_L2_HOT_MB=0)
+  int32_t* col_hint = nullptr;
+  int64_t class_rows[8] = {};         // [q] = vertices of class >= q (host)
   // directed patterns (world == 1): the transposed pattern (CSC of the local
   // matrix) and its work lists, for the column role of the backward
   // (PAPER.md:252 Psi^T; reading A4).  Plan-owned; null for symmetric plans.

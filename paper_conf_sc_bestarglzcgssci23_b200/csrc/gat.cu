@@ -38,7 +38,7 @@ __device__ __forceinline__ void merge_softmax(float& m, float& l, float4& acc, f
   const float mn = fmaxf(m, m2);
   if (mn == NEG_INF) return;
   const float x = ex2(m - mn), y = ex2(m2 - mn);
-  l = l * x + l2 * y;
+  l = fmaf(l, x, l2 * y);  // explicit: no contraction choice left to the compiler
   acc = make_float4(fmaf(acc.x, x, acc2.x * y), fmaf(acc.y, x, acc2.y * y),
                     fmaf(acc.z, x, acc2.z * y), fmaf(acc.w, x, acc2.w * y));
   m = mn;
@@ -192,7 +192,8 @@ gat_fwd_kernel(Items it, const float* __restrict__ P, const float* __restrict__ 
   }
 }
 
-// heavy rows: fold chunk partials in ascending chunk order
+// heavy rows: fold chunk partials in ascending chunk order (with o.Q: the factored
+// backward's u and C partials too, rescaled by the same factors)
 template <int K, int NH>
 __global__ void __launch_bounds__(kSparseThreads)
 gat_fwd_merge_kernel(Items it, int act, FwdOut o) {
@@ -201,23 +202,44 @@ gat_fwd_merge_kernel(Items it, int act, FwdOut o) {
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
   for (int64_t h = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; h < it.n_heavy; h += nw) {
     const int64_t row = it.heavy_rows[h];
-    float m[L::VPL], l[L::VPL];
-    float4 acc[L::VPL];
+    float m[L::VPL], l[L::VPL], lc[L::VPL];
+    float4 acc[L::VPL], accu[L::VPL];
 #pragma unroll
     for (int v = 0; v < L::VPL; ++v) {
       m[v] = NEG_INF;
-      l[v] = 0.f;
-      acc[v] = f4(0.f);
+      l[v] = lc[v] = 0.f;
+      acc[v] = accu[v] = f4(0.f);
     }
     for (int64_t s = it.heavy_off[h]; s < it.heavy_off[h + 1]; ++s) {
 #pragma unroll
       for (int v = 0; v < L::VPL; ++v) {
         const int c = L::col(v, q), hh = c / L::D;
-        merge_softmax(m[v], l[v], acc[v], o.pm[s * NH + hh], o.pl[s * NH + hh],
-                      ldg4(o.pacc + s * K + c));
+        const float m2 = o.pm[s * NH + hh];
+        const float mn = fmaxf(m[v], m2);
+        if (mn == NEG_INF) continue;
+        const float x = ex2(m[v] - mn), y = ex2(m2 - mn);
+        const float4 a2 = ldg4(o.pacc + s * K + c);
+        l[v] = fmaf(l[v], x, o.pl[s * NH + hh] * y);
+        acc[v] = make_float4(fmaf(acc[v].x, x, a2.x * y), fmaf(acc[v].y, x, a2.y * y),
+                             fmaf(acc[v].z, x, a2.z * y), fmaf(acc[v].w, x, a2.w * y));
+        if (o.Q) {
+          const float4 u2 = ldg4(o.pu + s * K + c);
+          lc[v] = fmaf(lc[v], x, o.pc[s * NH + hh] * y);
+          accu[v] = make_float4(fmaf(accu[v].x, x, u2.x * y), fmaf(accu[v].y, x, u2.y * y),
+                                fmaf(accu[v].z, x, u2.z * y), fmaf(accu[v].w, x, u2.w * y));
+        }
+        m[v] = mn;
       }
     }
-    if (g == 0) fwd_finish<K, NH>(row, m, l, acc, q, act, o);
+    if (g != 0) continue;
+    fwd_finish<K, NH>(row, m, l, acc, q, act, o);
+    if (o.Q) {
+#pragma unroll
+      for (int v = 0; v < L::VPL; ++v) {
+        const float inv = l[v] > 0.f ? 1.f / l[v] : 0.f, r = l[v] > 0.f ? lc[v] / l[v] : 0.f;
+        st4(o.Q + row * K + L::col(v, q), mul4(inv, fma4(-r, acc[v], accu[v])));
+      }
+    }
   }
 }
 
@@ -446,7 +468,8 @@ __global__ void __launch_bounds__(kSparseThreads)
 gat_bwd_prologue_kernel(int64_t n_local, int64_t row_begin, const float* __restrict__ dHout,
                         const float* __restrict__ Z, const float* __restrict__ st,
                         const float* __restrict__ mrow, const float* __restrict__ lrow, int act,
-                        TG* __restrict__ G, float4* __restrict__ rec, PeerRows peers) {
+                        TG* __restrict__ G, float4* __restrict__ rec, PeerRows peers,
+                        const float* __restrict__ Q, float* __restrict__ ds_row) {
   using L = RowLayout<K, NH>;
   const int lane = threadIdx.x & 31, g = lane / L::LANES, q = lane % L::LANES;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
@@ -454,22 +477,25 @@ gat_bwd_prologue_kernel(int64_t n_local, int64_t row_begin, const float* __restr
   for (int64_t rs = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; rs < slots; rs += nw) {
     const int64_t row = rs * L::GROUPS + g;
     const bool ok = row < n_local;
-    float dl[L::VPL];
+    float dl[L::VPL], dq[L::VPL];
     float4 gv[L::VPL];
 #pragma unroll
     for (int v = 0; v < L::VPL; ++v) {
       const int c = L::col(v, q);
-      float4 z = f4(0.f), dh = f4(0.f);
+      float4 z = f4(0.f), dh = f4(0.f), qv = f4(0.f);
       if (ok) {
         z = ldg4(Z + row * K + c);
         dh = ldg4(dHout + row * K + c);
+        if (Q) qv = ldg4(Q + row * K + c);
       }
       gv[v] = make_float4(dh.x * act_grad(act, z.x), dh.y * act_grad(act, z.y),
                           dh.z * act_grad(act, z.z), dh.w * act_grad(act, z.w));
       if constexpr (sizeof(TG) == 2) gv[v] = round_bf4(gv[v]);
       dl[v] = dot4(gv[v], z);
+      dq[v] = dot4(gv[v], qv);  // factored backward: ds_j = G_j . Q_j (gat_args.cuh)
     }
     L::head_reduce(dl);
+    if (Q) L::head_reduce(dq);
     if (!ok) continue;
     const int64_t grow = row_begin + row;
 #pragma unroll
@@ -485,6 +511,7 @@ gat_bwd_prologue_kernel(int64_t n_local, int64_t row_begin, const float* __restr
         rec[grow * NH + h] = r4;
         for (int pi = 0; pi < peers.n; ++pi)
           reinterpret_cast<float4*>(peers.b[pi])[grow * NH + h] = r4;
+        if (Q) ds_row[row * NH + h] = dq[v];
       }
     }
   }
@@ -563,9 +590,16 @@ __global__ void gat_debug_alpha_kernel(const int64_t* __restrict__ rp, int64_t n
 }
 
 // ---------------------------------------------------------------- layout
+// the factored backward (gat_args.cuh) runs where the k' = 128 kernels do, on
+// symmetric patterns
+bool factored(const Plan& p, const GatShape& g) {
+  return gat_factored_enabled() && gat_k128_supported(g.k_out, g.heads) && !p.directed();
+}
+
 struct SavedGat {
   float *P, *st, *Z, *m, *l;
   bf16* P16;  // BF16 mode: P stored as bfloat16 (P == NULL)
+  float* Q;   // factored backward: [n_local x K] (NULL otherwise)
 };
 SavedGat carve_saved(const Plan& p, const GatShape& g, void* base) {
   Carver c(base);
@@ -580,6 +614,7 @@ SavedGat carve_saved(const Plan& p, const GatShape& g, void* base) {
   s.Z = c.take<float>((size_t)p.n_local * g.k_out);
   s.m = c.take<float>((size_t)p.n_local * g.heads);
   s.l = c.take<float>((size_t)p.n_local * g.heads);
+  s.Q = factored(p, g) ? c.take<float>((size_t)p.n_local * g.k_out) : nullptr;
   return s;
 }
 size_t saved_size(const Plan& p, const GatShape& g) {
@@ -592,11 +627,12 @@ size_t saved_size(const Plan& p, const GatShape& g) {
   c.take<float>((size_t)p.n_local * g.k_out);
   c.take<float>((size_t)p.n_local * g.heads);
   c.take<float>((size_t)p.n_local * g.heads);
+  if (factored(p, g)) c.take<float>((size_t)p.n_local * g.k_out);
   return c.off + 256;
 }
 
 struct WsGat {
-  float *Wext, *pacc, *pm, *pl, *G, *dP, *da_part, *gemm, *ds_dir;
+  float *Wext, *pacc, *pm, *pl, *G, *dP, *da_part, *gemm, *ds_dir, *ds_row;
   bf16* G16;  // BF16 mode: G stored as bfloat16 (G == NULL)
   float4* rec;
   void* saved_inf;  // saved-layout scratch for inference
@@ -622,6 +658,7 @@ WsGat carve_ws(const Plan& p, const GatShape& g, void* base, size_t* total) {
   w.pm = c.take<float>((size_t)p.max_chunks() * g.heads);
   w.pl = c.take<float>((size_t)p.max_chunks() * g.heads);
   w.ds_dir = c.take<float>(p.csc_ptr ? (size_t)p.n_local * g.heads : 0);
+  w.ds_row = c.take<float>(factored(p, g) ? (size_t)p.n_local * g.heads : 0);
   w.dP = c.take<float>((size_t)p.n_local * g.k_out);
   w.da_part = c.take<float>((size_t)da_rows() * 2 * g.k_out);
   w.gemm = c.take<float>(gemm_tn_ws_floats(g.k_in, g.k_out));
@@ -630,6 +667,14 @@ WsGat carve_ws(const Plan& p, const GatShape& g, void* base, size_t* total) {
 }
 
 }  // namespace
+
+bool gat_factored_enabled() {
+  static const int v = [] {
+    const char* e = getenv("AGNN_GAT_FACTORED");
+    return e ? atoi(e) : 1;
+  }();
+  return v != 0;
+}
 
 size_t gat_saved_bytes(const Plan& p, const GatShape& g) { return saved_size(p, g); }
 size_t gat_workspace_bytes(const Plan& p, const GatShape& g) {
@@ -678,7 +723,8 @@ agnn_status gat_forward(const Plan& p, const GatShape& g, const float* W, const 
     // from the same (unrounded) accumulators; then the plain all-gather of P~ | st
     Items it = items_of(p);
     FwdOut o{saved ? sv.Z : nullptr, H_out, saved ? sv.m : nullptr, saved ? sv.l : nullptr,
-             w.pacc, w.pm, w.pl};
+             w.pacc, w.pm, w.pl, saved ? sv.Q : nullptr, w.pacc + p.max_chunks() * g.k_out,
+             w.pacc + 2 * p.max_chunks() * g.k_out};
     if ((st = gemm_rows_bf16(H_in, p.n_local, g.k_in, w.Wext, NEs, sv.P16 + p.row_begin * g.k_out,
                              g.k_out, stloc, w.dP, s)) != AGNN_OK)
       return st;
@@ -687,7 +733,9 @@ agnn_status gat_forward(const Plan& p, const GatShape& g, const float* W, const 
         return st;
       if ((st = allgather_rows(p, sv.st, 2 * g.heads, s)) != AGNN_OK) return st;
     }
-    if ((st = gat_fwd_k128_bf16(it, g.heads, sv.P16, sv.st, g.slope, g.act, o, s)) != AGNN_OK)
+    // gathered per edge: a bf16 row of P and the t_j of the heads
+    const Items ith = l2_hinted(it, p, 2 * (int64_t)g.k_out + 4 * g.heads);
+    if ((st = gat_fwd_k128_bf16(ith, g.heads, sv.P16, sv.st, g.slope, g.act, o, s)) != AGNN_OK)
       return st;
     if (it.n_heavy > 0) {
       AGNN_GAT_DISPATCH(K_, NH_, (gat_fwd_merge_kernel<K, NH>
@@ -735,9 +783,12 @@ agnn_status gat_forward(const Plan& p, const GatShape& g, const float* W, const 
   }
   Items it = items_of(p);
   FwdOut o{saved ? sv.Z : nullptr, H_out, saved ? sv.m : nullptr, saved ? sv.l : nullptr,
-           w.pacc, w.pm, w.pl};
+           w.pacc, w.pm, w.pl, saved ? sv.Q : nullptr, w.pacc + p.max_chunks() * g.k_out,
+           w.pacc + 2 * p.max_chunks() * g.k_out};
   if (gat_k128_supported(g.k_out, g.heads)) {
-    if ((st = gat_fwd_k128(it, g.heads, sv.P, sv.st, g.slope, g.act, o, p.n, s)) != AGNN_OK) return st;
+    const Items ith = l2_hinted(it, p, 4 * (int64_t)g.k_out + 4 * g.heads);
+    if ((st = gat_fwd_k128(ith, g.heads, sv.P, sv.st, g.slope, g.act, o, p.n, s)) != AGNN_OK)
+      return st;
   } else if (it.n_chunks + it.n_light > 0) {
     AGNN_GAT_DISPATCH(K_, NH_, (gat_fwd_kernel<K, NH, fwd_unroll<K>()>
                                 <<<grid_of(gat_fwd_kernel<K, NH, fwd_unroll<K>()>), kSparseThreads,
@@ -786,12 +837,12 @@ agnn_status gat_backward(const Plan& p, const GatShape& g, const float* W, const
     AGNN_GAT_DISPATCH(K_, NH_, (gat_bwd_prologue_kernel<K, NH, bf16>
                                 <<<grid_of(gat_bwd_prologue_kernel<K, NH, bf16>), kSparseThreads, 0,
                                    s>>>(p.n_local, p.row_begin, dH_out, sv.Z, sv.st, sv.m, sv.l,
-                                        g.act, w.G16, w.rec, pr)));
+                                        g.act, w.G16, w.rec, pr, sv.Q, w.ds_row)));
   } else {
     AGNN_GAT_DISPATCH(K_, NH_, (gat_bwd_prologue_kernel<K, NH>
                                 <<<grid_of(gat_bwd_prologue_kernel<K, NH>), kSparseThreads, 0, s>>>(
                                     p.n_local, p.row_begin, dH_out, sv.Z, sv.st, sv.m, sv.l, g.act,
-                                    w.G, w.rec, pr)));
+                                    w.G, w.rec, pr, sv.Q, w.ds_row)));
   }
   AGNN_LAUNCH_CHECK("gat_bwd_prologue_kernel");
   if (p.world > 1) {
@@ -809,7 +860,7 @@ agnn_status gat_backward(const Plan& p, const GatShape& g, const float* W, const
     }
   }
   BwdArgs A{sv.P, sv.st, w.G, w.rec, a, g.slope, w.dP, w.pacc, w.pm, w.pl, w.da_part,
-            nullptr, nullptr, w.ds_dir, sv.P16, w.G16};
+            nullptr, nullptr, w.ds_dir, sv.P16, w.G16, w.ds_row};
   int64_t main_warps = 0, merge_warps = 0;
   if (directed) {
     // row role over the CSR (ds_j), then the column role over the CSC (dt_j, acc_j, dP_j)
@@ -835,8 +886,15 @@ agnn_status gat_backward(const Plan& p, const GatShape& g, const float* W, const
                                 <<<(unsigned)(merge_warps / 8), kSparseThreads, 0, s>>>(
                                     it, A, main_warps)));
     AGNN_LAUNCH_CHECK("gat_bwd_merge_kernel");
+  } else if (sv.Q) {
+    // factored: gathered per edge only G_i and the records rec_i of the heads
+    const Items ith = l2_hinted(it, p, (g.bf16 ? 2 : 4) * (int64_t)g.k_out + 16 * g.heads);
+    if ((st = gat_bwd_k128f(ith, g.heads, A, &main_warps, s)) != AGNN_OK) return st;
   } else if (gat_k128_supported(g.k_out, g.heads)) {
-    if ((st = gat_bwd_k128(it, g.heads, A, &main_warps, s)) != AGNN_OK) return st;
+    // gathered per edge: rows P_i and G_i, the record rec_i and t_i of the heads
+    const Items ith =
+        l2_hinted(it, p, 2 * (g.bf16 ? 2 : 4) * (int64_t)g.k_out + 20 * g.heads);
+    if ((st = gat_bwd_k128(ith, g.heads, A, &main_warps, s)) != AGNN_OK) return st;
   } else {
     AGNN_GAT_DISPATCH(K_, NH_, (main_warps = (int64_t)grid_of(gat_bwd_kernel<K, NH, bwd_unroll<K>()>) *
                                              (kSparseThreads / 32)));

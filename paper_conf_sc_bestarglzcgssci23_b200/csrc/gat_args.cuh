@@ -12,6 +12,11 @@ struct GatFwdOut {
   float* pacc;   // [n_chunks x K]
   float* pm;     // [n_chunks x NH]
   float* pl;     // [n_chunks x NH]
+  // factored backward (gat_factored()): Q_i = sum_j c_ij P_j - (sum_j c_ij) Z_i with
+  // c_ij = alpha_ij lambda_ij, so that ds_i = G_i . Q_i (per head) needs no gathers
+  float* Q;      // [n_local x K]   nullable (inference, or the unfactored path)
+  float* pu;     // [n_chunks x K]  chunk partials of sum_j p_ij lambda_ij P_j
+  float* pc;     // [n_chunks x NH] chunk partials of sum_j p_ij lambda_ij
 };
 
 struct GatBwdArgs {
@@ -31,7 +36,20 @@ struct GatBwdArgs {
   float* ds_dir;       // [n_local x NH] directed patterns: row-pass ds for the column pass
   const bf16* P16;     // BF16 mode (reading B1): P and G stored as bfloat16 (P, G unused)
   const bf16* G16;
+  const float* ds_row; // [n_local x NH] factored backward: ds_j = G_j . Q_j (prologue)
 };
+
+// The factored GAT backward (k' = 128, symmetric pattern; AGNN_GAT_FACTORED=0
+// disables it).  With c_ji = alpha_ji lambda_ji (lambda = LReLU slope of the
+// entry), the row-role sum of PAPER.md:250-254 is linear in the gathered rows,
+//   ds_j = sum_i c_ji (G_j . P_i - delta_j) = G_j . (sum_i c_ji P_i - (sum_i c_ji) Z_j)
+//        = G_j . Q_j,
+// and the forward already gathers every P_i with its alpha_ji: it accumulates
+// Q_j alongside Z_j, the backward prologue forms ds_j = G_j . Q_j, and the
+// backward edge pass gathers only G_i and rec_i (column role):
+//   dt_j = sum_i c'_ij (G_i . P_j - delta_i) = P_j . v_j - sum_i c'_ij delta_i,
+//   v_j = sum_i c'_ij G_i,  acc_j = sum_i alpha_ij G_i.
+bool gat_factored_enabled();
 
 // k' = 128 kernels (gat_k128.cu): lane-parallel scalar work, warp-parallel rows
 bool gat_k128_supported(int k_out, int heads);
@@ -61,5 +79,10 @@ agnn_status gat_fwd_k128_bf16(const Items& it, int heads, const bf16* P, const f
                               float slope, int act, const GatFwdOut& o, cudaStream_t s);
 agnn_status gat_bwd_k128(const Items& it, int heads, const GatBwdArgs& A, int64_t* warps,
                          cudaStream_t s);  // A.P16 != NULL: BF16 mode
+// factored backward edge pass (A.ds_row set): gathers G_i, rec_i only
+agnn_status gat_bwd_k128f(const Items& it, int heads, const GatBwdArgs& A, int64_t* warps,
+                          cudaStream_t s);
+agnn_status gat_bwd_short_f(const Items& it, int heads, const GatBwdArgs& A, int64_t da_row0,
+                            int64_t* warps, cudaStream_t s);
 
 }  // namespace agnn

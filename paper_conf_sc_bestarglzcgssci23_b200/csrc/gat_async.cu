@@ -141,7 +141,7 @@ gat_bwd_async_kernel(Items it, GatBwdArgs A) {
     };
     auto col_of = [&](int t) -> int {
       const int64_t e = beg + (int64_t)t * B + pe;
-      return (t < nst && e < end) ? __ldg(it.col + e) : 0;
+      return (t < nst && e < end) ? (int)((uint32_t)__ldg(it.col + e) & it.col_mask) : 0;
     };
     // prologue: stages 0 .. NS-2 in flight, the ids of stage NS-1 loading
     {

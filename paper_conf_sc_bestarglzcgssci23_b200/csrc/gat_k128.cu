@@ -54,6 +54,28 @@ __device__ __forceinline__ void load_n(const float* p, float (&x)[N]) {
   }
 }
 
+// the same with an explicit L2 policy (gathered rows of other vertices)
+template <int N>
+__device__ __forceinline__ void load_n(const float* p, float (&x)[N], uint64_t pol) {
+  if constexpr (N % 4 == 0) {
+#pragma unroll
+    for (int i = 0; i < N; i += 4) {
+      const float4 v = ldg4_pol(p + i, pol);
+      x[i] = v.x;
+      x[i + 1] = v.y;
+      x[i + 2] = v.z;
+      x[i + 3] = v.w;
+    }
+  } else if constexpr (N == 2) {
+    const uint2 v = ldg8_pol(p, pol);
+    x[0] = __uint_as_float(v.x);
+    x[1] = __uint_as_float(v.y);
+  } else {
+#pragma unroll
+    for (int i = 0; i < N; ++i) x[i] = ldg1_pol(p + i, pol);
+  }
+}
+
 // fp32 rows, or bfloat16 rows (BF16 mode, reading B1): same code, the gathers
 // widen 4 bf16 (8 bytes) to a float4 (common.cuh ldg4 overloads)
 template <typename TP>
@@ -69,29 +91,38 @@ __device__ __forceinline__ const bf16* pick<bf16>(const float*, const bf16* h) {
 template <typename TP>
 constexpr int fwd_group() { return sizeof(TP) == 2 ? 8 : 4; }
 
-template <typename TP, int NH, int U, int MINB>
+// QF (training, factored backward): also accumulate u_i = sum_j p_ij lambda_ij P_j and
+// C_i = sum_j p_ij lambda_ij with the same online rescaling, and store
+// Q_i = (u_i - (C_i / l_i) acc_i) / l_i  (= sum_j c_ij P_j - (sum_j c_ij) Z_i, gat_args.cuh);
+// when every lambda_ij = 1 (all pre-activations > 0) u = acc and C = l bitwise, so
+// Q = 0 and ds = 0 exactly, as in exact arithmetic.
+template <typename TP, int NH, int U, int MINB, bool QF>
 __global__ void __launch_bounds__(256, MINB)
 gat_fwd_k128_kernel(Items it, const TP* __restrict__ P, const float* __restrict__ st,
                     float slope, int act, GatFwdOut o) {
   constexpr int D = K / NH, HL = D / 4;
-  __shared__ float sPw[8][NH][33];  // +1: heads read different rows without bank conflicts
+  // +1: heads read different rows without bank conflicts; QF: {p, p lambda} pairs
+  __shared__ float sPw[QF ? 1 : 8][NH][33];
+  __shared__ float2 sP2[QF ? 8 : 1][NH][33];
   __shared__ int sJ[8][32];
   const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
   const int hv = lane / HL, cq = lane * 4;
   const int64_t nitems = it.n_chunks + it.n_light;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const Gath ga(it);
   for (int64_t w = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; w < nitems; w += nw) {
     int64_t row, beg, end, slot;
     item_of(it, w, row, beg, end, slot);
     const int64_t grow = it.row_begin + row;
-    float si[NH], mr[NH], lp[NH];
+    float si[NH], mr[NH], lp[NH], lc[NH];
     load_n<NH>(st + grow * (2 * NH), si);
 #pragma unroll
     for (int h = 0; h < NH; ++h) {
       mr[h] = -INFINITY;
       lp[h] = 0.f;
+      lc[h] = 0.f;
     }
-    float4 acc = f4(0.f);
+    float4 acc = f4(0.f), accu = f4(0.f);
     // column ids one batch ahead: the next batch's ids load during this batch
     int jpre = beg + lane < end ? __ldg(it.col + beg + lane) : 0;
     for (int64_t b0 = beg; b0 < end; b0 += 32) {
@@ -106,9 +137,10 @@ gat_fwd_k128_kernel(Items it, const TP* __restrict__ P, const float* __restrict_
       typename SL::raw pv[U];
 #pragma unroll
       for (int u = 0; u < U; ++u)
-        pv[u] = u < cnt ? SL::load(P + (int64_t)sJ[wib][u] * K + cq) : SL::zero();
+        pv[u] = u < cnt ? SL::load(P + ga.row(sJ[wib][u]) * K + cq, ga.policy(sJ[wib][u]))
+                        : SL::zero();
       float tj[NH];
-      load_n<NH>(st + (int64_t)j * (2 * NH) + NH, tj);
+      load_n<NH>(st + ga.row(j) * (2 * NH) + NH, tj, ga.policy(j));
       float sch = 1.f;
 #pragma unroll
       for (int h = 0; h < NH; ++h) {
@@ -119,15 +151,35 @@ gat_fwd_k128_kernel(Items it, const TP* __restrict__ P, const float* __restrict_
         for (int off = 16; off > 0; off >>= 1) bm = fmaxf(bm, __shfl_xor_sync(FULL, bm, off));
         const float mn = fmaxf(mr[h], bm);
         const float sc = ex2(mr[h] - mn);  // 0 on the first batch (mr = -inf)
-        lp[h] *= sc;
+        // rounded multiply then add, never contracted: the training (QF) and inference
+        // variants must produce bitwise the same l, and lc the same ops as lp
+        lp[h] = __fmul_rn(lp[h], sc);
         if (h == hv) sch = sc;
         mr[h] = mn;
         const float p = valid ? ex2(e - mn) : 0.f;
-        lp[h] += p;
-        sPw[wib][h][lane] = p;
+        lp[h] = __fadd_rn(lp[h], p);
+        if constexpr (QF) {
+          const float pc = pre > 0.f ? p : p * slope;
+          lc[h] = __fadd_rn(__fmul_rn(lc[h], sc), pc);
+          sP2[wib][h][lane] = make_float2(p, pc);
+        } else {
+          sPw[wib][h][lane] = p;
+        }
       }
       acc = mul4(sch, acc);
+      if constexpr (QF) accu = mul4(sch, accu);
       __syncwarp();
+      // one gathered row: both accumulations
+      auto axpy = [&](int e, const typename SL::raw& r) {
+        const float4 x = SL::f(r);
+        if constexpr (QF) {
+          const float2 pw = sP2[wib][hv][e];
+          acc = fma4(pw.x, x, acc);
+          accu = fma4(pw.y, x, accu);
+        } else {
+          acc = fma4(sPw[wib][hv][e], x, acc);
+        }
+      };
       if (cnt == 32) {
         // full batch: 32/GR groups of GR rows, the next group in flight during this
         // group's FMAs
@@ -140,62 +192,77 @@ gat_fwd_k128_kernel(Items it, const TP* __restrict__ P, const float* __restrict_
 #pragma unroll
         for (int g = 0; g < NGR; g += 2) {
 #pragma unroll
-          for (int u = 0; u < GR; ++u)
-            qb[u] = SL::load(Pl + (int64_t)(uint32_t)__shfl_sync(FULL, j, GR * g + GR + u) * K);
-#pragma unroll
-          for (int u = 0; u < GR; ++u) acc = fma4(sPw[wib][hv][GR * g + u], SL::f(qa[u]), acc);
-          if (g + 2 < NGR) {
-#pragma unroll
-            for (int u = 0; u < GR; ++u)
-              qa[u] = SL::load(Pl + (int64_t)(uint32_t)__shfl_sync(FULL, j, GR * g + 2 * GR + u) * K);
+          for (int u = 0; u < GR; ++u) {
+            const int c = __shfl_sync(FULL, j, GR * g + GR + u);
+            qb[u] = SL::load(Pl + ga.row(c) * K, ga.policy(c));
           }
 #pragma unroll
-          for (int u = 0; u < GR; ++u)
-            acc = fma4(sPw[wib][hv][GR * g + GR + u], SL::f(qb[u]), acc);
+          for (int u = 0; u < GR; ++u) axpy(GR * g + u, qa[u]);
+          if (g + 2 < NGR) {
+#pragma unroll
+            for (int u = 0; u < GR; ++u) {
+              const int c = __shfl_sync(FULL, j, GR * g + 2 * GR + u);
+              qa[u] = SL::load(Pl + ga.row(c) * K, ga.policy(c));
+            }
+          }
+#pragma unroll
+          for (int u = 0; u < GR; ++u) axpy(GR * g + GR + u, qb[u]);
         }
       } else {
         for (int k = 0; k < cnt; k += U) {
-          float pw[U];
 #pragma unroll
           for (int u = 0; u < U; ++u) {
             const int kk = k + u;
-            if (k > 0) pv[u] = kk < cnt ? SL::load(P + (int64_t)sJ[wib][kk] * K + cq) : SL::zero();
-            pw[u] = kk < cnt ? sPw[wib][hv][kk] : 0.f;
+            if (k > 0)
+              pv[u] = kk < cnt ? SL::load(P + ga.row(sJ[wib][kk]) * K + cq, ga.policy(sJ[wib][kk]))
+                               : SL::zero();
           }
 #pragma unroll
-          for (int u = 0; u < U; ++u) acc = fma4(pw[u], SL::f(pv[u]), acc);
+          for (int u = 0; u < U; ++u)
+            if (k + u < cnt) axpy(k + u, pv[u]);
         }
       }
       __syncwarp();
     }
-    float l[NH];
+    float l[NH], cs[NH];
 #pragma unroll
     for (int h = 0; h < NH; ++h) {
-      float x = lp[h];
+      float x = lp[h], y = lc[h];
 #pragma unroll
-      for (int off = 16; off > 0; off >>= 1) x += __shfl_xor_sync(FULL, x, off);
+      for (int off = 16; off > 0; off >>= 1) {
+        x += __shfl_xor_sync(FULL, x, off);
+        if constexpr (QF) y += __shfl_xor_sync(FULL, y, off);
+      }
       l[h] = x;
+      cs[h] = y;
     }
-    float lh = l[0], mh = mr[0];
+    float lh = l[0], ch = cs[0];
 #pragma unroll
     for (int h = 1; h < NH; ++h)
       if (h == hv) {
         lh = l[h];
-        mh = mr[h];
+        ch = cs[h];
       }
     if (slot >= 0) {
       st4(o.pacc + slot * K + cq, acc);
+      if constexpr (QF) st4(o.pu + slot * K + cq, accu);
       if (lane == 0) {
 #pragma unroll
         for (int h = 0; h < NH; ++h) {
           o.pm[slot * NH + h] = mr[h];
           o.pl[slot * NH + h] = l[h];
+          if constexpr (QF) o.pc[slot * NH + h] = cs[h];
         }
       }
     } else {
-      const float4 z = mul4(lh > 0.f ? 1.f / lh : 0.f, acc);
+      const float inv = lh > 0.f ? 1.f / lh : 0.f;
+      const float4 z = mul4(inv, acc);
       if (o.Z) st4(o.Z + row * K + cq, z);
       st4(o.Hout + row * K + cq, act_fwd4(act, z));
+      if constexpr (QF) {
+        const float r = lh > 0.f ? ch / lh : 0.f;
+        st4(o.Q + row * K + cq, mul4(inv, fma4(-r, acc, accu)));
+      }
       if (o.m && lane == 0) {
 #pragma unroll
         for (int h = 0; h < NH; ++h) {
@@ -203,7 +270,6 @@ gat_fwd_k128_kernel(Items it, const TP* __restrict__ P, const float* __restrict_
           o.l[row * NH + h] = l[h];
         }
       }
-      (void)mh;
     }
   }
 }
@@ -271,7 +337,7 @@ gat_fwd_tma_kernel(const __grid_constant__ CUtensorMap mapP, Items it, const flo
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
   // load the column ids of a batch and (lane 0) start its gathers into ring half `hb`
   auto issue = [&](int64_t b0, int cnt, int hb) -> int {
-    const int j = lane < cnt ? __ldg(it.col + b0 + lane) : 0;
+    const int j = lane < cnt ? (int)((uint32_t)__ldg(it.col + b0 + lane) & it.col_mask) : 0;
     const int jl = __shfl_sync(FULL, j, cnt - 1);        // pad the last gather4 with a valid row
     const int jj = lane < cnt ? j : jl;
     if (lane < TB) sJ[wib][hb][lane] = jj;
@@ -407,6 +473,7 @@ gat_bwd_k128_kernel(Items it, GatBwdArgs A) {
   const TP* Pl = Pb + cq;
   const TP* Gl = Gb + cq;
   float4 da1 = f4(0.f), da2 = f4(0.f);
+  const Gath ga(it);
 
   for (int64_t w = gw; w < nitems; w += nw) {
     int64_t row, beg, end, slot;
@@ -424,18 +491,22 @@ gat_bwd_k128_kernel(Items it, GatBwdArgs A) {
     auto load = [&](BwdBatch<TP, B>& q, int cidx, int off, int cnt) {
 #pragma unroll
       for (int b = 0; b < B; ++b) {
-        const uint32_t i = (uint32_t)__shfl_sync(FULL, cidx, off + b);
+        const int c = __shfl_sync(FULL, cidx, off + b);
         if (b < cnt) {
-          q.Pi[b] = SL::load(Pl + (int64_t)i * K);
-          q.Gi[b] = SL::load(Gl + (int64_t)i * K);
+          const int64_t i = ga.row(c);
+          const uint64_t pol = ga.policy(c);
+          q.Pi[b] = SL::load(Pl + i * K, pol);
+          q.Gi[b] = SL::load(Gl + i * K, pol);
         } else {
           q.Pi[b] = q.Gi[b] = SL::zero();
         }
       }
-      const uint32_t im = (uint32_t)__shfl_sync(FULL, cidx, off + my_b);
+      const int cm = __shfl_sync(FULL, cidx, off + my_b);
       const bool vm = my_b < cnt;
-      q.ri = vm ? __ldg(A.rec + (int64_t)im * NH + hv) : f4(0.f);
-      q.ti = vm ? __ldg(A.st + (int64_t)im * (2 * NH) + NH + hv) : 0.f;
+      const int64_t im = ga.row(cm);
+      const uint64_t polm = ga.policy(cm);
+      q.ri = vm ? ldg4_pol(reinterpret_cast<const float*>(A.rec + im * NH + hv), polm) : f4(0.f);
+      q.ti = vm ? ldg1_pol(A.st + im * (2 * NH) + NH + hv, polm) : 0.f;
     };
     auto body = [&](const BwdBatch<TP, B>& q, int cnt) {
       float x1[B], x2[B];
@@ -520,6 +591,151 @@ gat_bwd_k128_kernel(Items it, GatBwdArgs A) {
   st4(A.da_part + gw * 2 * K + K + cq, da2);
 }
 
+// ---------------------------------------------------------------- factored backward
+// Column role only (the row role's ds_j = G_j . Q_j comes from the prologue,
+// gat_args.cuh): per row j, edges in windows of 32 (one edge per lane) —
+//   lane e: rec_i of all heads -> alpha_ij = 2^(LReLU(s_i + t_j) - m_i) / l_i,
+//   c'_ij = alpha_ij lambda_ij, partial sums of c'_ij delta_i;
+//   then the warp walks the window: lane q owns columns 4q..4q+3 of G_i and
+//   accumulates acc_j += alpha_ij G_i and v_j += c'_ij G_i (16-byte gather, 8 FMAs).
+// Per row: dt_j = P_j . v_j - sum_i c'_ij delta_i, dP_j = acc_j + ds_j a1 + dt_j a2.
+// Per edge it moves the index, one G row and the NH records (4 + K f + 16 NH bytes).
+template <typename TP, int NH, int MINB>
+__global__ void __launch_bounds__(256, MINB)
+gat_bwd_k128f_kernel(Items it, GatBwdArgs A) {
+  constexpr int D = K / NH, HL = D / 4;
+  __shared__ float2 sAC[8][NH][33];  // {alpha_ij, c'_ij}
+  __shared__ int sJ[8][32];
+  const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  const int hv = lane / HL, cq = lane * 4;
+  const int64_t nitems = it.n_chunks + it.n_light;
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const TP* Pb = pick<TP>(A.P, A.P16);
+  const TP* Gb = pick<TP>(A.G, A.G16);
+  const float slope = A.slope;
+  const Gath ga(it);
+  using SL = Slice<TP>;
+  float4 da1 = f4(0.f), da2 = f4(0.f);
+  for (int64_t w = gw; w < nitems; w += nw) {
+    int64_t row, beg, end, slot;
+    item_of(it, w, row, beg, end, slot);
+    const int64_t grow = it.row_begin + row;
+    float tj[NH], sd[NH];
+    load_n<NH>(A.st + grow * (2 * NH) + NH, tj);
+#pragma unroll
+    for (int h = 0; h < NH; ++h) sd[h] = 0.f;
+    float4 acc = f4(0.f), accv = f4(0.f);
+    int jpre = beg + lane < end ? __ldg(it.col + beg + lane) : 0;
+    for (int64_t b0 = beg; b0 < end; b0 += 32) {
+      const int cnt = (int)(end - b0 < 32 ? end - b0 : 32);
+      const bool valid = lane < cnt;
+      const int j = jpre;
+      jpre = b0 + 32 + lane < end ? __ldg(it.col + b0 + 32 + lane) : 0;
+      sJ[wib][lane] = j;
+      __syncwarp();
+      constexpr int GR = fwd_group<TP>(), NGR = 32 / GR;
+      typename SL::raw qa[GR], qb[GR];
+      // the first group of G rows is in flight while the weights are computed
+#pragma unroll
+      for (int u = 0; u < GR; ++u)
+        qa[u] = u < cnt ? SL::load(Gb + ga.row(sJ[wib][u]) * K + cq, ga.policy(sJ[wib][u]))
+                        : SL::zero();
+      {
+        const int64_t ir = ga.row(j);
+        const uint64_t pol = ga.policy(j);
+#pragma unroll
+        for (int h = 0; h < NH; ++h) {
+          const float4 r = valid ? ldg4_pol(reinterpret_cast<const float*>(A.rec + ir * NH + h), pol)
+                                 : f4(0.f);  // {s_i, m_i, 1/l_i, delta_i}
+          const float pre = r.x + tj[h];
+          const float e = fmaxf(pre, slope * pre);
+          const float al = valid ? ex2(e - r.y) * r.z : 0.f;
+          const float cc = pre > 0.f ? al : al * slope;
+          sd[h] = fmaf(cc, r.w, sd[h]);
+          sAC[wib][h][lane] = make_float2(al, cc);
+        }
+      }
+      __syncwarp();
+      auto axpy = [&](int e, const typename SL::raw& r) {
+        const float4 x = SL::f(r);
+        const float2 ac = sAC[wib][hv][e];
+        acc = fma4(ac.x, x, acc);
+        accv = fma4(ac.y, x, accv);
+      };
+      const TP* Gl = Gb + cq;
+      if (cnt == 32) {
+#pragma unroll
+        for (int g = 0; g < NGR; g += 2) {
+#pragma unroll
+          for (int u = 0; u < GR; ++u) {
+            const int c = __shfl_sync(FULL, j, GR * g + GR + u);
+            qb[u] = SL::load(Gl + ga.row(c) * K, ga.policy(c));
+          }
+#pragma unroll
+          for (int u = 0; u < GR; ++u) axpy(GR * g + u, qa[u]);
+          if (g + 2 < NGR) {
+#pragma unroll
+            for (int u = 0; u < GR; ++u) {
+              const int c = __shfl_sync(FULL, j, GR * g + 2 * GR + u);
+              qa[u] = SL::load(Gl + ga.row(c) * K, ga.policy(c));
+            }
+          }
+#pragma unroll
+          for (int u = 0; u < GR; ++u) axpy(GR * g + GR + u, qb[u]);
+        }
+      } else {
+        for (int k = 0; k < cnt; k += GR) {
+          if (k > 0) {
+#pragma unroll
+            for (int u = 0; u < GR; ++u) {
+              const int kk = k + u;
+              qa[u] = kk < cnt ? SL::load(Gl + ga.row(sJ[wib][kk]) * K, ga.policy(sJ[wib][kk]))
+                               : SL::zero();
+            }
+          }
+#pragma unroll
+          for (int u = 0; u < GR; ++u)
+            if (k + u < cnt) axpy(k + u, qa[u]);
+        }
+      }
+      __syncwarp();
+    }
+    // per row: dt_j = P_j . v_j - sum_i c'_ij delta_i  (head of lane hv)
+    const float4 Pj = SL::f(SL::load(Pb + grow * K + cq));
+    float x = dot4(Pj, accv);
+#pragma unroll
+    for (int o = 1; o < HL; o <<= 1) x += __shfl_xor_sync(FULL, x, o);
+    float sdh = 0.f;
+#pragma unroll
+    for (int h = 0; h < NH; ++h) {
+      float y = sd[h];
+#pragma unroll
+      for (int off = 16; off > 0; off >>= 1) y += __shfl_xor_sync(FULL, y, off);
+      if (h == hv) sdh = y;
+    }
+    const float dt = x - sdh;
+    if (slot >= 0) {
+      st4(A.pacc + slot * K + cq, acc);
+      if ((lane % HL) == 0) {
+        A.pdt[slot * NH + hv] = dt;
+        A.pds[slot * NH + hv] = it.chunk_idx[slot] == 0 ? A.ds_row[row * NH + hv] : 0.f;
+      }
+    } else {
+      const float ds = A.ds_row[row * NH + hv];
+      const float4 a1v = ldg4(A.a + hv * 2 * D + cq % D);
+      const float4 a2v = ldg4(A.a + hv * 2 * D + D + cq % D);
+      float4 dp = fma4(ds, a1v, acc);
+      dp = fma4(dt, a2v, dp);
+      st4(A.dP + row * K + cq, dp);
+      da1 = fma4(ds, Pj, da1);
+      da2 = fma4(dt, Pj, da2);
+    }
+  }
+  st4(A.da_part + gw * 2 * K + cq, da1);
+  st4(A.da_part + gw * 2 * K + K + cq, da2);
+}
+
 template <typename F>
 int grid_for(F* f) {
   return persistent_blocks(reinterpret_cast<const void*>(f));
@@ -590,7 +806,7 @@ agnn_status gat_fwd_k128(const Items& it_all, int heads, const float* P, const f
   const Items it = long_items(it_all);
   if (it.n_chunks + it.n_light == 0) return AGNN_OK;
   CUtensorMap map;
-  if (fwd_tma_enabled() && row_gather_map(&map, P, n_rows)) {
+  if (!o.Q && fwd_tma_enabled() && row_gather_map(&map, P, n_rows)) {
     AGNN_K128_DISPATCH(heads, ({
       constexpr int smem = TW * TRING;
       static bool attr = false;
@@ -608,22 +824,10 @@ agnn_status gat_fwd_k128(const Items& it_all, int heads, const float* P, const f
     }));
     return AGNN_OK;
   }
-  static int minb = -1;
-  if (minb < 0) {
-    const char* e = getenv("AGNN_FWD_MINB");
-    minb = e ? atoi(e) : 3;
-  }
   AGNN_K128_DISPATCH(heads, ({
-    if (minb == 4) {
-      gat_fwd_k128_kernel<float, NH, 4, 4><<<grid_for(gat_fwd_k128_kernel<float, NH, 4, 4>), 256,
-                                             0, s>>>(it, P, st, slope, act, o);
-    } else if (minb == 2) {
-      gat_fwd_k128_kernel<float, NH, 4, 2><<<grid_for(gat_fwd_k128_kernel<float, NH, 4, 2>), 256,
-                                             0, s>>>(it, P, st, slope, act, o);
-    } else {
-      gat_fwd_k128_kernel<float, NH, 4, 3><<<grid_for(gat_fwd_k128_kernel<float, NH, 4, 3>), 256,
-                                             0, s>>>(it, P, st, slope, act, o);
-    }
+    auto* kern = o.Q ? gat_fwd_k128_kernel<float, NH, 4, 3, true>
+                     : gat_fwd_k128_kernel<float, NH, 4, 3, false>;
+    kern<<<grid_for(kern), 256, 0, s>>>(it, P, st, slope, act, o);
     AGNN_LAUNCH_CHECK("gat_fwd_kernel");
   }));
   return AGNN_OK;
@@ -635,19 +839,10 @@ agnn_status gat_fwd_k128_bf16(const Items& it_all, int heads, const bf16* P, con
   if (sst != AGNN_OK) return sst;
   const Items it = long_items(it_all);
   if (it.n_chunks + it.n_light == 0) return AGNN_OK;
-  static int minb = -1;
-  if (minb < 0) {
-    const char* e = getenv("AGNN_FWD_MINB");
-    minb = e ? atoi(e) : 3;
-  }
   AGNN_K128_DISPATCH(heads, ({
-    if (minb == 4) {
-      gat_fwd_k128_kernel<bf16, NH, 8, 4><<<grid_for(gat_fwd_k128_kernel<bf16, NH, 8, 4>), 256, 0,
-                                            s>>>(it, P, st, slope, act, o);
-    } else {
-      gat_fwd_k128_kernel<bf16, NH, 8, 3><<<grid_for(gat_fwd_k128_kernel<bf16, NH, 8, 3>), 256, 0,
-                                            s>>>(it, P, st, slope, act, o);
-    }
+    auto* kern = o.Q ? gat_fwd_k128_kernel<bf16, NH, 8, 3, true>
+                     : gat_fwd_k128_kernel<bf16, NH, 8, 3, false>;
+    kern<<<grid_for(kern), 256, 0, s>>>(it, P, st, slope, act, o);
     AGNN_LAUNCH_CHECK("gat_fwd_kernel");
   }));
   return AGNN_OK;
@@ -695,6 +890,25 @@ agnn_status gat_bwd_k128(const Items& it_all, int heads, const GatBwdArgs& A, in
   // short rows: their da partials follow the main kernel's rows
   int64_t sw = 0;
   agnn_status sst = gat_bwd_short(it_all, heads, A, *warps, &sw, s);
+  *warps += sw;
+  return sst;
+}
+
+agnn_status gat_bwd_k128f(const Items& it_all, int heads, const GatBwdArgs& A, int64_t* warps,
+                          cudaStream_t s) {
+  *warps = 0;
+  const Items it = long_items(it_all);
+  AGNN_K128_DISPATCH(heads, ({
+    auto* kern = A.P16 ? (void (*)(Items, GatBwdArgs))gat_bwd_k128f_kernel<bf16, NH, 3>
+                       : (void (*)(Items, GatBwdArgs))gat_bwd_k128f_kernel<float, NH, 3>;
+    const int grid = grid_for(kern);
+    kern<<<grid, 256, 0, s>>>(it, A);
+    AGNN_LAUNCH_CHECK("gat_bwd_kernel");
+    *warps = (int64_t)grid * 8;
+  }));
+  // short rows: their da partials follow the main kernel's rows
+  int64_t sw = 0;
+  agnn_status sst = gat_bwd_short_f(it_all, heads, A, *warps, &sw, s);
   *warps += sw;
   return sst;
 }

@@ -41,6 +41,10 @@ struct Cols<float, V4> {
 #pragma unroll
     for (int i = 0; i < V4; ++i) v[i] = ldg4(p + 4 * i);
   }
+  __device__ __forceinline__ void load(const float* p, uint64_t pol) {
+#pragma unroll
+    for (int i = 0; i < V4; ++i) v[i] = ldg4_pol(p + 4 * i, pol);
+  }
   __device__ __forceinline__ void zero() {
 #pragma unroll
     for (int i = 0; i < V4; ++i) v[i] = f4(0.f);
@@ -54,6 +58,10 @@ struct Cols<bf16, V4> {
   __device__ __forceinline__ void load(const bf16* p) {
 #pragma unroll
     for (int i = 0; i < V4 / 2; ++i) v[i] = __ldg(reinterpret_cast<const uint4*>(p) + i);
+  }
+  __device__ __forceinline__ void load(const bf16* p, uint64_t pol) {
+#pragma unroll
+    for (int i = 0; i < V4 / 2; ++i) v[i] = ldg16_pol(reinterpret_cast<const uint4*>(p) + i, pol);
   }
   __device__ __forceinline__ void zero() {
 #pragma unroll
@@ -109,11 +117,13 @@ struct RowPipe {
 };
 
 // ---------------------------------------------------------------- forward
-template <typename TP, int NH, int SUB, int MINB, int U16>
+// QF: also u_i, C_i and Q_i of the factored backward (gat_k128.cu forward, gat_args.cuh)
+template <typename TP, int NH, int SUB, int MINB, int U16, bool QF>
 __global__ void __launch_bounds__(256, MINB)
 gat_fwd_short_kernel(const int4* __restrict__ meta, const int32_t* __restrict__ col,
                      int64_t n_rows, int64_t row_begin, const TP* __restrict__ P,
-                     const float* __restrict__ st, float slope, int act, GatFwdOut o) {
+                     const float* __restrict__ st, float slope, int act, GatFwdOut o,
+                     uint32_t col_mask, int hot_min, int cold_first) {
   using LY = Lay<SUB>;
   using RP = RowPipe<SUB>;
   constexpr int RPW = LY::RPW, CPL = LY::CPL, V4 = LY::V4, CW = RP::CW;
@@ -126,6 +136,7 @@ gat_fwd_short_kernel(const int4* __restrict__ meta, const int32_t* __restrict__ 
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
   const int64_t step = nw * RPW;
   const RP rp{meta, col, n_rows, g, q};
+  const Gath ga(col_mask, hot_min, cold_first);
   int64_t base = gw * RPW;
   int4 m_cur = rp.rec(base), m_nxt = rp.rec(base + step);
   int c_cur[CW];
@@ -140,10 +151,10 @@ gat_fwd_short_kernel(const int4* __restrict__ meta, const int32_t* __restrict__ 
     const int maxdeg = __reduce_max_sync(FULL, deg);
     const int64_t grow = row_begin + row;
     const float si = ok ? __ldg(st + grow * (2 * NH) + h) : 0.f;
-    float m = -INFINITY, l = 0.f;
-    float4 acc[V4];
+    float m = -INFINITY, l = 0.f, lc = 0.f;
+    float4 acc[V4], accu[V4];
 #pragma unroll
-    for (int v = 0; v < V4; ++v) acc[v] = f4(0.f);
+    for (int v = 0; v < V4; ++v) acc[v] = accu[v] = f4(0.f);
 #pragma unroll 1
     for (int b0 = 0; b0 < maxdeg; b0 += U) {
       {
@@ -155,43 +166,57 @@ gat_fwd_short_kernel(const int4* __restrict__ meta, const int32_t* __restrict__ 
 #pragma unroll
         for (int u = 0; u < U; ++u) {
           if (j[u] >= 0) {
-            tj[u] = __ldg(st + (int64_t)j[u] * (2 * NH) + NH + h);
-            pj[u].load(P + (int64_t)j[u] * K + c0);
+            const int64_t jr = ga.row(j[u]);
+            const uint64_t pol = ga.policy(j[u]);
+            tj[u] = ldg1_pol(st + jr * (2 * NH) + NH + h, pol);
+            pj[u].load(P + jr * K + c0, pol);
           } else {
             tj[u] = 0.f;
             pj[u].zero();
           }
         }
-        float e[U], bm = m;
+        float e[U], pre[U], bm = m;
 #pragma unroll
         for (int u = 0; u < U; ++u) {
-          const float pre = si + tj[u];
-          e[u] = j[u] >= 0 ? fmaxf(pre, slope * pre) : -INFINITY;  // LReLU, 0 <= slope <= 1
+          pre[u] = si + tj[u];
+          e[u] = j[u] >= 0 ? fmaxf(pre[u], slope * pre[u]) : -INFINITY;  // LReLU, 0 <= slope <= 1
           bm = fmaxf(bm, e[u]);
         }
         if (bm != -INFINITY) {  // this row has edges in the batch
           const float sc = ex2(m - bm);  // 0 on the first batch (m = -inf)
-          l *= sc;
+          l = __fmul_rn(l, sc);  // never contracted (training and inference variants agree)
+          if constexpr (QF) lc = __fmul_rn(lc, sc);
 #pragma unroll
-          for (int v = 0; v < V4; ++v) acc[v] = mul4(sc, acc[v]);
+          for (int v = 0; v < V4; ++v) {
+            acc[v] = mul4(sc, acc[v]);
+            if constexpr (QF) accu[v] = mul4(sc, accu[v]);
+          }
           m = bm;
 #pragma unroll
           for (int u = 0; u < U; ++u) {
             const float p = ex2(e[u] - m);  // 0 for padding edges
-            l += p;
+            l = __fadd_rn(l, p);
+            const float pc = pre[u] > 0.f ? p : p * slope;
+            if constexpr (QF) lc = __fadd_rn(lc, pc);
 #pragma unroll
-            for (int v = 0; v < V4; ++v) acc[v] = fma4(p, pj[u].get(v), acc[v]);
+            for (int v = 0; v < V4; ++v) {
+              const float4 x = pj[u].get(v);
+              acc[v] = fma4(p, x, acc[v]);
+              if constexpr (QF) accu[v] = fma4(pc, x, accu[v]);
+            }
           }
         }
       }
     }
     if (ok) {
       const float inv = l > 0.f ? 1.f / l : 0.f;
+      const float r = l > 0.f ? lc / l : 0.f;
 #pragma unroll
       for (int v = 0; v < V4; ++v) {
         const float4 z = mul4(inv, acc[v]);
         if (o.Z) st4(o.Z + row * K + c0 + 4 * v, z);
         st4(o.Hout + row * K + c0 + 4 * v, act_fwd4(act, z));
+        if constexpr (QF) st4(o.Q + row * K + c0 + 4 * v, mul4(inv, fma4(-r, acc[v], accu[v])));
       }
       if (o.m && (c0 % D) == 0) {
         o.m[row * NH + h] = l > 0.f ? m : 0.f;
@@ -216,7 +241,8 @@ __device__ __forceinline__ const bf16* pick_rows<bf16>(const float*, const bf16*
 template <typename TP, int NH, int SUB, int U, int MINB>
 __global__ void __launch_bounds__(256, MINB)
 gat_bwd_short_kernel(const int4* __restrict__ meta, const int32_t* __restrict__ col,
-                     int64_t n_rows, int64_t row_begin, GatBwdArgs A, int64_t da_row0) {
+                     int64_t n_rows, int64_t row_begin, GatBwdArgs A, int64_t da_row0,
+                     uint32_t col_mask, int hot_min, int cold_first) {
   using LY = Lay<SUB>;
   using RP = RowPipe<SUB>;
   constexpr int RPW = LY::RPW, CPL = LY::CPL, V4 = LY::V4, CW = RP::CW;
@@ -232,6 +258,7 @@ gat_bwd_short_kernel(const int4* __restrict__ meta, const int32_t* __restrict__ 
   const TP* Gb = pick_rows<TP>(A.G, A.G16);
   const float slope = A.slope;
   const RP rp{meta, col, n_rows, g, q};
+  const Gath ga(col_mask, hot_min, cold_first);
   float4 da1[V4], da2[V4];
 #pragma unroll
   for (int v = 0; v < V4; ++v) da1[v] = da2[v] = f4(0.f);
@@ -277,10 +304,12 @@ gat_bwd_short_kernel(const int4* __restrict__ meta, const int32_t* __restrict__ 
 #pragma unroll
         for (int u = 0; u < U; ++u) {
           if (i[u] >= 0) {
-            pi[u].load(Pb + (int64_t)i[u] * K + c0);
-            gi[u].load(Gb + (int64_t)i[u] * K + c0);
-            ri[u] = __ldg(A.rec + (int64_t)i[u] * NH + h);
-            ti[u] = __ldg(A.st + (int64_t)i[u] * (2 * NH) + NH + h);
+            const int64_t ir = ga.row(i[u]);
+            const uint64_t pol = ga.policy(i[u]);
+            pi[u].load(Pb + ir * K + c0, pol);
+            gi[u].load(Gb + ir * K + c0, pol);
+            ri[u] = ldg4_pol(reinterpret_cast<const float*>(A.rec + ir * NH + h), pol);
+            ti[u] = ldg1_pol(A.st + ir * (2 * NH) + NH + h, pol);
           } else {
             pi[u].zero();
             gi[u].zero();
@@ -373,6 +402,144 @@ gat_bwd_short_kernel(const int4* __restrict__ meta, const int32_t* __restrict__ 
   }
 }
 
+// factored backward (column role only; ds_j from the prologue, gat_args.cuh): per
+// edge the lane gathers its slice of G_i and the record of its head, recomputes
+// alpha_ij, c'_ij = alpha_ij lambda_ij, and accumulates acc += alpha G_i, v += c' G_i,
+// sd += c' delta_i (every lane of a head the same scalars); per row
+// dt_j = P_j . v_j - sd, dP_j = acc + ds_j a1 + dt_j a2.
+template <typename TP, int NH, int SUB, int U, int MINB>
+__global__ void __launch_bounds__(256, MINB)
+gat_bwd_short_f_kernel(const int4* __restrict__ meta, const int32_t* __restrict__ col,
+                       int64_t n_rows, int64_t row_begin, GatBwdArgs A, int64_t da_row0,
+                       uint32_t col_mask, int hot_min, int cold_first) {
+  using LY = Lay<SUB>;
+  using RP = RowPipe<SUB>;
+  constexpr int CPL = LY::CPL, V4 = LY::V4, CW = RP::CW;
+  constexpr int D = K / NH, HLS = D / CPL;  // HLS lanes share a head
+  static_assert(D >= CPL, "a lane's columns lie in one head");
+  static_assert(kMaxShort % U == 0, "whole batches");
+  const int lane = threadIdx.x & 31, g = lane / SUB, q = lane % SUB;
+  const int c0 = q * CPL, h = c0 / D;
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const int64_t step = nw * LY::RPW;
+  const TP* Pb = pick_rows<TP>(A.P, A.P16);
+  const TP* Gb = pick_rows<TP>(A.G, A.G16);
+  const float slope = A.slope;
+  const RP rp{meta, col, n_rows, g, q};
+  const Gath ga(col_mask, hot_min, cold_first);
+  float4 da1[V4], da2[V4];
+#pragma unroll
+  for (int v = 0; v < V4; ++v) da1[v] = da2[v] = f4(0.f);
+  int64_t base = gw * LY::RPW;
+  int4 m_cur = rp.rec(base), m_nxt = rp.rec(base + step);
+  int c_cur[CW];
+  rp.cols(m_cur, c_cur);
+  for (; base < n_rows; base += step) {
+    int c_nxt[CW];
+    rp.cols(m_nxt, c_nxt);
+    const int4 m_nn = rp.rec(base + 2 * step);
+    const bool ok = base + g < n_rows;
+    const int64_t row = m_cur.x;
+    const int deg = min(m_cur.y, kMaxShort);
+    const int maxdeg = __reduce_max_sync(FULL, deg);  // warp-uniform trip count
+    const int64_t grow = row_begin + row;
+    const float tj = __ldg(A.st + grow * (2 * NH) + NH + h);
+    float4 acc[V4], accv[V4];
+#pragma unroll
+    for (int v = 0; v < V4; ++v) acc[v] = accv[v] = f4(0.f);
+    float sd = 0.f;
+#pragma unroll 1
+    for (int b0 = 0; b0 < maxdeg; b0 += U) {
+      int i[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) i[u] = rp.id(c_cur, b0 + u, lane);
+      Cols<TP, V4> gi[U];
+      float4 ri[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        if (i[u] >= 0) {
+          const int64_t ir = ga.row(i[u]);
+          const uint64_t pol = ga.policy(i[u]);
+          gi[u].load(Gb + ir * K + c0, pol);
+          ri[u] = ldg4_pol(reinterpret_cast<const float*>(A.rec + ir * NH + h), pol);
+        } else {
+          gi[u].zero();
+          ri[u] = f4(0.f);
+        }
+      }
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        if (i[u] >= 0) {
+          const float pre = ri[u].x + tj;
+          const float e = fmaxf(pre, slope * pre);
+          const float al = ex2(e - ri[u].y) * ri[u].z;
+          const float cc = pre > 0.f ? al : al * slope;
+          sd = fmaf(cc, ri[u].w, sd);
+#pragma unroll
+          for (int v = 0; v < V4; ++v) {
+            const float4 x = gi[u].get(v);
+            acc[v] = fma4(al, x, acc[v]);
+            accv[v] = fma4(cc, x, accv[v]);
+          }
+        }
+      }
+    }
+    float4 Pj[V4];
+    {
+      Cols<TP, V4> cp;
+      cp.load(Pb + grow * K + c0);
+#pragma unroll
+      for (int v = 0; v < V4; ++v) Pj[v] = cp.get(v);
+    }
+    float x = 0.f;
+#pragma unroll
+    for (int v = 0; v < V4; ++v) x += dot4(Pj[v], accv[v]);
+#pragma unroll
+    for (int o = 1; o < HLS; o <<= 1) x += __shfl_xor_sync(FULL, x, o);
+    if (ok) {
+      const float dt = x - sd;
+      const float ds = A.ds_row[row * NH + h];
+#pragma unroll
+      for (int v = 0; v < V4; ++v) {
+        const int cc = (c0 % D) + 4 * v;
+        const float4 a1v = ldg4(A.a + h * 2 * D + cc);
+        const float4 a2v = ldg4(A.a + h * 2 * D + D + cc);
+        float4 dp = fma4(ds, a1v, acc[v]);
+        dp = fma4(dt, a2v, dp);
+        st4(A.dP + row * K + c0 + 4 * v, dp);
+        da1[v] = fma4(ds, Pj[v], da1[v]);
+        da2[v] = fma4(dt, Pj[v], da2[v]);
+      }
+    }
+    m_cur = m_nxt;
+    m_nxt = m_nn;
+#pragma unroll
+    for (int k = 0; k < CW; ++k) c_cur[k] = c_nxt[k];
+  }
+#pragma unroll
+  for (int o = SUB; o < 32; o <<= 1) {
+#pragma unroll
+    for (int v = 0; v < V4; ++v) {
+      da1[v].x += __shfl_xor_sync(FULL, da1[v].x, o);
+      da1[v].y += __shfl_xor_sync(FULL, da1[v].y, o);
+      da1[v].z += __shfl_xor_sync(FULL, da1[v].z, o);
+      da1[v].w += __shfl_xor_sync(FULL, da1[v].w, o);
+      da2[v].x += __shfl_xor_sync(FULL, da2[v].x, o);
+      da2[v].y += __shfl_xor_sync(FULL, da2[v].y, o);
+      da2[v].z += __shfl_xor_sync(FULL, da2[v].z, o);
+      da2[v].w += __shfl_xor_sync(FULL, da2[v].w, o);
+    }
+  }
+  if (g == 0) {
+#pragma unroll
+    for (int v = 0; v < V4; ++v) {
+      st4(A.da_part + (da_row0 + gw) * 2 * K + c0 + 4 * v, da1[v]);
+      st4(A.da_part + (da_row0 + gw) * 2 * K + K + c0 + 4 * v, da2[v]);
+    }
+  }
+}
+
 template <typename F>
 int grid_for(F* f) {
   return persistent_blocks(reinterpret_cast<const void*>(f));
@@ -401,10 +568,12 @@ agnn_status gat_fwd_short(const Items& it, int heads, const TP* P, const float* 
     }
     // 3 blocks / SM with 4 bf16 rows per batch, or 2 blocks / SM with 8
     // (fp32: 2 blocks / SM, 4 rows per batch; the 3-block variant spills)
-    auto* kern = (sizeof(TP) == 4 || minb == 2) ? gat_fwd_short_kernel<TP, NH, 8, 2, 8>
-                                                : gat_fwd_short_kernel<TP, NH, 8, 3, 4>;
+    auto* kern = o.Q ? ((sizeof(TP) == 4 || minb == 2) ? gat_fwd_short_kernel<TP, NH, 8, 2, 8, true>
+                                                       : gat_fwd_short_kernel<TP, NH, 8, 3, 4, true>)
+                     : ((sizeof(TP) == 4 || minb == 2) ? gat_fwd_short_kernel<TP, NH, 8, 2, 8, false>
+                                                       : gat_fwd_short_kernel<TP, NH, 8, 3, 4, false>);
     kern<<<grid_for(kern), 256, 0, s>>>(it.short_meta, it.col, it.n_short, it.row_begin, P, st,
-                                         slope, act, o);
+                                         slope, act, o, it.col_mask, it.hot_min, it.cold_first);
     AGNN_LAUNCH_CHECK("gat_fwd_short_kernel");
   }));
   return AGNN_OK;
@@ -430,7 +599,8 @@ agnn_status gat_bwd_short(const Items& it, int heads, const GatBwdArgs& A, int64
     if (A.P16) {
       auto launch = [&](auto* kern) {
         grid = grid_for(kern);
-        kern<<<grid, 256, 0, s>>>(it.short_meta, it.col, it.n_short, it.row_begin, A, da_row0);
+        kern<<<grid, 256, 0, s>>>(it.short_meta, it.col, it.n_short, it.row_begin, A, da_row0,
+                                  it.col_mask, it.hot_min, it.cold_first);
       };
       if (variant == 1)
         launch(gat_bwd_short_kernel<bf16, NH, 8, 4, 1>);
@@ -441,8 +611,26 @@ agnn_status gat_bwd_short(const Items& it, int heads, const GatBwdArgs& A, int64
     } else {
       auto* kern = gat_bwd_short_kernel<float, NH, 16, 2, 2>;
       grid = grid_for(kern);
-      kern<<<grid, 256, 0, s>>>(it.short_meta, it.col, it.n_short, it.row_begin, A, da_row0);
+      kern<<<grid, 256, 0, s>>>(it.short_meta, it.col, it.n_short, it.row_begin, A, da_row0,
+                                it.col_mask, it.hot_min, it.cold_first);
     }
+    AGNN_LAUNCH_CHECK("gat_bwd_short_kernel");
+    *warps = (int64_t)grid * 8;
+  }));
+  return AGNN_OK;
+}
+
+agnn_status gat_bwd_short_f(const Items& it, int heads, const GatBwdArgs& A, int64_t da_row0,
+                            int64_t* warps, cudaStream_t s) {
+  *warps = 0;
+  if (it.n_short == 0) return AGNN_OK;
+  AGNN_SHORT_DISPATCH(heads, ({
+    // 16 lanes per row (2 rows per warp), 8 (fp32) or 16 (bf16) edges per batch
+    auto* kern = A.P16 ? gat_bwd_short_f_kernel<bf16, NH, 16, 8, 2>
+                       : gat_bwd_short_f_kernel<float, NH, 16, 4, 2>;
+    const int grid = grid_for(kern);
+    kern<<<grid, 256, 0, s>>>(it.short_meta, it.col, it.n_short, it.row_begin, A, da_row0,
+                              it.col_mask, it.hot_min, it.cold_first);
     AGNN_LAUNCH_CHECK("gat_bwd_short_kernel");
     *warps = (int64_t)grid * 8;
   }));

@@ -45,7 +45,96 @@ __global__ void validate_kernel(const int64_t* __restrict__ rp, const int32_t* _
   }
 }
 
+// occurrences of every column id in the local CSR (how often a pass gathers row j)
+__global__ void col_count_kernel(const int32_t* __restrict__ col, int64_t nnz,
+                                 int32_t* __restrict__ cnt) {
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < nnz;
+       e += (int64_t)gridDim.x * blockDim.x)
+    atomicAdd(cnt + col[e], 1);
+}
+
+struct ClassThresholds {
+  int32_t t[8];  // t[q], q = 1..7: class >= q iff count >= t[q]
+};
+
+// col_hint[e] = col[e] | class(col[e]) << kColHintShift
+__global__ void col_class_kernel(const int32_t* __restrict__ col, int64_t nnz,
+                                 const int32_t* __restrict__ cnt, ClassThresholds th,
+                                 int32_t* __restrict__ out) {
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < nnz;
+       e += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t c = col[e], k = cnt[c];
+    int q = 0;
+#pragma unroll
+    for (int x = 1; x < 8; ++x) q += k >= th.t[x];
+    out[e] = c | (q << kColHintShift);
+  }
+}
+
+// L2 budget (MB) for evict_last rows per pass; 0 disables the column classes
+int64_t l2_hot_budget() {
+  static const int64_t v = [] {
+    const char* e = getenv("AGNN_L2_HOT_MB");
+    return e ? (int64_t)atoll(e) : (int64_t)128;
+  }();
+  return v;
+}
+
+// Column classes for the L2 residency hints.  Class q (1..7) = the column is among
+// the 2^(21-q) vertices this rank gathers most often (ties at a threshold are all
+// left out; a vertex gathered once is never hot).  Plan time only; synchronises.
+agnn_status build_col_classes(Plan& p, cudaStream_t s) {
+  if (p.n > ((int64_t)1 << kColHintShift) || p.nnz == 0 || l2_hot_budget() <= 0) return AGNN_OK;
+  int32_t* cnt = nullptr;
+  AGNN_CUDA_TRY(cudaMallocAsync(&cnt, sizeof(int32_t) * (size_t)p.n, s));
+  AGNN_CUDA_TRY(cudaMemsetAsync(cnt, 0, sizeof(int32_t) * (size_t)p.n, s));
+  col_count_kernel<<<kNumSMs * 8, 256, 0, s>>>(p.col_idx, p.nnz, cnt);
+  AGNN_LAUNCH_CHECK("col_count_kernel");
+  std::vector<int32_t> hc((size_t)p.n);
+  AGNN_CUDA_TRY(cudaMemcpyAsync(hc.data(), cnt, sizeof(int32_t) * hc.size(),
+                                cudaMemcpyDeviceToHost, s));
+  AGNN_CUDA_TRY(cudaStreamSynchronize(s));
+  int32_t maxc = 0;
+  for (int32_t c : hc) maxc = std::max(maxc, c);
+  std::vector<int64_t> ge((size_t)maxc + 2, 0);  // ge[t] = #{count >= t}
+  for (int32_t c : hc) ++ge[(size_t)c];
+  for (int64_t t = maxc - 1; t >= 0; --t) ge[(size_t)t] += ge[(size_t)t + 1];
+  ClassThresholds th;
+  th.t[0] = 0;
+  p.class_rows[0] = p.n;
+  for (int q = 1; q < 8; ++q) {
+    const int64_t R = (int64_t)1 << (21 - q);
+    int64_t t = 2;
+    while (t <= maxc && ge[(size_t)t] > R) ++t;
+    th.t[q] = (int32_t)std::min<int64_t>(t, (int64_t)maxc + 1);
+    p.class_rows[q] = th.t[q] <= maxc ? ge[(size_t)th.t[q]] : 0;
+  }
+  AGNN_CUDA_TRY(cudaMalloc(&p.col_hint, sizeof(int32_t) * (size_t)p.nnz));
+  col_class_kernel<<<kNumSMs * 8, 256, 0, s>>>(p.col_idx, p.nnz, cnt, th, p.col_hint);
+  AGNN_LAUNCH_CHECK("col_class_kernel");
+  AGNN_CUDA_TRY(cudaFreeAsync(cnt, s));
+  AGNN_CUDA_TRY(cudaStreamSynchronize(s));
+  return AGNN_OK;
+}
+
 }  // namespace
+
+Items l2_hinted(const Items& it, const Plan& p, int64_t row_bytes) {
+  static const int cold_first = [] {
+    const char* e = getenv("AGNN_L2_COLD");
+    return e ? atoi(e) : 1;
+  }();
+  if (!p.col_hint || it.col != p.col_idx || row_bytes <= 0) return it;
+  const int64_t budget = l2_hot_budget() << 20;
+  int q = 1;
+  while (q < 8 && p.class_rows[q] * row_bytes > budget) ++q;
+  Items r = it;
+  r.col = p.col_hint;
+  r.col_mask = (1u << kColHintShift) - 1u;
+  r.hot_min = q;
+  r.cold_first = cold_first;
+  return r;
+}
 
 int persistent_blocks(const void* func) {
   static std::mutex mu;
@@ -268,6 +357,11 @@ agnn_status plan_build(Plan& p, cudaStream_t s) {
     AGNN_CUDA_TRY(cudaStreamSynchronize(s));
   }
   p.meta_block = L.block;
+  // L2 residency classes of the columns (symmetric or directed; the row pass's gathers)
+  if (const char* e = getenv("AGNN_L2_SETASIDE_MB")) {  // measurement: persisting L2 carve-out
+    cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)atoll(e) << 20);
+  }
+  if ((st = build_col_classes(p, s)) != AGNN_OK) return st;
   // 4. directed pattern on one GPU: the CSC and its work lists (column role of the backward)
   if (p.directed() && p.world == 1 && p.n_local == p.n) {
     const size_t ptr_bytes = ((sizeof(int64_t) * (size_t)(p.n + 1)) + 255) & ~size_t(255);

@@ -1,0 +1,14 @@
+# factored GAT backward: parity tests + C5 A/B (fp32, bf16)
+timeout 900 python -m pytest tests -m gpu -x -q 2>&1 | tail -15 > gpurun_out/fact_pytest.txt
+run() {
+  for p in fp32 bf16; do
+    timeout 300 python bench.py --prec $p --steps 5 --no-cpu-baseline --no-e2e --no-bf16-line 2>gpurun_out/fact_err_$p.txt | python -c "
+import json,sys
+d=json.loads([l for l in sys.stdin if l.startswith('{')][-1])
+print('$p', '$*', round(d['value']/1e9,3), round(d['ms_per_step'],1), {k:round(v['ms_per_step'],2) for k,v in d['kernels'].items() if v['ms_per_step']>1}, d['clocks']['sm_mhz'])
+" >> gpurun_out/fact_sweep.txt
+  done
+}
+AGNN_GAT_FACTORED=0 run fact=0
+run fact=1
+AGNN_GAT_FACTORED=0 run fact=0
