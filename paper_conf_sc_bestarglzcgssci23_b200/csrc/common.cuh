@@ -250,11 +250,13 @@ struct Plan {
   int32_t* empty_rows = nullptr;      // [n_empty] local rows without stored entries
   int64_t n_empty = 0;
   // L2 residency classes of the gathered rows (plan.cu "column classes"): a
-  // plan-owned copy of col_idx whose bits [28, 31) hold the class c in 0..7 of
-  // the column (c >= q: among the 2^(21-q) most-gathered vertices of this rank);
-  // null when n > 2^28 or disabled (AGNN_L2_HOT_MB=0)
+  // plan-owned copy of col_idx whose bits [hint_shift, 31) hold the class c of
+  // the column (c >= q: among the ~2^(21 - (q-1)/4) most-gathered vertices of
+  // this rank); null when n > 2^28 or disabled (AGNN_L2_HOT_MB=0)
   int32_t* col_hint = nullptr;
-  int64_t class_rows[8] = {};         // [q] = vertices of class >= q (host)
+  int hint_shift = 0;
+  int n_classes = 0;                  // classes 1..n_classes-1 in use
+  int64_t class_rows[64] = {};        // [q] = vertices of class >= q (host)
   // directed patterns (world == 1): the transposed pattern (CSC of the local
   // matrix) and its work lists, for the column role of the backward
   // (PAPER.md:252 Psi^T; reading A4).  Plan-owned; null for symmetric plans.

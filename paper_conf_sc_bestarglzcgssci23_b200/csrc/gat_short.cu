@@ -123,7 +123,7 @@ __global__ void __launch_bounds__(256, MINB)
 gat_fwd_short_kernel(const int4* __restrict__ meta, const int32_t* __restrict__ col,
                      int64_t n_rows, int64_t row_begin, const TP* __restrict__ P,
                      const float* __restrict__ st, float slope, int act, GatFwdOut o,
-                     uint32_t col_mask, int hot_min, int cold_first) {
+                     uint32_t col_mask, uint32_t hot_thr, int cold_first) {
   using LY = Lay<SUB>;
   using RP = RowPipe<SUB>;
   constexpr int RPW = LY::RPW, CPL = LY::CPL, V4 = LY::V4, CW = RP::CW;
@@ -136,7 +136,7 @@ gat_fwd_short_kernel(const int4* __restrict__ meta, const int32_t* __restrict__ 
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
   const int64_t step = nw * RPW;
   const RP rp{meta, col, n_rows, g, q};
-  const Gath ga(col_mask, hot_min, cold_first);
+  const Gath ga(col_mask, hot_thr, cold_first);
   int64_t base = gw * RPW;
   int4 m_cur = rp.rec(base), m_nxt = rp.rec(base + step);
   int c_cur[CW];
@@ -242,7 +242,7 @@ template <typename TP, int NH, int SUB, int U, int MINB>
 __global__ void __launch_bounds__(256, MINB)
 gat_bwd_short_kernel(const int4* __restrict__ meta, const int32_t* __restrict__ col,
                      int64_t n_rows, int64_t row_begin, GatBwdArgs A, int64_t da_row0,
-                     uint32_t col_mask, int hot_min, int cold_first) {
+                     uint32_t col_mask, uint32_t hot_thr, int cold_first) {
   using LY = Lay<SUB>;
   using RP = RowPipe<SUB>;
   constexpr int RPW = LY::RPW, CPL = LY::CPL, V4 = LY::V4, CW = RP::CW;
@@ -258,7 +258,7 @@ gat_bwd_short_kernel(const int4* __restrict__ meta, const int32_t* __restrict__ 
   const TP* Gb = pick_rows<TP>(A.G, A.G16);
   const float slope = A.slope;
   const RP rp{meta, col, n_rows, g, q};
-  const Gath ga(col_mask, hot_min, cold_first);
+  const Gath ga(col_mask, hot_thr, cold_first);
   float4 da1[V4], da2[V4];
 #pragma unroll
   for (int v = 0; v < V4; ++v) da1[v] = da2[v] = f4(0.f);
@@ -411,7 +411,7 @@ template <typename TP, int NH, int SUB, int U, int MINB>
 __global__ void __launch_bounds__(256, MINB)
 gat_bwd_short_f_kernel(const int4* __restrict__ meta, const int32_t* __restrict__ col,
                        int64_t n_rows, int64_t row_begin, GatBwdArgs A, int64_t da_row0,
-                       uint32_t col_mask, int hot_min, int cold_first) {
+                       uint32_t col_mask, uint32_t hot_thr, int cold_first) {
   using LY = Lay<SUB>;
   using RP = RowPipe<SUB>;
   constexpr int CPL = LY::CPL, V4 = LY::V4, CW = RP::CW;
@@ -427,7 +427,7 @@ gat_bwd_short_f_kernel(const int4* __restrict__ meta, const int32_t* __restrict_
   const TP* Gb = pick_rows<TP>(A.G, A.G16);
   const float slope = A.slope;
   const RP rp{meta, col, n_rows, g, q};
-  const Gath ga(col_mask, hot_min, cold_first);
+  const Gath ga(col_mask, hot_thr, cold_first);
   float4 da1[V4], da2[V4];
 #pragma unroll
   for (int v = 0; v < V4; ++v) da1[v] = da2[v] = f4(0.f);
@@ -568,12 +568,30 @@ agnn_status gat_fwd_short(const Items& it, int heads, const TP* P, const float* 
     }
     // 3 blocks / SM with 4 bf16 rows per batch, or 2 blocks / SM with 8
     // (fp32: 2 blocks / SM, 4 rows per batch; the 3-block variant spills)
-    auto* kern = o.Q ? ((sizeof(TP) == 4 || minb == 2) ? gat_fwd_short_kernel<TP, NH, 8, 2, 8, true>
-                                                       : gat_fwd_short_kernel<TP, NH, 8, 3, 4, true>)
-                     : ((sizeof(TP) == 4 || minb == 2) ? gat_fwd_short_kernel<TP, NH, 8, 2, 8, false>
-                                                       : gat_fwd_short_kernel<TP, NH, 8, 3, 4, false>);
+    // AGNN_FWD_SHORT_VARIANT (measurement): 0 = default (fp32: 8 lanes per row, 2 blocks
+    // / SM; bf16: as 1); 1 = 16 lanes per row, 3 blocks / SM; 2 = 16 lanes, 2 blocks /
+    // SM, 8-edge bf16 batches; 3 = 8 lanes per row for bf16 too
+    static int variant = -1;
+    if (variant < 0) {
+      const char* e = getenv("AGNN_FWD_SHORT_VARIANT");
+      variant = e ? atoi(e) : 0;
+    }
+    using KF = void (*)(const int4*, const int32_t*, int64_t, int64_t, const TP*, const float*,
+                        float, int, GatFwdOut, uint32_t, uint32_t, int);
+    KF kern;
+    if (variant == 1 || (variant == 0 && sizeof(TP) == 2))  // bf16 default (measured C5)
+      kern = o.Q ? (KF)gat_fwd_short_kernel<TP, NH, 16, 3, 4, true>
+                 : (KF)gat_fwd_short_kernel<TP, NH, 16, 3, 4, false>;
+    else if (variant == 2)
+      kern = o.Q ? (KF)gat_fwd_short_kernel<TP, NH, 16, 2, 8, true>
+                 : (KF)gat_fwd_short_kernel<TP, NH, 16, 2, 8, false>;
+    else  // variant 0 (fp32) or 3
+      kern = o.Q ? ((sizeof(TP) == 4 || minb == 2) ? (KF)gat_fwd_short_kernel<TP, NH, 8, 2, 8, true>
+                                                   : (KF)gat_fwd_short_kernel<TP, NH, 8, 3, 4, true>)
+                 : ((sizeof(TP) == 4 || minb == 2) ? (KF)gat_fwd_short_kernel<TP, NH, 8, 2, 8, false>
+                                                   : (KF)gat_fwd_short_kernel<TP, NH, 8, 3, 4, false>);
     kern<<<grid_for(kern), 256, 0, s>>>(it.short_meta, it.col, it.n_short, it.row_begin, P, st,
-                                         slope, act, o, it.col_mask, it.hot_min, it.cold_first);
+                                         slope, act, o, it.col_mask, it.hot_thr, it.cold_first);
     AGNN_LAUNCH_CHECK("gat_fwd_short_kernel");
   }));
   return AGNN_OK;
@@ -600,7 +618,7 @@ agnn_status gat_bwd_short(const Items& it, int heads, const GatBwdArgs& A, int64
       auto launch = [&](auto* kern) {
         grid = grid_for(kern);
         kern<<<grid, 256, 0, s>>>(it.short_meta, it.col, it.n_short, it.row_begin, A, da_row0,
-                                  it.col_mask, it.hot_min, it.cold_first);
+                                  it.col_mask, it.hot_thr, it.cold_first);
       };
       if (variant == 1)
         launch(gat_bwd_short_kernel<bf16, NH, 8, 4, 1>);
@@ -612,7 +630,7 @@ agnn_status gat_bwd_short(const Items& it, int heads, const GatBwdArgs& A, int64
       auto* kern = gat_bwd_short_kernel<float, NH, 16, 2, 2>;
       grid = grid_for(kern);
       kern<<<grid, 256, 0, s>>>(it.short_meta, it.col, it.n_short, it.row_begin, A, da_row0,
-                                it.col_mask, it.hot_min, it.cold_first);
+                                it.col_mask, it.hot_thr, it.cold_first);
     }
     AGNN_LAUNCH_CHECK("gat_bwd_short_kernel");
     *warps = (int64_t)grid * 8;
@@ -625,12 +643,33 @@ agnn_status gat_bwd_short_f(const Items& it, int heads, const GatBwdArgs& A, int
   *warps = 0;
   if (it.n_short == 0) return AGNN_OK;
   AGNN_SHORT_DISPATCH(heads, ({
-    // 16 lanes per row (2 rows per warp), 8 (fp32) or 16 (bf16) edges per batch
-    auto* kern = A.P16 ? gat_bwd_short_f_kernel<bf16, NH, 16, 8, 2>
-                       : gat_bwd_short_f_kernel<float, NH, 16, 4, 2>;
+    // 16 lanes per row (2 rows per warp); AGNN_BWD_SHORT_VARIANT (measurement):
+    // 3 (default) = 2-edge fp32 / 4-edge bf16 batches with 3 blocks / SM;
+    // 4 = 4 / 8-edge batches, 2 blocks / SM; 1 = 4 / 8-edge, 3 blocks / SM; 2 = 8 lanes per row
+    static int variant = -1;
+    if (variant < 0) {
+      const char* e = getenv("AGNN_BWD_SHORT_VARIANT");
+      variant = e ? atoi(e) : 0;
+    }
+    using KB = void (*)(const int4*, const int32_t*, int64_t, int64_t, GatBwdArgs, int64_t,
+                        uint32_t, uint32_t, int);
+    KB kern;
+    if (variant == 0) variant = 3;  // default (measured C5: 14.7 -> 13.5 ms fp32)
+    if (variant == 1)
+      kern = A.P16 ? (KB)gat_bwd_short_f_kernel<bf16, NH, 16, 8, 3>
+                   : (KB)gat_bwd_short_f_kernel<float, NH, 16, 4, 3>;
+    else if (variant == 2)
+      kern = A.P16 ? (KB)gat_bwd_short_f_kernel<bf16, NH, 8, 4, 2>
+                   : (KB)gat_bwd_short_f_kernel<float, NH, 8, 4, 2>;
+    else if (variant == 3)
+      kern = A.P16 ? (KB)gat_bwd_short_f_kernel<bf16, NH, 16, 4, 3>
+                   : (KB)gat_bwd_short_f_kernel<float, NH, 16, 2, 3>;
+    else  // 4
+      kern = A.P16 ? (KB)gat_bwd_short_f_kernel<bf16, NH, 16, 8, 2>
+                   : (KB)gat_bwd_short_f_kernel<float, NH, 16, 4, 2>;
     const int grid = grid_for(kern);
     kern<<<grid, 256, 0, s>>>(it.short_meta, it.col, it.n_short, it.row_begin, A, da_row0,
-                              it.col_mask, it.hot_min, it.cold_first);
+                              it.col_mask, it.hot_thr, it.cold_first);
     AGNN_LAUNCH_CHECK("gat_bwd_short_kernel");
     *warps = (int64_t)grid * 8;
   }));

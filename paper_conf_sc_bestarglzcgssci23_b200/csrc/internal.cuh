@@ -26,31 +26,29 @@ struct Items {
   int64_t n_short;
   const int32_t* long_rows;
   int64_t n_long;
-  // L2 residency hints (see l2_hinted): col entries carry the column class in bits
-  // [28, 31) when col_mask = 0x0fffffff; gathered rows of class >= hot_min are
-  // loaded with evict_last, the others with evict_first (cold_first) or normal
+  // L2 residency hints (see l2_hinted): col entries carry the column class in the
+  // bits above col_mask; a gathered row is loaded with evict_last iff its entry
+  // (class bits included) is >= hot_thr, else with evict_first (cold_first) or normal
   uint32_t col_mask = 0x7fffffffu;
-  int hot_min = 8;
+  uint32_t hot_thr = 0xffffffffu;
   int cold_first = 0;
 };
-// kColHintShift: bit position of the column class in Plan::col_hint entries
-constexpr int kColHintShift = 28;
+constexpr int kMaxColClasses = 64;
 // the items `it` of plan `p` with L2 hints for gathered rows of `row_bytes` bytes
 // per pass (the hot class is the largest set of rows that fits the L2 budget)
 Items l2_hinted(const Items& it, const Plan& p, int64_t row_bytes);
 // device side of the hints: decode a (possibly classed) column entry c >= 0 into the
 // row id and the L2 policy of its gather
 struct Gath {
-  uint32_t mask;
-  int hot_min;
+  uint32_t mask, thr;
   L2Pol pol;
   __device__ __forceinline__ explicit Gath(const Items& it)
-      : mask(it.col_mask), hot_min(it.hot_min), pol(make_l2pol(it.cold_first)) {}
-  __device__ __forceinline__ Gath(uint32_t m, int h, int cf)
-      : mask(m), hot_min(h), pol(make_l2pol(cf)) {}
+      : mask(it.col_mask), thr(it.hot_thr), pol(make_l2pol(it.cold_first)) {}
+  __device__ __forceinline__ Gath(uint32_t m, uint32_t t, int cf)
+      : mask(m), thr(t), pol(make_l2pol(cf)) {}
   __device__ __forceinline__ int64_t row(int c) const { return (int64_t)((uint32_t)c & mask); }
   __device__ __forceinline__ uint64_t policy(int c) const {
-    return (c >> kColHintShift) >= hot_min ? pol.hot : pol.cold;
+    return (uint32_t)c >= thr ? pol.hot : pol.cold;
   }
 };
 Items items_of(const Plan& p);

@@ -10,6 +10,7 @@
 // any launch geometry and any number of GPUs (the row is always computed by its
 // owner in the same order).
 #include <algorithm>
+#include <cmath>
 #include <cstdlib>
 #include <mutex>
 #include <unordered_map>
@@ -54,10 +55,11 @@ __global__ void col_count_kernel(const int32_t* __restrict__ col, int64_t nnz,
 }
 
 struct ClassThresholds {
-  int32_t t[8];  // t[q], q = 1..7: class >= q iff count >= t[q]
+  int32_t t[kMaxColClasses];  // t[q], q = 1..nq-1: class >= q iff count >= t[q] (nondecreasing)
+  int nq, shift;
 };
 
-// col_hint[e] = col[e] | class(col[e]) << kColHintShift
+// col_hint[e] = col[e] | class(col[e]) << shift
 __global__ void col_class_kernel(const int32_t* __restrict__ col, int64_t nnz,
                                  const int32_t* __restrict__ cnt, ClassThresholds th,
                                  int32_t* __restrict__ out) {
@@ -65,9 +67,8 @@ __global__ void col_class_kernel(const int32_t* __restrict__ col, int64_t nnz,
        e += (int64_t)gridDim.x * blockDim.x) {
     const int32_t c = col[e], k = cnt[c];
     int q = 0;
-#pragma unroll
-    for (int x = 1; x < 8; ++x) q += k >= th.t[x];
-    out[e] = c | (q << kColHintShift);
+    while (q + 1 < th.nq && k >= th.t[q + 1]) ++q;
+    out[e] = (int32_t)((uint32_t)c | ((uint32_t)q << th.shift));
   }
 }
 
@@ -75,16 +76,21 @@ __global__ void col_class_kernel(const int32_t* __restrict__ col, int64_t nnz,
 int64_t l2_hot_budget() {
   static const int64_t v = [] {
     const char* e = getenv("AGNN_L2_HOT_MB");
-    return e ? (int64_t)atoll(e) : (int64_t)128;
+    return e ? (int64_t)atoll(e) : (int64_t)96;
   }();
   return v;
 }
 
-// Column classes for the L2 residency hints.  Class q (1..7) = the column is among
-// the 2^(21-q) vertices this rank gathers most often (ties at a threshold are all
-// left out; a vertex gathered once is never hot).  Plan time only; synchronises.
+// Column classes for the L2 residency hints.  Class >= q (q = 1, 2, ...) = the
+// column is among the R_q = 2^21 / 2^((q-1)/4) vertices this rank gathers most
+// often (ties at a threshold are all left out; a vertex gathered once is never
+// hot).  The classes sit in the free high bits of the column ids.  Plan time
+// only; synchronises.
 agnn_status build_col_classes(Plan& p, cudaStream_t s) {
-  if (p.n > ((int64_t)1 << kColHintShift) || p.nnz == 0 || l2_hot_budget() <= 0) return AGNN_OK;
+  int shift = 1;
+  while (((int64_t)1 << shift) < p.n) ++shift;
+  const int nq = std::min(kMaxColClasses, 1 << std::max(0, 31 - shift));
+  if (p.nnz == 0 || l2_hot_budget() <= 0 || nq < 2) return AGNN_OK;
   int32_t* cnt = nullptr;
   AGNN_CUDA_TRY(cudaMallocAsync(&cnt, sizeof(int32_t) * (size_t)p.n, s));
   AGNN_CUDA_TRY(cudaMemsetAsync(cnt, 0, sizeof(int32_t) * (size_t)p.n, s));
@@ -100,15 +106,19 @@ agnn_status build_col_classes(Plan& p, cudaStream_t s) {
   for (int32_t c : hc) ++ge[(size_t)c];
   for (int64_t t = maxc - 1; t >= 0; --t) ge[(size_t)t] += ge[(size_t)t + 1];
   ClassThresholds th;
+  th.nq = nq;
+  th.shift = shift;
   th.t[0] = 0;
   p.class_rows[0] = p.n;
-  for (int q = 1; q < 8; ++q) {
-    const int64_t R = (int64_t)1 << (21 - q);
-    int64_t t = 2;
-    while (t <= maxc && ge[(size_t)t] > R) ++t;
+  int64_t t = 2;
+  for (int q = 1; q < nq; ++q) {
+    const double R = std::ldexp(1.0, 21) / std::pow(2.0, (q - 1) / 4.0);
+    while (t <= maxc && (double)ge[(size_t)t] > R) ++t;
     th.t[q] = (int32_t)std::min<int64_t>(t, (int64_t)maxc + 1);
     p.class_rows[q] = th.t[q] <= maxc ? ge[(size_t)th.t[q]] : 0;
   }
+  p.hint_shift = shift;
+  p.n_classes = nq;
   AGNN_CUDA_TRY(cudaMalloc(&p.col_hint, sizeof(int32_t) * (size_t)p.nnz));
   col_class_kernel<<<kNumSMs * 8, 256, 0, s>>>(p.col_idx, p.nnz, cnt, th, p.col_hint);
   AGNN_LAUNCH_CHECK("col_class_kernel");
@@ -127,11 +137,11 @@ Items l2_hinted(const Items& it, const Plan& p, int64_t row_bytes) {
   if (!p.col_hint || it.col != p.col_idx || row_bytes <= 0) return it;
   const int64_t budget = l2_hot_budget() << 20;
   int q = 1;
-  while (q < 8 && p.class_rows[q] * row_bytes > budget) ++q;
+  while (q < p.n_classes && p.class_rows[q] * row_bytes > budget) ++q;
   Items r = it;
   r.col = p.col_hint;
-  r.col_mask = (1u << kColHintShift) - 1u;
-  r.hot_min = q;
+  r.col_mask = (1u << p.hint_shift) - 1u;
+  r.hot_thr = q < p.n_classes ? (uint32_t)q << p.hint_shift : 0xffffffffu;
   r.cold_first = cold_first;
   return r;
 }
