@@ -12,6 +12,7 @@ namespace agnn {
 
 constexpr float kLog2e = 1.4426950408889634f;
 constexpr int kNumSMs = 148;
+constexpr int kBundleEdges = 32;  // stored entries per short-row bundle (one warp batch)
 
 // ---- error plumbing (host) -------------------------------------------------
 void set_error(const std::string& msg);
@@ -245,7 +246,11 @@ struct Plan {
   int64_t n_short = 0, n_long = 0;
   int32_t* short_rows = nullptr;
   int32_t* long_rows = nullptr;
-  int4* short_meta = nullptr;         // [n_short] {row, degree, beg lo, beg hi}: one 16-B load
+  int4* short_meta = nullptr;         // [n_short] {row, degree, beg lo, beg hi}: one 16-B load;
+                                      // the n_short_nz non-empty rows first
+  int64_t n_short_nz = 0;
+  int4* bundles = nullptr;            // [n_bundles] {first short record, rows, entries, 0}
+  int64_t n_bundles = 0;
   void* short_block = nullptr;        // backs short_meta
   int32_t* empty_rows = nullptr;      // [n_empty] local rows without stored entries
   int64_t n_empty = 0;

@@ -84,5 +84,13 @@ agnn_status gat_bwd_k128f(const Items& it, int heads, const GatBwdArgs& A, int64
                           cudaStream_t s);
 agnn_status gat_bwd_short_f(const Items& it, int heads, const GatBwdArgs& A, int64_t da_row0,
                             int64_t* warps, cudaStream_t s);
+// bundles of short rows (gat_bundle.cu): the short rows as 32-entry warp batches;
+// AGNN_SHORT_BUNDLES=0 falls back to the row-group short kernels (gat_short.cu)
+bool gat_bundles_enabled(bool bf16_storage);
+template <typename TP>
+agnn_status gat_fwd_bundle(const Items& it, int heads, const TP* P, const float* st, float slope,
+                           int act, const GatFwdOut& o, cudaStream_t s);
+agnn_status gat_bwd_bundle(const Items& it, int heads, const GatBwdArgs& A, int64_t da_row0,
+                           int64_t* warps, cudaStream_t s);
 
 }  // namespace agnn

@@ -801,7 +801,9 @@ bool fwd_tma_enabled() {
 
 agnn_status gat_fwd_k128(const Items& it_all, int heads, const float* P, const float* st,
                          float slope, int act, const GatFwdOut& o, int64_t n_rows, cudaStream_t s) {
-  agnn_status sst = gat_fwd_short<float>(it_all, heads, P, st, slope, act, o, s);
+  agnn_status sst = (gat_bundles_enabled(false) && it_all.bundles)
+                        ? gat_fwd_bundle<float>(it_all, heads, P, st, slope, act, o, s)
+                        : gat_fwd_short<float>(it_all, heads, P, st, slope, act, o, s);
   if (sst != AGNN_OK) return sst;
   const Items it = long_items(it_all);
   if (it.n_chunks + it.n_light == 0) return AGNN_OK;
@@ -835,7 +837,9 @@ agnn_status gat_fwd_k128(const Items& it_all, int heads, const float* P, const f
 
 agnn_status gat_fwd_k128_bf16(const Items& it_all, int heads, const bf16* P, const float* st,
                               float slope, int act, const GatFwdOut& o, cudaStream_t s) {
-  agnn_status sst = gat_fwd_short<bf16>(it_all, heads, P, st, slope, act, o, s);
+  agnn_status sst = (gat_bundles_enabled(true) && it_all.bundles)
+                        ? gat_fwd_bundle<bf16>(it_all, heads, P, st, slope, act, o, s)
+                        : gat_fwd_short<bf16>(it_all, heads, P, st, slope, act, o, s);
   if (sst != AGNN_OK) return sst;
   const Items it = long_items(it_all);
   if (it.n_chunks + it.n_light == 0) return AGNN_OK;
@@ -908,7 +912,9 @@ agnn_status gat_bwd_k128f(const Items& it_all, int heads, const GatBwdArgs& A, i
   }));
   // short rows: their da partials follow the main kernel's rows
   int64_t sw = 0;
-  agnn_status sst = gat_bwd_short_f(it_all, heads, A, *warps, &sw, s);
+  agnn_status sst = (gat_bundles_enabled(A.P16 != nullptr) && it_all.bundles)
+                        ? gat_bwd_bundle(it_all, heads, A, *warps, &sw, s)
+                        : gat_bwd_short_f(it_all, heads, A, *warps, &sw, s);
   *warps += sw;
   return sst;
 }

@@ -22,8 +22,11 @@ struct Items {
   // the light rows split by degree (kernels with a short-row variant): rows of degree
   // <= the plan's short_max (short) and the others (long); items_of_csc: none
   const int32_t* short_rows;
-  const int4* short_meta;     // per short row {row, degree, beg lo, beg hi}
+  const int4* short_meta;     // per short row {row, degree, beg lo, beg hi}; non-empty first
   int64_t n_short;
+  int64_t n_short_nz;         // short rows with stored entries
+  const int4* bundles;        // {first short record, rows, entries, 0} (gat_short.cu)
+  int64_t n_bundles;
   const int32_t* long_rows;
   int64_t n_long;
   // L2 residency hints (see l2_hinted): col entries carry the column class in the

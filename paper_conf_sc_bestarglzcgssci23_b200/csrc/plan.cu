@@ -182,6 +182,9 @@ Items items_of(const Plan& p) {
   it.short_rows = p.short_rows;
   it.short_meta = p.short_meta;
   it.n_short = p.n_short;
+  it.n_short_nz = p.n_short_nz;
+  it.bundles = p.bundles;
+  it.n_bundles = p.n_bundles;
   it.long_rows = p.long_rows;
   it.n_long = p.n_long;
   return it;
@@ -275,6 +278,8 @@ Items items_of_csc(const Plan& p) {
   it.n_local = p.n;
   it.short_rows = it.long_rows = nullptr;
   it.short_meta = nullptr;
+  it.bundles = nullptr;
+  it.n_bundles = it.n_short_nz = 0;
   it.n_short = it.n_long = 0;
   return it;
 }
@@ -350,20 +355,42 @@ agnn_status plan_build(Plan& p, cudaStream_t s) {
   if (p.n_short > 0) {
     // {row, degree, beg} of every short row in one 16-byte record (the short-row
     // kernels prefetch the next rows' records and column ids a step ahead)
-    std::vector<int4> meta((size_t)p.n_short);
+    std::vector<int4> meta;
     std::vector<int32_t> srows((size_t)p.n_short);
     AGNN_CUDA_TRY(cudaMemcpyAsync(srows.data(), p.short_rows, sizeof(int32_t) * srows.size(),
                                   cudaMemcpyDeviceToHost, s));
     AGNN_CUDA_TRY(cudaStreamSynchronize(s));
-    for (size_t x = 0; x < srows.size(); ++x) {
-      const int64_t r = srows[x], b = rp[(size_t)r];
-      meta[x] = make_int4(srows[x], (int)(rp[(size_t)r + 1] - b), (int)(uint32_t)(uint64_t)b,
-                          (int)(uint32_t)((uint64_t)b >> 32));
+    // rows with stored entries first (ascending), then the empty rows: the bundles
+    // below cover exactly the first n_short_nz records
+    meta.reserve(srows.size());
+    for (int pass = 0; pass < 2; ++pass)
+      for (size_t x = 0; x < srows.size(); ++x) {
+        const int64_t r = srows[x], b = rp[(size_t)r], d = rp[(size_t)r + 1] - b;
+        if ((d > 0) != (pass == 0)) continue;
+        meta.push_back(make_int4(srows[x], (int)d, (int)(uint32_t)(uint64_t)b,
+                                 (int)(uint32_t)((uint64_t)b >> 32)));
+      }
+    p.n_short_nz = 0;
+    while (p.n_short_nz < (int64_t)meta.size() && meta[(size_t)p.n_short_nz].y > 0) ++p.n_short_nz;
+    // bundles: consecutive non-empty short rows packed greedily into groups of at most
+    // kBundleEdges stored entries, {first record, rows, entries, 0}; a warp takes one
+    // bundle as one batch (the bundle kernels, gat_short.cu)
+    std::vector<int4> bund;
+    for (int64_t x = 0; x < p.n_short_nz;) {
+      int64_t e = 0, y = x;
+      while (y < p.n_short_nz && e + meta[(size_t)y].y <= kBundleEdges) e += meta[(size_t)y++].y;
+      bund.push_back(make_int4((int)x, (int)(y - x), (int)e, 0));
+      x = y;
     }
-    AGNN_CUDA_TRY(cudaMalloc(&p.short_block, sizeof(int4) * meta.size()));
+    p.n_bundles = (int64_t)bund.size();
+    AGNN_CUDA_TRY(cudaMalloc(&p.short_block, sizeof(int4) * (meta.size() + bund.size())));
     p.short_meta = static_cast<int4*>(p.short_block);
+    p.bundles = p.short_meta + meta.size();
     AGNN_CUDA_TRY(cudaMemcpyAsync(p.short_meta, meta.data(), sizeof(int4) * meta.size(),
                                   cudaMemcpyHostToDevice, s));
+    if (!bund.empty())
+      AGNN_CUDA_TRY(cudaMemcpyAsync(p.bundles, bund.data(), sizeof(int4) * bund.size(),
+                                    cudaMemcpyHostToDevice, s));
     AGNN_CUDA_TRY(cudaStreamSynchronize(s));
   }
   p.meta_block = L.block;

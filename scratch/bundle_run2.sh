@@ -1,0 +1,11 @@
+run() {
+  for p in fp32 bf16; do
+    timeout 300 python bench.py --prec $p --steps 5 --no-cpu-baseline --no-e2e --no-bf16-line 2>gpurun_out/bundle_err_$p.txt | python -c "
+import json,sys
+d=json.loads([l for l in sys.stdin if l.startswith('{')][-1])
+print('$p', '$*', round(d['value']/1e9,3), round(d['ms_per_step'],1), {k:round(v['ms_per_step'],2) for k,v in d['kernels'].items() if 'short' in k}, d['clocks']['sm_mhz'])
+" >> gpurun_out/bundle_ab2.txt
+  done
+}
+AGNN_SHORT_BUNDLES=0 run bundles=0
+run bundles=1

@@ -5,7 +5,8 @@ GAT backward (Eq. 6 with Psi^T) into the forward:
 ds_j = G_j . Q_j with Q_j = sum_i c_ji P_i - (sum_i c_ji) Z_j, c = alpha lambda.
 Its parity against the FP64 oracle is covered by every GAT k' = 128 case of
 test_gpu_parity.py / test_gpu_bf16.py (it is the default path); here:
-  * the unfactored path (AGNN_GAT_FACTORED=0) still meets the same bar;
+  * the unfactored path (AGNN_GAT_FACTORED=0) still meets the same bar, and so do
+    both short-row decompositions (row groups, bundles) for both storage types;
   * the factored path gives da1 = 0 EXACTLY when LeakyReLU is linear on every
     stored entry (the a-orientation identity of test_oracle_pins.py: each row's
     softmax is invariant to s_i), where the unfactored sum only reaches ~eps;
@@ -70,6 +71,14 @@ def _child(tmp_path, env, tag, prec="fp32", check=True):
 @pytest.mark.parametrize("prec", ["fp32", "bf16"])
 def test_unfactored_path_parity(tmp_path, prec):
     _child(tmp_path, {"AGNN_GAT_FACTORED": "0"}, "unf", prec)
+
+
+@pytest.mark.parametrize("prec", ["fp32", "bf16"])
+@pytest.mark.parametrize("bundles", ["0", "2"])
+def test_short_row_paths_parity(tmp_path, prec, bundles):
+    """Short rows through the row-group kernels (0) or the bundle kernels (2 = for
+    both storage types; the default uses bundles for fp32 only)."""
+    _child(tmp_path, {"AGNN_SHORT_BUNDLES": bundles}, f"b{bundles}", prec)
 
 
 def test_l2_hints_change_no_bit(tmp_path):
