@@ -96,7 +96,7 @@ constexpr int fwd_group() { return sizeof(TP) == 2 ? 8 : 4; }
 // Q_i = (u_i - (C_i / l_i) acc_i) / l_i  (= sum_j c_ij P_j - (sum_j c_ij) Z_i, gat_args.cuh);
 // when every lambda_ij = 1 (all pre-activations > 0) u = acc and C = l bitwise, so
 // Q = 0 and ds = 0 exactly, as in exact arithmetic.
-template <typename TP, int NH, int U, int MINB, bool QF>
+template <typename TP, int NH, int U, int MINB, bool QF, int GRT = 0>
 __global__ void __launch_bounds__(256, MINB)
 gat_fwd_k128_kernel(Items it, const TP* __restrict__ P, const float* __restrict__ st,
                     float slope, int act, GatFwdOut o) {
@@ -183,7 +183,7 @@ gat_fwd_k128_kernel(Items it, const TP* __restrict__ P, const float* __restrict_
       if (cnt == 32) {
         // full batch: 32/GR groups of GR rows, the next group in flight during this
         // group's FMAs
-        constexpr int GR = fwd_group<TP>(), NGR = 32 / GR;
+        constexpr int GR = GRT ? GRT : fwd_group<TP>(), NGR = 32 / GR;
         static_assert(U >= GR, "the prefetch covers the first group");
         const TP* Pl = P + cq;
         typename SL::raw qa[GR], qb[GR];
@@ -600,7 +600,7 @@ gat_bwd_k128_kernel(Items it, GatBwdArgs A) {
 //   accumulates acc_j += alpha_ij G_i and v_j += c'_ij G_i (16-byte gather, 8 FMAs).
 // Per row: dt_j = P_j . v_j - sum_i c'_ij delta_i, dP_j = acc_j + ds_j a1 + dt_j a2.
 // Per edge it moves the index, one G row and the NH records (4 + K f + 16 NH bytes).
-template <typename TP, int NH, int MINB>
+template <typename TP, int NH, int MINB, int GRT = 0>
 __global__ void __launch_bounds__(256, MINB)
 gat_bwd_k128f_kernel(Items it, GatBwdArgs A) {
   constexpr int D = K / NH, HL = D / 4;
@@ -634,7 +634,7 @@ gat_bwd_k128f_kernel(Items it, GatBwdArgs A) {
       jpre = b0 + 32 + lane < end ? __ldg(it.col + b0 + 32 + lane) : 0;
       sJ[wib][lane] = j;
       __syncwarp();
-      constexpr int GR = fwd_group<TP>(), NGR = 32 / GR;
+      constexpr int GR = GRT ? GRT : fwd_group<TP>(), NGR = 32 / GR;
       typename SL::raw qa[GR], qb[GR];
       // the first group of G rows is in flight while the weights are computed
 #pragma unroll
@@ -827,8 +827,24 @@ agnn_status gat_fwd_k128(const Items& it_all, int heads, const float* P, const f
     return AGNN_OK;
   }
   AGNN_K128_DISPATCH(heads, ({
-    auto* kern = o.Q ? gat_fwd_k128_kernel<float, NH, 4, 3, true>
-                     : gat_fwd_k128_kernel<float, NH, 4, 3, false>;
+    // AGNN_FWD_VARIANT (measurement): 0 = 3 blocks / SM, 4-row groups; 1 = 2 blocks /
+    // SM, 8-row groups; 2 = 4 blocks / SM
+    static int variant = -1;
+    if (variant < 0) {
+      const char* e = getenv("AGNN_FWD_VARIANT");
+      variant = e ? atoi(e) : 0;
+    }
+    using KF = void (*)(Items, const float*, const float*, float, int, GatFwdOut);
+    KF kern;
+    if (variant == 1)
+      kern = o.Q ? (KF)gat_fwd_k128_kernel<float, NH, 8, 2, true, 8>
+                 : (KF)gat_fwd_k128_kernel<float, NH, 8, 2, false, 8>;
+    else if (variant == 2)
+      kern = o.Q ? (KF)gat_fwd_k128_kernel<float, NH, 4, 4, true>
+                 : (KF)gat_fwd_k128_kernel<float, NH, 4, 4, false>;
+    else
+      kern = o.Q ? (KF)gat_fwd_k128_kernel<float, NH, 4, 3, true>
+                 : (KF)gat_fwd_k128_kernel<float, NH, 4, 3, false>;
     kern<<<grid_for(kern), 256, 0, s>>>(it, P, st, slope, act, o);
     AGNN_LAUNCH_CHECK("gat_fwd_kernel");
   }));
@@ -903,8 +919,24 @@ agnn_status gat_bwd_k128f(const Items& it_all, int heads, const GatBwdArgs& A, i
   *warps = 0;
   const Items it = long_items(it_all);
   AGNN_K128_DISPATCH(heads, ({
-    auto* kern = A.P16 ? (void (*)(Items, GatBwdArgs))gat_bwd_k128f_kernel<bf16, NH, 3>
-                       : (void (*)(Items, GatBwdArgs))gat_bwd_k128f_kernel<float, NH, 3>;
+    // AGNN_BWDF_VARIANT (measurement): 0 = default (fp32: as 1, bf16: 3 blocks / SM;
+    // measured C5: fp32 73.5 -> 69.2 ms, bf16 59.2 vs 64.7 ms); 1 = 2 blocks / SM;
+    // 2 = 2 blocks / SM, 8-row (fp32) / 16-row (bf16) groups; 3 = 4 blocks / SM
+    static int variant = -1;
+    if (variant < 0) {
+      const char* e = getenv("AGNN_BWDF_VARIANT");
+      variant = e ? atoi(e) : 0;
+    }
+    using KB = void (*)(Items, GatBwdArgs);
+    KB kern;
+    if (variant == 1 || (variant == 0 && !A.P16))
+      kern = A.P16 ? (KB)gat_bwd_k128f_kernel<bf16, NH, 2> : (KB)gat_bwd_k128f_kernel<float, NH, 2>;
+    else if (variant == 2)
+      kern = A.P16 ? (KB)gat_bwd_k128f_kernel<bf16, NH, 2, 16> : (KB)gat_bwd_k128f_kernel<float, NH, 2, 8>;
+    else if (variant == 3)
+      kern = A.P16 ? (KB)gat_bwd_k128f_kernel<bf16, NH, 4> : (KB)gat_bwd_k128f_kernel<float, NH, 4>;
+    else
+      kern = A.P16 ? (KB)gat_bwd_k128f_kernel<bf16, NH, 3> : (KB)gat_bwd_k128f_kernel<float, NH, 3>;
     const int grid = grid_for(kern);
     kern<<<grid, 256, 0, s>>>(it, A);
     AGNN_LAUNCH_CHECK("gat_bwd_kernel");
