@@ -525,7 +525,9 @@ agnn_status av_forward(const Plan& p, const agnn_layer_desc& d, const float* W, 
   Items it = items_of(p);
   AvFwd A{Hf, sv.nu, d.beta, fabsf(d.beta), sv.X, sv.l, w.pacc, w.pl};
   if ((K_ == 128 || K_ == 256) && !k128_disabled()) {
-    if ((st = av_fwd_batched(it, K_, ag, A, s)) != AGNN_OK) return st;
+    // gathered per entry: an H_j row (+ nu_j)
+    const Items ith = l2_hinted(it, p, 4 * (int64_t)K_ + (ag ? 4 : 0));
+    if ((st = av_fwd_batched(ith, K_, ag, A, s)) != AGNN_OK) return st;
   } else if (it.n_chunks + it.n_light > 0) {
     if (ag) AGNN_AV_DISPATCH(K_, (av_fwd_kernel<K, AG, av_fwd_unroll<K>()>
                                   <<<grid_of(av_fwd_kernel<K, AG, av_fwd_unroll<K>()>),
@@ -627,7 +629,9 @@ agnn_status av_backward(const Plan& p, const agnn_layer_desc& d, const float* W,
     return AGNN_OK;
   }
   if ((K_ == 128 || K_ == 256) && !k128_disabled()) {
-    if ((st = av_bwd_batched(it, K_, ag, A, s)) != AGNN_OK) return st;
+    // gathered per entry: the H_i and M_i rows (+ the record)
+    const Items ith = l2_hinted(it, p, 8 * (int64_t)K_ + (ag ? 16 : 0));
+    if ((st = av_bwd_batched(ith, K_, ag, A, s)) != AGNN_OK) return st;
   } else if (it.n_chunks + it.n_light > 0) {
     if (ag) AGNN_AV_DISPATCH(K_, (av_bwd_kernel<K, AG, av_bwd_unroll<K>()>
                                   <<<grid_of(av_bwd_kernel<K, AG, av_bwd_unroll<K>()>),

@@ -49,6 +49,7 @@ __global__ void __launch_bounds__(256, MINB) av_fwd_batched_kernel(Items it, AvF
   const int64_t nitems = it.n_chunks + it.n_light;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
   const float* Hl = A.H + cq;
+  const Gath ga(it);  // L2 residency hints of the gathered rows (plan column classes)
   for (int64_t w = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; w < nitems; w += nw) {
     int64_t row, beg, end, slot;
     item_of(it, w, row, beg, end, slot);
@@ -64,14 +65,16 @@ __global__ void __launch_bounds__(256, MINB) av_fwd_batched_kernel(Items it, AvF
     auto load = [&](FwdBatch<B, V>& q, int cidx, int off, int cnt) {
 #pragma unroll
       for (int b = 0; b < B; ++b) {
-        const uint32_t j = (uint32_t)__shfl_sync(FULL, cidx, off + b);
+        const int c = __shfl_sync(FULL, cidx, off + b);
+        const int64_t j = ga.row(c);
+        const uint64_t pol = ga.policy(c);
 #pragma unroll
         for (int v = 0; v < V; ++v)
-          q.Hj[b][v] = b < cnt ? ldg4(Hl + (int64_t)j * K + v * 128) : f4(0.f);
+          q.Hj[b][v] = b < cnt ? ldg4_pol(Hl + j * K + v * 128, pol) : f4(0.f);
       }
       if (MODEL == AV_AG) {
-        const uint32_t jm = (uint32_t)__shfl_sync(FULL, cidx, off + my_b);
-        q.nuj = my_b < cnt ? __ldg(A.nu + jm) : 1.f;
+        const int cm = __shfl_sync(FULL, cidx, off + my_b);
+        q.nuj = my_b < cnt ? ldg1_pol(A.nu + ga.row(cm), ga.policy(cm)) : 1.f;
       }
     };
     auto body = [&](const FwdBatch<B, V>& q, int cnt) {
@@ -150,6 +153,7 @@ __global__ void __launch_bounds__(256, MINB) av_bwd_batched_kernel(Items it, AvB
   const int my_b = TR::edge_of(lane);
   const float beta = A.beta;
   const int64_t nitems = it.n_chunks + it.n_light;
+  const Gath ga(it);
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
   const float* Hl = A.H + cq;
   const float* Ml = A.M + cq;
@@ -169,20 +173,23 @@ __global__ void __launch_bounds__(256, MINB) av_bwd_batched_kernel(Items it, AvB
     auto load = [&](BwdBatchAV<B, V>& q, int cidx, int off, int cnt) {
 #pragma unroll
       for (int b = 0; b < B; ++b) {
-        const uint32_t i = (uint32_t)__shfl_sync(FULL, cidx, off + b);
+        const int c = __shfl_sync(FULL, cidx, off + b);
+        const int64_t i = ga.row(c);
+        const uint64_t pol = ga.policy(c);
 #pragma unroll
         for (int v = 0; v < V; ++v) {
           if (b < cnt) {
-            q.Hi[b][v] = ldg4(Hl + (int64_t)i * K + v * 128);
-            q.Mi[b][v] = ldg4(Ml + (int64_t)i * K + v * 128);
+            q.Hi[b][v] = ldg4_pol(Hl + i * K + v * 128, pol);
+            q.Mi[b][v] = ldg4_pol(Ml + i * K + v * 128, pol);
           } else {
             q.Hi[b][v] = q.Mi[b][v] = f4(0.f);
           }
         }
       }
       if (MODEL == AV_AG) {
-        const uint32_t im = (uint32_t)__shfl_sync(FULL, cidx, off + my_b);
-        q.ri = my_b < cnt ? __ldg(A.rec + im) : f4(1.f);
+        const int cm = __shfl_sync(FULL, cidx, off + my_b);
+        q.ri = my_b < cnt ? ldg4_pol(reinterpret_cast<const float*>(A.rec + ga.row(cm)), ga.policy(cm))
+                          : f4(1.f);
       }
     };
     auto body = [&](const BwdBatchAV<B, V>& q, int cnt) {
