@@ -152,7 +152,13 @@ agnn_status agnn_partition(int64_t n, const int64_t* row_ptr_host, int world, in
                            int64_t* bounds_host);
 
 /* Validate the CSR on the device, build the work lists (light rows + heavy-row
- * chunks), and (world > 1) create the NCCL communicator.  Synchronises once. */
+ * chunks, short-row bundles), and (world > 1) create the NCCL communicator.
+ * Also builds the L2 residency classes of the columns: a plan-owned copy of
+ * col_idx (nnz x 4 bytes of device memory) whose free high bits rank every
+ * column by how often this rank gathers it; the sparse kernels load the rows of
+ * the most-gathered columns with an evict_last L2 policy (
+ * environment AGNN_L2_HOT_MB = L2 budget in MB, 0 disables).  The classes are
+ * performance metadata only: no result depends on them.  Synchronises. */
 agnn_status agnn_plan_create(const agnn_csr* csr, const agnn_dist* dist /* NULL => 1 GPU */,
                              cudaStream_t stream, agnn_plan_t* out);
 agnn_status agnn_plan_destroy(agnn_plan_t plan);
@@ -176,7 +182,10 @@ agnn_status agnn_model_create(agnn_plan_t plan, int n_layers, const agnn_layer_d
 agnn_status agnn_model_destroy(agnn_model_t model);
 
 /* bytes of the per-layer `saved` buffer (intermediates kept for backward)
- * and of the scratch `workspace` shared by forward and backward.            */
+ * and of the scratch `workspace` shared by forward and backward.  For GAT with
+ * k_out = 128 on a symmetric pattern `saved` also holds Q [n_local x k_out]
+ * (the factored backward: ds_j = G_j . Q_j); the layout is
+ * internal, only the size is part of the contract.                          */
 agnn_status agnn_saved_bytes(agnn_model_t model, int layer, size_t* bytes);
 agnn_status agnn_workspace_bytes(agnn_model_t model, int layer, size_t* bytes);
 
