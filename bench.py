@@ -225,9 +225,11 @@ def run_reference(args):
 
 # ----------------------------------------------------------------------------- ours
 def gat_factored(w):
-    """The factored GAT backward runs for k' = 128 on symmetric patterns (gat_args.cuh)."""
-    return (w.model == "gat" and w.k == 128 and w.heads in (1, 2, 4, 8)
-            and os.environ.get("AGNN_GAT_FACTORED", "1") != "0")
+    """The factored GAT backward (gat_args.cuh) on symmetric patterns: k' = 128 by
+    default, every width with AGNN_GAT_FACTORED=2, never with 0."""
+    mode = os.environ.get("AGNN_GAT_FACTORED", "1")
+    k128 = w.k == 128 and w.heads in (1, 2, 4, 8)
+    return w.model == "gat" and (mode == "2" or (mode == "1" and k128))
 
 
 def pass_bytes(w, m, n):

@@ -81,7 +81,26 @@ __device__ __forceinline__ void fwd_finish(int64_t row, const float (&m)[RowLayo
 }
 
 // ---------------------------------------------------------------- forward
-template <int K, int NH, int U>
+// merge of two online-softmax states that also carry the factored backward's
+// (lc, accu) = (sum p lambda, sum p lambda P) with the same rescale factors
+__device__ __forceinline__ void merge_softmax_q(float& m, float& l, float4& acc, float& lc,
+                                                float4& accu, float m2, float l2, float4 acc2,
+                                                float lc2, float4 accu2) {
+  const float mn = fmaxf(m, m2);
+  if (mn == NEG_INF) return;
+  const float x = ex2(m - mn), y = ex2(m2 - mn);
+  l = fmaf(l, x, l2 * y);
+  acc = make_float4(fmaf(acc.x, x, acc2.x * y), fmaf(acc.y, x, acc2.y * y),
+                    fmaf(acc.z, x, acc2.z * y), fmaf(acc.w, x, acc2.w * y));
+  lc = fmaf(lc, x, lc2 * y);
+  accu = make_float4(fmaf(accu.x, x, accu2.x * y), fmaf(accu.y, x, accu2.y * y),
+                     fmaf(accu.z, x, accu2.z * y), fmaf(accu.w, x, accu2.w * y));
+  m = mn;
+}
+
+// QF (training, factored backward; gat_args.cuh): also u_i = sum_j c_ij P_j and
+// C_i = sum_j c_ij (c = p lambda) with the same rescaling; Q_i = (u - (C/l) acc) / l.
+template <int K, int NH, int U, bool QF>
 __global__ void __launch_bounds__(kSparseThreads)
 gat_fwd_kernel(Items it, const float* __restrict__ P, const float* __restrict__ st, float slope,
                int act, FwdOut o) {
@@ -93,14 +112,14 @@ gat_fwd_kernel(Items it, const float* __restrict__ P, const float* __restrict__ 
     int64_t row, beg, end, slot;
     item_range<K, NH>(it, w, row, beg, end, slot);
     const int64_t grow = it.row_begin + row;
-    float si[L::VPL], m[L::VPL], l[L::VPL];
-    float4 acc[L::VPL];
+    float si[L::VPL], m[L::VPL], l[L::VPL], lc[L::VPL];
+    float4 acc[L::VPL], accu[L::VPL];
 #pragma unroll
     for (int v = 0; v < L::VPL; ++v) {
       si[v] = __ldg(st + grow * (2 * NH) + L::head(v, q));
       m[v] = NEG_INF;
-      l[v] = 0.f;
-      acc[v] = f4(0.f);
+      l[v] = lc[v] = 0.f;
+      acc[v] = accu[v] = f4(0.f);
     }
     for (int64_t e0 = beg; e0 < end; e0 += 32) {
       const int cnt = (int)(end - e0 < 32 ? end - e0 : 32);
@@ -127,24 +146,35 @@ gat_fwd_kernel(Items it, const float* __restrict__ P, const float* __restrict__ 
         }
 #pragma unroll
         for (int v = 0; v < L::VPL; ++v) {
-          float ev[U];
+          float ev[U], pre[U];
           float mn = m[v];
 #pragma unroll
           for (int u = 0; u < U; ++u) {
-            const float pre = si[v] + tj[u][v];
-            ev[u] = pre > 0.f ? pre : slope * pre;
+            pre[u] = si[v] + tj[u][v];
+            ev[u] = pre[u] > 0.f ? pre[u] : slope * pre[u];
             if (val[u]) mn = fmaxf(mn, ev[u]);
           }
           if (mn != NEG_INF) {
             const float sc = ex2(m[v] - mn);
-            l[v] *= sc;
+            // rounded mul / add, never contracted: the QF and inference variants agree
+            // bitwise, and lc follows the same operations as l
+            l[v] = __fmul_rn(l[v], sc);
             acc[v] = mul4(sc, acc[v]);
+            if constexpr (QF) {
+              lc[v] = __fmul_rn(lc[v], sc);
+              accu[v] = mul4(sc, accu[v]);
+            }
 #pragma unroll
             for (int u = 0; u < U; ++u) {
               if (val[u]) {
                 const float p = ex2(ev[u] - mn);
-                l[v] += p;
+                l[v] = __fadd_rn(l[v], p);
                 acc[v] = fma4(p, pj[u][v], acc[v]);
+                if constexpr (QF) {
+                  const float pc = pre[u] > 0.f ? p : p * slope;
+                  lc[v] = __fadd_rn(lc[v], pc);
+                  accu[v] = fma4(pc, pj[u][v], accu[v]);
+                }
               }
             }
             m[v] = mn;
@@ -158,20 +188,36 @@ gat_fwd_kernel(Items it, const float* __restrict__ P, const float* __restrict__ 
 #pragma unroll
       for (int v = 0; v < L::VPL; ++v) {
         const float m2 = __shfl_xor_sync(FULL, m[v], off), l2 = __shfl_xor_sync(FULL, l[v], off);
-        float4 a2;
+        float4 a2, u2 = f4(0.f);
+        float lc2 = 0.f;
         a2.x = __shfl_xor_sync(FULL, acc[v].x, off);
         a2.y = __shfl_xor_sync(FULL, acc[v].y, off);
         a2.z = __shfl_xor_sync(FULL, acc[v].z, off);
         a2.w = __shfl_xor_sync(FULL, acc[v].w, off);
+        if constexpr (QF) {
+          lc2 = __shfl_xor_sync(FULL, lc[v], off);
+          u2.x = __shfl_xor_sync(FULL, accu[v].x, off);
+          u2.y = __shfl_xor_sync(FULL, accu[v].y, off);
+          u2.z = __shfl_xor_sync(FULL, accu[v].z, off);
+          u2.w = __shfl_xor_sync(FULL, accu[v].w, off);
+        }
         if (g & (off / L::LANES)) {  // canonical order: the lower group's state goes first
-          float mt = m2, lt = l2;
-          float4 at = a2;
-          merge_softmax(mt, lt, at, m[v], l[v], acc[v]);
+          float mt = m2, lt = l2, lct = lc2;
+          float4 at = a2, ut = u2;
+          if constexpr (QF)
+            merge_softmax_q(mt, lt, at, lct, ut, m[v], l[v], acc[v], lc[v], accu[v]);
+          else
+            merge_softmax(mt, lt, at, m[v], l[v], acc[v]);
           m[v] = mt;
           l[v] = lt;
           acc[v] = at;
+          lc[v] = lct;
+          accu[v] = ut;
         } else {
-          merge_softmax(m[v], l[v], acc[v], m2, l2, a2);
+          if constexpr (QF)
+            merge_softmax_q(m[v], l[v], acc[v], lc[v], accu[v], m2, l2, a2, lc2, u2);
+          else
+            merge_softmax(m[v], l[v], acc[v], m2, l2, a2);
         }
       }
     }
@@ -181,13 +227,22 @@ gat_fwd_kernel(Items it, const float* __restrict__ P, const float* __restrict__ 
       for (int v = 0; v < L::VPL; ++v) {
         const int c = L::col(v, q);
         st4(o.pacc + slot * K + c, acc[v]);
+        if constexpr (QF) st4(o.pu + slot * K + c, accu[v]);
         if ((c % L::D) == 0) {
           o.pm[slot * NH + c / L::D] = m[v];
           o.pl[slot * NH + c / L::D] = l[v];
+          if constexpr (QF) o.pc[slot * NH + c / L::D] = lc[v];
         }
       }
     } else {
       fwd_finish<K, NH>(row, m, l, acc, q, act, o);
+      if constexpr (QF) {
+#pragma unroll
+        for (int v = 0; v < L::VPL; ++v) {
+          const float inv = l[v] > 0.f ? 1.f / l[v] : 0.f, r = l[v] > 0.f ? lc[v] / l[v] : 0.f;
+          st4(o.Q + row * K + L::col(v, q), mul4(inv, fma4(-r, acc[v], accu[v])));
+        }
+      }
     }
   }
 }
@@ -590,10 +645,15 @@ __global__ void gat_debug_alpha_kernel(const int64_t* __restrict__ rp, int64_t n
 }
 
 // ---------------------------------------------------------------- layout
-// the factored backward (gat_args.cuh) runs where the k' = 128 kernels do, on
-// symmetric patterns
+// the factored backward (gat_args.cuh) runs on symmetric patterns: the k' = 128
+// kernels, or the generic ones (forward with QF, backward = the column-role pass
+// over the CSR, which for a symmetric pattern lists every column's entries)
+// AGNN_GAT_FACTORED: 1 (default) = k' = 128 only; 2 = every width; 0 = never.
+// Measured: k' = 128 at C5 1.45x faster step; k' = 64 at C2 (L2-resident, so the
+// gathered bytes it saves cost nothing) 0.81 -> 0.87 ms, hence k' = 128 only by default.
 bool factored(const Plan& p, const GatShape& g) {
-  return gat_factored_enabled() && gat_k128_supported(g.k_out, g.heads) && !p.directed();
+  const int mode = gat_factored_mode();
+  return mode > 0 && !p.directed() && (mode == 2 || gat_k128_supported(g.k_out, g.heads));
 }
 
 struct SavedGat {
@@ -668,12 +728,12 @@ WsGat carve_ws(const Plan& p, const GatShape& g, void* base, size_t* total) {
 
 }  // namespace
 
-bool gat_factored_enabled() {
+int gat_factored_mode() {
   static const int v = [] {
     const char* e = getenv("AGNN_GAT_FACTORED");
     return e ? atoi(e) : 1;
   }();
-  return v != 0;
+  return v;
 }
 
 size_t gat_saved_bytes(const Plan& p, const GatShape& g) { return saved_size(p, g); }
@@ -790,9 +850,14 @@ agnn_status gat_forward(const Plan& p, const GatShape& g, const float* W, const 
     if ((st = gat_fwd_k128(ith, g.heads, sv.P, sv.st, g.slope, g.act, o, p.n, s)) != AGNN_OK)
       return st;
   } else if (it.n_chunks + it.n_light > 0) {
-    AGNN_GAT_DISPATCH(K_, NH_, (gat_fwd_kernel<K, NH, fwd_unroll<K>()>
-                                <<<grid_of(gat_fwd_kernel<K, NH, fwd_unroll<K>()>), kSparseThreads,
-                                   0, s>>>(it, sv.P, sv.st, g.slope, g.act, o)));
+    if (o.Q)
+      AGNN_GAT_DISPATCH(K_, NH_, (gat_fwd_kernel<K, NH, fwd_unroll<K>(), true>
+                                  <<<grid_of(gat_fwd_kernel<K, NH, fwd_unroll<K>(), true>),
+                                     kSparseThreads, 0, s>>>(it, sv.P, sv.st, g.slope, g.act, o)));
+    else
+      AGNN_GAT_DISPATCH(K_, NH_, (gat_fwd_kernel<K, NH, fwd_unroll<K>(), false>
+                                  <<<grid_of(gat_fwd_kernel<K, NH, fwd_unroll<K>(), false>),
+                                     kSparseThreads, 0, s>>>(it, sv.P, sv.st, g.slope, g.act, o)));
     AGNN_LAUNCH_CHECK("gat_fwd_kernel");
   }
   if (it.n_heavy > 0) {
@@ -862,6 +927,7 @@ agnn_status gat_backward(const Plan& p, const GatShape& g, const float* W, const
   BwdArgs A{sv.P, sv.st, w.G, w.rec, a, g.slope, w.dP, w.pacc, w.pm, w.pl, w.da_part,
             nullptr, nullptr, w.ds_dir, sv.P16, w.G16, w.ds_row};
   int64_t main_warps = 0, merge_warps = 0;
+  bool merged = false;  // the branch below ran its own heavy-row merge
   if (directed) {
     // row role over the CSR (ds_j), then the column role over the CSC (dt_j, acc_j, dP_j)
     Items itc = items_of_csc(p);
@@ -886,10 +952,26 @@ agnn_status gat_backward(const Plan& p, const GatShape& g, const float* W, const
                                 <<<(unsigned)(merge_warps / 8), kSparseThreads, 0, s>>>(
                                     it, A, main_warps)));
     AGNN_LAUNCH_CHECK("gat_bwd_merge_kernel");
-  } else if (sv.Q) {
+  } else if (sv.Q && gat_k128_supported(g.k_out, g.heads)) {
     // factored: gathered per edge only G_i and the records rec_i of the heads
     const Items ith = l2_hinted(it, p, (g.bf16 ? 2 : 4) * (int64_t)g.k_out + 16 * g.heads);
     if ((st = gat_bwd_k128f(ith, g.heads, A, &main_warps, s)) != AGNN_OK) return st;
+  } else if (sv.Q) {
+    // factored, generic widths: the column-role pass of the directed backward over the
+    // (symmetric) CSR, with ds_j = G_j . Q_j from the prologue in place of the row pass
+    merged = true;
+    A.ds_dir = w.ds_row;
+    AGNN_GAT_DISPATCH(K_, NH_, (main_warps = (int64_t)grid_of(gat_bwd_kernel<K, NH, bwd_unroll<K>(), 2>) *
+                                             (kSparseThreads / 32)));
+    AGNN_GAT_DISPATCH(K_, NH_, (gat_bwd_kernel<K, NH, bwd_unroll<K>(), 2>
+                                <<<(unsigned)(main_warps / 8), kSparseThreads, 0, s>>>(it, A)));
+    AGNN_LAUNCH_CHECK("gat_bwd_kernel");
+    AGNN_GAT_DISPATCH(K_, NH_, (merge_warps = (int64_t)grid_of(gat_bwd_merge_kernel<K, NH, 2>) *
+                                              (kSparseThreads / 32)));
+    AGNN_GAT_DISPATCH(K_, NH_, (gat_bwd_merge_kernel<K, NH, 2>
+                                <<<(unsigned)(merge_warps / 8), kSparseThreads, 0, s>>>(
+                                    it, A, main_warps)));
+    AGNN_LAUNCH_CHECK("gat_bwd_merge_kernel");
   } else if (gat_k128_supported(g.k_out, g.heads)) {
     // gathered per edge: rows P_i and G_i, the record rec_i and t_i of the heads
     const Items ith =
@@ -902,7 +984,7 @@ agnn_status gat_backward(const Plan& p, const GatShape& g, const float* W, const
                                 <<<(unsigned)(main_warps / 8), kSparseThreads, 0, s>>>(it, A)));
     AGNN_LAUNCH_CHECK("gat_bwd_kernel");
   }
-  if (!directed) {
+  if (!directed && !merged) {
     AGNN_GAT_DISPATCH(K_, NH_, (merge_warps = (int64_t)grid_of(gat_bwd_merge_kernel<K, NH>) *
                                               (kSparseThreads / 32)));
     AGNN_GAT_DISPATCH(K_, NH_, (gat_bwd_merge_kernel<K, NH>

@@ -39,8 +39,8 @@ struct GatBwdArgs {
   const float* ds_row; // [n_local x NH] factored backward: ds_j = G_j . Q_j (prologue)
 };
 
-// The factored GAT backward (k' = 128, symmetric pattern; AGNN_GAT_FACTORED=0
-// disables it).  With c_ji = alpha_ji lambda_ji (lambda = LReLU slope of the
+// The factored GAT backward (symmetric patterns; k' = 128 by default, every width
+// with AGNN_GAT_FACTORED=2, off with 0).  With c_ji = alpha_ji lambda_ji (lambda = LReLU slope of the
 // entry), the row-role sum of PAPER.md:250-254 is linear in the gathered rows,
 //   ds_j = sum_i c_ji (G_j . P_i - delta_j) = G_j . (sum_i c_ji P_i - (sum_i c_ji) Z_j)
 //        = G_j . Q_j,
@@ -49,7 +49,7 @@ struct GatBwdArgs {
 // backward edge pass gathers only G_i and rec_i (column role):
 //   dt_j = sum_i c'_ij (G_i . P_j - delta_i) = P_j . v_j - sum_i c'_ij delta_i,
 //   v_j = sum_i c'_ij G_i,  acc_j = sum_i alpha_ij G_i.
-bool gat_factored_enabled();
+int gat_factored_mode();  // AGNN_GAT_FACTORED: 0 off, 1 k' = 128 (default), 2 all widths
 
 // k' = 128 kernels (gat_k128.cu): lane-parallel scalar work, warp-parallel rows
 bool gat_k128_supported(int k_out, int heads);

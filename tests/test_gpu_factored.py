@@ -32,9 +32,9 @@ from paper_conf_sc_bestarglzcgssci23_b200 import gen, runner  # noqa: E402
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
-def W(graph, scale, ef, heads, prec="fp32", act="relu", chunk=None):
+def W(graph, scale, ef, heads, prec="fp32", act="relu", k=128):
     n = 1 << scale
-    return gen.Workload(f"gat-{graph}{scale}-h{heads}-{prec}", "gat", graph, scale, n, ef * n, 128,
+    return gen.Workload(f"gat-{graph}{scale}-h{heads}-{prec}", "gat", graph, scale, n, ef * n, k,
                         heads, 1, act=act, prec=prec)
 
 
@@ -43,7 +43,7 @@ import sys, numpy as np, torch
 sys.path[:0] = [{root!r}, {tests!r}, {root!r} + "/oracle"]
 import parity_utils as pu
 from paper_conf_sc_bestarglzcgssci23_b200 import gen
-w = gen.Workload("gat-kron14-h4", "gat", "kron", 14, 1 << 14, 8 << 14, 128, 4, 1, act="elu",
+w = gen.Workload("gat-kron14-h4", "gat", "kron", 14, 1 << 14, 8 << 14, {k}, 4, 1, act="elu",
                  prec={prec!r})
 src, dst, rp, ci = pu.host_graph(w)
 g = pu.device_graph(w, src, dst)
@@ -57,10 +57,10 @@ np.savez({out!r}, H=st.H[1].cpu().numpy(), dH=st.dH[0].cpu().numpy(),
 """
 
 
-def _child(tmp_path, env, tag, prec="fp32", check=True):
+def _child(tmp_path, env, tag, prec="fp32", check=True, k=128):
     out = str(tmp_path / f"{tag}.npz")
     code = _CHILD.format(root=ROOT, tests=os.path.join(ROOT, "tests"), prec=prec, check=check,
-                         out=out)
+                         out=out, k=k)
     e = dict(os.environ, AGNN_CHUNK_EDGES="256", **env)  # heavy rows too
     r = subprocess.run([sys.executable, "-c", code], env=e, capture_output=True, text=True,
                        timeout=600)
@@ -68,9 +68,17 @@ def _child(tmp_path, env, tag, prec="fp32", check=True):
     return dict(np.load(out))
 
 
-@pytest.mark.parametrize("prec", ["fp32", "bf16"])
-def test_unfactored_path_parity(tmp_path, prec):
-    _child(tmp_path, {"AGNN_GAT_FACTORED": "0"}, "unf", prec)
+@pytest.mark.parametrize("prec,k", [("fp32", 128), ("bf16", 128), ("fp32", 64), ("fp32", 256)])
+def test_unfactored_path_parity(tmp_path, prec, k):
+    """k' = 128: the k128 kernels; other widths: the generic row-group kernels."""
+    _child(tmp_path, {"AGNN_GAT_FACTORED": "0"}, "unf", prec, k=k)
+
+
+@pytest.mark.parametrize("k", [32, 64, 256])
+def test_factored_generic_widths_parity(tmp_path, k):
+    """The factored backward on the generic kernels (forward with QF, then the
+    column-role pass over the symmetric CSR), heavy rows included."""
+    _child(tmp_path, {"AGNN_GAT_FACTORED": "2"}, f"fac{k}", "fp32", k=k)
 
 
 @pytest.mark.parametrize("prec", ["fp32", "bf16"])
@@ -89,10 +97,10 @@ def test_l2_hints_change_no_bit(tmp_path):
         assert np.array_equal(a[k], b[k]) and np.array_equal(a[k], c[k]), k
 
 
-@pytest.mark.parametrize("prec", ["fp32", "bf16"])
-def test_factored_da1_exactly_zero_when_leaky_relu_linear(prec):
+@pytest.mark.parametrize("prec,k", [("fp32", 128), ("bf16", 128)])
+def test_factored_da1_exactly_zero_when_leaky_relu_linear(prec, k):
     """H, W, a > 0 => P, s, t > 0 => every pre-activation > 0 => ds = 0 exactly."""
-    w = W("kron", 13, 8, 4, prec=prec, act="none")
+    w = W("kron", 13, 8, 4, prec=prec, act="none", k=k)
     st = runner.Stack(w, "cuda")
     g = torch.Generator(device="cpu").manual_seed(7)
     st.H[0].copy_(torch.rand(st.H[0].shape, generator=g) * 0.9 + 0.1)
