@@ -645,15 +645,16 @@ __global__ void gat_debug_alpha_kernel(const int64_t* __restrict__ rp, int64_t n
 }
 
 // ---------------------------------------------------------------- layout
-// the factored backward (gat_args.cuh) runs on symmetric patterns: the k' = 128
-// kernels, or the generic ones (forward with QF, backward = the column-role pass
-// over the CSR, which for a symmetric pattern lists every column's entries)
+// the factored backward (gat_args.cuh): symmetric patterns run the k' = 128
+// kernels or the generic ones (forward with QF, backward = the column-role pass
+// over the CSR, which for a symmetric pattern lists every column's entries);
+// directed patterns skip their row pass (column pass over the CSC only)
 // AGNN_GAT_FACTORED: 1 (default) = k' = 128 only; 2 = every width; 0 = never.
 // Measured: k' = 128 at C5 1.45x faster step; k' = 64 at C2 (L2-resident, so the
 // gathered bytes it saves cost nothing) 0.81 -> 0.87 ms, hence k' = 128 only by default.
 bool factored(const Plan& p, const GatShape& g) {
   const int mode = gat_factored_mode();
-  return mode > 0 && !p.directed() && (mode == 2 || gat_k128_supported(g.k_out, g.heads));
+  return mode > 0 && (mode == 2 || gat_k128_supported(g.k_out, g.heads));
 }
 
 struct SavedGat {
@@ -929,16 +930,22 @@ agnn_status gat_backward(const Plan& p, const GatShape& g, const float* W, const
   int64_t main_warps = 0, merge_warps = 0;
   bool merged = false;  // the branch below ran its own heavy-row merge
   if (directed) {
-    // row role over the CSR (ds_j), then the column role over the CSC (dt_j, acc_j, dP_j)
+    // row role over the CSR (ds_j), then the column role over the CSC (dt_j, acc_j, dP_j);
+    // factored (Q saved by the forward): ds_j = G_j . Q_j from the prologue replaces
+    // the whole row pass (the forward visited exactly row j's entries)
     Items itc = items_of_csc(p);
-    AGNN_GAT_DISPATCH(K_, NH_, (gat_bwd_kernel<K, NH, bwd_unroll<K>(), 1>
-                                <<<grid_of(gat_bwd_kernel<K, NH, bwd_unroll<K>(), 1>),
-                                   kSparseThreads, 0, s>>>(it, A)));
-    AGNN_LAUNCH_CHECK("gat_bwd_row_kernel");
-    if (it.n_heavy > 0) {
-      AGNN_GAT_DISPATCH(K_, NH_, (gat_bwd_merge_kernel<K, NH, 1>
-                                  <<<kNumSMs * 2, kSparseThreads, 0, s>>>(it, A, 0)));
-      AGNN_LAUNCH_CHECK("gat_bwd_merge_kernel");
+    if (sv.Q) {
+      A.ds_dir = w.ds_row;
+    } else {
+      AGNN_GAT_DISPATCH(K_, NH_, (gat_bwd_kernel<K, NH, bwd_unroll<K>(), 1>
+                                  <<<grid_of(gat_bwd_kernel<K, NH, bwd_unroll<K>(), 1>),
+                                     kSparseThreads, 0, s>>>(it, A)));
+      AGNN_LAUNCH_CHECK("gat_bwd_row_kernel");
+      if (it.n_heavy > 0) {
+        AGNN_GAT_DISPATCH(K_, NH_, (gat_bwd_merge_kernel<K, NH, 1>
+                                    <<<kNumSMs * 2, kSparseThreads, 0, s>>>(it, A, 0)));
+        AGNN_LAUNCH_CHECK("gat_bwd_merge_kernel");
+      }
     }
     it = itc;
     AGNN_GAT_DISPATCH(K_, NH_, (main_warps = (int64_t)grid_of(gat_bwd_kernel<K, NH, bwd_unroll<K>(), 2>) *

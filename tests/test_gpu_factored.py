@@ -57,6 +57,34 @@ np.savez({out!r}, H=st.H[1].cpu().numpy(), dH=st.dH[0].cpu().numpy(),
 """
 
 
+_CHILD_DIRECTED = r"""
+import sys, numpy as np, torch
+sys.path[:0] = [{root!r}, {tests!r}, {root!r} + "/oracle"]
+import oracle, parity_utils as pu
+from paper_conf_sc_bestarglzcgssci23_b200 import agnn, gen, runner
+w = gen.Workload("gat-dir", "gat", "kron", 13, 1 << 13, 8 << 13, {k}, 2, 1, act="elu")
+flags = agnn.BUILD_SELF_LOOPS | agnn.BUILD_CONNECT_ISOLATED
+src, dst = w.host_edges()
+rp, ci = oracle.csr_build(w.n, src, dst, flags=flags)
+drp, dci = agnn.csr_build(w.n, torch.from_numpy(src.view(np.int32)).cuda(),
+                          torch.from_numpy(dst.view(np.int32)).cuda(), flags)
+g = runner.Graph(w.n, drp, dci, int(dci.numel()))
+st = pu.gpu_step(w, graph=g, symmetric=False)
+H, Ws, As, R = w.host_inputs()
+print("ERRS", pu.compare(w, st, pu.oracle_step(w, rp, ci, H, Ws, As, R)))
+"""
+
+
+@pytest.mark.parametrize("mode,k", [("2", 64), ("0", 128), ("1", 128)])
+def test_directed_factored_and_unfactored(mode, k):
+    """Directed patterns: factored (row pass replaced by ds = G.Q) and two-pass."""
+    code = _CHILD_DIRECTED.format(root=ROOT, tests=os.path.join(ROOT, "tests"), k=k)
+    e = dict(os.environ, AGNN_CHUNK_EDGES="128", AGNN_GAT_FACTORED=mode)
+    r = subprocess.run([sys.executable, "-c", code], env=e, capture_output=True, text=True,
+                       timeout=600)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
+
+
 def _child(tmp_path, env, tag, prec="fp32", check=True, k=128):
     out = str(tmp_path / f"{tag}.npz")
     code = _CHILD.format(root=ROOT, tests=os.path.join(ROOT, "tests"), prec=prec, check=check,
