@@ -345,6 +345,19 @@ def run_ours(args):
     w = workload(args)
     agnn.lib()
     uid = None
+    if world > 1 and args.comm == "peer" and not same_gpu:
+        # the peer-memory exchange maps the other GPUs' buffers (CUDA IPC over
+        # NVLink): every rank checks P2P access to every other visible GPU, and if
+        # any pair lacks it all ranks fall back to the NCCL exchange together
+        ok = all(torch.cuda.can_device_access_peer(local, d)
+                 for d in range(torch.cuda.device_count()) if d != local)
+        flag = torch.tensor([1 if ok else 0], device=dev, dtype=torch.int32)
+        dist.all_reduce(flag, op=dist.ReduceOp.MIN)
+        if int(flag.item()) == 0:
+            if rank == 0:
+                print("bench: no P2P access between some GPUs; using the NCCL exchange",
+                      file=sys.stderr)
+            args.comm = "nccl"
     if world > 1 and args.comm == "nccl":
         obj = [agnn.nccl_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
