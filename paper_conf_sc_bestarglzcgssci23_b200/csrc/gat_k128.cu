@@ -11,7 +11,11 @@
 //   warp max; running max / rescale once per batch; p_ij = 2^(e_ij - m).
 //   Then the warp walks the batch: lane q owns columns 4q..4q+3 of P_j and
 //   accumulates p_ij(head(q)) P_j.  Per edge: one 16-byte gather and 4 FMAs.
-// Backward, per row j, edges in batches of B (<= lanes per head):
+// Factored backward (default, gat_args.cuh): the forward also accumulates Q_j, and
+//   the backward row kernel (gat_bwd_k128f_kernel) keeps only the column role —
+//   32-entry windows, lane-parallel alpha_ij / c'_ij from the gathered records,
+//   then warp-parallel acc += alpha G_i, v += c' G_i; no per-edge dot products.
+// Unfactored backward (AGNN_GAT_FACTORED=0), per row j, edges in batches of B (<= lanes per head):
 //   warp-parallel: gather P_i, G_i slices; partial dots G_j.P_i and G_i.P_j;
 //   a transposed butterfly reduction leaves each lane with both full dots of
 //   ONE edge of its head; lane-parallel scalar work (the two alpha recomputes,
