@@ -212,7 +212,7 @@ def run_reference(args):
               f"{args.config} ({gen.describe(w)})")
     line = {"impl": "reference", "metric": metric_name(w), "value": val, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": T * 1e3,
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
             "data": "synthetic",
             "config": {"workload": args.config, "model": w.model, "graph": w.graph,
                        "n": ws.n, "edges": m, "k": w.k, "heads": w.heads, "layers": w.layers,
