@@ -13,9 +13,11 @@ Default workload: C5 = GAT, 4 heads, k = 128, Kronecker n = 2^24 / ~1.0e9
 edges, 1 layer — the north_star target (fits one B200).  Inputs (8.6 GB per
 feature matrix) are far larger than the 126 MB L2, so no explicit flush.
 
-Multi-GPU: launched by torch.distributed.run, one rank per GPU; 1D row blocks,
-NCCL all-gather of P / G and all-reduce of dW, da inside libagnn.so; rank 0
-prints the JSON line; time = max over ranks of CUDA-event time.
+Multi-GPU: launched by torch.distributed.run, one rank per GPU; 1D row blocks;
+the all-gathers of P / G are fused into the producing kernels as NVLink peer
+stores and dW, da are all-reduced through peer memory (--comm peer, default;
+--comm nccl or missing P2P access: NCCL inside libagnn.so); rank 0 prints the
+JSON line; time = max over ranks of CUDA-event time.
 """
 from __future__ import annotations
 
