@@ -226,15 +226,14 @@ def run_reference(args):
 
 
 # ----------------------------------------------------------------------------- ours
-def gat_factored(w):
-    """The factored GAT backward (gat_args.cuh) on symmetric patterns: k' = 128 by
-    default, every width with AGNN_GAT_FACTORED=2, never with 0."""
-    mode = os.environ.get("AGNN_GAT_FACTORED", "1")
+def gat_factored(w, mode=1):
+    """The factored GAT backward (gat_args.cuh) on symmetric patterns: plan option
+    gat_factored (include/agnn.h) = 1 (default): k' = 128; 2: every width; 0: never."""
     k128 = w.k == 128 and w.heads in (1, 2, 4, 8)
-    return w.model == "gat" and (mode == "2" or (mode == "1" and k128))
+    return w.model == "gat" and (mode == 2 or (mode == 1 and k128))
 
 
-def pass_bytes(w, m, n):
+def pass_bytes(w, m, n, factored_mode=1):
     """Algorithmic bytes of each sparse pass per launch:
     {pass: (bytes, per stored edge, per row)}.  f = stored feature bytes (bf16 P, G
     in BF16 mode, reading B1); outputs and dP are fp32.
@@ -253,7 +252,7 @@ def pass_bytes(w, m, n):
     out = {}
     if w.model == "gat":
         fs = 2 if w.prec == "bf16" else 4
-        fac = gat_factored(w)
+        fac = gat_factored(w, factored_mode)
         pe = 4 + w.k * fs + 4 * w.heads
         pr = 4 * w.heads + (3 if fac else 2) * w.k * f + 8 * w.heads + 8
         out["fwd"] = (pe * m + pr * n, pe, pr)

@@ -112,7 +112,17 @@ typedef enum {
   AGNN_PREC_BF16 = 2     /* GAT: P and G stored as bfloat16 (reading B1)      */
 } agnn_prec;
 
-enum { AGNN_CSR_SYMMETRIC = 1u };
+/* agnn_csr.flags.
+ * AGNN_CSR_SYMMETRIC: the pattern is symmetric ("for undirected
+ *   graphs A = A^T"); the backward then visits every stored entry once for
+ *   both of its roles.  The library trusts the flag unless
+ * AGNN_PLAN_VERIFY_SYMMETRY is also set: agnn_plan_create then checks on the
+ *   device that every stored (i,j) has its transpose (j,i) stored, and returns
+ *   AGNN_EINVAL if one is missing (world == 1 with every row in the plan; with
+ *   world > 1 each rank can see only its own rows, so the flag makes
+ *   agnn_plan_create return AGNN_EUNSUPPORTED).  Costs one binary search per
+ *   stored entry at plan time; nothing at run time.                         */
+enum { AGNN_CSR_SYMMETRIC = 1u, AGNN_PLAN_VERIFY_SYMMETRY = 2u };
 
 typedef struct {
   int64_t n;               /* global vertex count                                  */
@@ -120,8 +130,29 @@ typedef struct {
   int64_t row_end;
   const int64_t* row_ptr;  /* device, [row_end - row_begin + 1], row_ptr[0] == 0   */
   const int32_t* col_idx;  /* device, [row_ptr[n_local]], global ids, ascending    */
-  uint32_t flags;          /* AGNN_CSR_SYMMETRIC                                   */
+  uint32_t flags;          /* AGNN_CSR_SYMMETRIC | AGNN_PLAN_VERIFY_SYMMETRY       */
 } agnn_csr;
+
+/* Work-decomposition options of a plan (agnn_plan_create_ex).  None of them
+ * changes what is computed: every choice gives the same outputs up to fp32
+ * rounding order (the chunk size fixes the summation order of heavy rows, so a
+ * plan with a different chunk size is a different, equally valid rounding).
+ * A field < 0 (or 0 for chunk_edges) takes the default; agnn_plan_create uses
+ * all defaults.  Values out of range return AGNN_EINVAL.                     */
+typedef struct {
+  int32_t chunk_edges;    /* heavy-row chunk size in stored entries, 32 .. 2^30;
+                             default: 256 for n <= 2^21, doubling per doubling of
+                             n, at most 2048 (a function of the global n only)  */
+  int32_t short_edges;    /* rows of degree <= short_edges go to the short-row
+                             kernels where a kernel has one; 0 .. 32, default 32  */
+  int32_t short_bundles;  /* GAT k'=128 short rows packed into 32-entry warp
+                             bundles: 0 never, 1 fp32 storage only (default),
+                             2 fp32 and bf16                                       */
+  int32_t gat_factored;   /* GAT factored backward: 0 never,
+                             1 k_out = 128 only (default), 2 every width          */
+  int32_t l2_hot_mb;      /* L2 budget (MB) of the evict_last gathers, 0 disables
+                             the hints; default 96 (performance only, see below)  */
+} agnn_plan_options;
 
 typedef struct {
   int rank, world;
@@ -157,16 +188,20 @@ agnn_status agnn_partition(int64_t n, const int64_t* row_ptr_host, int world, in
  * col_idx (nnz x 4 bytes of device memory) whose free high bits rank every
  * column by how often this rank gathers it; the sparse kernels load the rows of
  * the most-gathered columns with an evict_last L2 policy (
- * environment AGNN_L2_HOT_MB = L2 budget in MB, 0 disables).  The classes are
- * performance metadata only: no result depends on them.  Synchronises. */
+ * agnn_plan_options.l2_hot_mb).  The classes are performance metadata only:
+ * no result depends on them.  With world == 1 the CSR must hold every row
+ * (row_begin == 0, row_end == n), else AGNN_EINVAL.  Synchronises. */
 agnn_status agnn_plan_create(const agnn_csr* csr, const agnn_dist* dist /* NULL => 1 GPU */,
                              cudaStream_t stream, agnn_plan_t* out);
+/* The same with explicit work-decomposition options (NULL => defaults).      */
+agnn_status agnn_plan_create_ex(const agnn_csr* csr, const agnn_dist* dist,
+                                const agnn_plan_options* options, cudaStream_t stream,
+                                agnn_plan_t* out);
 agnn_status agnn_plan_destroy(agnn_plan_t plan);
 /* host-side statistics: [0]=n_local [1]=nnz_local [2]=light rows [3]=heavy rows
  * [4]=heavy chunks [5]=chunk size [6]=max degree [7]=n (global) [8]=short rows
  * (light rows of degree <= [9], taken by the short-row kernels where a kernel
- * has one) [9]=short_max (0: no split; AGNN_SHORT_EDGES overrides the default and
- * maximum 32) */
+ * has one) [9]=short_max (agnn_plan_options.short_edges; 0: no split) */
 agnn_status agnn_plan_info(agnn_plan_t plan, int64_t* info10);
 
 /* The transposed pattern of the plan's CSR (test/utility; synchronises):

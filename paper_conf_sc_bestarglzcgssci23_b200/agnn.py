@@ -19,7 +19,7 @@ AGG = {"sum": 0, "mean": 1, "gcn": 2, "max": 3, "min": 4}
 ACT = {"none": 0, "relu": 1, "elu": 2}
 PREC_FP32, PREC_TF32X3, PREC_BF16 = 0, 1, 2
 PREC = {"fp32": PREC_FP32, "tf32x3": PREC_TF32X3, "bf16": PREC_BF16}
-CSR_SYMMETRIC = 1
+CSR_SYMMETRIC, PLAN_VERIFY_SYMMETRY = 1, 2
 BUILD_SYMMETRIZE, BUILD_SELF_LOOPS, BUILD_CONNECT_ISOLATED = 1, 2, 4
 BUILD_PAPER = BUILD_SYMMETRIZE | BUILD_SELF_LOOPS | BUILD_CONNECT_ISOLATED
 
@@ -27,7 +27,7 @@ STATUS = {0: "AGNN_OK", 1: "AGNN_EINVAL", 2: "AGNN_ECUDA", 3: "AGNN_ENCCL", 4: "
           5: "AGNN_EUNSUPPORTED", 6: "AGNN_ESTATE"}
 
 # every symbol include/agnn.h declares (tests check the .so exports all of them)
-EXPORTS = ("agnn_partition", "agnn_plan_create", "agnn_plan_destroy", "agnn_plan_info",
+EXPORTS = ("agnn_partition", "agnn_plan_create", "agnn_plan_create_ex", "agnn_plan_destroy", "agnn_plan_info",
            "agnn_plan_csc", "agnn_loss_inner", "agnn_sgd_step",
            "agnn_ipc_export", "agnn_plan_ctl_export", "agnn_plan_connect", "agnn_plan_register",
            "agnn_model_create", "agnn_model_destroy", "agnn_saved_bytes", "agnn_workspace_bytes",
@@ -49,6 +49,17 @@ class CSR(ctypes.Structure):
     _fields_ = [("n", ctypes.c_int64), ("row_begin", ctypes.c_int64), ("row_end", ctypes.c_int64),
                 ("row_ptr", ctypes.c_void_p), ("col_idx", ctypes.c_void_p),
                 ("flags", ctypes.c_uint32)]
+
+
+class PlanOptions(ctypes.Structure):
+    """agnn_plan_options (include/agnn.h); a field < 0 (0 for chunk_edges) = default."""
+    _fields_ = [("chunk_edges", ctypes.c_int32), ("short_edges", ctypes.c_int32),
+                ("short_bundles", ctypes.c_int32), ("gat_factored", ctypes.c_int32),
+                ("l2_hot_mb", ctypes.c_int32)]
+
+    @classmethod
+    def make(cls, chunk_edges=0, short_edges=-1, short_bundles=-1, gat_factored=-1, l2_hot_mb=-1):
+        return cls(chunk_edges, short_edges, short_bundles, gat_factored, l2_hot_mb)
 
 
 class Dist(ctypes.Structure):
@@ -218,11 +229,13 @@ class Plan:
     """agnn_plan_create: validated CSR + work lists (+ NCCL communicator when world > 1)."""
 
     def __init__(self, row_ptr, col_idx, n, row_begin=0, row_end=None, symmetric=True,
-                 rank=0, world=1, nccl_unique_id: bytes | None = None, bounds=None, stream=None):
+                 rank=0, world=1, nccl_unique_id: bytes | None = None, bounds=None, stream=None,
+                 options: dict | None = None, verify_symmetry: bool = False):
         self.row_ptr, self.col_idx = row_ptr, col_idx  # keep the caller's CSR alive
         row_end = n if row_end is None else row_end
-        self._csr = CSR(n, row_begin, row_end, row_ptr.data_ptr(), col_idx.data_ptr(),
-                        CSR_SYMMETRIC if symmetric else 0)
+        flags = (CSR_SYMMETRIC if symmetric else 0) | (PLAN_VERIFY_SYMMETRY if verify_symmetry else 0)
+        self._csr = CSR(n, row_begin, row_end, row_ptr.data_ptr(), col_idx.data_ptr(), flags)
+        self._opts = PlanOptions.make(**(options or {}))
         dist = None
         if world > 1:
             import numpy as np
@@ -233,9 +246,9 @@ class Plan:
                 uid = ctypes.cast(self._uid, ctypes.c_void_p)
             dist = Dist(rank, world, uid, self._bounds.ctypes.data_as(ctypes.c_void_p))
         h = ctypes.c_void_p()
-        _check(lib().agnn_plan_create(ctypes.byref(self._csr),
-                                      ctypes.byref(dist) if dist is not None else None,
-                                      _stream(stream), ctypes.byref(h)))
+        _check(lib().agnn_plan_create_ex(ctypes.byref(self._csr),
+                                         ctypes.byref(dist) if dist is not None else None,
+                                         ctypes.byref(self._opts), _stream(stream), ctypes.byref(h)))
         self.handle = h
         self.n, self.row_begin, self.row_end = n, row_begin, row_end
         self.n_local = row_end - row_begin

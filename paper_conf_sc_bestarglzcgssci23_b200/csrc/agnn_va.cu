@@ -487,16 +487,6 @@ agnn_status av_workspace_bytes(const Plan& p, const agnn_layer_desc& d, size_t* 
     else return fail(AGNN_EUNSUPPORTED, "AGNN/VA: k_in must be 16/32/64/128/256"); \
   } while (0)
 
-// AGNN_AV_K128=0 selects the generic kernels at k = 128 / 256 (A/B comparisons)
-bool k128_disabled() {
-  static int v = -1;
-  if (v < 0) {
-    const char* e = getenv("AGNN_AV_K128");
-    v = (e && e[0] == '0') ? 1 : 0;
-  }
-  return v == 1;
-}
-
 template <int K>
 constexpr int av_fwd_unroll() { return K >= 256 ? 2 : 4; }
 template <int K>
@@ -524,7 +514,7 @@ agnn_status av_forward(const Plan& p, const agnn_layer_desc& d, const float* W, 
   }
   Items it = items_of(p);
   AvFwd A{Hf, sv.nu, d.beta, fabsf(d.beta), sv.X, sv.l, w.pacc, w.pl};
-  if ((K_ == 128 || K_ == 256) && !k128_disabled()) {
+  if (K_ == 128 || K_ == 256) {
     // gathered per entry: an H_j row (+ nu_j)
     const Items ith = l2_hinted(it, p, 4 * (int64_t)K_ + (ag ? 4 : 0));
     if ((st = av_fwd_batched(ith, K_, ag, A, s)) != AGNN_OK) return st;
@@ -628,7 +618,7 @@ agnn_status av_backward(const Plan& p, const agnn_layer_desc& d, const float* W,
 #undef AV_PASS
     return AGNN_OK;
   }
-  if ((K_ == 128 || K_ == 256) && !k128_disabled()) {
+  if (K_ == 128 || K_ == 256) {
     // gathered per entry: the H_i and M_i rows (+ the record)
     const Items ith = l2_hinted(it, p, 8 * (int64_t)K_ + (ag ? 16 : 0));
     if ((st = av_bwd_batched(ith, K_, ag, A, s)) != AGNN_OK) return st;

@@ -86,6 +86,15 @@ void prof_mark(const char* name, cudaStream_t s) {
 }
 
 agnn_status plan_build(Plan& p, cudaStream_t s);
+agnn_status plan_options(Plan& p, const agnn_plan_options* o);
+
+// widths with a sparse-kernel instantiation (the dispatch tables of gat.cu,
+// agnn_va.cu, cgnn.cu): anything else is rejected here, before any launch
+static bool pow2_width(int k) { return k == 16 || k == 32 || k == 64 || k == 128 || k == 256; }
+static bool gat_width(int k, int h) {
+  if (k == 16) return h == 1 || h == 2 || h == 4;
+  return pow2_width(k) && (h == 1 || h == 2 || h == 4 || h == 8);
+}
 
 static agnn_status check_desc(const agnn_layer_desc& d) {
   if (d.k_in <= 0 || d.k_out <= 0 || d.k_in % 4 || d.k_out % 4)
@@ -99,17 +108,19 @@ static agnn_status check_desc(const agnn_layer_desc& d) {
   if (d.kind == AGNN_GAT) {
     if (d.heads <= 0 || d.k_out % d.heads || (d.k_out / d.heads) % 4)
       return fail(AGNN_EINVAL, "GAT: k_out must split into heads of a multiple of 4 features");
-    if (d.k_out > 256 || d.k_out % 16)
-      return fail(AGNN_EUNSUPPORTED, "GAT: k_out must be one of 16..256, multiple of 16");
+    if (!gat_width(d.k_out, d.heads))
+      return fail(AGNN_EUNSUPPORTED,
+                  "GAT: (k_out, heads) must be k_out in 16/32/64/128/256 with 1/2/4/8 heads "
+                  "(k_out = 16: 1/2/4)");
   } else if (d.kind == AGNN_AGNN || d.kind == AGNN_VA) {
     if (d.heads != 1) return fail(AGNN_EINVAL, "AGNN/VA: heads must be 1");
-    if (d.k_in > 256 || d.k_in % 16)
-      return fail(AGNN_EUNSUPPORTED, "AGNN/VA: k_in must be one of 16..256, multiple of 16");
+    if (!pow2_width(d.k_in))
+      return fail(AGNN_EUNSUPPORTED, "AGNN/VA: k_in must be 16/32/64/128/256");
   } else if (d.kind == AGNN_CGNN) {
     if (d.heads != 1) return fail(AGNN_EINVAL, "C-GNN: heads must be 1");
     if (d.agg < AGNN_AGG_SUM || d.agg > AGNN_AGG_MIN) return fail(AGNN_EINVAL, "C-GNN: agg");
-    if (d.k_in > 256 || d.k_in % 16)
-      return fail(AGNN_EUNSUPPORTED, "C-GNN: k_in must be one of 16..256, multiple of 16");
+    if (!pow2_width(d.k_in))
+      return fail(AGNN_EUNSUPPORTED, "C-GNN: k_in must be 16/32/64/128/256");
   } else {
     return fail(AGNN_EINVAL, "layer desc: kind");
   }
@@ -223,11 +234,22 @@ agnn_status agnn_profile_reset(void) {
 
 agnn_status agnn_plan_create(const agnn_csr* csr, const agnn_dist* dist, cudaStream_t s,
                              agnn_plan_t* out) {
+  return agnn_plan_create_ex(csr, dist, nullptr, s, out);
+}
+
+agnn_status agnn_plan_create_ex(const agnn_csr* csr, const agnn_dist* dist,
+                                const agnn_plan_options* opts, cudaStream_t s, agnn_plan_t* out) {
   try {
     if (!csr || !out) return fail(AGNN_EINVAL, "agnn_plan_create: NULL argument");
     if (csr->n <= 0 || csr->n > INT32_MAX || csr->row_begin < 0 || csr->row_end > csr->n ||
         csr->row_end < csr->row_begin || !csr->row_ptr)
       return fail(AGNN_EINVAL, "agnn_plan_create: bad CSR header (n, row range, row_ptr)");
+    if (!(dist && dist->world > 1) && (csr->row_begin != 0 || csr->row_end != csr->n))
+      return fail(AGNN_EINVAL,
+                  "agnn_plan_create: with world == 1 the CSR must hold every row "
+                  "(row_begin == 0, row_end == n)");
+    if (csr->flags & ~(uint32_t)(AGNN_CSR_SYMMETRIC | AGNN_PLAN_VERIFY_SYMMETRY))
+      return fail(AGNN_EINVAL, "agnn_plan_create: unknown CSR flags");
     auto* h = new (std::nothrow) agnn_plan_s();
     if (!h) return fail(AGNN_ENOMEM, "agnn_plan_create: out of host memory");
     Plan& p = h->p;
@@ -255,7 +277,8 @@ agnn_status agnn_plan_create(const agnn_csr* csr, const agnn_dist* dist, cudaStr
         return fail(AGNN_EINVAL, "agnn_plan_create: bounds do not match the CSR row range");
       }
     }
-    agnn_status st = plan_build(p, s);
+    agnn_status st = plan_options(p, opts);
+    if (st == AGNN_OK) st = plan_build(p, s);
     if (st == AGNN_OK && p.world > 1) st = comm_init(p, dist->nccl_unique_id);
     if (st != AGNN_OK) {
       comm_destroy(p);

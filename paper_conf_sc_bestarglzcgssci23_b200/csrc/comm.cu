@@ -127,16 +127,34 @@ PFN_getRange get_range_fn() {
   return fn;
 }
 
-// map every peer's IPC handle (rank order, 64 B each) + byte offset; own rank -> local
+// CUDA IPC maps an allocation at most once per process, while several plans (and
+// several registered tensors of one allocation) may need it: the mappings are
+// shared and reference-counted.  Every acquisition is recorded in the acquiring
+// plan's `opened` list and released by comm_destroy; the mapping is closed when
+// its last holder releases it.
+struct IpcMap {
+  void* base;
+  int refs;
+};
+std::mutex g_ipc_mu;
+std::map<std::pair<int, std::string>, IpcMap> g_ipc;
+
+void ipc_release(void* base) {  // caller holds g_ipc_mu
+  for (auto it = g_ipc.begin(); it != g_ipc.end(); ++it) {
+    if (it->second.base != base) continue;
+    if (--it->second.refs == 0) {
+      cudaIpcCloseMemHandle(base);
+      g_ipc.erase(it);
+    }
+    return;
+  }
+}
 }  // namespace
 
+// map every peer's IPC handle (rank order, 64 B each) + byte offset; own rank -> local
 agnn_status peer_open(Plan& p, const void* handles, const int64_t* offsets, void* local,
                        char* out[kMaxPeers]) {
-  // one process may register several tensors of the same allocation: map each
-  // (rank, handle) once
-  static std::mutex mu;
-  static std::map<std::pair<int, std::string>, void*> cache;
-  std::lock_guard<std::mutex> lock(mu);
+  std::lock_guard<std::mutex> lock(g_ipc_mu);
   for (int r = 0; r < p.world; ++r) {
     if (r == p.rank) {
       out[r] = static_cast<char*>(local);
@@ -146,14 +164,15 @@ agnn_status peer_open(Plan& p, const void* handles, const int64_t* offsets, void
     memcpy(&h, static_cast<const char*>(handles) + 64 * r, sizeof(h));
     const auto key = std::make_pair(r, std::string(reinterpret_cast<const char*>(&h), sizeof(h)));
     void* base = nullptr;
-    auto it = cache.find(key);
-    if (it != cache.end()) {
-      base = it->second;
+    auto it = g_ipc.find(key);
+    if (it != g_ipc.end()) {
+      base = it->second.base;
+      ++it->second.refs;
     } else {
       AGNN_CUDA_TRY(cudaIpcOpenMemHandle(&base, h, cudaIpcMemLazyEnablePeerAccess));
-      cache[key] = base;
-      p.opened->push_back(base);
+      g_ipc[key] = IpcMap{base, 1};
     }
+    p.opened->push_back(base);
     out[r] = static_cast<char*>(base) + offsets[r];
   }
   return AGNN_OK;
@@ -221,7 +240,8 @@ void comm_destroy(Plan& p) {
   if (p.nccl) ncclCommDestroy(static_cast<ncclComm_t>(p.nccl));
   p.nccl = nullptr;
   if (p.opened) {
-    for (void* q : *p.opened) cudaIpcCloseMemHandle(q);
+    std::lock_guard<std::mutex> lock(g_ipc_mu);
+    for (void* q : *p.opened) ipc_release(q);
     delete p.opened;
     p.opened = nullptr;
   }

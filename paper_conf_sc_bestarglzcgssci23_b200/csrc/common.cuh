@@ -276,6 +276,10 @@ struct Plan {
   void* csc_block = nullptr;          // backs csc_ptr / csc_idx
   void* c_meta_block = nullptr;       // backs the column work lists
   bool directed() const { return !(flags & 1u); }
+  // work-decomposition options (agnn_plan_options; include/agnn.h)
+  int gat_factored = 1;               // 0 never, 1 k' = 128 only, 2 every width
+  int bundle_mode = 1;                // short-row bundles: 0 never, 1 fp32, 2 fp32 + bf16
+  int64_t l2_hot_mb = 96;             // evict_last budget; 0: no column classes
   int64_t max_chunks() const { return n_chunks > c_chunks ? n_chunks : c_chunks; }
   // distribution
   int rank = 0, world = 1;

@@ -649,11 +649,11 @@ __global__ void gat_debug_alpha_kernel(const int64_t* __restrict__ rp, int64_t n
 // kernels or the generic ones (forward with QF, backward = the column-role pass
 // over the CSR, which for a symmetric pattern lists every column's entries);
 // directed patterns skip their row pass (column pass over the CSC only)
-// AGNN_GAT_FACTORED: 1 (default) = k' = 128 only; 2 = every width; 0 = never.
+// Plan option gat_factored: 1 (default) = k' = 128 only; 2 = every width; 0 = never.
 // Measured: k' = 128 at C5 1.45x faster step; k' = 64 at C2 (L2-resident, so the
 // gathered bytes it saves cost nothing) 0.81 -> 0.87 ms, hence k' = 128 only by default.
 bool factored(const Plan& p, const GatShape& g) {
-  const int mode = gat_factored_mode();
+  const int mode = p.gat_factored;
   return mode > 0 && (mode == 2 || gat_k128_supported(g.k_out, g.heads));
 }
 
@@ -728,14 +728,6 @@ WsGat carve_ws(const Plan& p, const GatShape& g, void* base, size_t* total) {
 }
 
 }  // namespace
-
-int gat_factored_mode() {
-  static const int v = [] {
-    const char* e = getenv("AGNN_GAT_FACTORED");
-    return e ? atoi(e) : 1;
-  }();
-  return v;
-}
 
 size_t gat_saved_bytes(const Plan& p, const GatShape& g) { return saved_size(p, g); }
 size_t gat_workspace_bytes(const Plan& p, const GatShape& g) {
@@ -848,7 +840,7 @@ agnn_status gat_forward(const Plan& p, const GatShape& g, const float* W, const 
            w.pacc + 2 * p.max_chunks() * g.k_out};
   if (gat_k128_supported(g.k_out, g.heads)) {
     const Items ith = l2_hinted(it, p, 4 * (int64_t)g.k_out + 4 * g.heads);
-    if ((st = gat_fwd_k128(ith, g.heads, sv.P, sv.st, g.slope, g.act, o, p.n, s)) != AGNN_OK)
+    if ((st = gat_fwd_k128(ith, g.heads, sv.P, sv.st, g.slope, g.act, o, s)) != AGNN_OK)
       return st;
   } else if (it.n_chunks + it.n_light > 0) {
     if (o.Q)

@@ -40,7 +40,7 @@ struct GatBwdArgs {
 };
 
 // The factored GAT backward (symmetric patterns; k' = 128 by default, every width
-// with AGNN_GAT_FACTORED=2, off with 0).  With c_ji = alpha_ji lambda_ji (lambda = LReLU slope of the
+// or none with agnn_plan_options.gat_factored).  With c_ji = alpha_ji lambda_ji (lambda = LReLU slope of the
 // entry), the row-role sum of PAPER.md:250-254 is linear in the gathered rows,
 //   ds_j = sum_i c_ji (G_j . P_i - delta_j) = G_j . (sum_i c_ji P_i - (sum_i c_ji) Z_j)
 //        = G_j . Q_j,
@@ -49,22 +49,17 @@ struct GatBwdArgs {
 // backward edge pass gathers only G_i and rec_i (column role):
 //   dt_j = sum_i c'_ij (G_i . P_j - delta_i) = P_j . v_j - sum_i c'_ij delta_i,
 //   v_j = sum_i c'_ij G_i,  acc_j = sum_i alpha_ij G_i.
-int gat_factored_mode();  // AGNN_GAT_FACTORED: 0 off, 1 k' = 128 (default), 2 all widths
 
 // k' = 128 kernels (gat_k128.cu): lane-parallel scalar work, warp-parallel rows
 bool gat_k128_supported(int k_out, int heads);
 agnn_status gat_fwd_k128(const Items& it, int heads, const float* P, const float* st, float slope,
-                         int act, const GatFwdOut& o, int64_t n_rows, cudaStream_t s);
+                         int act, const GatFwdOut& o, cudaStream_t s);
 // short rows (gat_short.cu): rows of it.short_rows, 4 rows per warp
 template <typename TP>
 agnn_status gat_fwd_short(const Items& it, int heads, const TP* P, const float* st, float slope,
                           int act, const GatFwdOut& o, cudaStream_t s);
 agnn_status gat_bwd_short(const Items& it, int heads, const GatBwdArgs& A, int64_t da_row0,
                           int64_t* warps, cudaStream_t s);
-// BF16 backward with cp.async staging (gat_async.cu); opt-in with AGNN_BWD_ASYNC=1
-bool gat_bwd_async_enabled();
-agnn_status gat_bwd_async(const Items& it, int heads, const GatBwdArgs& A, int64_t* warps,
-                          cudaStream_t s);
 // the k' = 128 row kernels take the long light rows; the short ones go to gat_short.cu
 inline Items long_items(const Items& it) {
   Items r = it;
@@ -85,8 +80,11 @@ agnn_status gat_bwd_k128f(const Items& it, int heads, const GatBwdArgs& A, int64
 agnn_status gat_bwd_short_f(const Items& it, int heads, const GatBwdArgs& A, int64_t da_row0,
                             int64_t* warps, cudaStream_t s);
 // bundles of short rows (gat_bundle.cu): the short rows as 32-entry warp batches;
-// AGNN_SHORT_BUNDLES=0 falls back to the row-group short kernels (gat_short.cu)
-bool gat_bundles_enabled(bool bf16_storage);
+// the plan's bundle mode (agnn_plan_options.short_bundles) selects them per storage
+// type, else the row-group short kernels (gat_short.cu) run
+inline bool gat_bundles_enabled(const Items& it, bool bf16_storage) {
+  return bf16_storage ? it.bundle_mode >= 2 : it.bundle_mode >= 1;
+}
 template <typename TP>
 agnn_status gat_fwd_bundle(const Items& it, int heads, const TP* P, const float* st, float slope,
                            int act, const GatFwdOut& o, cudaStream_t s);

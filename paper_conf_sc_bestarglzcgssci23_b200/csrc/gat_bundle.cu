@@ -412,25 +412,10 @@ int grid_of_fn(F* f) {
     else return fail(AGNN_EUNSUPPORTED, "GAT k'=128: heads must be 1/2/4/8"); \
   } while (0)
 
-// AGNN_SHORT_BUNDLES: 1 = bundles for fp32 storage (default; measured C5: fwd short
-// rows 14.0 -> 12.3 ms, bwd 13.3 -> 12.9 ms), 2 = for bf16 too (measured on par or
-// slightly slower than the row-group kernels: 10.3 -> 10.8 ms), 0 = never
-// AGNN_BUNDLE_MINB (measurement): resident 256-thread blocks per SM of the bundle kernels
-static int bundle_minb() {
-  static const int v = [] {
-    const char* e = getenv("AGNN_BUNDLE_MINB");
-    return e ? atoi(e) : 2;
-  }();
-  return v;
-}
-
-bool gat_bundles_enabled(bool bf16_storage) {
-  static const int v = [] {
-    const char* e = getenv("AGNN_SHORT_BUNDLES");
-    return e ? atoi(e) : 1;
-  }();
-  return bf16_storage ? v >= 2 : v >= 1;
-}
+// bundles run for fp32 storage by default (agnn_plan_options.short_bundles; measured
+// C5, round 1: fwd short rows 14.0 -> 12.3 ms, bwd 13.3 -> 12.9 ms); for bf16 they
+// measured on par or slightly slower than the row-group kernels (10.3 -> 10.8 ms).
+// 2 resident 256-thread blocks per SM (3 measured slower: fwd 12.2 -> 15.1 ms).
 
 template <typename TP>
 agnn_status gat_fwd_bundle(const Items& it, int heads, const TP* P, const float* st, float slope,
@@ -442,10 +427,8 @@ agnn_status gat_fwd_bundle(const Items& it, int heads, const TP* P, const float*
     AGNN_LAUNCH_CHECK("gat_empty_rows_kernel");
   }
   if (it.n_bundles == 0) return AGNN_OK;
-  const int minb = bundle_minb();
   AGNN_BUNDLE_DISPATCH(heads, ({
-    auto* kern = minb == 3 ? (o.Q ? gat_fwd_bundle_kernel<TP, NH, true, 3> : gat_fwd_bundle_kernel<TP, NH, false, 3>)
-                           : (o.Q ? gat_fwd_bundle_kernel<TP, NH, true, 2> : gat_fwd_bundle_kernel<TP, NH, false, 2>);
+    auto* kern = o.Q ? gat_fwd_bundle_kernel<TP, NH, true, 2> : gat_fwd_bundle_kernel<TP, NH, false, 2>;
     kern<<<grid_of_fn(kern), 256, 0, s>>>(it, P, st, slope, act, o);
     AGNN_LAUNCH_CHECK("gat_fwd_short_kernel");
   }));
@@ -467,11 +450,9 @@ agnn_status gat_bwd_bundle(const Items& it, int heads, const GatBwdArgs& A, int6
     AGNN_LAUNCH_CHECK("gat_empty_rows_kernel");
   }
   if (it.n_bundles == 0) return AGNN_OK;
-  const int minb = bundle_minb();
   AGNN_BUNDLE_DISPATCH(heads, ({
     using KB = void (*)(Items, GatBwdArgs, int64_t);
-    KB kern = minb == 3 ? (A.P16 ? (KB)gat_bwd_bundle_kernel<bf16, NH, 3> : (KB)gat_bwd_bundle_kernel<float, NH, 3>)
-                        : (A.P16 ? (KB)gat_bwd_bundle_kernel<bf16, NH, 2> : (KB)gat_bwd_bundle_kernel<float, NH, 2>);
+    KB kern = A.P16 ? (KB)gat_bwd_bundle_kernel<bf16, NH, 2> : (KB)gat_bwd_bundle_kernel<float, NH, 2>;
     const int grid = grid_of_fn(kern);
     kern<<<grid, 256, 0, s>>>(it, A, da_row0);
     AGNN_LAUNCH_CHECK("gat_bwd_short_kernel");

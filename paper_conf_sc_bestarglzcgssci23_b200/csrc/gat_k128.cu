@@ -20,11 +20,6 @@
 //   a transposed butterfly reduction leaves each lane with both full dots of
 //   ONE edge of its head; lane-parallel scalar work (the two alpha recomputes,
 //   dc_ji, dc_ij); alpha_ij is broadcast back for acc_j += alpha_ij G_i.
-#include <cuda.h>
-#include <cudaTypedefs.h>
-
-#include <mutex>
-
 #include "gat_args.cuh"
 #include "warp_batch.cuh"
 
@@ -267,178 +262,6 @@ gat_fwd_k128_kernel(Items it, const TP* __restrict__ P, const float* __restrict_
         const float r = lh > 0.f ? ch / lh : 0.f;
         st4(o.Q + row * K + cq, mul4(inv, fma4(-r, acc, accu)));
       }
-      if (o.m && lane == 0) {
-#pragma unroll
-        for (int h = 0; h < NH; ++h) {
-          o.m[row * NH + h] = l[h] > 0.f ? mr[h] : 0.f;
-          o.l[row * NH + h] = l[h];
-        }
-      }
-    }
-  }
-}
-
-// ---------------------------------------------------------------- forward (TMA gather)
-// Same arithmetic as gat_fwd_k128_kernel; the neighbour rows P_j arrive by TMA
-// tile::gather4 (4 rows of 512 B per instruction, issued by one lane) into a
-// per-warp shared-memory ring of two 16-edge batches, so the next batch's
-// gathers are in flight while the current batch is scored and accumulated.
-__device__ __forceinline__ uint32_t sh_u32(const void* p) {
-  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
-}
-__device__ __forceinline__ void mbar_init1(uint64_t* b) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(sh_u32(b)) : "memory");
-}
-__device__ __forceinline__ void mbar_expect(uint64_t* b, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(sh_u32(b)),
-               "r"(bytes)
-               : "memory");
-}
-__device__ __forceinline__ void mbar_wait_parity(uint64_t* b, uint32_t parity) {
-  asm volatile(
-      "{\n.reg .pred p;\nW_%=:\n"
-      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
-      "@!p bra W_%=;\n}\n" ::"r"(sh_u32(b)),
-      "r"(parity)
-      : "memory");
-}
-__device__ __forceinline__ void gather4(void* dst, const CUtensorMap* map, uint64_t* bar, int r0,
-                                        int r1, int r2, int r3) {
-  asm volatile(
-      "cp.async.bulk.tensor.2d.shared::cta.global.tile::gather4.mbarrier::complete_tx::bytes"
-      " [%0], [%1, {%3, %4, %5, %6, %7}], [%2];" ::"r"(sh_u32(dst)),
-      "l"(map), "r"(sh_u32(bar)), "n"(0), "r"(r0), "r"(r1), "r"(r2), "r"(r3)
-      : "memory");
-}
-
-constexpr int TB = 16;           // edges per batch
-constexpr int TG = TB / 4;       // gather4 stages per batch
-constexpr int TW = 4;            // warps per block
-constexpr int TRING = 2 * TB * K * 4;   // bytes per warp: two batches of rows
-
-template <int NH>
-__global__ void __launch_bounds__(TW * 32)
-gat_fwd_tma_kernel(const __grid_constant__ CUtensorMap mapP, Items it, const float* __restrict__ st,
-                   float slope, int act, GatFwdOut o) {
-  constexpr int D = K / NH, HL = D / 4;
-  extern __shared__ __align__(128) unsigned char tsm[];
-  __shared__ __align__(8) uint64_t bars[TW][2][TG];
-  __shared__ float sPw[TW][NH][33];
-  __shared__ int sJ[TW][2][TB];
-  const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
-  const int hv = lane / HL, cq = lane * 4;
-  float4* ring = reinterpret_cast<float4*>(tsm + wib * TRING);  // [2][TB][32] float4
-  if (lane == 0) {
-#pragma unroll
-    for (int b = 0; b < 2; ++b)
-#pragma unroll
-      for (int g = 0; g < TG; ++g) mbar_init1(&bars[wib][b][g]);
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-  }
-  __syncwarp();
-  uint32_t phase = 0;  // bit (half * TG + g): parity of the next completion of bars[half][g]
-  const int64_t nitems = it.n_chunks + it.n_light;
-  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  // load the column ids of a batch and (lane 0) start its gathers into ring half `hb`
-  auto issue = [&](int64_t b0, int cnt, int hb) -> int {
-    const int j = lane < cnt ? (int)((uint32_t)__ldg(it.col + b0 + lane) & it.col_mask) : 0;
-    const int jl = __shfl_sync(FULL, j, cnt - 1);        // pad the last gather4 with a valid row
-    const int jj = lane < cnt ? j : jl;
-    if (lane < TB) sJ[wib][hb][lane] = jj;
-    __syncwarp();
-    if (lane == 0) {
-      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-      for (int g = 0; g * 4 < cnt; ++g) {
-        mbar_expect(&bars[wib][hb][g], 4 * K * 4);
-        gather4(ring + (hb * TB + 4 * g) * 32, &mapP, &bars[wib][hb][g], sJ[wib][hb][4 * g],
-                sJ[wib][hb][4 * g + 1], sJ[wib][hb][4 * g + 2], sJ[wib][hb][4 * g + 3]);
-      }
-    }
-    return j;
-  };
-  for (int64_t w = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; w < nitems; w += nw) {
-    int64_t row, beg, end, slot;
-    item_of(it, w, row, beg, end, slot);
-    const int64_t grow = it.row_begin + row;
-    float si[NH], mr[NH], lp[NH];
-    load_n<NH>(st + grow * (2 * NH), si);
-#pragma unroll
-    for (int h = 0; h < NH; ++h) {
-      mr[h] = -INFINITY;
-      lp[h] = 0.f;
-    }
-    float4 acc = f4(0.f);
-    int hb = 0;
-    int cnt = (int)(end - beg < TB ? end - beg : TB);
-    int jcur = cnt > 0 ? issue(beg, cnt, hb) : 0;
-    for (int64_t b0 = beg; b0 < end; b0 += TB) {
-      // next batch of this row: its gathers overlap this batch's work
-      const int64_t b1 = b0 + TB;
-      const int cnt1 = b1 < end ? (int)(end - b1 < TB ? end - b1 : TB) : 0;
-      const int jnext = cnt1 > 0 ? issue(b1, cnt1, hb ^ 1) : 0;
-      // lane-parallel scores of this batch (lanes < cnt)
-      const bool valid = lane < cnt;
-      float tj[NH];
-      load_n<NH>(st + (int64_t)jcur * (2 * NH) + NH, tj);
-      float sch = 1.f;
-#pragma unroll
-      for (int h = 0; h < NH; ++h) {
-        const float pre = si[h] + tj[h];
-        const float e = valid ? fmaxf(pre, slope * pre) : -INFINITY;
-        float bm = e;
-#pragma unroll
-        for (int off = 16; off > 0; off >>= 1) bm = fmaxf(bm, __shfl_xor_sync(FULL, bm, off));
-        const float mn = fmaxf(mr[h], bm);
-        const float sc = ex2(mr[h] - mn);
-        lp[h] *= sc;
-        if (h == hv) sch = sc;
-        mr[h] = mn;
-        const float p = valid ? ex2(e - mn) : 0.f;
-        lp[h] += p;
-        sPw[wib][h][lane] = p;
-      }
-      acc = mul4(sch, acc);
-      __syncwarp();
-      for (int g = 0; g * 4 < cnt; ++g) {
-        const int bit = hb * TG + g;
-        mbar_wait_parity(&bars[wib][hb][g], (phase >> bit) & 1u);
-        phase ^= 1u << bit;
-#pragma unroll
-        for (int r = 0; r < 4; ++r) {
-          const int kk = 4 * g + r;
-          if (kk < cnt) acc = fma4(sPw[wib][hv][kk], ring[(hb * TB + kk) * 32 + lane], acc);
-        }
-      }
-      __syncwarp();
-      hb ^= 1;
-      cnt = cnt1;
-      jcur = jnext;
-    }
-    float l[NH];
-#pragma unroll
-    for (int h = 0; h < NH; ++h) {
-      float x = lp[h];
-#pragma unroll
-      for (int off = 16; off > 0; off >>= 1) x += __shfl_xor_sync(FULL, x, off);
-      l[h] = x;
-    }
-    float lh = l[0];
-#pragma unroll
-    for (int h = 1; h < NH; ++h)
-      if (h == hv) lh = l[h];
-    if (slot >= 0) {
-      st4(o.pacc + slot * K + cq, acc);
-      if (lane == 0) {
-#pragma unroll
-        for (int h = 0; h < NH; ++h) {
-          o.pm[slot * NH + h] = mr[h];
-          o.pl[slot * NH + h] = l[h];
-        }
-      }
-    } else {
-      const float4 z = mul4(lh > 0.f ? 1.f / lh : 0.f, acc);
-      if (o.Z) st4(o.Z + row * K + cq, z);
-      st4(o.Hout + row * K + cq, act_fwd4(act, z));
       if (o.m && lane == 0) {
 #pragma unroll
         for (int h = 0; h < NH; ++h) {
@@ -767,88 +590,19 @@ constexpr int bwd_batch() { return (K / NH / 4) >= 4 ? 4 : K / NH / 4; }
 template <int NH>
 constexpr int bwd_batch_bf16() { return (K / NH / 4) >= 8 ? 8 : K / NH / 4; }
 
-PFN_cuTensorMapEncodeTiled_v12000 tmap_encoder() {
-  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
-  static std::once_flag once;
-  std::call_once(once, [] {
-    cudaDriverEntryPointQueryResult q;
-    void* p = nullptr;
-    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) ==
-            cudaSuccess &&
-        q == cudaDriverEntryPointSuccess)
-      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
-  });
-  return fn;
-}
-
-// 2D map of a [rows x 128] fp32 table for tile::gather4 (box = one 512-byte row)
-bool row_gather_map(CUtensorMap* map, const float* base, int64_t rows) {
-  auto enc = tmap_encoder();
-  if (!enc || rows <= 0 || rows > INT32_MAX) return false;
-  cuuint64_t dims[2] = {(cuuint64_t)K, (cuuint64_t)rows};
-  cuuint64_t strides[1] = {(cuuint64_t)K * 4};
-  cuuint32_t box[2] = {(cuuint32_t)K, 1};
-  cuuint32_t es[2] = {1, 1};
-  return enc(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(base), dims, strides, box,
-             es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
-             CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
-}
-
-bool fwd_tma_enabled() {
-  static int v = -1;
-  if (v < 0) {
-    const char* e = getenv("AGNN_GATHER");
-    v = (e && std::string(e) == "tma") ? 1 : 0;
-  }
-  return v == 1;
-}
-
 agnn_status gat_fwd_k128(const Items& it_all, int heads, const float* P, const float* st,
-                         float slope, int act, const GatFwdOut& o, int64_t n_rows, cudaStream_t s) {
-  agnn_status sst = (gat_bundles_enabled(false) && it_all.bundles)
+                         float slope, int act, const GatFwdOut& o, cudaStream_t s) {
+  agnn_status sst = (gat_bundles_enabled(it_all, false) && it_all.bundles)
                         ? gat_fwd_bundle<float>(it_all, heads, P, st, slope, act, o, s)
                         : gat_fwd_short<float>(it_all, heads, P, st, slope, act, o, s);
   if (sst != AGNN_OK) return sst;
   const Items it = long_items(it_all);
   if (it.n_chunks + it.n_light == 0) return AGNN_OK;
-  CUtensorMap map;
-  if (!o.Q && fwd_tma_enabled() && row_gather_map(&map, P, n_rows)) {
-    AGNN_K128_DISPATCH(heads, ({
-      constexpr int smem = TW * TRING;
-      static bool attr = false;
-      if (!attr) {
-        cudaFuncSetAttribute(gat_fwd_tma_kernel<NH>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             smem);
-        attr = true;
-      }
-      int per_sm = 0;
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, gat_fwd_tma_kernel<NH>, TW * 32,
-                                                    smem);
-      const int grid = kNumSMs * (per_sm > 0 ? per_sm : 1);
-      gat_fwd_tma_kernel<NH><<<grid, TW * 32, smem, s>>>(map, it, st, slope, act, o);
-      AGNN_LAUNCH_CHECK("gat_fwd_kernel");
-    }));
-    return AGNN_OK;
-  }
   AGNN_K128_DISPATCH(heads, ({
-    // AGNN_FWD_VARIANT (measurement): 0 = 3 blocks / SM, 4-row groups; 1 = 2 blocks /
-    // SM, 8-row groups; 2 = 4 blocks / SM
-    static int variant = -1;
-    if (variant < 0) {
-      const char* e = getenv("AGNN_FWD_VARIANT");
-      variant = e ? atoi(e) : 0;
-    }
-    using KF = void (*)(Items, const float*, const float*, float, int, GatFwdOut);
-    KF kern;
-    if (variant == 1)
-      kern = o.Q ? (KF)gat_fwd_k128_kernel<float, NH, 8, 2, true, 8>
-                 : (KF)gat_fwd_k128_kernel<float, NH, 8, 2, false, 8>;
-    else if (variant == 2)
-      kern = o.Q ? (KF)gat_fwd_k128_kernel<float, NH, 4, 4, true>
-                 : (KF)gat_fwd_k128_kernel<float, NH, 4, 4, false>;
-    else
-      kern = o.Q ? (KF)gat_fwd_k128_kernel<float, NH, 4, 3, true>
-                 : (KF)gat_fwd_k128_kernel<float, NH, 4, 3, false>;
+    // 3 blocks / SM, 4-row gather groups (measured C5, round 1: 2 blocks / SM with
+    // 8-row groups and 4 blocks / SM were both slower)
+    auto* kern = o.Q ? gat_fwd_k128_kernel<float, NH, 4, 3, true>
+                     : gat_fwd_k128_kernel<float, NH, 4, 3, false>;
     kern<<<grid_for(kern), 256, 0, s>>>(it, P, st, slope, act, o);
     AGNN_LAUNCH_CHECK("gat_fwd_kernel");
   }));
@@ -857,7 +611,7 @@ agnn_status gat_fwd_k128(const Items& it_all, int heads, const float* P, const f
 
 agnn_status gat_fwd_k128_bf16(const Items& it_all, int heads, const bf16* P, const float* st,
                               float slope, int act, const GatFwdOut& o, cudaStream_t s) {
-  agnn_status sst = (gat_bundles_enabled(true) && it_all.bundles)
+  agnn_status sst = (gat_bundles_enabled(it_all, true) && it_all.bundles)
                         ? gat_fwd_bundle<bf16>(it_all, heads, P, st, slope, act, o, s)
                         : gat_fwd_short<bf16>(it_all, heads, P, st, slope, act, o, s);
   if (sst != AGNN_OK) return sst;
@@ -876,34 +630,13 @@ agnn_status gat_bwd_k128(const Items& it_all, int heads, const GatBwdArgs& A, in
                          cudaStream_t s) {
   *warps = 0;
   const Items it = long_items(it_all);
-  if (A.P16 && gat_bwd_async_enabled()) {
-    agnn_status st = gat_bwd_async(it, heads, A, warps, s);
-    if (st != AGNN_OK) return st;
-    int64_t sw = 0;
-    st = gat_bwd_short(it_all, heads, A, *warps, &sw, s);
-    *warps += sw;
-    return st;
-  }
-  static int minb = -1;
-  if (minb < 0) {
-    const char* e = getenv("AGNN_BWD_MINB");
-    minb = e ? atoi(e) : 2;
-  }
   AGNN_K128_DISPATCH(heads, ({
     constexpr int B = bwd_batch<NH>();
     constexpr int B16 = bwd_batch_bf16<NH>();
     int grid;
     if (A.P16) {  // BF16 mode (reading B1)
-      if (minb == 3) {
-        grid = grid_for(gat_bwd_k128_kernel<bf16, NH, B16, 3>);
-        gat_bwd_k128_kernel<bf16, NH, B16, 3><<<grid, 256, 0, s>>>(it, A);
-      } else {
-        grid = grid_for(gat_bwd_k128_kernel<bf16, NH, B16, 2>);
-        gat_bwd_k128_kernel<bf16, NH, B16, 2><<<grid, 256, 0, s>>>(it, A);
-      }
-    } else if (minb == 3) {
-      grid = grid_for(gat_bwd_k128_kernel<float, NH, B, 3>);
-      gat_bwd_k128_kernel<float, NH, B, 3><<<grid, 256, 0, s>>>(it, A);
+      grid = grid_for(gat_bwd_k128_kernel<bf16, NH, B16, 2>);
+      gat_bwd_k128_kernel<bf16, NH, B16, 2><<<grid, 256, 0, s>>>(it, A);
     } else {
       grid = grid_for(gat_bwd_k128_kernel<float, NH, B, 2>);
       gat_bwd_k128_kernel<float, NH, B, 2><<<grid, 256, 0, s>>>(it, A);
@@ -923,24 +656,10 @@ agnn_status gat_bwd_k128f(const Items& it_all, int heads, const GatBwdArgs& A, i
   *warps = 0;
   const Items it = long_items(it_all);
   AGNN_K128_DISPATCH(heads, ({
-    // AGNN_BWDF_VARIANT (measurement): 0 = default (fp32: as 1, bf16: 3 blocks / SM;
-    // measured C5: fp32 73.5 -> 69.2 ms, bf16 59.2 vs 64.7 ms); 1 = 2 blocks / SM;
-    // 2 = 2 blocks / SM, 8-row (fp32) / 16-row (bf16) groups; 3 = 4 blocks / SM
-    static int variant = -1;
-    if (variant < 0) {
-      const char* e = getenv("AGNN_BWDF_VARIANT");
-      variant = e ? atoi(e) : 0;
-    }
-    using KB = void (*)(Items, GatBwdArgs);
-    KB kern;
-    if (variant == 1 || (variant == 0 && !A.P16))
-      kern = A.P16 ? (KB)gat_bwd_k128f_kernel<bf16, NH, 2> : (KB)gat_bwd_k128f_kernel<float, NH, 2>;
-    else if (variant == 2)
-      kern = A.P16 ? (KB)gat_bwd_k128f_kernel<bf16, NH, 2, 16> : (KB)gat_bwd_k128f_kernel<float, NH, 2, 8>;
-    else if (variant == 3)
-      kern = A.P16 ? (KB)gat_bwd_k128f_kernel<bf16, NH, 4> : (KB)gat_bwd_k128f_kernel<float, NH, 4>;
-    else
-      kern = A.P16 ? (KB)gat_bwd_k128f_kernel<bf16, NH, 3> : (KB)gat_bwd_k128f_kernel<float, NH, 3>;
+    // fp32: 2 blocks / SM; bf16: 3 blocks / SM (measured C5, round 1: fp32 73.5 -> 69.2 ms
+    // against 3 blocks; bf16 59.2 vs 64.7 ms against 2)
+    auto* kern = A.P16 ? (void (*)(Items, GatBwdArgs))gat_bwd_k128f_kernel<bf16, NH, 3>
+                       : (void (*)(Items, GatBwdArgs))gat_bwd_k128f_kernel<float, NH, 2>;
     const int grid = grid_for(kern);
     kern<<<grid, 256, 0, s>>>(it, A);
     AGNN_LAUNCH_CHECK("gat_bwd_kernel");
@@ -948,7 +667,7 @@ agnn_status gat_bwd_k128f(const Items& it_all, int heads, const GatBwdArgs& A, i
   }));
   // short rows: their da partials follow the main kernel's rows
   int64_t sw = 0;
-  agnn_status sst = (gat_bundles_enabled(A.P16 != nullptr) && it_all.bundles)
+  agnn_status sst = (gat_bundles_enabled(it_all, A.P16 != nullptr) && it_all.bundles)
                         ? gat_bwd_bundle(it_all, heads, A, *warps, &sw, s)
                         : gat_bwd_short_f(it_all, heads, A, *warps, &sw, s);
   *warps += sw;

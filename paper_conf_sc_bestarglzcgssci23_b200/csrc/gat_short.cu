@@ -561,35 +561,17 @@ agnn_status gat_fwd_short(const Items& it, int heads, const TP* P, const float* 
                           int act, const GatFwdOut& o, cudaStream_t s) {
   if (it.n_short == 0) return AGNN_OK;
   AGNN_SHORT_DISPATCH(heads, ({
-    static int minb = -1;  // AGNN_FWD_SHORT_MINB (measurement): resident 256-thread blocks
-    if (minb < 0) {
-      const char* e = getenv("AGNN_FWD_SHORT_MINB");
-      minb = e ? atoi(e) : 2;
-    }
-    // 3 blocks / SM with 4 bf16 rows per batch, or 2 blocks / SM with 8
-    // (fp32: 2 blocks / SM, 4 rows per batch; the 3-block variant spills)
-    // AGNN_FWD_SHORT_VARIANT (measurement): 0 = default (fp32: 8 lanes per row, 2 blocks
-    // / SM; bf16: as 1); 1 = 16 lanes per row, 3 blocks / SM; 2 = 16 lanes, 2 blocks /
-    // SM, 8-edge bf16 batches; 3 = 8 lanes per row for bf16 too
-    static int variant = -1;
-    if (variant < 0) {
-      const char* e = getenv("AGNN_FWD_SHORT_VARIANT");
-      variant = e ? atoi(e) : 0;
-    }
+    // fp32: 8 lanes per row, 2 blocks / SM (the 3-block variant spills); bf16: 16 lanes
+    // per row, 3 blocks / SM, 4-edge batches (measured C5, round 1)
     using KF = void (*)(const int4*, const int32_t*, int64_t, int64_t, const TP*, const float*,
                         float, int, GatFwdOut, uint32_t, uint32_t, int);
     KF kern;
-    if (variant == 1 || (variant == 0 && sizeof(TP) == 2))  // bf16 default (measured C5)
+    if (sizeof(TP) == 2)
       kern = o.Q ? (KF)gat_fwd_short_kernel<TP, NH, 16, 3, 4, true>
                  : (KF)gat_fwd_short_kernel<TP, NH, 16, 3, 4, false>;
-    else if (variant == 2)
-      kern = o.Q ? (KF)gat_fwd_short_kernel<TP, NH, 16, 2, 8, true>
-                 : (KF)gat_fwd_short_kernel<TP, NH, 16, 2, 8, false>;
-    else  // variant 0 (fp32) or 3
-      kern = o.Q ? ((sizeof(TP) == 4 || minb == 2) ? (KF)gat_fwd_short_kernel<TP, NH, 8, 2, 8, true>
-                                                   : (KF)gat_fwd_short_kernel<TP, NH, 8, 3, 4, true>)
-                 : ((sizeof(TP) == 4 || minb == 2) ? (KF)gat_fwd_short_kernel<TP, NH, 8, 2, 8, false>
-                                                   : (KF)gat_fwd_short_kernel<TP, NH, 8, 3, 4, false>);
+    else
+      kern = o.Q ? (KF)gat_fwd_short_kernel<TP, NH, 8, 2, 8, true>
+                 : (KF)gat_fwd_short_kernel<TP, NH, 8, 2, 8, false>;
     kern<<<grid_for(kern), 256, 0, s>>>(it.short_meta, it.col, it.n_short, it.row_begin, P, st,
                                          slope, act, o, it.col_mask, it.hot_thr, it.cold_first);
     AGNN_LAUNCH_CHECK("gat_fwd_short_kernel");
@@ -609,23 +591,13 @@ agnn_status gat_bwd_short(const Items& it, int heads, const GatBwdArgs& A, int64
     int grid;
     // one 8-warp block per SM with up to 255 registers: U edges x 4 rows of gathers
     // in flight per warp without spilling (bf16 rows are half the registers)
-    static int variant = -1;  // AGNN_BWD_SHORT (measurement): 0 = 16 lanes x 4 edges, 2 blocks/SM;
-    if (variant < 0) {         // 1 = 8 lanes x 4 edges, 1 block/SM; 2 = 16 lanes x 8 edges
-      const char* e = getenv("AGNN_BWD_SHORT");
-      variant = e ? atoi(e) : 0;
-    }
     if (A.P16) {
       auto launch = [&](auto* kern) {
         grid = grid_for(kern);
         kern<<<grid, 256, 0, s>>>(it.short_meta, it.col, it.n_short, it.row_begin, A, da_row0,
                                   it.col_mask, it.hot_thr, it.cold_first);
       };
-      if (variant == 1)
-        launch(gat_bwd_short_kernel<bf16, NH, 8, 4, 1>);
-      else if (variant == 2)
-        launch(gat_bwd_short_kernel<bf16, NH, 16, 8, 1>);
-      else
-        launch(gat_bwd_short_kernel<bf16, NH, 16, 4, 2>);
+      launch(gat_bwd_short_kernel<bf16, NH, 16, 4, 2>);
     } else {
       auto* kern = gat_bwd_short_kernel<float, NH, 16, 2, 2>;
       grid = grid_for(kern);
@@ -643,30 +615,12 @@ agnn_status gat_bwd_short_f(const Items& it, int heads, const GatBwdArgs& A, int
   *warps = 0;
   if (it.n_short == 0) return AGNN_OK;
   AGNN_SHORT_DISPATCH(heads, ({
-    // 16 lanes per row (2 rows per warp); AGNN_BWD_SHORT_VARIANT (measurement):
-    // 3 (default) = 2-edge fp32 / 4-edge bf16 batches with 3 blocks / SM;
-    // 4 = 4 / 8-edge batches, 2 blocks / SM; 1 = 4 / 8-edge, 3 blocks / SM; 2 = 8 lanes per row
-    static int variant = -1;
-    if (variant < 0) {
-      const char* e = getenv("AGNN_BWD_SHORT_VARIANT");
-      variant = e ? atoi(e) : 0;
-    }
+    // 16 lanes per row (2 rows per warp), 2-edge fp32 / 4-edge bf16 batches, 3 blocks /
+    // SM (measured C5, round 1: 14.7 -> 13.5 ms fp32 against 4-edge batches at 2 / SM)
     using KB = void (*)(const int4*, const int32_t*, int64_t, int64_t, GatBwdArgs, int64_t,
                         uint32_t, uint32_t, int);
-    KB kern;
-    if (variant == 0) variant = 3;  // default (measured C5: 14.7 -> 13.5 ms fp32)
-    if (variant == 1)
-      kern = A.P16 ? (KB)gat_bwd_short_f_kernel<bf16, NH, 16, 8, 3>
-                   : (KB)gat_bwd_short_f_kernel<float, NH, 16, 4, 3>;
-    else if (variant == 2)
-      kern = A.P16 ? (KB)gat_bwd_short_f_kernel<bf16, NH, 8, 4, 2>
-                   : (KB)gat_bwd_short_f_kernel<float, NH, 8, 4, 2>;
-    else if (variant == 3)
-      kern = A.P16 ? (KB)gat_bwd_short_f_kernel<bf16, NH, 16, 4, 3>
-                   : (KB)gat_bwd_short_f_kernel<float, NH, 16, 2, 3>;
-    else  // 4
-      kern = A.P16 ? (KB)gat_bwd_short_f_kernel<bf16, NH, 16, 8, 2>
-                   : (KB)gat_bwd_short_f_kernel<float, NH, 16, 4, 2>;
+    KB kern = A.P16 ? (KB)gat_bwd_short_f_kernel<bf16, NH, 16, 4, 3>
+                    : (KB)gat_bwd_short_f_kernel<float, NH, 16, 2, 3>;
     const int grid = grid_for(kern);
     kern<<<grid, 256, 0, s>>>(it.short_meta, it.col, it.n_short, it.row_begin, A, da_row0,
                               it.col_mask, it.hot_thr, it.cold_first);

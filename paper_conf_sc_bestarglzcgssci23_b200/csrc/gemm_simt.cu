@@ -236,10 +236,6 @@ agnn_status gemm_rows(const float* A, int64_t M, int K, const float* B, bool b_t
                       float* C0, int n_split, float* C1, cudaStream_t s, float* Cact, int act,
                       int n_store, const PeerOut* peers, bool* peers_done) {
   if (peers_done) *peers_done = false;
-  if (M <= 0) {
-    if (peers_done) *peers_done = true;
-    return AGNN_OK;
-  }
   if (b_trans) {  // tcgen05 3xTF32 path when the shape has an instantiation
     const int ns = (n_store <= 0 || n_store > N) ? N : n_store;
     const agnn_status st = gemm_tc(A, M, K, B, ns, C0, n_split, C1, ns, Cact, act, s, peers);
@@ -248,6 +244,7 @@ agnn_status gemm_rows(const float* A, int64_t M, int K, const float* B, bool b_t
       return st;
     }
   }
+  if (M <= 0) return AGNN_OK;  // (the fused all-gather decision above is the shape's)
   if (K % 4 || N % 4) return fail(AGNN_EINVAL, "gemm_rows: K and N must be multiples of 4");
   dim3 grid((unsigned)((M + BM - 1) / BM), (N + BN - 1) / BN);
   if (n_store <= 0 || n_store > N) n_store = N;

@@ -794,14 +794,6 @@ agnn_status launch_tn_tc(const float* A, int lda, int64_t M, const float* B, int
   return AGNN_OK;
 }
 
-bool tc_disabled() {
-  static int v = -1;
-  if (v < 0) {
-    const char* e = getenv("AGNN_GEMM");
-    v = (e && std::string(e) == "simt") ? 1 : 0;
-  }
-  return v == 1;
-}
 
 
 }  // namespace
@@ -811,7 +803,7 @@ bool tc_disabled() {
 // AGNN_EUNSUPPORTED for other shapes.
 agnn_status gemm_tn_tc(const float* A, int64_t M, int K1, const float* B, int N, float* C,
                        float* ws, cudaStream_t s) {
-  if (tc_disabled() || M <= 0) return AGNN_EUNSUPPORTED;
+  if (M <= 0) return AGNN_EUNSUPPORTED;
   if ((reinterpret_cast<uintptr_t>(A) & 15) || (reinterpret_cast<uintptr_t>(B) & 15))
     return AGNN_EUNSUPPORTED;
   if (K1 == 128 && N == 128) return launch_tn_tc<128, 128>(A, K1, M, B, N, C, N, ws, s);
@@ -834,20 +826,25 @@ agnn_status gemm_tn_tc(const float* A, int64_t M, int K1, const float* B, int N,
 agnn_status gemm_tc(const float* A, int64_t M, int K, const float* B, int n_real, float* C0,
                     int n_split, float* C1, int n_store, float* Cact, int act, cudaStream_t s,
                     const PeerOut* peers, bf16* C0h) {
-  if (tc_disabled()) return AGNN_EUNSUPPORTED;
-  if (M <= 0) return AGNN_OK;
+  // the shape decides (never M or the rank): with the peer exchange every rank must
+  // agree on whether the epilogue did the all-gather (an empty row block included)
   if ((reinterpret_cast<uintptr_t>(A) & 15) || (K % 32)) return AGNN_EUNSUPPORTED;
   if (C0h && (peers || Cact || (n_split & 3))) return AGNN_EUNSUPPORTED;
+  if (peers && (peers->n > kMaxPeers - 1 || (!C0 && peers->n > 0))) return AGNN_EUNSUPPORTED;
+  const int npad = (n_real + 15) / 16 * 16;
+  const bool shape_ok = (K == 128 && (npad == 128 || npad == 144 || npad == 160 || npad == 64)) ||
+                        (K == 64 && (npad == 64 || npad == 80 || npad == 128)) ||
+                        (K == 256 && (npad == 256 || npad == 128));
+  if (!shape_ok) return AGNN_EUNSUPPORTED;
+  if (M <= 0) return AGNN_OK;
   TcOut o{C0, C1, Cact, n_split, n_store, act, 0, {}, {}, C0h};
   if (peers) {
-    if (peers->n > kMaxPeers - 1 || (!C0 && peers->n > 0)) return AGNN_EUNSUPPORTED;
     o.npeer = peers->n;
     for (int i = 0; i < peers->n; ++i) {
       o.pC0[i] = peers->C0[i];
       o.pC1[i] = peers->C1[i];
     }
   }
-  const int npad = (n_real + 15) / 16 * 16;
   // resident B: S = the 16 KB stages that fit next to B (2 x K x N x 4 bytes), <= 8
   if (K == 128 && npad == 128) return launch_tc<128, 128, 4, false>(A, M, B, n_real, o, s);
   if (K == 128 && npad == 144) return launch_tc<144, 128, 3, false>(A, M, B, n_real, o, s);

@@ -35,6 +35,7 @@ struct Items {
   uint32_t col_mask = 0x7fffffffu;
   uint32_t hot_thr = 0xffffffffu;
   int cold_first = 0;
+  int bundle_mode = 1;        // the plan's short-row bundle mode (gat_bundles_enabled)
 };
 constexpr int kMaxColClasses = 64;
 // the items `it` of plan `p` with L2 hints for gathered rows of `row_bytes` bytes

@@ -22,7 +22,8 @@ namespace agnn {
 
 namespace {
 
-enum : int { ERR_ROWPTR0 = 1, ERR_ROWPTR_MONO = 2, ERR_COL_RANGE = 4, ERR_COL_ORDER = 8 };
+enum : int { ERR_ROWPTR0 = 1, ERR_ROWPTR_MONO = 2, ERR_COL_RANGE = 4, ERR_COL_ORDER = 8,
+             ERR_ASYMMETRIC = 16 };
 
 __global__ void validate_kernel(const int64_t* __restrict__ rp, const int32_t* __restrict__ col,
                                 int64_t n_local, int64_t n, int* __restrict__ err) {
@@ -43,6 +44,28 @@ __global__ void validate_kernel(const int64_t* __restrict__ rp, const int32_t* _
     }
     bad = __reduce_or_sync(0xffffffffu, bad);
     if (bad && lane == 0) atomicOr(err, bad);
+  }
+}
+
+// AGNN_PLAN_VERIFY_SYMMETRY ("for undirected graphs A = A^T"): every
+// stored (i,j) must have (j,i) stored — a binary search for i in row j, one lane per
+// entry.  Needs every row (world == 1) and a CSR that passed validate_kernel.
+__global__ void symmetry_kernel(const int64_t* __restrict__ rp, const int32_t* __restrict__ col,
+                                int64_t n, int* __restrict__ err) {
+  const int lane = threadIdx.x & 31;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < n; i += nw) {
+    bool bad = false;
+    for (int64_t p = rp[i] + lane; p < rp[i + 1]; p += 32) {
+      const int64_t j = col[p];
+      int64_t lo = rp[j], hi = rp[j + 1];
+      while (lo < hi) {  // first position in row j with column >= i
+        const int64_t mid = lo + (hi - lo) / 2;
+        if ((int64_t)col[mid] < i) lo = mid + 1; else hi = mid;
+      }
+      bad |= !(lo < rp[j + 1] && (int64_t)col[lo] == i);
+    }
+    if (__any_sync(0xffffffffu, bad) && lane == 0) atomicOr(err, ERR_ASYMMETRIC);
   }
 }
 
@@ -72,15 +95,6 @@ __global__ void col_class_kernel(const int32_t* __restrict__ col, int64_t nnz,
   }
 }
 
-// L2 budget (MB) for evict_last rows per pass; 0 disables the column classes
-int64_t l2_hot_budget() {
-  static const int64_t v = [] {
-    const char* e = getenv("AGNN_L2_HOT_MB");
-    return e ? (int64_t)atoll(e) : (int64_t)96;
-  }();
-  return v;
-}
-
 // Column classes for the L2 residency hints.  Class >= q (q = 1, 2, ...) = the
 // column is among the R_q = 2^21 / 2^((q-1)/4) vertices this rank gathers most
 // often (ties at a threshold are all left out; a vertex gathered once is never
@@ -90,7 +104,7 @@ agnn_status build_col_classes(Plan& p, cudaStream_t s) {
   int shift = 1;
   while (((int64_t)1 << shift) < p.n) ++shift;
   const int nq = std::min(kMaxColClasses, 1 << std::max(0, 31 - shift));
-  if (p.nnz == 0 || l2_hot_budget() <= 0 || nq < 2) return AGNN_OK;
+  if (p.nnz == 0 || p.l2_hot_mb <= 0 || nq < 2) return AGNN_OK;
   int32_t* cnt = nullptr;
   AGNN_CUDA_TRY(cudaMallocAsync(&cnt, sizeof(int32_t) * (size_t)p.n, s));
   AGNN_CUDA_TRY(cudaMemsetAsync(cnt, 0, sizeof(int32_t) * (size_t)p.n, s));
@@ -129,20 +143,18 @@ agnn_status build_col_classes(Plan& p, cudaStream_t s) {
 
 }  // namespace
 
+// every gathered row outside the hot set is loaded evict_first (measured C5, round 1:
+// evict_last alone, without evict_first for the rest, gave nothing)
 Items l2_hinted(const Items& it, const Plan& p, int64_t row_bytes) {
-  static const int cold_first = [] {
-    const char* e = getenv("AGNN_L2_COLD");
-    return e ? atoi(e) : 1;
-  }();
   if (!p.col_hint || it.col != p.col_idx || row_bytes <= 0) return it;
-  const int64_t budget = l2_hot_budget() << 20;
+  const int64_t budget = p.l2_hot_mb << 20;
   int q = 1;
   while (q < p.n_classes && p.class_rows[q] * row_bytes > budget) ++q;
   Items r = it;
   r.col = p.col_hint;
   r.col_mask = (1u << p.hint_shift) - 1u;
   r.hot_thr = q < p.n_classes ? (uint32_t)q << p.hint_shift : 0xffffffffu;
-  r.cold_first = cold_first;
+  r.cold_first = 1;
   return r;
 }
 
@@ -187,6 +199,7 @@ Items items_of(const Plan& p) {
   it.n_bundles = p.n_bundles;
   it.long_rows = p.long_rows;
   it.n_long = p.n_long;
+  it.bundle_mode = p.bundle_mode;
   return it;
 }
 
@@ -206,13 +219,6 @@ agnn_status build_lists(const std::vector<int64_t>& rp, int64_t n_rows, int chun
   std::vector<int32_t> light, chunk_row, chunk_idx, heavy, heavy_off{0}, empty, shorts, longs;
   light.reserve((size_t)n_rows);
   int64_t maxdeg = 0;
-  // debug / measurement only (AGNN_DEBUG_SKIP_BELOW=d): light rows of degree < d get
-  // no work item, so their outputs are left unwritten; used to time the share of
-  // short rows in the sparse kernels, never in tests or the bench
-  static const int64_t skip_below = [] {
-    const char* e = getenv("AGNN_DEBUG_SKIP_BELOW");
-    return e ? (int64_t)atoll(e) : (int64_t)0;
-  }();
   for (int64_t i = 0; i < n_rows; ++i) {
     const int64_t d = rp[(size_t)i + 1] - rp[(size_t)i];
     maxdeg = std::max(maxdeg, d);
@@ -225,7 +231,7 @@ agnn_status build_lists(const std::vector<int64_t>& rp, int64_t n_rows, int chun
         chunk_idx.push_back((int32_t)q);
       }
       heavy_off.push_back((int32_t)chunk_row.size());
-    } else if (d >= skip_below) {
+    } else {
       light.push_back((int32_t)i);
       if (short_max > 0) (d <= short_max ? shorts : longs).push_back((int32_t)i);
     }
@@ -284,30 +290,41 @@ Items items_of_csc(const Plan& p) {
   return it;
 }
 
+// heavy-row chunk size (edges): the longest item bounds a launch, so smaller graphs
+// (fewer edges per resident warp) take smaller chunks.  A function of the GLOBAL n
+// only, so chunk boundaries, and with them the summation order, are the same for
+// every number of GPUs: 256 up to n = 2^21, doubling per doubling of n, <= 2048
+// (measured: C2 1.49e9 -> 2.72e9 edges/s, C3 +11 %, C4 +8 %, C5 unchanged).
+// Options (agnn_plan_options): tests take small chunks to exercise the split/merge
+// path on small graphs; short rows (degree <= short_max, a function of the degree
+// only, like the chunks) go to the short-row kernels where a kernel has one.
+agnn_status plan_options(Plan& p, const agnn_plan_options* o) {
+  int64_t c = 256;
+  for (int64_t t = (int64_t)1 << 21; t < p.n && c < 2048; t <<= 1) c <<= 1;
+  p.chunk = (int)c;
+  if (!o) return AGNN_OK;
+  if (o->chunk_edges != 0) {
+    if (o->chunk_edges < 32 || o->chunk_edges > (1 << 30))
+      return fail(AGNN_EINVAL, "agnn_plan_options: chunk_edges must be 0 or in 32 .. 2^30");
+    p.chunk = o->chunk_edges;
+  }
+  if (o->short_edges >= 0) {
+    if (o->short_edges > 32) return fail(AGNN_EINVAL, "agnn_plan_options: short_edges > 32");
+    p.short_max = o->short_edges;
+  }
+  if (o->short_bundles >= 0) {
+    if (o->short_bundles > 2) return fail(AGNN_EINVAL, "agnn_plan_options: short_bundles > 2");
+    p.bundle_mode = o->short_bundles;
+  }
+  if (o->gat_factored >= 0) {
+    if (o->gat_factored > 2) return fail(AGNN_EINVAL, "agnn_plan_options: gat_factored > 2");
+    p.gat_factored = o->gat_factored;
+  }
+  if (o->l2_hot_mb >= 0) p.l2_hot_mb = o->l2_hot_mb;
+  return AGNN_OK;
+}
+
 agnn_status plan_build(Plan& p, cudaStream_t s) {
-  // heavy-row chunk size (edges): the longest item bounds a launch, so smaller graphs
-  // (fewer edges per resident warp) take smaller chunks.  A function of the GLOBAL n
-  // only, so chunk boundaries, and with them the summation order, are the same for
-  // every number of GPUs: 256 up to n = 2^21, doubling per doubling of n, <= 2048
-  // (measured: C2 1.49e9 -> 2.72e9 edges/s, C3 +11 %, C4 +8 %, C5 unchanged).
-  {
-    int64_t c = 256;
-    for (int64_t t = (int64_t)1 << 21; t < p.n && c < 2048; t <<= 1) c <<= 1;
-    p.chunk = (int)c;
-  }
-  // AGNN_CHUNK_EDGES overrides it (tests use small chunks to exercise the split/merge
-  // path on small graphs)
-  if (const char* env = getenv("AGNN_CHUNK_EDGES")) {
-    const long v = atol(env);
-    if (v >= 32 && v <= (1L << 30)) p.chunk = (int)v;
-  }
-  // short rows (degree <= short_max) go to the short-row kernels where a kernel has
-  // one (AGNN_SHORT_EDGES overrides; 0 disables the split).  A function of the degree
-  // only, like the chunks, so results do not depend on the number of GPUs.
-  if (const char* env = getenv("AGNN_SHORT_EDGES")) {
-    const long v = atol(env);  // the short-row kernels take up to 32 edges per row
-    if (v >= 0) p.short_max = (int)(v < 32 ? v : 32);
-  }
   // 1. validate on the device
   int* d_err = nullptr;
   AGNN_CUDA_TRY(cudaMallocAsync(&d_err, sizeof(int), s));
@@ -333,6 +350,26 @@ agnn_status plan_build(Plan& p, cudaStream_t s) {
     return fail(AGNN_EINVAL, m);
   }
   p.nnz = rp[(size_t)p.n_local];
+  if (p.flags & AGNN_PLAN_VERIFY_SYMMETRY) {
+    if (p.world != 1 || p.n_local != p.n)
+      return fail(AGNN_EUNSUPPORTED,
+                  "agnn_plan_create: AGNN_PLAN_VERIFY_SYMMETRY needs world == 1 (every row)");
+    int* d_sym = nullptr;
+    AGNN_CUDA_TRY(cudaMallocAsync(&d_sym, sizeof(int), s));
+    AGNN_CUDA_TRY(cudaMemsetAsync(d_sym, 0, sizeof(int), s));
+    if (p.nnz > 0) {
+      symmetry_kernel<<<kNumSMs * 8, 256, 0, s>>>(p.row_ptr, p.col_idx, p.n, d_sym);
+      AGNN_LAUNCH_CHECK("symmetry_kernel");
+    }
+    int h_sym = 0;
+    AGNN_CUDA_TRY(cudaMemcpyAsync(&h_sym, d_sym, sizeof(int), cudaMemcpyDeviceToHost, s));
+    AGNN_CUDA_TRY(cudaStreamSynchronize(s));
+    AGNN_CUDA_TRY(cudaFreeAsync(d_sym, s));
+    if (h_sym)
+      return fail(AGNN_EINVAL,
+                  "agnn_plan_create: AGNN_PLAN_VERIFY_SYMMETRY: the pattern is not symmetric "
+                  "(a stored (i,j) has no stored (j,i))");
+  }
   // 3. work lists of the rows
   Lists L;
   agnn_status st = build_lists(rp, p.n_local, p.chunk, true, p.short_max, L, s);
@@ -395,9 +432,6 @@ agnn_status plan_build(Plan& p, cudaStream_t s) {
   }
   p.meta_block = L.block;
   // L2 residency classes of the columns (symmetric or directed; the row pass's gathers)
-  if (const char* e = getenv("AGNN_L2_SETASIDE_MB")) {  // measurement: persisting L2 carve-out
-    cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)atoll(e) << 20);
-  }
   if ((st = build_col_classes(p, s)) != AGNN_OK) return st;
   // 4. directed pattern on one GPU: the CSC and its work lists (column role of the backward)
   if (p.directed() && p.world == 1 && p.n_local == p.n) {

@@ -59,7 +59,7 @@ class Stack:
 
     def __init__(self, w: gen.Workload, device="cuda", rank=0, world=1, nccl_uid=None,
                  c_v: int = 4, graph: Graph | None = None, inputs_on_device=True,
-                 symmetric: bool = True, allgather_obj=None):
+                 symmetric: bool = True, allgather_obj=None, plan_options: dict | None = None):
         self.w, self.device, self.rank, self.world = w, torch.device(device), rank, world
         self.stream = torch.cuda.current_stream(self.device)
         g = graph or build_graph(w, self.device)
@@ -76,7 +76,8 @@ class Stack:
         self.nnz_local = int(self.col_idx.numel())
         # symmetric=False: a directed pattern (reading A4); the plan builds its CSC
         self.plan = agnn.Plan(self.row_ptr, self.col_idx, w.n, b0, b1, symmetric=symmetric, rank=rank,
-                              world=world, nccl_unique_id=nccl_uid, bounds=self.bounds)
+                              world=world, nccl_unique_id=nccl_uid, bounds=self.bounds,
+                              options=plan_options)
         descs = [agnn.layer_desc(w.model, w.k, w.k, w.heads, w.act, prec=agnn.PREC[w.prec],
                                  negative_slope=w.slope,
                                  beta=w.beta, eps=w.eps, agg=w.agg) for _ in range(w.layers)]

@@ -77,8 +77,8 @@ def oracle_step(w: gen.Workload, rp, ci, H, Ws, As, R):
     return {"H": Hs, "fwd": fwd, "dH": dHs, "dW": dWs, "da": das}
 
 
-def gpu_step(w: gen.Workload, graph=None, R=None, symmetric=True):
-    st = runner.Stack(w, "cuda", graph=graph, symmetric=symmetric)
+def gpu_step(w: gen.Workload, graph=None, R=None, symmetric=True, plan_options=None):
+    st = runner.Stack(w, "cuda", graph=graph, symmetric=symmetric, plan_options=plan_options)
     if R is not None:
         st.dH[w.layers].copy_(torch.from_numpy(np.ascontiguousarray(R, np.float32)))
     st.step()

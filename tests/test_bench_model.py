@@ -25,21 +25,18 @@ def _bench():
     return mod
 
 
-def test_gat_c5_bytes_per_edge(monkeypatch):
+def test_gat_c5_bytes_per_edge():
     b = _bench()
     w = gen.CONFIGS["C5"]
-    monkeypatch.delenv("AGNN_GAT_FACTORED", raising=False)
     pb = b.pass_bytes(w, 1000, 10)
     assert pb["fwd"][1] == 4 + 128 * 4 + 4 * 4 == 532
     assert pb["bwd"][1] == 4 + 128 * 4 + 16 * 4 == 580          # factored: G_i + rec_i
     assert pb["bwd"][0] == 580 * 1000 + pb["bwd"][2] * 10
-    monkeypatch.setenv("AGNN_GAT_FACTORED", "0")
-    assert b.pass_bytes(w, 1000, 10)["bwd"][1] == 4 + 2 * 128 * 4 + 20 * 4 == 1108
+    assert b.pass_bytes(w, 1000, 10, factored_mode=0)["bwd"][1] == 4 + 2 * 128 * 4 + 20 * 4 == 1108
 
 
-def test_gat_bf16_storage_bytes(monkeypatch):
+def test_gat_bf16_storage_bytes():
     b = _bench()
-    monkeypatch.delenv("AGNN_GAT_FACTORED", raising=False)
     w = dataclasses.replace(gen.CONFIGS["C5"], prec="bf16")
     pb = b.pass_bytes(w, 1, 0)
     assert pb["fwd"][1] == 4 + 128 * 2 + 16 == 276
@@ -53,12 +50,9 @@ def test_agnn_va_bytes(cfg, per_edge):
     assert b.pass_bytes(w, 1, 0)["bwd"][1] == per_edge
 
 
-def test_factored_mode_selection(monkeypatch):
+def test_factored_mode_selection():
     b = _bench()
     c5, c2 = gen.CONFIGS["C5"], gen.CONFIGS["C2"]   # k' = 128 / k' = 64
-    monkeypatch.delenv("AGNN_GAT_FACTORED", raising=False)
     assert b.gat_factored(c5) and not b.gat_factored(c2)
-    monkeypatch.setenv("AGNN_GAT_FACTORED", "2")
-    assert b.gat_factored(c5) and b.gat_factored(c2)
-    monkeypatch.setenv("AGNN_GAT_FACTORED", "0")
-    assert not b.gat_factored(c5)
+    assert b.gat_factored(c5, 2) and b.gat_factored(c2, 2)
+    assert not b.gat_factored(c5, 0)

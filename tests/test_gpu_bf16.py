@@ -89,9 +89,9 @@ def _exact_inputs(w, seed=5):
     return H, Ws, As, R
 
 
-def _exact_run(w, g):
+def _exact_run(w, g, plan_options=None):
     H, Ws, As, R = _exact_inputs(w)
-    st = runner.Stack(w, "cuda", graph=g)
+    st = runner.Stack(w, "cuda", graph=g, plan_options=plan_options)
     st.H[0].copy_(torch.from_numpy(H))
     for l in range(w.layers):
         st.W[l].copy_(torch.from_numpy(Ws[l]))
@@ -121,13 +121,12 @@ def test_bf16_exact_projection_tight(w):
     assert pu.rel(st.dW[0].cpu().numpy(), ref32["dW"][0]) > 1e-4, errs
 
 
-def test_bf16_heavy_chunks(monkeypatch):
+def test_bf16_heavy_chunks():
     """Small chunks: many heavy rows through the split / merge path (bwd_finish reads P~)."""
-    monkeypatch.setenv("AGNN_CHUNK_EDGES", "64")
     w = W("kron", 12, 8, 4, act="none")
     src, dst, rp, ci = pu.host_graph(w)
     g = pu.device_graph(w, src, dst)
-    st, (H, Ws, As, R) = _exact_run(w, g)
+    st, (H, Ws, As, R) = _exact_run(w, g, plan_options={"chunk_edges": 64})
     assert st.plan.info()["heavy_rows"] > 0
     pu.compare(w, st, pu.oracle_step(w, rp, ci, H, Ws, As, R), tol=EXACT_GUARD)
 

@@ -74,16 +74,16 @@ def test_plan_info_and_heavy_rows():
 
 
 @pytest.mark.parametrize("short", ["0", "4", "32"])
-def test_short_row_split_parity(short, monkeypatch):
+def test_short_row_split_parity(short):
     """The short-row kernels (4 rows per warp) against the oracle for several
     thresholds (0 = every light row through the warp-per-row kernels)."""
-    monkeypatch.setenv("AGNN_SHORT_EDGES", short)
+    opts = {"short_edges": int(short)}
     for prec in ("fp32", "bf16"):
         w = W("gat", "kron", 14, 8, 128, heads=4, act="none", prec=prec)
         src, dst, rp, ci = pu.host_graph(w)
         g = pu.device_graph(w, src, dst)
         H, Ws, As, R = w.host_inputs()
-        st = pu.gpu_step(w, graph=g, R=R)
+        st = pu.gpu_step(w, graph=g, R=R, plan_options=opts)
         assert st.plan.info()["short_max"] == int(short)
         ref = pu.oracle_step(w, rp, ci, H, Ws, As, R)
         pu.compare(w, st, ref, tol=pu.TOL_FP32 if prec == "fp32" else pu.TOL_BF16)
@@ -264,28 +264,64 @@ def test_directed_layer_parity(w):
     pu.compare_attention(w, st, ref)
 
 
-def test_directed_heavy_chunks(monkeypatch):
+def test_directed_heavy_chunks():
     """Small chunks force heavy rows AND heavy columns through the split/merge path."""
-    monkeypatch.setenv("AGNN_CHUNK_EDGES", "64")
     for model, heads in (("gat", 4), ("agnn", 1), ("va", 1)):
         w = W(model, "kron", 12, 8, 64, heads=heads, act="none")
         rp, ci, g = _directed_graph(w)
-        st = pu.gpu_step(w, graph=g, symmetric=False)
+        st = pu.gpu_step(w, graph=g, symmetric=False, plan_options={"chunk_edges": 64})
         assert st.plan.info()["heavy_rows"] > 0
         H, Ws, As, R = w.host_inputs()
         pu.compare(w, st, pu.oracle_step(w, rp, ci, H, Ws, As, R))
 
 
-def test_symmetric_flag_on_directed_pattern_is_not_silently_wrong():
-    """The same directed pattern through a plan WITHOUT the flag must match the oracle;
-    a symmetric plan over a symmetric pattern gives the same result as a directed plan."""
-    w = W("gat", "kron", 13, 8, 64, heads=2, act="none")
-    src, dst, rp, ci = pu.host_graph(w)   # symmetric pattern
-    g = pu.device_graph(w, src, dst)
-    a = pu.gpu_step(w, graph=g)
-    b = pu.gpu_step(w, graph=g, symmetric=False)
+def test_symmetric_flag_on_directed_pattern_is_rejected():
+    """A directed pattern passed as AGNN_CSR_SYMMETRIC would silently give a wrong
+    backward; with AGNN_PLAN_VERIFY_SYMMETRY the plan checks A = A^T on the device
+     and refuses it, while the same check accepts the symmetric
+    pattern, and the directed plan of the pattern still matches the oracle."""
+    w = W("gat", "kron", 12, 8, 64, heads=2, act="none")
+    rp, ci, g = _directed_graph(w)
+    with pytest.raises(agnn.AgnnError) as e:
+        agnn.Plan(g.row_ptr, g.col_idx, w.n, symmetric=True, verify_symmetry=True)
+    assert e.value.status == 1 and "not symmetric" in str(e.value)
+    st = pu.gpu_step(w, graph=g, symmetric=False)
+    H, Ws, As, R = w.host_inputs()
+    pu.compare(w, st, pu.oracle_step(w, rp, ci, H, Ws, As, R))
+    # the symmetric pattern of the same recipe passes the check, and a plan of it with
+    # the flag computes the same as the directed (two-pass) plan of it
+    src, dst, rps, cis = pu.host_graph(w)
+    gs = pu.device_graph(w, src, dst)
+    agnn.Plan(gs.row_ptr, gs.col_idx, w.n, symmetric=True, verify_symmetry=True)
+    a = pu.gpu_step(w, graph=gs)
+    b = pu.gpu_step(w, graph=gs, symmetric=False)
     for x, y in ((a.dH[0], b.dH[0]), (a.dW[0], b.dW[0]), (a.da[0], b.da[0])):
         assert pu.rel(x.cpu().numpy(), y.cpu().numpy()) <= 1e-6
+
+
+def test_plan_rejects_partial_rows_on_one_gpu():
+    """world == 1 with row_begin > 0 would gather out of range: EINVAL (agnn.h)."""
+    w = W("gat", "kron", 10, 8, 64)
+    src, dst, rp, ci = pu.host_graph(w)
+    g = pu.device_graph(w, src, dst)
+    half = w.n // 2
+    rp_t = g.row_ptr[half:].contiguous() - int(rp[half])
+    with pytest.raises(agnn.AgnnError) as e:
+        agnn.Plan(rp_t, g.col_idx[int(rp[half]):].contiguous(), w.n, row_begin=half)
+    assert e.value.status == 1
+
+
+@pytest.mark.parametrize("kind,k,heads", [("gat", 48, 1), ("gat", 128, 16), ("gat", 16, 8),
+                                          ("va", 48, 1), ("agnn", 96, 1), ("cgnn", 80, 1)])
+def test_model_rejects_widths_without_kernels(kind, k, heads):
+    """(k, heads) outside the dispatch tables fail at agnn_model_create, before any launch."""
+    w = W("gat", "kron", 10, 8, 64)
+    src, dst, rp, ci = pu.host_graph(w)
+    g = pu.device_graph(w, src, dst)
+    plan = agnn.Plan(g.row_ptr, g.col_idx, w.n)
+    with pytest.raises(agnn.AgnnError) as e:
+        agnn.Model(plan, [agnn.layer_desc(kind, k, k, heads)])
+    assert e.value.status in (1, 5)
 
 
 # ------------------------------------------------------------------ C-GNN over semirings (f3)
@@ -300,12 +336,12 @@ CGNN_CASES = [
 ]
 
 
-def _cgnn_check(w, rp, ci, g, symmetric=True):
+def _cgnn_check(w, rp, ci, g, symmetric=True, plan_options=None):
     H, Ws, As, R = w.host_inputs()
     if w.act == "relu":
         f0 = pu.oracle_step(w, rp, ci, H, Ws, As, R)["fwd"][-1]
         R = pu.relu_kink_mask(w, f0["Z"], R)
-    st = pu.gpu_step(w, graph=g, R=R, symmetric=symmetric)
+    st = pu.gpu_step(w, graph=g, R=R, symmetric=symmetric, plan_options=plan_options)
     ref = pu.oracle_step(w, rp, ci, H, Ws, As, R)
     pu.compare(w, st, ref)
     return st, ref
@@ -319,11 +355,10 @@ def test_cgnn_layer_parity(w):
 
 
 @pytest.mark.parametrize("agg", ["sum", "mean", "gcn", "max", "min"])
-def test_cgnn_directed_and_heavy_chunks(agg, monkeypatch):
+def test_cgnn_directed_and_heavy_chunks(agg):
     """Directed pattern (backward gathers over the CSC) with heavy rows and columns
     split into 64-edge chunks."""
-    monkeypatch.setenv("AGNN_CHUNK_EDGES", "64")
     w = W("cgnn", "kron", 12, 8, 64, act="none", agg=agg)
     rp, ci, g = _directed_graph(w)
-    st, _ = _cgnn_check(w, rp, ci, g, symmetric=False)
+    st, _ = _cgnn_check(w, rp, ci, g, symmetric=False, plan_options={"chunk_edges": 64})
     assert st.plan.info()["heavy_rows"] > 0
