@@ -40,7 +40,8 @@ def lib():
     if _lib is None:
         so = _build.build_gen()
         _lib = ctypes.CDLL(so)
-        for f in ("agen_edges_host", "agen_fill_host", "agen_edges_device", "agen_fill_device"):
+        for f in ("agen_edges_host", "agen_fill_host", "agen_fill_rows_host", "agen_edges_device",
+                  "agen_fill_device"):
             getattr(_lib, f).restype = ctypes.c_int
     return _lib
 
@@ -66,6 +67,17 @@ def fill(seed: int, stream: int, shape, scale: float = 1.0, offset: int = 0) -> 
     lib().agen_fill_host(ctypes.c_uint64(seed), ctypes.c_uint64(stream), ctypes.c_uint64(offset),
                          ctypes.c_uint64(out.size), ctypes.c_float(scale),
                          out.ctypes.data_as(ctypes.c_void_p))
+    return out
+
+
+def fill_rows(seed: int, stream: int, ids, width: int, scale: float = 1.0) -> np.ndarray:
+    """Host rows `ids` of a [*, width] fill() tensor (same values, without the rest)."""
+    ids = np.ascontiguousarray(ids, dtype=np.int64)
+    out = np.empty((len(ids), width), dtype=np.float32)
+    lib().agen_fill_rows_host(ctypes.c_uint64(seed), ctypes.c_uint64(stream),
+                              ids.ctypes.data_as(ctypes.c_void_p), ctypes.c_int64(len(ids)),
+                              ctypes.c_int64(width), ctypes.c_float(scale),
+                              out.ctypes.data_as(ctypes.c_void_p))
     return out
 
 

@@ -28,6 +28,17 @@ int agen_fill_host(uint64_t seed, uint64_t stream, uint64_t offset, uint64_t cou
   return 0;
 }
 
+/* rows of a [*, width] tensor: out[r][c] = U[-1,1)(seed, stream, ids[r] * width + c) * scale
+ * (host) — the same values agen_fill_host gives at those rows of the whole tensor. */
+int agen_fill_rows_host(uint64_t seed, uint64_t stream, const int64_t* ids, int64_t nrows,
+                        int64_t width, float scale, float* out) {
+#pragma omp parallel for schedule(static)
+  for (int64_t r = 0; r < nrows; ++r)
+    for (int64_t c = 0; c < width; ++c)
+      out[r * width + c] = agen_unif_pm1(seed, stream, (uint64_t)(ids[r] * width + c)) * scale;
+  return 0;
+}
+
 }  // extern "C"
 
 __global__ void agen_edges_kernel(int kind, uint64_t seed, int scale, uint64_t n, uint64_t n_samples,

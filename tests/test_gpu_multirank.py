@@ -4,9 +4,12 @@ The gpurun pool gives one B200, and NCCL refuses two ranks on one device, but
 CUDA IPC maps memory between two processes on the same device exactly as
 between two GPUs on an NVSwitch.  So the peer transport — IPC setup, the
 row-pushing all-gather, the flag barrier, the slot all-reduce — runs here for
-real, and every output must match the single-process run: H_out and dH bitwise
-for the row-local outputs (the chunk order does not depend on the number of
-ranks), dW / da within fp32 rounding of the different partial-sum grouping.
+real.  Every rank's outputs are checked against the FP64 ORACLE (the same
+normwise 1e-5 bar and per-row bound as the single-GPU parity tests, on the
+rank's row block for H_out and dH, on the all-reduced dW / da), and in addition
+against the single-process GPU run: H_out and dH bitwise (the chunk order does
+not depend on the number of ranks — P-invariance), dW / da within fp32 rounding
+of the different partial-sum grouping, and bitwise equal on every rank.
 """
 from __future__ import annotations
 
@@ -24,10 +27,12 @@ from paper_conf_sc_bestarglzcgssci23_b200 import gen  # noqa: E402
 
 CASES = {
     "gat-k64h2": gen.Workload("mr-gat", "gat", "kron", 13, 1 << 13, 8 << 13, 64, 2, 1, act="elu"),
+    # seed 4: min |s_i + t_j| = 4.4e-6 rms, so fp32 and fp64 take the same LeakyReLU
+    # branch on every entry (reading A5'; seed 1 has an entry at 8e-7 rms)
     "gat-k128h4": gen.Workload("mr-gat128", "gat", "kron", 14, 1 << 14, 8 << 14, 128, 4, 1,
-                               act="none"),
+                               act="none", seed=4),
     "gat-k128h4-bf16": gen.Workload("mr-gat128b", "gat", "kron", 14, 1 << 14, 8 << 14, 128, 4, 1,
-                                    act="elu", prec="bf16"),
+                                    act="elu", prec="bf16", seed=4),
     "agnn-k128-L2": gen.Workload("mr-agnn", "agnn", "rmat", 13, 1 << 13, 8 << 13, 128, 1, 2,
                                  act="elu"),
     "va-k64": gen.Workload("mr-va", "va", "kron", 13, 1 << 13, 8 << 13, 64, 1, 1, act="none"),
@@ -47,9 +52,31 @@ def _free_port():
 def _outputs(st):
     L = st.w.layers
     out = {"H": st.H[L].cpu().numpy(), "dH": st.dH[0].cpu().numpy(),
+           "Hl": [x.cpu().numpy() for x in st.H[1:]], "dHl": [x.cpu().numpy() for x in st.dH],
            "dW": [x.cpu().numpy() for x in st.dW]}
     out["da"] = [x.cpu().numpy() for x in st.da if x is not None]
     return out
+
+
+def _check_oracle(w, allout):
+    """Every rank's row block of H^l, dH^l and its dW, da against the FP64 oracle."""
+    import oracle  # noqa: F401  (tests/ and oracle/ are on sys.path via conftest)
+    import parity_utils as pu
+    src, dst, rp, ci = pu.host_graph(w)
+    H, Ws, As, R = w.host_inputs()
+    ref = pu.oracle_step(w, rp, ci, H, Ws, As, R)
+    tol = pu.TOL_BF16 if w.prec == "bf16" else pu.TOL_FP32
+    for o in allout:
+        b0, b1 = o["rows"]
+        pairs = {}
+        for l in range(w.layers):
+            pairs[f"H{l + 1}"] = (o["Hl"][l], ref["H"][l + 1][b0:b1])
+            pairs[f"dW{l}"] = (o["dW"][l], ref["dW"][l])
+        for l in range(w.layers + 1):
+            pairs[f"dH{l}"] = (o["dHl"][l], ref["dH"][l][b0:b1])
+        for l, x in enumerate(o["da"]):
+            pairs[f"da{l}"] = (x, ref["da"][l])
+        pu.compare_arrays(pairs, tol, rowwise=[k for k in pairs if not k.startswith("da")])
 
 
 def _worker(rank, world, port, name):
@@ -74,6 +101,7 @@ def _worker(rank, world, port, name):
     allout = [None] * world
     dist.all_gather_object(allout, mine)
     if rank == 0:
+        _check_oracle(w, allout)
         ref = runner.Stack(w, "cuda")
         for _ in range(2):
             ref.step()

@@ -275,6 +275,35 @@ def test_directed_heavy_chunks():
         pu.compare(w, st, pu.oracle_step(w, rp, ci, H, Ws, As, R))
 
 
+@pytest.mark.parametrize("k", [64, 128])
+def test_agnn_eps_branch(k):
+    """Reading A8 on the GPU: zero rows and rows of norm < eps = 1e-12 take
+    nu_i = eps (constant), with the gradient dHhat_j / eps of the oracle
+    (pinned in test_oracle_pins.py::test_agnn_eps_branch)."""
+    w = W("agnn", "kron", 12, 8, k, layers=1, act="elu")
+    src, dst, rp, ci = pu.host_graph(w)
+    g = pu.device_graph(w, src, dst)
+    H, Ws, As, R = w.host_inputs()
+    deg = np.diff(rp)
+    zero = [int(np.argmax(deg)), 5, 77]          # the hub row among them
+    tiny = [300, 1001]
+    H = H.copy()
+    H[zero] = 0.0
+    H[tiny] *= np.float32(1e-14)
+    st = runner.Stack(w, "cuda", graph=g)
+    st.H[0].copy_(torch.from_numpy(H))
+    st.dH[1].copy_(torch.from_numpy(R))
+    st.step()
+    torch.cuda.synchronize()
+    ref = pu.oracle_step(w, rp, ci, H, Ws, As, R)
+    pu.compare(w, st, ref)
+    # the branch rows carry the 1/eps-scaled gradients; check them on their own too
+    pu.compare_arrays({"dH_eps": (st.dH[0].cpu().numpy()[zero + tiny], ref["dH"][0][zero + tiny]),
+                       "H_eps": (st.H[1].cpu().numpy()[zero + tiny], ref["H"][1][zero + tiny])},
+                      rowwise=["dH_eps", "H_eps"])
+    pu.compare_attention(w, st, ref)
+
+
 def test_symmetric_flag_on_directed_pattern_is_rejected():
     """A directed pattern passed as AGNN_CSR_SYMMETRIC would silently give a wrong
     backward; with AGNN_PLAN_VERIFY_SYMMETRY the plan checks A = A^T on the device

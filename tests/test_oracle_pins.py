@@ -100,6 +100,37 @@ def test_agnn_local_equals_global(beta, kind, symmetric):
     assert rel(b["dW"], ref["dW"]) < 1e-12
 
 
+@pytest.mark.parametrize("kind", ["none", "elu"])
+@pytest.mark.parametrize("symmetric", [True, False])
+def test_agnn_eps_branch(kind, symmetric):
+    """Reading A8: nu_i = max(|H_i|, eps), constant on the eps branch.  A zero row and a
+    row of norm ~1e-14 < eps = 1e-12 take the branch: the oracle matches autograd of
+    the dense formulation with a clamped norm (torch.clamp passes no gradient below
+    eps), and the closed forms of the branch hold: the zero row scores c_ij = 0, so its
+    attention is uniform (mean aggregation), and its input gradient is
+    exactly dHhat_j / eps (no projection term, since d(H/eps)/dH = I/eps)."""
+    rng = np.random.default_rng(21)
+    n, k, kout = 12, 6, 4
+    rp, ci = rand_graph(n, 0.35, rng, symmetric=symmetric)
+    H, W, _, R = rand_inputs(n, k, kout, 1, rng)
+    H[3] = 0.0
+    H[7] *= 1e-14
+    assert np.linalg.norm(H[7]) < 1e-12
+    f, b = oracle.layer("agnn", rp, ci, H, W, dHout=R, act=kind, beta=1.3)
+    ref = dense_ref.agnn(rp, ci, H, W, R, beta=1.3, kind=kind)
+    assert np.abs(alpha_dense(rp, ci, f["alpha"], n) - ref["Psi"]).max() < 1e-13
+    assert rel(f["Z"], ref["Z"]) < 1e-13
+    assert rel(b["dH"], ref["dH"]) < 1e-12 and rel(b["dH"][3], ref["dH"][3]) < 1e-12
+    assert rel(b["dH"][7], ref["dH"][7]) < 1e-12
+    assert rel(b["dW"], ref["dW"]) < 1e-12
+    # zero row: uniform attention over its stored entries, X_3 = mean of its neighbours
+    row = slice(rp[3], rp[4])
+    np.testing.assert_allclose(f["alpha"][row], 1.0 / (rp[4] - rp[3]), rtol=1e-14)
+    np.testing.assert_allclose(f["X"][3], H[ci[row]].mean(0), rtol=1e-12, atol=1e-15)
+    # the branch's gradient scale: |dH_j| ~ |dHhat_j| / eps >> the other rows
+    assert np.linalg.norm(b["dH"][3]) > 1e6 * np.linalg.norm(b["dH"][0])
+
+
 @pytest.mark.parametrize("kind", ["none", "relu", "elu"])
 @pytest.mark.parametrize("symmetric", [True, False])
 def test_va_local_equals_global_and_eq11_13(kind, symmetric):
