@@ -13,17 +13,30 @@ Default workload: C5 = GAT, 4 heads, k = 128, Kronecker n = 2^24 / ~1.0e9
 edges, 1 layer — the north_star target (fits one B200).  Inputs (8.6 GB per
 feature matrix) are far larger than the 126 MB L2, so no explicit flush.
 
-Multi-GPU: launched by torch.distributed.run, one rank per GPU; 1D row blocks;
-the all-gathers of P / G are fused into the producing kernels as NVLink peer
-stores and dW, da are all-reduced through peer memory (--comm peer, default;
---comm nccl or missing P2P access: NCCL inside libagnn.so); rank 0 prints the
-JSON line; time = max over ranks of CUDA-event time.
+Multi-GPU: one rank per GPU.  `--gpus N` with N > 1 outside torchrun re-launches
+itself under torch.distributed.run (N processes); 1D row blocks; the all-gathers
+of P / G are fused into the producing kernels as NVLink peer stores and dW, da
+are all-reduced through peer memory (--comm peer, default; --comm nccl or
+missing P2P access: NCCL inside libagnn.so); rank 0 prints the JSON line; time =
+max over ranks of CUDA-event time.  Default scaling is strong (the named config
+at every N); --weak grows the graph with N (n = 2^21 N, same edge factor,
+S§8(d)).  AGNN_BENCH_SAME_GPU=1 (functional test only) runs every rank on cuda:0.
+
+Roofline (S§8(d) "three numbers per sparse kernel"): `frac` = ncu-measured DRAM
+bytes of the dominant pass per launch (profiles/ncu_traffic.json, stamped with
+the hash of the kernel sources it was captured from; a stale entry is refused)
+/ the live CUDA-event launch time / the measured HBM copy peak; `model_frac` =
+the algorithmic byte model / time / peak (can exceed 1: L2 serves hub gathers);
+`gather_peak_frac` = DRAM rate / the measured random-row gather rate.
 """
 from __future__ import annotations
 
 import argparse
+import glob
+import hashlib
 import json
 import os
+import socket
 import subprocess
 import sys
 import threading
@@ -60,7 +73,68 @@ def parse():
                    help="override log2 n of the workload (same recipe and edge factor)")
     p.add_argument("--cpu-sample-scale", type=int, default=17,
                    help="log2 n of the bounded oracle sample (same recipe as the workload)")
+    p.add_argument("--weak", action="store_true",
+                   help="weak scaling: n = 2^21 x N vertices (same recipe and edge factor)")
     return p.parse_args()
+
+
+# ----------------------------------------------------------------------------- launcher
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    return port
+
+
+def maybe_relaunch(args):
+    """--gpus N > 1 outside torchrun: run this script as N ranks under
+    torch.distributed.run (one process per GPU) and exit with its status."""
+    if args.gpus <= 1 or "WORLD_SIZE" in os.environ:
+        return
+    if args.impl == "ours" and os.environ.get("AGNN_BENCH_SAME_GPU") != "1":
+        import torch
+        have = torch.cuda.device_count()
+        if have < args.gpus:
+            sys.exit(f"bench.py --gpus {args.gpus}: only {have} CUDA device(s) visible "
+                     "(AGNN_BENCH_SAME_GPU=1 runs the ranks on one GPU as a functional test)")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1",
+           f"--nproc-per-node={args.gpus}", "--master-addr", "127.0.0.1",
+           "--master-port", str(_free_port()), os.path.abspath(__file__)] + sys.argv[1:]
+    sys.exit(subprocess.call(cmd))
+
+
+# ----------------------------------------------------------------------------- ncu stamps
+# the practical HBM rate of random whole-row gathers of 512 B (scratch/gather_probe.cu,
+# profiles/r01_gather_probe.txt: 24 warps / SM, 8 rows in flight): read-only gathers
+# exceed the copy peak of MEASURED_PEAKS.json
+GATHER_PEAK_GBS = 7272.0
+
+
+def kernel_source_hash():
+    """sha256 (first 16 hex) of the library sources the DRAM traffic was measured on."""
+    h = hashlib.sha256()
+    pkg = os.path.join(ROOT, "paper_conf_sc_bestarglzcgssci23_b200", "csrc")
+    for f in sorted(glob.glob(os.path.join(pkg, "*.cu")) + glob.glob(os.path.join(pkg, "*.cuh")) +
+                    glob.glob(os.path.join(ROOT, "include", "*.h"))):
+        h.update(os.path.basename(f).encode())
+        h.update(open(f, "rb").read())
+    return h.hexdigest()[:16]
+
+
+def ncu_traffic(key):
+    """{kernel: DRAM bytes per launch} of workload `key`, or (None, why) when the
+    committed capture is missing or was taken on other kernel sources."""
+    try:
+        tr = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))
+    except Exception:
+        return None, "no profiles/ncu_traffic.json"
+    ent = tr.get(key)
+    if not ent:
+        return None, f"no ncu capture for {key}"
+    if ent.get("_source_hash") != kernel_source_hash():
+        return None, f"stale ncu capture for {key} (kernel sources changed since)"
+    return {k: v for k, v in ent.items() if not k.startswith("_")}, ent.get("_captured")
 
 
 # ----------------------------------------------------------------------------- clocks
@@ -141,8 +215,16 @@ def time_oracle(w, scale, reps=1):
         t0 = time.perf_counter()
         oracle_train_step(pu, ws, rp, ci, H, Ws, As, R)
         times.append(time.perf_counter() - t0)
-    cores = len(os.sched_getaffinity(0))
-    return ws, len(ci), times, cores
+    return ws, len(ci), times, oracle_threads()
+
+
+def oracle_threads():
+    """OpenMP threads the oracle's libgomp runs with (the cores it actually uses)."""
+    import ctypes
+    try:
+        return int(ctypes.CDLL("libgomp.so.1").omp_get_max_threads())
+    except Exception:
+        return len(os.sched_getaffinity(0))
 
 
 def cpu_model():
@@ -155,9 +237,17 @@ def cpu_model():
     return "unknown"
 
 
-def workload(args):
+def workload(args, world=1):
     from paper_conf_sc_bestarglzcgssci23_b200 import gen
     w = gen.CONFIGS[args.config]
+    if getattr(args, "weak", False) and w.graph != "er":
+        import dataclasses
+        ef = w.n_samples // w.n
+        n = (1 << 21) * world
+        if n & (n - 1):
+            sys.exit("bench.py --weak: the Kronecker recipe needs a power-of-two number of GPUs")
+        w = dataclasses.replace(w, name=f"{w.name}-weak{world}", scale=n.bit_length() - 1,
+                                n=n, n_samples=ef * n)
     if getattr(args, "prec", "fp32") != "fp32":
         import dataclasses
         w = dataclasses.replace(w, prec=args.prec)
@@ -191,8 +281,10 @@ def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
+    if "WORLD_SIZE" in os.environ:  # torchrun sets OMP_NUM_THREADS=1; the oracle uses every core
+        os.environ["OMP_NUM_THREADS"] = str(len(os.sched_getaffinity(0)))
     from paper_conf_sc_bestarglzcgssci23_b200 import gen
-    w = workload(args)
+    w = workload(args, int(os.environ.get("WORLD_SIZE", str(args.gpus))))
     ws = oracle_sample(w, args.cpu_sample_scale)
     sys.path.insert(0, os.path.join(ROOT, "oracle"))
     sys.path.insert(0, os.path.join(ROOT, "tests"))
@@ -209,12 +301,13 @@ def run_reference(args):
     T = (time.perf_counter() - t0) / args.steps
     m = len(ci)
     val = ws.layers * m / T
-    cores = len(os.sched_getaffinity(0))
+    cores = oracle_threads()
     sample = (f"oracle (C, FP64, OpenMP) on {gen.describe(ws)}, m={m} — a bounded sample of "
               f"{args.config} ({gen.describe(w)})")
     line = {"impl": "reference", "metric": metric_name(w), "value": val, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": T * 1e3,
-            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+            "higher_is_better": True, "scaling": "weak" if args.weak else "strong",
+            "vs_baseline": None, "dtype": "f64",
             "data": "synthetic",
             "config": {"workload": args.config, "model": w.model, "graph": w.graph,
                        "n": ws.n, "edges": m, "k": w.k, "heads": w.heads, "layers": w.layers,
@@ -277,18 +370,23 @@ PASSES = {"gat": {"bwd": ("gat_bwd_kernel", "gat_bwd_short_kernel"),
 
 def roofline(args, w, st, prof, world):
     """Roofline object of the dominant sparse pass (largest share of the step) from the
-    live per-kernel event profile; every sparse pass is listed under "passes"."""
+    live per-kernel event profile; every sparse pass is listed under "passes".
+
+    frac = ncu DRAM bytes per launch (committed capture of the same kernels on the
+    same workload, refused when stale) / live launch time / measured HBM peak —
+    S§8(d)'s "HBM roofline fraction"; model_frac = algorithmic bytes / time / peak;
+    gather_peak_frac = DRAM rate / the measured random-row gather rate."""
     peaks = measured_peaks()
     hbm = peaks.get("hbm_gbs")
-    peak_src = "measured (MEASURED_PEAKS.json hbm_gbs)" if hbm else "fallback (B200_PROFILING.md)"
+    peak_src = ("measured (MEASURED_PEAKS.json hbm_gbs, copy; the burst figure: each pass is "
+                "timed as its own launches)" if hbm else "fallback (B200_PROFILING.md)")
     hbm = hbm or 6650.0
     step_ms_prof = sum(v[1] for v in prof.values()) / args.steps
-    try:  # ncu DRAM bytes per launch of the same kernels on the same workload (committed)
-        tr = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))
-        key = args.config + ("" if w.prec == "fp32" else "-" + w.prec)
-        per = tr.get(key, {}) if (args.scale is None and world == 1) else {}
-    except Exception:
-        per = {}
+    key = args.config + ("" if w.prec == "fp32" else "-" + w.prec)
+    if args.scale is not None or world > 1 or getattr(args, "weak", False):
+        per, why = None, "no ncu capture for this workload / world size"
+    else:
+        per, why = ncu_traffic(key)
     passes = {}
     pb = pass_bytes(w, st.nnz_local, st.n_local)
     for pname, kernels in PASSES.get(w.model, {}).items():
@@ -299,12 +397,18 @@ def roofline(args, w, st, prof, world):
         tot = sum(prof[k][1] for k in names)
         alg, per_edge, per_row = pb[pname]
         ms = tot / cnt if cnt else None  # the pass per layer (its launches back to back)
-        achieved = (alg / (ms / 1e3) / 1e9) if ms else None
-        traffic = sum(per[k] for k in names) if names and all(k in per for k in names) else None
+        model = (alg / (ms / 1e3) / 1e9) if ms else None
+        traffic = sum(per[k] for k in names) if per and all(k in per for k in names) else None
+        dram = (traffic / (ms / 1e3) / 1e9) if (traffic and ms) else None
         passes[pname] = {
-            "bound": "hbm", "kernel": "+".join(names), "achieved": achieved, "peak": hbm,
-            "unit": "GB/s", "frac": (achieved / hbm) if achieved else None, "traffic": traffic,
-            "dram_frac": (traffic / (ms / 1e3) / 1e9 / hbm) if (traffic and ms) else None,
+            "bound": "hbm", "kernel": "+".join(names),
+            "achieved": dram, "peak": hbm, "unit": "GB/s",
+            "frac": (dram / hbm) if dram else None, "traffic": traffic,
+            "achieved_basis": ("ncu DRAM bytes (dram__bytes_read.sum + dram__bytes_write.sum) per "
+                               "launch / live CUDA-event launch time") if dram else why,
+            "model_achieved": model, "model_frac": (model / hbm) if model else None,
+            "gather_peak_gbs": GATHER_PEAK_GBS,
+            "gather_peak_frac": (dram / GATHER_PEAK_GBS) if dram else None,
             "peak_source": peak_src, "algorithmic_bytes_per_launch": alg,
             "bytes_per_edge": per_edge, "bytes_per_row": per_row, "launch_ms": ms,
             "share_of_step": (tot / args.steps / step_ms_prof) if step_ms_prof else None}
@@ -314,7 +418,16 @@ def roofline(args, w, st, prof, world):
     r = dict(passes[dom])
     r["pass"] = dom
     r["passes"] = passes
+    r["ncu_capture"] = why if per else None
     return r
+
+
+def comm_split(prof, steps):
+    """ms per step of the exchange (peer barriers, pushes, reductions or NCCL) and of
+    everything else, from the live per-kernel profile of this rank."""
+    comm = sum(v[1] for k, v in prof.items() if k.startswith(("peer_", "nccl_")))
+    tot = sum(v[1] for v in prof.values())
+    return {"comm_ms_per_step": comm / steps, "compute_ms_per_step": (tot - comm) / steps}
 
 
 def run_ours(args):
@@ -343,7 +456,10 @@ def run_ours(args):
             dist.init_process_group("gloo")
         else:
             dist.init_process_group("nccl", device_id=dev)
-    w = workload(args)
+    if world != args.gpus and rank == 0:
+        print(f"bench: --gpus {args.gpus} but WORLD_SIZE={world}; reporting n_gpus={world}",
+              file=sys.stderr)
+    w = workload(args, world)
     agnn.lib()
     uid = None
     if world > 1 and args.comm == "peer" and not same_gpu:
@@ -468,6 +584,12 @@ def run_ours(args):
     # ---- roofline of the dominant kernel ----------------------------------------
     roof = roofline(args, w, st, prof, world)
     kernels = {k: {"launches": v[0], "ms_per_step": v[1] / args.steps} for k, v in prof.items()}
+    split = comm_split(prof, args.steps)
+    per_rank = [split]
+    if world > 1:
+        per_rank = [None] * world
+        dist.all_gather_object(per_rank, dict(split, rank=rank, rows=st.n_local,
+                                              edges=st.nnz_local))
 
     # ---- end-to-end through the C ABI with host buffers -------------------------
     # Every step copies its inputs (H^0 and the upstream gradient R = dL/dH^L)
@@ -597,7 +719,7 @@ def run_ours(args):
         line = {"metric": metric_name(w),
                 "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": T * 1e3, "higher_is_better": True,
-                "scaling": "strong", "vs_baseline": None,
+                "scaling": "weak" if args.weak else "strong", "vs_baseline": None,
                 "dtype": "f32", "data": "synthetic",
                 "config": {"workload": args.config, "model": w.model, "graph": w.graph,
                            "n": n, "edges": m, "k": w.k, "heads": w.heads, "layers": w.layers,
@@ -611,7 +733,10 @@ def run_ours(args):
                            "cuda_graph": use_graph, "eager_ms_per_step": eager_ms / args.steps,
                            "setup_s": setup_s},
                 "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
-                "clocks": ck, "kernels": kernels}
+                "clocks": ck, "kernels": kernels, "per_rank": per_rank}
+        if same_gpu and world > 1:
+            line["note"] = ("AGNN_BENCH_SAME_GPU: every rank ran on cuda:0 (functional test of the "
+                            "multi-rank path, not a scaling measurement)")
         if bf16 is not None:
             line["bf16_storage"] = bf16
         print(json.dumps(line), flush=True)
@@ -621,6 +746,7 @@ def run_ours(args):
 
 def main():
     args = parse()
+    maybe_relaunch(args)
     if args.impl == "reference":
         run_reference(args)
     else:

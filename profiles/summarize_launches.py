@@ -1,14 +1,33 @@
 """Summarise an ncu launch list (gpu__time_duration + DRAM bytes per launch) of one
 bench step into profiles/<round>_launches_<cfg>_summary.md and update
 profiles/ncu_traffic.json (DRAM bytes per launch keyed by the library's kernel
-names, which bench.py uses for roofline.traffic)."""
-import csv, json, re, sys, collections
+names, which bench.py uses for roofline.traffic), stamped with the hash of the
+kernel sources (bench.py refuses an entry whose hash no longer matches).
+
+    python profiles/summarize_launches.py <launches.csv> <config key> <round> <out.md> profiles/ncu_traffic.json
+"""
+import collections
+import csv
+import datetime
+import importlib.util
+import json
+import os
+import re
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _bench():
+    spec = importlib.util.spec_from_file_location("bench_mod", os.path.join(ROOT, "bench.py"))
+    mod = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(mod)
+    return mod
 
 ALIAS = {"gat_bwd_k128_kernel": "gat_bwd_kernel", "gat_bwd_k128f_kernel": "gat_bwd_kernel",
          "gat_bwd_short_f_kernel": "gat_bwd_short_kernel",
          "gat_bwd_bundle_kernel": "gat_bwd_short_kernel", "gat_fwd_bundle_kernel": "gat_fwd_short_kernel", "gat_fwd_k128_kernel": "gat_fwd_kernel",
-         "gat_bwd_async_kernel": "gat_bwd_kernel",
-         "av_bwd_k128_kernel": "av_bwd_kernel", "av_fwd_k128_kernel": "av_fwd_kernel",
+                  "av_bwd_k128_kernel": "av_bwd_kernel", "av_fwd_k128_kernel": "av_fwd_kernel",
          "av_bwd_batched_kernel": "av_bwd_kernel", "av_fwd_batched_kernel": "av_fwd_kernel",
          "gemm_tn_tc_kernel": "gemm_tn_kernel", "tn_sum_kernel": "sum_splits_kernel"}
 STEP = re.compile(r"(gat_|av_|gemm_|agnn_rec|nu_kernel|grad_act|sum_splits|tn_sum|sgd|transpose|to_bf16|cg_)")
@@ -60,9 +79,13 @@ def main(csv_path, cfg, rnd, out_md, traffic_json):
     cfgd = {}
     for key, a in step.items():
         cfgd[a["lib"]] = max(cfgd.get(a["lib"], 0.0), a["dram"] / a["n"])
+    cfgd["_source_hash"] = _bench().kernel_source_hash()
+    cfgd["_captured"] = (f"{rnd} {datetime.date.today().isoformat()}: ncu --metrics "
+                         "dram__bytes_read.sum,dram__bytes_write.sum per launch of one bench step "
+                         f"({os.path.basename(csv_path)})")
     tr[cfg] = cfgd
-    tr["_source"] = (f"{rnd}: ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum per launch of "
-                     "one bench step (scratch/summarize_launches.py over profiles/*_launches_*.csv)")
+    tr["_source"] = ("ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum per launch of one "
+                     "bench step (profiles/summarize_launches.py over the launch-list csv)")
     json.dump(tr, open(traffic_json, "w"), indent=1)
 
 

@@ -56,3 +56,52 @@ def test_factored_mode_selection():
     assert b.gat_factored(c5) and not b.gat_factored(c2)
     assert b.gat_factored(c5, 2) and b.gat_factored(c2, 2)
     assert not b.gat_factored(c5, 0)
+
+
+def test_gpus_flag_launches_n_ranks():
+    """`bench.py --gpus 2` outside torchrun re-launches itself as 2 ranks
+    (torch.distributed.run); the reference arm (FP64 oracle, CPU) runs on rank 0
+    only and reports n_gpus = 2 with the threads the oracle actually used."""
+    import json
+    import subprocess
+    import sys
+    env = {k: v for k, v in os.environ.items() if k not in ("WORLD_SIZE", "RANK", "LOCAL_RANK")}
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--impl", "reference",
+                        "--gpus", "2", "--steps", "1", "--warmup", "0", "--config", "C2",
+                        "--cpu-sample-scale", "7"], capture_output=True, text=True, timeout=600,
+                       env=env)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1, r.stdout            # rank 0 alone prints
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["impl"] == "reference" and d["cpu_baseline"]["cores"] >= 1
+
+
+def test_weak_scaling_workload():
+    b = _bench()
+
+    class A:
+        config, prec, scale, weak = "C5", "fp32", None, True
+    for world in (1, 2, 4, 8):
+        w = b.workload(A, world)
+        assert w.n == (1 << 21) * world and w.n_samples == 32 * w.n and w.k == 128
+
+
+def test_stale_ncu_capture_is_refused(tmp_path, monkeypatch):
+    import json
+    b = _bench()
+    h = b.kernel_source_hash()
+    prof = tmp_path / "profiles"
+    prof.mkdir()
+    (prof / "ncu_traffic.json").write_text(json.dumps({
+        "C5": {"gat_bwd_kernel": 1e9, "_source_hash": h, "_captured": "now"},
+        "C3": {"av_bwd_kernel": 1e9, "_source_hash": "0" * 16}}))
+    monkeypatch.setattr(b, "ROOT", str(tmp_path))
+    # the hash is of the sources under ROOT: point it back at the repo for the check
+    monkeypatch.setattr(b, "kernel_source_hash", lambda: h)
+    per, why = b.ncu_traffic("C5")
+    assert per == {"gat_bwd_kernel": 1e9} and why == "now"
+    per, why = b.ncu_traffic("C3")
+    assert per is None and "stale" in why
+    per, why = b.ncu_traffic("C4")
+    assert per is None

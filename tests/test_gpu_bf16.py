@@ -67,8 +67,8 @@ def _run(w):
 def test_bf16_layer_parity(w):
     st, (rp, ci, H, Ws, As, R) = _run(w)
     ref = pu.oracle_step(w, rp, ci, H, Ws, As, R)
-    errs = pu.compare(w, st, ref, tol=pu.TOL_BF16)
-    fwd = {k: v for k, v in errs.items() if k.startswith("H")}
+    errs = pu.compare(w, st, ref, tol=pu.TOL_BF16, row_tol=1e-2)
+    fwd = {k: v for k, v in errs.items() if k.startswith("H") and not k.endswith(":row")}
     assert max(fwd.values()) <= FWD_GUARD, errs
     # alpha depends only on the fp32 scores and stats: the fp32 bar still holds
     pu.compare_attention(w, st, ref)
@@ -115,7 +115,7 @@ def test_bf16_exact_projection_tight(w):
     P = H.astype(np.float64) @ Ws[0].astype(np.float64)
     assert np.abs(P).max() < 256 and np.all(P * 8 == np.round(P * 8))  # bf16-exact
     ref = pu.oracle_step(w, rp, ci, H, Ws, As, R)
-    errs = pu.compare(w, st, ref, tol=EXACT_GUARD)
+    errs = pu.compare(w, st, ref, tol=EXACT_GUARD, all_rows=True, row_tol=1e-3)
     # G~ really is rounded: the fp32 oracle on the same inputs is visibly off
     ref32 = pu.oracle_step(dataclasses.replace(w, prec="fp32"), rp, ci, H, Ws, As, R)
     assert pu.rel(st.dW[0].cpu().numpy(), ref32["dW"][0]) > 1e-4, errs
@@ -128,7 +128,8 @@ def test_bf16_heavy_chunks():
     g = pu.device_graph(w, src, dst)
     st, (H, Ws, As, R) = _exact_run(w, g, plan_options={"chunk_edges": 64})
     assert st.plan.info()["heavy_rows"] > 0
-    pu.compare(w, st, pu.oracle_step(w, rp, ci, H, Ws, As, R), tol=EXACT_GUARD)
+    pu.compare(w, st, pu.oracle_step(w, rp, ci, H, Ws, As, R), tol=EXACT_GUARD, all_rows=True,
+               row_tol=1e-3)
 
 
 def test_bf16_inference_and_determinism():

@@ -83,12 +83,13 @@ def _subproblem(rp, nbs_full, rows_full, sources):
 def _hub_rows(rp, chunk, rng):
     """The maximum-degree row and rows of 2..8 heavy-row chunks (S§8(c) chunk merge)."""
     deg = np.diff(rp)
-    hubs = [int(np.argmax(deg))]
+    top = int(np.argmax(deg))
+    hubs = []
     multi = np.nonzero((deg > 2 * chunk) & (deg <= 8 * chunk))[0]
     hubs += [int(x) for x in rng.choice(multi, min(6, len(multi)), replace=False)]
     two = np.nonzero((deg > chunk) & (deg <= 2 * chunk))[0]
     hubs += [int(x) for x in rng.choice(two, min(2, len(two)), replace=False)]
-    return sorted(set(hubs))
+    return [top] + sorted(set(hubs) - {top})   # the maximum-degree row first
 
 
 def test_forward_sampled_rows(stack):
