@@ -27,6 +27,7 @@ def rel(x, y):
 # wrong row (a dropped term, a wrong chunk merge) is off by O(1).  DESIGN.md §3.
 ROW_TOL = {"fwd": 1e-4, "bwd": 1e-3}
 ROW_FLOOR = 1e-2    # rows far below the typical row norm are compared absolutely
+BF16_ROW_TOL = 1e-2  # BF16 storage (random inputs): forward rows, measured <= 1.6e-3
 
 
 def row_err(x, y):
@@ -165,6 +166,8 @@ def compare(w, st, ref, tol=TOL_FP32, rows=None, row_tol=None, all_rows=False):
         if w.model == "gat":
             pairs[f"da{l}"] = (st.da[l].cpu().numpy(), ref["da"][l])
     keys = [k for k in pairs if not k.startswith("da")] if all_rows else rowwise_keys(w, pairs)
+    if row_tol is None and w.prec == "bf16":
+        row_tol = BF16_ROW_TOL
     return compare_arrays(pairs, tol, rowwise=keys, row_tol=row_tol)
 
 

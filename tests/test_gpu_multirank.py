@@ -77,7 +77,7 @@ def _check_oracle(w, allout):
         for l, x in enumerate(o["da"]):
             pairs[f"da{l}"] = (x, ref["da"][l])
         pu.compare_arrays(pairs, tol, rowwise=pu.rowwise_keys(w, pairs),
-                          row_tol=1e-2 if w.prec == "bf16" else None)
+                          row_tol=pu.BF16_ROW_TOL if w.prec == "bf16" else None)
 
 
 def _worker(rank, world, port, name):
