@@ -66,18 +66,23 @@ def agnn_deps():
         sorted(glob.glob(os.path.join(INCLUDE, "*.h")))
 
 
-def build_agnn(force: bool = False, verbose_ptxas: bool = False) -> str:
-    """Compile every csrc/*.cu to an object (in parallel) and link libagnn.so."""
-    if not (force or _stale(AGNN_SO, agnn_deps())):
-        return AGNN_SO
+def build_agnn(force: bool = False, verbose_ptxas: bool = False, out: str | None = None,
+               defines=()) -> str:
+    """Compile every csrc/*.cu to an object (in parallel) and link libagnn.so.
+    out / defines: an extra build (e.g. -D experiment switches) at another path."""
+    so = out or AGNN_SO
+    if not (force or _stale(so, agnn_deps())):
+        return so
     nccl_inc, nccl_lib = _nccl_dirs()
-    objdir = os.path.join(ROOT, "build", "agnn")
+    objdir = os.path.join(ROOT, "build", "agnn" if not out else
+                          "agnn_" + os.path.basename(out).replace(".so", ""))
     os.makedirs(objdir, exist_ok=True)
     headers = [d for d in agnn_deps() if not d.endswith(".cu")]
     flags = [*ARCH, "-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC",
              "--expt-relaxed-constexpr", "-I", INCLUDE, "-I", CSRC, "-I", nccl_inc]
     if verbose_ptxas:
         flags.append("-Xptxas=-v")
+    flags += ["-D" + d for d in defines]
     jobs = []
     for src in agnn_sources():
         obj = os.path.join(objdir, os.path.basename(src)[:-3] + ".o")
@@ -87,9 +92,9 @@ def build_agnn(force: bool = False, verbose_ptxas: bool = False) -> str:
     with ThreadPoolExecutor(max_workers=max(1, min(8, os.cpu_count() or 1))) as ex:
         list(ex.map(_run, jobs))
     objs = [os.path.join(objdir, os.path.basename(s)[:-3] + ".o") for s in agnn_sources()]
-    _run([NVCC, *ARCH, "-shared", "-o", AGNN_SO, *objs, "-L", nccl_lib, "-l:libnccl.so.2",
+    _run([NVCC, *ARCH, "-shared", "-o", so, *objs, "-L", nccl_lib, "-l:libnccl.so.2",
           "-Xlinker", "-rpath," + nccl_lib])
-    return AGNN_SO
+    return so
 
 
 def build_all(force: bool = False):

@@ -81,7 +81,8 @@ def lib(build: bool = True):
     """Load libagnn.so (building it in-tree if stale).  Raises if unavailable."""
     global _lib
     if _lib is None:
-        so = _build.build_agnn() if build else _build.AGNN_SO
+        # AGNN_LIB: an explicit libagnn.so (e.g. a build of another revision for A/B timing)
+        so = os.environ.get("AGNN_LIB") or (_build.build_agnn() if build else _build.AGNN_SO)
         if not os.path.exists(so):
             raise RuntimeError(f"libagnn.so not found at {so}; run __graft_entry__.build()")
         L = ctypes.CDLL(so)

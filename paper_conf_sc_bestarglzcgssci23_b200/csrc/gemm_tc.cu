@@ -66,7 +66,10 @@ __device__ __forceinline__ void tma_prefetch_2d(const CUtensorMap* map, int c0, 
                "r"(c0), "r"(c1)
                : "memory");
 }
-constexpr int TC_PF = 6;  // chunks prefetched ahead into L2
+#ifndef AGNN_EXP_PF
+#define AGNN_EXP_PF 6
+#endif
+constexpr int TC_PF = AGNN_EXP_PF;  // chunks prefetched ahead into L2
 
 __device__ __forceinline__ void fence_proxy_async() {
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
@@ -114,6 +117,27 @@ __device__ __forceinline__ void mma_commit(uint64_t* bar) {
   asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
                    s_addr(bar))
                : "memory");
+}
+// 16 columns into r[0..15] without waiting (several loads in flight, one wait)
+__device__ __forceinline__ void tmem_ld16_issue(uint32_t taddr, uint32_t* r) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,"
+      "%15}, [%16];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
+        "=r"(r[7]), "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]),
+        "=r"(r[14]), "=r"(r[15])
+      : "r"(taddr));
+}
+__device__ __forceinline__ void tmem_ld_wait() {
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+// after tmem_ld_wait: ties 16 loaded registers to a point after the wait, so no use of
+// them can be scheduled before it (volatile asm statements keep their order)
+__device__ __forceinline__ void tmem_reg_fence16(uint32_t* r) {
+  asm volatile(""
+               : "+r"(r[0]), "+r"(r[1]), "+r"(r[2]), "+r"(r[3]), "+r"(r[4]), "+r"(r[5]),
+                 "+r"(r[6]), "+r"(r[7]), "+r"(r[8]), "+r"(r[9]), "+r"(r[10]), "+r"(r[11]),
+                 "+r"(r[12]), "+r"(r[13]), "+r"(r[14]), "+r"(r[15]));
 }
 __device__ __forceinline__ void tmem_ld16(uint32_t taddr, float (&v)[16]) {
   uint32_t r[16];
@@ -295,7 +319,8 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
   // LOT (resident B): the A lo part goes to TMEM (2 slots of 32 columns) instead of
   // shared memory, so a stage is 16 KB and the ring holds S - 1 chunks in flight
   constexpr bool LOT = !SB;
-  constexpr int LO_COLS = LOT ? 64 : 0;
+  constexpr int LO_SLOTS = 2;  // 32-column TMEM slots of A lo (chunk g uses slot g % 2)
+  constexpr int LO_COLS = LOT ? 32 * LO_SLOTS : 0;
   constexpr int NG0 = N <= 128 ? 4 : N <= 160 ? 3 : 2;
   constexpr int NGT = (NG0 * N + LO_COLS <= 512) ? NG0 : (NG0 - 1) * N + LO_COLS <= 512 ? NG0 - 1 : 2;
   constexpr int NG = KCH < NGT ? KCH : NGT;
@@ -307,13 +332,14 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
   constexpr uint32_t IDESC = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(N >> 3) << 17) |
                              ((uint32_t)(TC_BM >> 4) << 24);
   extern __shared__ __align__(1024) uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
-                                             ~uintptr_t(1023));
+  // 1024-byte aligned by an offset from the __shared__ array, so every access stays
+  // in the shared address space (LDS/STS, not generic loads and stores)
+  uint8_t* smem = smem_raw + ((1024u - (s_addr(smem_raw) & 1023u)) & 1023u);
   uint8_t* Bh = smem;                  // resident B (SB = false)
   uint8_t* Bl = smem + BRES;
   uint8_t* ring = smem + 2 * BRES;     // S stages
   float* stg = reinterpret_cast<float*>(ring + S * STAGE);  // epilogue transpose, 4 x 32 x 36
-  __shared__ uint64_t tma_bar[S], mma_bar[S], acc_full, acc_empty;
+  __shared__ uint64_t tma_bar[S], mma_bar[S], acc_full, acc_empty[NG];
   __shared__ uint32_t tmem_base_s;
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const bool math = warp < 4;
@@ -332,7 +358,8 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       mbar_init(&mma_bar[i], 1);
     }
     mbar_init(&acc_full, 1);
-    mbar_init(&acc_empty, 128);
+#pragma unroll
+    for (int i = 0; i < NG; ++i) mbar_init(&acc_empty[i], 128);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(&tmA) : "memory");
     if (SB) asm volatile("prefetch.tensormap [%0];" ::"l"(&tmB) : "memory");
@@ -378,28 +405,18 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       const uint32_t par = (uint32_t)((g / S) & 1);
       const int kc = (int)(g % KCH);
       const int64_t tl = g / KCH;  // this CTA's tile ordinal
-      if (tid == 0) {
-        if (g + S - 1 + TC_PF < nchunks) {
-          const int64_t gp = g + S - 1 + TC_PF;
-          tma_prefetch_2d(&tmA, (int)(gp % KCH) * TC_KC,
-                          (int)((first + (gp / KCH) * gridDim.x) * TC_BM));
-        }
-        if (g + S - 1 < nchunks) {
-          // the stage of chunk g+S-1 held chunk g-1: its MMAs must be done
-          if (g >= 1) mbar_wait(&mma_bar[(g - 1) % S], (uint32_t)(((g - 1) / S) & 1));
-          issue(g + S - 1);
-        }
-      }
       mbar_wait(&tma_bar[st], par);
       uint8_t* Ahi = ring + st * STAGE;
       uint8_t* Alo = Ahi + A_BYTES;  // SB only
-      const uint32_t lo_slot = LO_COL + (uint32_t)((g & 1) * 32);
+      const uint32_t lo_slot = LO_COL + (uint32_t)((g % LO_SLOTS) * 32);
       if (LOT) {
         // thread r splits row r of the tile: hi in place (swizzled 128-byte row),
-        // lo into TMEM lane r.  The slot was last read by chunk g-2's MMAs.
-        if (g >= 2) mbar_wait(&mma_bar[(g - 2) % S], (uint32_t)(((g - 2) / S) & 1));
+        // lo into TMEM lane r.  The slot was last read by chunk g-LO_SLOTS's MMAs.
+        if (g >= LO_SLOTS)
+          mbar_wait(&mma_bar[(g - LO_SLOTS) % S], (uint32_t)(((g - LO_SLOTS) / S) & 1));
         uint8_t* rowp = Ahi + tid * 128;
         float lo[32];
+#ifndef AGNN_EXP_NOSPLIT
 #pragma unroll
         for (int c = 0; c < 8; ++c) {
           float4* q = reinterpret_cast<float4*>(rowp + ((c ^ (tid & 7)) << 4));
@@ -413,6 +430,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
         }
         tc_fence_after();
         tmem_st32(tmem + ((uint32_t)(warp * 32) << 16) + lo_slot, lo);
+#endif
       } else {
         constexpr int SPLIT16 = (A_BYTES + (SB ? BC_BYTES : 0)) / 16;
 #pragma unroll 4
@@ -430,26 +448,42 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       tc_fence_before();
       math_barrier();
       if (tid == 0) {
-        // the first MMA of a tile overwrites the accumulators: the epilogue must have
-        // drained the previous tile
-        if (kc == 0 && tl >= 1) mbar_wait(&acc_empty, (uint32_t)((tl - 1) & 1));
+        const int grp = kc % NG;
+        // the first MMA into an accumulator group of a tile overwrites it: the epilogue
+        // must have drained that group of the previous tile (groups are released one by
+        // one, so the drain overlaps this tile's first chunks)
+        if (kc < NG && tl >= 1) mbar_wait(&acc_empty[grp], (uint32_t)((tl - 1) & 1));
         tc_fence_after();
         const uint32_t ah = s_addr(Ahi), al = s_addr(Alo);
         const uint32_t bh = SB ? s_addr(Ahi + 2 * A_BYTES) : s_addr(Bh + kc * BC_BYTES);
         const uint32_t bl = SB ? bh + BC_BYTES : s_addr(Bl + kc * BC_BYTES);
-        const int grp = kc % NG;
         const uint32_t tacc = tmem + (uint32_t)(grp * N);
 #pragma unroll
         for (int ks = 0; ks < TC_KC / 8; ++ks) {  // K = 8 tf32 (32 bytes) per MMA
           const uint32_t o = ks * 32;
           const uint32_t acc0 = (kc >= NG || ks > 0) ? 1u : 0u;  // first MMA of the group
           mma_tf32(tacc, sw128_desc(ah + o), sw128_desc(bh + o), IDESC, acc0);
+#ifdef AGNN_EXP_NOSPLIT
+          if (LOT) continue;
+#endif
           mma_tf32(tacc, sw128_desc(ah + o), sw128_desc(bl + o), IDESC, 1u);
           if (LOT) mma_tf32_ta(tacc, tmem + lo_slot + (uint32_t)(ks * 8), sw128_desc(bh + o), IDESC, 1u);
           else mma_tf32(tacc, sw128_desc(al + o), sw128_desc(bh + o), IDESC, 1u);
         }
         mma_commit(&mma_bar[st]);
         if (kc == KCH - 1) mma_commit(&acc_full);
+        // refill the stage of chunk g-1 with chunk g+S-1 once chunk g-1's MMAs are done:
+        // waiting here (after chunk g's MMAs are queued behind them) keeps the tensor
+        // pipe busy while the math warps split chunk g+1
+        if (g + S - 1 + TC_PF < nchunks) {
+          const int64_t gp = g + S - 1 + TC_PF;
+          tma_prefetch_2d(&tmA, (int)(gp % KCH) * TC_KC,
+                          (int)((first + (gp / KCH) * gridDim.x) * TC_BM));
+        }
+        if (g + S - 1 < nchunks) {
+          if (g >= 1) mbar_wait(&mma_bar[(g - 1) % S], (uint32_t)(((g - 1) / S) & 1));
+          issue(g + S - 1);
+        }
       }
     }
   } else {
@@ -461,30 +495,34 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       const int64_t t = first + tl * gridDim.x;
       const int64_t row0 = t * TC_BM + ew * 32;
       const int64_t row = row0 + lane;
-      // wide tiles drain in two halves (registers); TMEM is released after the last
+      // wide tiles drain in two halves (registers); the groups are released after the
+      // last half reads them
       constexpr int NP = N > 160 ? N / 2 : N;
 #pragma unroll 1
       for (int h0 = 0; h0 < N; h0 += NP) {
         float v[NP];
+        const bool last_half = h0 + NP >= N;
+        // group-major: all of group 0 (one wait), then each further group added with
+        // round-to-nearest FADDs; a group is released as soon as it has been read
 #pragma unroll
-        for (int c0 = 0; c0 < NP; c0 += 16) {
-          float a16[16];
-          tmem_ld16(tbase + h0 + c0, a16);
+        for (int gi = 0; gi < NG; ++gi) {
+          uint32_t r[NP];
 #pragma unroll
-          for (int gi = 1; gi < NG; ++gi) {
-            float w2[16];
-            tmem_ld16(tbase + (uint32_t)(gi * N) + h0 + c0, w2);
+          for (int c0 = 0; c0 < NP; c0 += 16) tmem_ld16_issue(tbase + (uint32_t)(gi * N) + h0 + c0, r + c0);
+          tmem_ld_wait();
 #pragma unroll
-            for (int x = 0; x < 16; ++x) a16[x] += w2[x];
+          for (int c0 = 0; c0 < NP; c0 += 16) tmem_reg_fence16(r + c0);
+          if (last_half) {
+            tc_fence_before();
+            mbar_arrive(&acc_empty[gi]);
           }
 #pragma unroll
-          for (int x = 0; x < 16; ++x) v[c0 + x] = a16[x];
-        }
-        if (h0 + NP >= N) {
-          tc_fence_before();
-          mbar_arrive(&acc_empty);
+          for (int x = 0; x < NP; ++x) v[x] = gi == 0 ? __uint_as_float(r[x]) : v[x] + __uint_as_float(r[x]);
         }
         const bool coal = (out.n_split & 3) == 0;
+#ifdef AGNN_EXP_NOSTORE
+        if (v[0] != 12345.f) continue;
+#endif
 #pragma unroll
         for (int c0 = 0; c0 < NP; c0 += 32) {
           if (c0 + 32 <= NP && coal && h0 + c0 + 32 <= out.n_split) {
@@ -549,8 +587,7 @@ gemm_tn_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
                              ((uint32_t)(N >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
   constexpr uint32_t TMEM_COLS = N <= 32 ? 32 : N <= 64 ? 64 : N <= 128 ? 128 : 256;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
-                                             ~uintptr_t(1023));
+  uint8_t* smem = smem_raw + ((1024u - (s_addr(smem_raw) & 1023u)) & 1023u);
   __shared__ uint64_t tma_bar[2], mma_bar[2];
   __shared__ uint32_t tmem_base_s;
   const int tid = threadIdx.x, warp = tid >> 5;
@@ -615,6 +652,7 @@ gemm_tn_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
     // CTA's slab: zero them before the split
     const int64_t rem = r_end - (r_beg + g * TN_ROWS);
     const int valid_rows = rem < TN_ROWS ? (int)rem : TN_ROWS;
+#pragma unroll 4
     for (int i = tid; i < (A_BYTES + B_BYTES) / 16; i += TC_THREADS) {
       const bool isA = i < A_BYTES / 16;
       const int li = isA ? i : i - A_BYTES / 16;

@@ -47,7 +47,10 @@ def test_gemm_against_fp64(M, K, N):
     assert np.linalg.norm(c - ref) / np.linalg.norm(ref) < (5e-7 if K <= 128 else 1.5e-6)
 
 
+# 3000017 rows: 367 slabs of 8192 rows, several per CTA (the chunk stream crosses
+# slab boundaries inside the kernel's ring and accumulator groups)
 @pytest.mark.parametrize("M,K1,N", [(1000, 128, 128), (65536, 128, 128), (300001, 128, 128),
+                                    (3000017, 128, 128), (2500000, 128, 64),
                                     (77, 128, 64), (20000, 64, 64), (12345, 128, 64),
                                     (100003, 256, 256), (3000, 256, 128)])
 def test_gemm_tn_against_fp64(M, K1, N):
