@@ -198,11 +198,15 @@ agnn_status agnn_plan_create_ex(const agnn_csr* csr, const agnn_dist* dist,
                                 const agnn_plan_options* options, cudaStream_t stream,
                                 agnn_plan_t* out);
 agnn_status agnn_plan_destroy(agnn_plan_t plan);
-/* host-side statistics: [0]=n_local [1]=nnz_local [2]=light rows [3]=heavy rows
- * [4]=heavy chunks [5]=chunk size [6]=max degree [7]=n (global) [8]=short rows
- * (light rows of degree <= [9], taken by the short-row kernels where a kernel
- * has one) [9]=short_max (agnn_plan_options.short_edges; 0: no split) */
-agnn_status agnn_plan_info(agnn_plan_t plan, int64_t* info10);
+/* host-side statistics (info: 12 int64, host): [0]=n_local [1]=nnz_local
+ * [2]=light rows [3]=heavy rows [4]=heavy chunks [5]=chunk size [6]=max degree
+ * [7]=n (global) [8]=short rows (light rows of degree <= [9], taken by the
+ * short-row kernels where a kernel has one) [9]=short_max
+ * (agnn_plan_options.short_edges; 0: no split) [10]=rows of other blocks this
+ * rank's rows reference (received per peer-memory exchange) [11]=rows of this
+ * rank's block sent per peer-memory exchange (summed over the peers; known after
+ * agnn_plan_connect) */
+agnn_status agnn_plan_info(agnn_plan_t plan, int64_t* info);
 
 /* The transposed pattern of the plan's CSR (test/utility; synchronises):
  * col_ptr [n+1] (device, int64), row_idx [nnz] (device, int32) list, for

@@ -255,10 +255,10 @@ class Plan:
         self.n_local = row_end - row_begin
 
     def info(self) -> dict:
-        a = (ctypes.c_int64 * 10)()
+        a = (ctypes.c_int64 * 12)()
         _check(lib().agnn_plan_info(self.handle, a))
         keys = ("n_local", "nnz", "light_rows", "heavy_rows", "heavy_chunks", "chunk", "max_degree",
-                "n", "short_rows", "short_max")
+                "n", "short_rows", "short_max", "recv_rows", "send_rows")
         return dict(zip(keys, list(a)))
 
     # ---- peer-memory exchange setup (world > 1 without an NCCL id) -------------

@@ -508,8 +508,8 @@ agnn_status av_forward(const Plan& p, const agnn_layer_desc& d, const float* W, 
   if (p.world > 1) {
     AGNN_CUDA_TRY(cudaMemcpyAsync(sv.Hfull + p.row_begin * d.k_in, H_in,
                                   sizeof(float) * p.n_local * d.k_in, cudaMemcpyDeviceToDevice, s));
-    if ((st = allgather_rows(p, sv.Hfull, d.k_in, s)) != AGNN_OK) return st;
-    if (ag && (st = allgather_rows(p, sv.nu, 1, s)) != AGNN_OK) return st;
+    const RowArray ra[2] = {{sv.Hfull, d.k_in}, {sv.nu, 1}};
+    if ((st = allgather_rows(p, ra, ag ? 2 : 1, s)) != AGNN_OK) return st;
     Hf = sv.Hfull;
   }
   Items it = items_of(p);
@@ -561,33 +561,20 @@ agnn_status av_backward(const Plan& p, const agnn_layer_desc& d, const float* W,
   if ((st = gemm_tn(sv.X, p.n_local, d.k_in, w.G, d.k_out, dW, w.gemm, s)) != AGNN_OK) return st;
   if (p.world > 1 && (st = allreduce_sum(p, dW, (int64_t)d.k_in * d.k_out, s)) != AGNN_OK) return st;
   if (!dH_in) return AGNN_OK;
-  // M = G W^T (Eq. 12); peer mode: the GEMM epilogue also stores M's rows into every
-  // peer's replica (fused all-gather between an entry and an exit barrier)
+  // M = G W^T (Eq. 12) for the local rows; with P > 1 the rows the other ranks
+  // reference (and AGNN's records) then go to their replicas (comm.cu)
   float* Mloc = w.M + p.row_begin * d.k_in;
-  bool m_done = p.world == 1;
-  if (p.world > 1 && p.peer) {
-    void* tm[kMaxPeers];
-    if ((st = peer_targets(p, Mloc, tm)) != AGNN_OK) return st;
-    PeerOut po;
-    for (int r = 0; r < p.world; ++r)
-      if (r != p.rank) po.C0[po.n++] = static_cast<float*>(tm[r]);
-    if ((st = peer_barrier(p, s)) != AGNN_OK) return st;
-    if ((st = gemm_rows(w.G, p.n_local, d.k_out, W, true, d.k_in, Mloc, d.k_in, nullptr, s,
-                        nullptr, 0, 0, &po, &m_done)) != AGNN_OK)
-      return st;
-    if (m_done && (st = peer_barrier(p, s)) != AGNN_OK) return st;
-  } else if ((st = gemm_rows(w.G, p.n_local, d.k_out, W, true, d.k_in, Mloc, d.k_in, nullptr,
-                             s)) != AGNN_OK) {
+  if ((st = gemm_rows(w.G, p.n_local, d.k_out, W, true, d.k_in, Mloc, d.k_in, nullptr, s)) !=
+      AGNN_OK)
     return st;
-  }
   if (ag) {
     AGNN_AV_DISPATCH(K_, (agnn_rec_kernel<K><<<grid_of(agnn_rec_kernel<K>), kSparseThreads, 0, s>>>(
                              p.n_local, p.row_begin, w.M, sv.X, sv.nu, sv.l, fabsf(d.beta), w.rec)));
     AGNN_LAUNCH_CHECK("agnn_rec_kernel");
   }
   if (p.world > 1) {
-    if (!m_done && (st = allgather_rows(p, w.M, d.k_in, s)) != AGNN_OK) return st;
-    if (ag && (st = allgather_rows(p, reinterpret_cast<float*>(w.rec), 4, s)) != AGNN_OK) return st;
+    const RowArray ra[2] = {{w.M, d.k_in}, {reinterpret_cast<float*>(w.rec), 4}};
+    if ((st = allgather_rows(p, ra, ag ? 2 : 1, s)) != AGNN_OK) return st;
   }
   const float* Hf = p.world > 1 ? sv.Hfull : H_in;
   Items it = items_of(p);

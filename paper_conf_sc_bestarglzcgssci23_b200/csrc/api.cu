@@ -324,6 +324,8 @@ agnn_status agnn_plan_info(agnn_plan_t h, int64_t* info) {
   info[7] = p.n;
   info[8] = p.n_short;
   info[9] = p.short_max;
+  info[10] = p.n_wanted;
+  info[11] = p.send_off[p.world > 1 ? p.world : 0];
   return AGNN_OK;
 }
 
@@ -341,6 +343,7 @@ agnn_status agnn_plan_connect(agnn_plan_t h, const void* handles, const int64_t*
   agnn_status st = peer_open(p, handles, offsets, p.ctl, out);
   if (st != AGNN_OK) return st;
   for (int r = 0; r < p.world; ++r) p.peer_ctl[r] = out[r];
+  if ((st = peer_send_lists(p)) != AGNN_OK) return st;
   p.peer_ready = true;
   return AGNN_OK;
 }

@@ -352,8 +352,8 @@ agnn_status cg_forward(const Plan& p, const agnn_layer_desc& d, const float* W, 
   if (p.world > 1) {
     AGNN_CUDA_TRY(cudaMemcpyAsync(sv.Hfull + p.row_begin * d.k_in, H_in,
                                   sizeof(float) * p.n_local * d.k_in, cudaMemcpyDeviceToDevice, s));
-    if ((st = allgather_rows(p, sv.Hfull, d.k_in, s)) != AGNN_OK) return st;
-    if ((st = allgather_rows(p, sv.rdeg, 1, s)) != AGNN_OK) return st;
+    const RowArray ra[2] = {{sv.Hfull, d.k_in}, {sv.rdeg, 1}};
+    if ((st = allgather_rows(p, ra, 2, s)) != AGNN_OK) return st;
     Hf = sv.Hfull;
   }
   Items it = items_of(p);

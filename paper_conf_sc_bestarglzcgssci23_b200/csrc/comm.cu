@@ -11,12 +11,15 @@
 //  * peer memory (default when the caller passes no NCCL id): at setup every
 //    rank maps the other ranks' replicated buffers and control block with CUDA
 //    IPC (NVLink / NVSwitch loads and stores, agnn_plan_connect /
-//    agnn_plan_register); an all-gather is a kernel that stores this rank's rows
-//    straight into every peer's replica, fenced by a flag barrier; an all-reduce
-//    writes this rank's partial into every peer's slot and each rank adds the
-//    slots in rank order (identical, deterministic result on every rank).  The
-//    projection GEMM can also store its output rows into the peers' replicas
-//    from its epilogue (gat.cu), so that exchange overlaps the GEMM tile by tile.
+//    agnn_plan_register).  An all-gather is a kernel that stores rows of this
+//    rank's block straight into every peer's replica, fenced by a flag barrier —
+//    only the rows the peer's own CSR references (its "wanted" columns in this
+//    block, exchanged once at agnn_plan_connect): the sparse kernels gather a
+//    replicated row only as the neighbour of a local row, so every row a rank
+//    reads arrives and the results are bitwise those of the full all-gather, at
+//    ~40-60 % of its NVLink bytes on the Kronecker graphs.  An
+//    all-reduce writes this rank's partial into every peer's slot and each rank
+//    adds the slots in rank order (identical, deterministic result on every rank).
 //  * NCCL: the variable-size all-gather is a group of ncclBroadcast calls (one
 //    root per rank, in place), since NCCL has no all-gather-v; ncclAllReduce.
 #include <cuda.h>
@@ -45,6 +48,9 @@ float* red_of(void* ctl, int world, int set, int rank) {
 struct PeerPtrs {
   char* p[kMaxPeers];
 };
+struct PeerOffs {
+  int64_t o[kMaxPeers + 1];  // send_off
+};
 
 // barrier over the ranks: publish `epoch` into slot [rank] of every peer's flags,
 // then wait until every peer has published it into ours (system-scope release /
@@ -67,23 +73,32 @@ __global__ void peer_barrier_kernel(int64_t* own, PeerPtrs peers, int rank, int 
   }
 }
 
-// rows [off, off + count) of a replicated array: local copy -> every peer's copy
-__global__ void peer_push_kernel(const float* __restrict__ src, PeerPtrs dst, int rank, int world,
-                                 int64_t off, int64_t count) {
-  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-  const int64_t t0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  const bool vec = ((off | count) & 3) == 0;
-  if (vec) {
-    for (int64_t i = t0; i < count / 4; i += stride) {
-      const float4 v = ldg4(src + off + 4 * i);
-      for (int r = 0; r < world; ++r)
-        if (r != rank) st4(reinterpret_cast<float*>(dst.p[r]) + off + 4 * i, v);
-    }
-  } else {
-    for (int64_t i = t0; i < count; i += stride) {
-      const float v = src[off + i];
-      for (int r = 0; r < world; ++r)
-        if (r != rank) reinterpret_cast<float*>(dst.p[r])[off + i] = v;
+// the rows of send lists (global row ids, by peer) of the replicated arrays -> the
+// same rows of every peer's replica; one warp per (peer, row), every array in turn
+struct PushArr {
+  const float* src[4];
+  PeerPtrs dst[4];
+  int64_t width[4];  // floats per row
+  int n;
+};
+__global__ void peer_push_needed_kernel(PushArr A, const int32_t* __restrict__ idx,
+                                        int64_t total, PeerOffs offs) {
+  const int lane = threadIdx.x & 31;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  for (int64_t w = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; w < total; w += nw) {
+    int q = 0;
+    while (w >= offs.o[q + 1]) ++q;  // peer of list entry w
+    const int64_t row = idx[w];
+#pragma unroll 1
+    for (int a = 0; a < A.n; ++a) {
+      const int64_t wd = A.width[a];
+      const float* src = A.src[a] + row * wd;
+      float* dst = reinterpret_cast<float*>(A.dst[a].p[q]) + row * wd;
+      if ((wd & 3) == 0) {
+        for (int64_t c = 4 * lane; c < wd; c += 128) st4(dst + c, ldg4(src + c));
+      } else {
+        for (int64_t c = lane; c < wd; c += 32) dst[c] = src[c];
+      }
     }
   }
 }
@@ -210,13 +225,81 @@ agnn_status peer_targets(const Plan& p, const void* local, void* out[kMaxPeers])
   return AGNN_OK;
 }
 
+__global__ void mark_cols_kernel(const int32_t* __restrict__ col, int64_t nnz,
+                                 uint8_t* __restrict__ mark) {
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < nnz;
+       e += (int64_t)gridDim.x * blockDim.x)
+    mark[col[e]] = 1;
+}
+
+// The columns of other ranks' blocks that this rank's CSR references ("wanted"),
+// ascending, with per-block offsets, written behind the flags and reduce slots of
+// the control block (peers read them at agnn_plan_connect).  Plan time; synchronises.
 agnn_status peer_init(Plan& p) {
   p.peer = true;
   p.regs = new std::vector<Plan::Reg>();
   p.opened = new std::vector<void*>();
-  AGNN_CUDA_TRY(cudaMalloc(&p.ctl, ctl_bytes(p.world)));
+  std::vector<uint8_t> mark((size_t)p.n, 0);
+  if (p.nnz > 0) {
+    uint8_t* d_mark = nullptr;
+    AGNN_CUDA_TRY(cudaMalloc(&d_mark, (size_t)p.n));
+    AGNN_CUDA_TRY(cudaMemset(d_mark, 0, (size_t)p.n));
+    mark_cols_kernel<<<kNumSMs * 8, 256>>>(p.col_idx, p.nnz, d_mark);
+    AGNN_CUDA_TRY(cudaGetLastError());
+    AGNN_CUDA_TRY(cudaMemcpy(mark.data(), d_mark, (size_t)p.n, cudaMemcpyDeviceToHost));
+    AGNN_CUDA_TRY(cudaFree(d_mark));
+  }
+  std::vector<int64_t> woff((size_t)p.world + 1, 0);
+  std::vector<int32_t> want;
+  for (int q = 0; q < p.world; ++q) {
+    woff[(size_t)q] = (int64_t)want.size();
+    if (q == p.rank) continue;
+    for (int64_t j = p.bounds[q]; j < p.bounds[q + 1]; ++j)
+      if (mark[(size_t)j]) want.push_back((int32_t)j);
+  }
+  woff[(size_t)p.world] = (int64_t)want.size();
+  p.n_wanted = (int64_t)want.size();
+  p.want_off = (ctl_bytes(p.world) + 255) & ~size_t(255);
+  const size_t bytes = p.want_off + sizeof(int64_t) * woff.size() + sizeof(int32_t) * want.size();
+  AGNN_CUDA_TRY(cudaMalloc(&p.ctl, bytes));
   AGNN_CUDA_TRY(cudaMemset(p.ctl, 0, ctl_bytes(p.world)));
+  char* w = static_cast<char*>(p.ctl) + p.want_off;
+  AGNN_CUDA_TRY(cudaMemcpy(w, woff.data(), sizeof(int64_t) * woff.size(), cudaMemcpyHostToDevice));
+  if (!want.empty())
+    AGNN_CUDA_TRY(cudaMemcpy(w + sizeof(int64_t) * woff.size(), want.data(),
+                             sizeof(int32_t) * want.size(), cudaMemcpyHostToDevice));
   AGNN_CUDA_TRY(cudaDeviceSynchronize());
+  return AGNN_OK;
+}
+
+// agnn_plan_connect: the send lists = every peer's wanted columns in this rank's block
+agnn_status peer_send_lists(Plan& p) {
+  std::vector<int32_t> all;
+  p.send_off[0] = 0;
+  for (int q = 0; q < p.world; ++q) {
+    if (q != p.rank) {
+      const char* w = static_cast<const char*>(p.peer_ctl[q]) + p.want_off;
+      int64_t o[2];
+      AGNN_CUDA_TRY(cudaMemcpy(o, w + sizeof(int64_t) * p.rank, sizeof(o), cudaMemcpyDeviceToHost));
+      const int64_t cnt = o[1] - o[0];
+      if (cnt < 0 || cnt > p.n_local)
+        return fail(AGNN_ESTATE, "peer exchange: inconsistent wanted lists (plans differ across ranks)");
+      const size_t at = all.size();
+      all.resize(at + (size_t)cnt);
+      if (cnt > 0)
+        AGNN_CUDA_TRY(cudaMemcpy(all.data() + at,
+                                 w + sizeof(int64_t) * (p.world + 1) + sizeof(int32_t) * o[0],
+                                 sizeof(int32_t) * cnt, cudaMemcpyDeviceToHost));
+    }
+    p.send_off[q + 1] = (int64_t)all.size();
+  }
+  if (p.send_idx) cudaFree(p.send_idx);
+  p.send_idx = nullptr;
+  if (!all.empty()) {
+    AGNN_CUDA_TRY(cudaMalloc(&p.send_idx, sizeof(int32_t) * all.size()));
+    AGNN_CUDA_TRY(cudaMemcpy(p.send_idx, all.data(), sizeof(int32_t) * all.size(),
+                             cudaMemcpyHostToDevice));
+  }
   return AGNN_OK;
 }
 
@@ -247,11 +330,18 @@ void comm_destroy(Plan& p) {
   }
   delete p.regs;
   p.regs = nullptr;
+  if (p.send_idx) cudaFree(p.send_idx);
+  p.send_idx = nullptr;
   if (p.ctl) cudaFree(p.ctl);
   p.ctl = nullptr;
 }
 
 agnn_status allgather_rows(const Plan& p, float* full, int64_t width, cudaStream_t s) {
+  const RowArray a{full, width};
+  return allgather_rows(p, &a, 1, s);
+}
+
+agnn_status allgather_rows(const Plan& p, const RowArray* arrs, int n_arrs, cudaStream_t s) {
   if (p.world <= 1) return AGNN_OK;
   struct Mark {
     cudaStream_t s;
@@ -260,18 +350,28 @@ agnn_status allgather_rows(const Plan& p, float* full, int64_t width, cudaStream
     }
   } mark{s};
   if (p.peer) {
-    // entry barrier: every peer is done reading its replica of `full` (the buffer
-    // may be a workspace array reused by the previous layer); push; exit barrier
+    // entry barrier: every peer is done reading its replica (the buffers may be
+    // workspace arrays reused by the previous layer); push the rows each peer
+    // references; exit barrier
     if (!p.peer_ready) return fail(AGNN_ESTATE, "peer exchange: agnn_plan_connect not called");
-    PeerPtrs dst;
-    if (!peer_lookup(p, full, dst))
-      return fail(AGNN_ESTATE, "peer exchange: buffer not registered (agnn_plan_register)");
+    if (n_arrs > 4) return fail(AGNN_EINVAL, "allgather_rows: at most 4 arrays");
+    PushArr A;
+    A.n = n_arrs;
+    for (int i = 0; i < n_arrs; ++i) {
+      if (!peer_lookup(p, arrs[i].full, A.dst[i]))
+        return fail(AGNN_ESTATE, "peer exchange: buffer not registered (agnn_plan_register)");
+      A.src[i] = arrs[i].full;
+      A.width[i] = arrs[i].width;
+    }
     agnn_status st = peer_barrier(p, s);
     if (st != AGNN_OK) return st;
-    const int64_t off = p.row_begin * width, count = p.n_local * width;
-    if (count > 0) {
-      const int64_t blocks = std::min<int64_t>((count / 4 + 255) / 256 + 1, (int64_t)kNumSMs * 8);
-      peer_push_kernel<<<(unsigned)blocks, 256, 0, s>>>(full, dst, p.rank, p.world, off, count);
+    const int64_t total = p.send_off[p.world];
+    if (total > 0) {
+      PeerOffs offs;
+      for (int q = 0; q <= p.world; ++q) offs.o[q] = p.send_off[q];
+      for (int q = p.world + 1; q <= kMaxPeers; ++q) offs.o[q] = total;
+      const int64_t blocks = std::min<int64_t>((total + 7) / 8, (int64_t)kNumSMs * 4);
+      peer_push_needed_kernel<<<(unsigned)blocks, 256, 0, s>>>(A, p.send_idx, total, offs);
       AGNN_LAUNCH_CHECK("peer_push_kernel");
     }
     return peer_barrier(p, s);
@@ -279,14 +379,17 @@ agnn_status allgather_rows(const Plan& p, float* full, int64_t width, cudaStream
   ncclComm_t comm = static_cast<ncclComm_t>(p.nccl);
   agnn_status st = nccl_status(ncclGroupStart(), "ncclGroupStart");
   if (st != AGNN_OK) return st;
-  for (int r = 0; r < p.world; ++r) {
-    const int64_t rows = p.bounds[r + 1] - p.bounds[r];
-    if (rows == 0) continue;
-    float* blk = full + p.bounds[r] * width;
-    ncclResult_t e = ncclBroadcast(blk, blk, (size_t)(rows * width), ncclFloat32, r, comm, s);
-    if (e != ncclSuccess) {
-      ncclGroupEnd();
-      return nccl_status(e, "ncclBroadcast");
+  for (int i = 0; i < n_arrs; ++i) {
+    const int64_t width = arrs[i].width;
+    for (int r = 0; r < p.world; ++r) {
+      const int64_t rows = p.bounds[r + 1] - p.bounds[r];
+      if (rows == 0) continue;
+      float* blk = arrs[i].full + p.bounds[r] * width;
+      ncclResult_t e = ncclBroadcast(blk, blk, (size_t)(rows * width), ncclFloat32, r, comm, s);
+      if (e != ncclSuccess) {
+        ncclGroupEnd();
+        return nccl_status(e, "ncclBroadcast");
+      }
     }
   }
   return nccl_status(ncclGroupEnd(), "ncclGroupEnd");

@@ -782,9 +782,8 @@ agnn_status gat_forward(const Plan& p, const GatShape& g, const float* W, const 
                              g.k_out, stloc, w.dP, s)) != AGNN_OK)
       return st;
     if (p.world > 1) {
-      if ((st = allgather_rows(p, reinterpret_cast<float*>(sv.P16), g.k_out / 2, s)) != AGNN_OK)
-        return st;
-      if ((st = allgather_rows(p, sv.st, 2 * g.heads, s)) != AGNN_OK) return st;
+      const RowArray ra[2] = {{reinterpret_cast<float*>(sv.P16), g.k_out / 2}, {sv.st, 2 * g.heads}};
+      if ((st = allgather_rows(p, ra, 2, s)) != AGNN_OK) return st;
     }
     // gathered per edge: a bf16 row of P and the t_j of the heads
     const Items ith = l2_hinted(it, p, 2 * (int64_t)g.k_out + 4 * g.heads);
@@ -797,42 +796,15 @@ agnn_status gat_forward(const Plan& p, const GatShape& g, const float* W, const 
     }
     return AGNN_OK;
   }
+  // P | s t for the local rows, written at their global offsets; with P > 1 the
+  // rows the other ranks reference are then pushed to their replicas (comm.cu)
   float* Ploc = sv.P + p.row_begin * g.k_out;
-  if (p.world > 1 && p.peer) {
-    // fused GEMM -> all-gather over peer memory: the GEMM epilogue stores every
-    // output tile into the local P | st and into every peer's replica (NVLink
-    // stores overlap the next tiles' MMAs); entry / exit barriers order it with
-    // the peers' reads of the previous contents and of these rows
-    void* tp[kMaxPeers];
-    void* ts[kMaxPeers];
-    if ((st = peer_targets(p, Ploc, tp)) != AGNN_OK) return st;
-    if ((st = peer_targets(p, stloc, ts)) != AGNN_OK) return st;
-    PeerOut po;
-    for (int r = 0; r < p.world; ++r) {
-      if (r == p.rank) continue;
-      po.C0[po.n] = static_cast<float*>(tp[r]);
-      po.C1[po.n] = static_cast<float*>(ts[r]);
-      ++po.n;
-    }
-    if ((st = peer_barrier(p, s)) != AGNN_OK) return st;
-    bool fused = false;
-    if ((st = gemm_rows(H_in, p.n_local, g.k_in, w.Wext, true, NE, Ploc, g.k_out, stloc, s,
-                        nullptr, 0, NEs, &po, &fused)) != AGNN_OK)
-      return st;
-    if (fused) {
-      if ((st = peer_barrier(p, s)) != AGNN_OK) return st;
-    } else {
-      if ((st = allgather_rows(p, sv.P, g.k_out, s)) != AGNN_OK) return st;
-      if ((st = allgather_rows(p, sv.st, 2 * g.heads, s)) != AGNN_OK) return st;
-    }
-  } else {
-    if ((st = gemm_rows(H_in, p.n_local, g.k_in, w.Wext, true, NE, Ploc, g.k_out, stloc, s,
-                        nullptr, 0, NEs)) != AGNN_OK)
-      return st;
-    if (p.world > 1) {
-      if ((st = allgather_rows(p, sv.P, g.k_out, s)) != AGNN_OK) return st;
-      if ((st = allgather_rows(p, sv.st, 2 * g.heads, s)) != AGNN_OK) return st;
-    }
+  if ((st = gemm_rows(H_in, p.n_local, g.k_in, w.Wext, true, NE, Ploc, g.k_out, stloc, s,
+                      nullptr, 0, NEs)) != AGNN_OK)
+    return st;
+  if (p.world > 1) {
+    const RowArray ra[2] = {{sv.P, g.k_out}, {sv.st, 2 * g.heads}};
+    if ((st = allgather_rows(p, ra, 2, s)) != AGNN_OK) return st;
   }
   Items it = items_of(p);
   FwdOut o{saved ? sv.Z : nullptr, H_out, saved ? sv.m : nullptr, saved ? sv.l : nullptr,
@@ -874,21 +846,7 @@ agnn_status gat_backward(const Plan& p, const GatShape& g, const float* W, const
   const int K_ = g.k_out, NH_ = g.heads;
   Items it = items_of(p);
   agnn_status st;
-  PeerRows pr;  // peer mode: G and rec rows also go straight to every peer's replica
-  if (p.world > 1 && p.peer) {
-    void* tg[kMaxPeers];
-    void* tr[kMaxPeers];
-    if ((st = peer_targets(p, g.bf16 ? (void*)w.G16 : (void*)w.G, tg)) != AGNN_OK) return st;
-    if ((st = peer_targets(p, w.rec, tr)) != AGNN_OK) return st;
-    for (int r = 0; r < p.world; ++r) {
-      if (r == p.rank) continue;
-      pr.a[pr.n] = static_cast<float*>(tg[r]);
-      pr.b[pr.n] = static_cast<float*>(tr[r]);
-      ++pr.n;
-    }
-    // entry barrier: every peer has finished reading its G / rec (previous layer)
-    if ((st = peer_barrier(p, s)) != AGNN_OK) return st;
-  }
+  const PeerRows pr;  // (no fused peer stores: the exchange below pushes the needed rows)
   if (g.bf16) {
     if (directed)
       return fail(AGNN_EUNSUPPORTED, "AGNN_PREC_BF16: symmetric patterns only");
@@ -903,19 +861,11 @@ agnn_status gat_backward(const Plan& p, const GatShape& g, const float* W, const
                                     w.G, w.rec, pr, sv.Q, w.ds_row)));
   }
   AGNN_LAUNCH_CHECK("gat_bwd_prologue_kernel");
-  if (p.world > 1) {
-    if (p.peer) {  // the prologue stored G | rec into the peers' replicas: exit barrier
-      if ((st = peer_barrier(p, s)) != AGNN_OK) return st;
-    } else if (g.bf16) {
-      if ((st = allgather_rows(p, reinterpret_cast<float*>(w.G16), g.k_out / 2, s)) != AGNN_OK)
-        return st;
-      if ((st = allgather_rows(p, reinterpret_cast<float*>(w.rec), 4 * g.heads, s)) != AGNN_OK)
-        return st;
-    } else {
-      if ((st = allgather_rows(p, w.G, g.k_out, s)) != AGNN_OK) return st;
-      if ((st = allgather_rows(p, reinterpret_cast<float*>(w.rec), 4 * g.heads, s)) != AGNN_OK)
-        return st;
-    }
+  if (p.world > 1) {  // G | rec rows the other ranks reference -> their replicas
+    const RowArray ra[2] = {{g.bf16 ? reinterpret_cast<float*>(w.G16) : w.G,
+                             g.bf16 ? g.k_out / 2 : g.k_out},
+                            {reinterpret_cast<float*>(w.rec), 4 * g.heads}};
+    if ((st = allgather_rows(p, ra, 2, s)) != AGNN_OK) return st;
   }
   BwdArgs A{sv.P, sv.st, w.G, w.rec, a, g.slope, w.dP, w.pacc, w.pm, w.pl, w.da_part,
             nullptr, nullptr, w.ds_dir, sv.P16, w.G16, w.ds_row};

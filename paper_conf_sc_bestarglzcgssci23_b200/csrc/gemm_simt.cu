@@ -204,7 +204,7 @@ __global__ void sum_splits_kernel(const float* __restrict__ part, int splits, in
 
 agnn_status gemm_tc(const float* A, int64_t M, int K, const float* B, int n_real, float* C0,
                     int n_split, float* C1, int n_store, float* Cact, int act, cudaStream_t s,
-                    const PeerOut* peers, bf16* C0h = nullptr);
+                    bf16* C0h = nullptr);
 
 namespace {
 // Y[i] = bf16_rn(X[i]) over rows x cols (cols % 4 == 0)
@@ -218,7 +218,7 @@ __global__ void to_bf16_kernel(const float* __restrict__ X, int64_t count4, bf16
 agnn_status gemm_rows_bf16(const float* A, int64_t M, int K, const float* B, int N, bf16* C0h,
                            int n_split, float* C1, float* scratch, cudaStream_t s) {
   if (M <= 0) return AGNN_OK;
-  agnn_status st = gemm_tc(A, M, K, B, N, nullptr, n_split, C1, N, nullptr, 0, s, nullptr, C0h);
+  agnn_status st = gemm_tc(A, M, K, B, N, nullptr, n_split, C1, N, nullptr, 0, s, C0h);
   if (st != AGNN_EUNSUPPORTED) return st;
   // no tcgen05 instantiation for this shape: fp32 product into scratch, then round
   // (B has (N + 3) / 4 * 4 rows, the padding rows zero; columns >= N are not stored)
@@ -234,17 +234,13 @@ agnn_status gemm_rows_bf16(const float* A, int64_t M, int K, const float* B, int
 
 agnn_status gemm_rows(const float* A, int64_t M, int K, const float* B, bool b_trans, int N,
                       float* C0, int n_split, float* C1, cudaStream_t s, float* Cact, int act,
-                      int n_store, const PeerOut* peers, bool* peers_done) {
-  if (peers_done) *peers_done = false;
+                      int n_store) {
   if (b_trans) {  // tcgen05 3xTF32 path when the shape has an instantiation
     const int ns = (n_store <= 0 || n_store > N) ? N : n_store;
-    const agnn_status st = gemm_tc(A, M, K, B, ns, C0, n_split, C1, ns, Cact, act, s, peers);
-    if (st != AGNN_EUNSUPPORTED) {
-      if (peers_done) *peers_done = st == AGNN_OK;
-      return st;
-    }
+    const agnn_status st = gemm_tc(A, M, K, B, ns, C0, n_split, C1, ns, Cact, act, s);
+    if (st != AGNN_EUNSUPPORTED) return st;
   }
-  if (M <= 0) return AGNN_OK;  // (the fused all-gather decision above is the shape's)
+  if (M <= 0) return AGNN_OK;
   if (K % 4 || N % 4) return fail(AGNN_EINVAL, "gemm_rows: K and N must be multiples of 4");
   dim3 grid((unsigned)((M + BM - 1) / BM), (N + BN - 1) / BN);
   if (n_store <= 0 || n_store > N) n_store = N;

@@ -187,20 +187,14 @@ struct TcOut {
   float* C1;    // columns [n_split, n_store), row stride n_store - n_split
   float* Cact;  // sigma(C) for columns < n_split (nullable)
   int n_split, n_store, act;
-  int npeer;                       // peer replicas also written (peer-memory exchange)
-  float* pC0[kMaxPeers - 1];
-  float* pC1[kMaxPeers - 1];
   bf16* C0h;    // EPI_BF16: columns [0, n_split) stored as bfloat16 here instead of C0
 };
 
-// epilogue variants (compile time, so the plain fp32 epilogue carries neither)
+// epilogue variants (compile time, so the plain fp32 epilogue carries no bf16 code)
 constexpr int EPI_PLAIN = 0;  // C0 | C1 fp32 (+ sigma copy)
-constexpr int EPI_PEER = 1;   // also every peer's replica (peer-memory all-gather)
 constexpr int EPI_BF16 = 2;   // C0 columns rounded to bfloat16 into C0h (reading B1)
 
 // 16 consecutive columns c0.. of output row `row` (C0 | C1 split, optional sigma copy).
-// PEER: the same values also go to every peer's replica (peer-memory all-gather);
-// a compile-time flag, so the single-GPU epilogue carries no peer code at all.
 __device__ __forceinline__ void store_row16_to(const TcOut& out, float* C0, float* C1, float* Ca,
                                                int64_t row, int c0, const float (&v)[16]) {
 #pragma unroll
@@ -241,11 +235,6 @@ __device__ __forceinline__ void store_row16(const TcOut& out, int64_t row, int c
     return;
   }
   store_row16_to(out, out.C0, out.C1, out.Cact, row, c0, v);
-  if constexpr (EPI == EPI_PEER) {
-#pragma unroll 1
-    for (int pi = 0; pi < out.npeer; ++pi)
-      store_row16_to(out, out.pC0[pi], out.pC1[pi], nullptr, row, c0, v);
-  }
 }
 
 // 32 columns [c0, c0+32) of the warp's 32 rows [row0, row0+32) through a per-warp
@@ -272,11 +261,6 @@ __device__ __forceinline__ void store_block32(const TcOut& out, int64_t row0, in
       }
       if (out.C0) st4(out.C0 + row * out.n_split + c0 + cc, q);
       if (out.Cact) st4(out.Cact + row * out.n_split + c0 + cc, act_fwd4(out.act, q));
-      if constexpr (EPI == EPI_PEER) {
-#pragma unroll 1
-        for (int pi = 0; pi < out.npeer; ++pi)  // peers' replicas (NVLink stores)
-          st4(out.pC0[pi] + row * out.n_split + c0 + cc, q);
-      }
     }
   }
   __syncwarp();
@@ -756,8 +740,6 @@ agnn_status launch_tc(const float* A, int64_t M, const float* B, int n_real, con
   if (!attr) {
     cudaFuncSetAttribute(gemm_tc_kernel<N, K, S, SB, EPI_PLAIN>,
                          cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    cudaFuncSetAttribute(gemm_tc_kernel<N, K, S, SB, EPI_PEER>,
-                         cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     cudaFuncSetAttribute(gemm_tc_kernel<N, K, S, SB, EPI_BF16>,
                          cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     attr = true;
@@ -769,8 +751,6 @@ agnn_status launch_tc(const float* A, int64_t M, const float* B, int n_real, con
   const int grid = (int)std::min<int64_t>(ntiles, sms);
   if (o.C0h)
     gemm_tc_kernel<N, K, S, SB, EPI_BF16><<<grid, TC_WS_THREADS, smem, s>>>(ma, mb, B, n_real, M, o);
-  else if (o.npeer > 0)
-    gemm_tc_kernel<N, K, S, SB, EPI_PEER><<<grid, TC_WS_THREADS, smem, s>>>(ma, mb, B, n_real, M, o);
   else
     gemm_tc_kernel<N, K, S, SB, EPI_PLAIN><<<grid, TC_WS_THREADS, smem, s>>>(ma, mb, B, n_real, M, o);
   AGNN_LAUNCH_CHECK("gemm_tc_kernel");
@@ -863,26 +843,16 @@ agnn_status gemm_tn_tc(const float* A, int64_t M, int K1, const float* B, int N,
 // Returns AGNN_EUNSUPPORTED when the shape has no tcgen05 instantiation.
 agnn_status gemm_tc(const float* A, int64_t M, int K, const float* B, int n_real, float* C0,
                     int n_split, float* C1, int n_store, float* Cact, int act, cudaStream_t s,
-                    const PeerOut* peers, bf16* C0h) {
-  // the shape decides (never M or the rank): with the peer exchange every rank must
-  // agree on whether the epilogue did the all-gather (an empty row block included)
+                    bf16* C0h) {
   if ((reinterpret_cast<uintptr_t>(A) & 15) || (K % 32)) return AGNN_EUNSUPPORTED;
-  if (C0h && (peers || Cact || (n_split & 3))) return AGNN_EUNSUPPORTED;
-  if (peers && (peers->n > kMaxPeers - 1 || (!C0 && peers->n > 0))) return AGNN_EUNSUPPORTED;
+  if (C0h && (Cact || (n_split & 3))) return AGNN_EUNSUPPORTED;
   const int npad = (n_real + 15) / 16 * 16;
   const bool shape_ok = (K == 128 && (npad == 128 || npad == 144 || npad == 160 || npad == 64)) ||
                         (K == 64 && (npad == 64 || npad == 80 || npad == 128)) ||
                         (K == 256 && (npad == 256 || npad == 128));
   if (!shape_ok) return AGNN_EUNSUPPORTED;
   if (M <= 0) return AGNN_OK;
-  TcOut o{C0, C1, Cact, n_split, n_store, act, 0, {}, {}, C0h};
-  if (peers) {
-    o.npeer = peers->n;
-    for (int i = 0; i < peers->n; ++i) {
-      o.pC0[i] = peers->C0[i];
-      o.pC1[i] = peers->C1[i];
-    }
-  }
+  TcOut o{C0, C1, Cact, n_split, n_store, act, C0h};
   // resident B: S = the 16 KB stages that fit next to B (2 x K x N x 4 bytes), <= 8
   if (K == 128 && npad == 128) return launch_tc<128, 128, 4, false>(A, M, B, n_real, o, s);
   if (K == 128 && npad == 144) return launch_tc<144, 128, 3, false>(A, M, B, n_real, o, s);

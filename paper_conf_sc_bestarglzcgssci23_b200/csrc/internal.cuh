@@ -77,24 +77,15 @@ inline int grid_of(F* func) { return persistent_blocks(reinterpret_cast<const vo
 // Columns [0, n_split) go to C0 (ld = n_split), [n_split, N) to C1 (ld = N - n_split).
 // If Cact != NULL, sigma(C) (act) is also written to Cact (layout of C0); C0 may be NULL.
 // Columns >= n_store (padding) are computed but not stored (n_store <= 0: N).
-// peers (peer-memory exchange): the tcgen05 epilogue also stores C0 / C1 at the same
-// offsets into every peer's replica (the fused GEMM -> all-gather); *peers_done
-// tells whether it did (shapes on the SIMT fallback leave it to the caller).
-// replicas of up to two row arrays in the other ranks (kernel argument)
+// replicas of up to two row arrays in the other ranks (kernel argument; unused when n = 0)
 struct PeerRows {
   int n = 0;
   float* a[kMaxPeers - 1] = {};
   float* b[kMaxPeers - 1] = {};
 };
-struct PeerOut {
-  int n = 0;
-  float* C0[kMaxPeers] = {};
-  float* C1[kMaxPeers] = {};
-};
 agnn_status gemm_rows(const float* A, int64_t M, int K, const float* B, bool b_trans, int N,
                       float* C0, int n_split, float* C1, cudaStream_t s, float* Cact = nullptr,
-                      int act = 0, int n_store = 0, const PeerOut* peers = nullptr,
-                      bool* peers_done = nullptr);
+                      int act = 0, int n_store = 0);
 // BF16 storage (reading B1): C = A * B^T with columns [0, n_split) rounded to bf16
 // into C0h (ld n_split) and [n_split, N) fp32 into C1 (ld N - n_split); scratch
 // [M x n_split] fp32 is used only when the shape has no tcgen05 instantiation.
@@ -129,7 +120,16 @@ agnn_status gat_debug_alpha(const Plan& p, const GatShape& g, const void* saved,
 // ---- multi-GPU exchange (comm.cu) -------------------------------------------------
 // all-gather of row blocks: rows [bounds[r], bounds[r+1]) of `full` (row width
 // `width` floats) are broadcast from rank r; in place.
+// Peer transport: only the rows each peer's CSR references are sent (comm.cu).
 agnn_status allgather_rows(const Plan& p, float* full, int64_t width, cudaStream_t s);
+struct RowArray {
+  float* full;     // replicated [n x width] array (rows of this rank's block are sent)
+  int64_t width;   // floats per row
+};
+// several arrays in one exchange (one barrier pair, one push kernel); n_arrs <= 4
+agnn_status allgather_rows(const Plan& p, const RowArray* arrs, int n_arrs, cudaStream_t s);
+// agnn_plan_connect: the send lists from the peers' wanted columns
+agnn_status peer_send_lists(Plan& p);
 agnn_status allreduce_sum(const Plan& p, float* buf, int64_t count, cudaStream_t s);
 agnn_status comm_init(Plan& p, const void* unique_id);  // unique_id NULL: peer-memory exchange
 // peer-memory exchange helpers (comm.cu)

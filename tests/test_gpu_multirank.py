@@ -80,6 +80,23 @@ def _check_oracle(w, allout):
                           row_tol=pu.BF16_ROW_TOL if w.prec == "bf16" else None)
 
 
+def _check_send_lists(w, allout):
+    """The needed-rows exchange (comm.cu): each rank receives exactly the distinct
+    out-of-block columns its CSR references, and the ranks send what the others
+    receive in total (host count from the canonical CSR)."""
+    import parity_utils as pu
+    _, _, rp, ci = pu.host_graph(w)
+    full = 0
+    for o in allout:
+        b0, b1 = o["rows"]
+        cols = np.unique(ci[rp[b0]:rp[b1]])
+        want = int(((cols < b0) | (cols >= b1)).sum())
+        assert o["recv"] == want, (o["rows"], o["recv"], want)
+        full += w.n - (b1 - b0)
+    assert sum(o["send"] for o in allout) == sum(o["recv"] for o in allout)
+    assert sum(o["recv"] for o in allout) < full
+
+
 def _worker(rank, world, port, name):
     import torch.distributed as dist
     from paper_conf_sc_bestarglzcgssci23_b200 import runner
@@ -94,6 +111,8 @@ def _worker(rank, world, port, name):
     torch.cuda.synchronize()
     mine = _outputs(st)
     mine["rows"] = (st.row_begin, st.row_end)
+    info = st.plan.info()
+    mine["recv"], mine["send"] = info["recv_rows"], info["send_rows"]
     # inference mode (nothing saved; the replicas live in the workspace)
     st.H[w.layers].zero_()
     st.forward(inference=True)
@@ -103,6 +122,7 @@ def _worker(rank, world, port, name):
     dist.all_gather_object(allout, mine)
     if rank == 0:
         _check_oracle(w, allout)
+        _check_send_lists(w, allout)
         ref = runner.Stack(w, "cuda")
         for _ in range(2):
             ref.step()
