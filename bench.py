@@ -524,15 +524,30 @@ def run_ours(args):
         barrier()
         return sum(a.elapsed_time(b) for a, b in evs)
 
+    busy_steps = {}
+
     def keep_busy(run_step, seconds=0.6):
         # short timed regions (C1, C2: < 1 ms) end before nvidia-smi takes its first
         # sample: keep the GPU under the same load for a moment first, so the clock
-        # samples straddle the timed steps
-        if small:
+        # samples straddle the timed steps.  Every rank must run the same number of
+        # steps (the exchange barriers pair up across ranks): the count is fixed from
+        # a timed step, the maximum over ranks.
+        if not small:
+            return
+        if seconds not in busy_steps:
+            torch.cuda.synchronize()
             t0 = time.perf_counter()
-            while time.perf_counter() - t0 < seconds:
-                run_step()
-                torch.cuda.synchronize()
+            run_step()
+            torch.cuda.synchronize()
+            cnt = max(1, int(seconds / max(time.perf_counter() - t0, 1e-5)))
+            if world > 1:
+                c = torch.tensor([cnt], device="cpu" if same_gpu else dev)
+                dist.all_reduce(c, op=dist.ReduceOp.MAX)
+                cnt = int(c.item())
+            busy_steps[seconds] = cnt
+        for _ in range(busy_steps[seconds]):
+            run_step()
+        torch.cuda.synchronize()
 
     clocks = ClockSampler(local)
     clocks.start()
