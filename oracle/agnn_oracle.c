@@ -188,6 +188,16 @@ static double bf16_round(double x) {
   return (double)f;
 }
 
+/* AGNN / VA BF16 storage mode (reading B2): the gathered operands
+ * are the layer input H and the backward's M = G W^T, both stored in bfloat16:
+ * the layer computes on H~ = bf16(fp32(H)) throughout (the caller rounds the
+ * input with oracle_bf16_round) and M~ = bf16(fp32(M)) replaces M everywhere. */
+int oracle_bf16_round(int64_t count, double* x) {
+#pragma omp parallel for schedule(static)
+  for (int64_t i = 0; i < count; ++i) x[i] = bf16_round(x[i]);
+  return 0;
+}
+
 static int gat_forward_impl(int64_t n, const int64_t* rp, const int32_t* ci, int k, int kout,
                             int heads, const double* H, const double* W, const double* a,
                             double slope, int act, double* P, double* s, double* t, double* alpha,
@@ -421,10 +431,11 @@ int oracle_agnn_forward(int64_t n, const int64_t* rp, const int32_t* ci, int k, 
  *   dH^_j = sum_{(j,i)} dc_ji H^_i + sum_{(i,j)} dc_ij H^_i
  *   dH_j  = sum_{(i,j)} alpha_ij M_i + (dH^_j - (dH^_j . H^_j) H^_j) / nu_j
  *           (nu_j == eps branch: dH^_j / nu_j, nu treated as constant)     */
-int oracle_agnn_backward(int64_t n, const int64_t* rp, const int32_t* ci, int k, int kout,
-                         const double* H, const double* W, double beta, double eps, int act,
-                         const double* nu, const double* alpha, const double* X, const double* Z,
-                         const double* dHout, double* dH, double* dW) {
+static int agnn_backward_impl(int64_t n, const int64_t* rp, const int32_t* ci, int k, int kout,
+                              const double* H, const double* W, double beta, double eps, int act,
+                              const double* nu, const double* alpha, const double* X,
+                              const double* Z, const double* dHout, double* dH, double* dW,
+                              int bf16) {
   const int64_t nnz = rp[n];
   double* G = (double*)malloc(sizeof(double) * (size_t)(n * kout + 1));
   double* M = (double*)malloc(sizeof(double) * (size_t)(n * k + 1));
@@ -437,6 +448,7 @@ int oracle_agnn_backward(int64_t n, const int64_t* rp, const int32_t* ci, int k,
   for (int64_t x = 0; x < n * kout; ++x) G[x] = dHout[x] * act_df(act, Z[x]);
   mm_tn(n, k, kout, X, G, dW);
   mm_nt(n, kout, k, G, W, M);
+  if (bf16) oracle_bf16_round(n * k, M);  /* BF16 mode (reading B2): M~ used throughout */
 #pragma omp parallel for schedule(dynamic, 64)
   for (int64_t i = 0; i < n; ++i) {
     double dl = 0.0;
@@ -477,6 +489,20 @@ int oracle_agnn_backward(int64_t n, const int64_t* rp, const int32_t* ci, int k,
   free(G); free(M); free(dc); free(cp); free(pos); free(erow);
   return 0;
 }
+int oracle_agnn_backward(int64_t n, const int64_t* rp, const int32_t* ci, int k, int kout,
+                         const double* H, const double* W, double beta, double eps, int act,
+                         const double* nu, const double* alpha, const double* X, const double* Z,
+                         const double* dHout, double* dH, double* dW) {
+  return agnn_backward_impl(n, rp, ci, k, kout, H, W, beta, eps, act, nu, alpha, X, Z, dHout, dH,
+                            dW, 0);
+}
+int oracle_agnn_backward_bf16(int64_t n, const int64_t* rp, const int32_t* ci, int k, int kout,
+                              const double* H, const double* W, double beta, double eps, int act,
+                              const double* nu, const double* alpha, const double* X,
+                              const double* Z, const double* dHout, double* dH, double* dW) {
+  return agnn_backward_impl(n, rp, ci, k, kout, H, W, beta, eps, act, nu, alpha, X, Z, dHout, dH,
+                            dW, 1);
+}
 
 /* ================================================================== */
 /* VA (PAPER.md:173 Psi = A (.) (H H^T), no softmax; Eq. 7 at :262):
@@ -508,10 +534,10 @@ int oracle_va_forward(int64_t n, const int64_t* rp, const int32_t* ci, int k, in
  *   G = dHout (.) sigma'(Z); M = G W^T (Eq. 12); N = A (.) (M H^T) (Eq. 12)
  *   Gamma = dH = (N + N^T) H + (A^T (.) H_x) M (Eq. 11)
  *   Y = dW = H^T (A^T (.) H_x) G = X^T G (Eq. 13)                        */
-int oracle_va_backward(int64_t n, const int64_t* rp, const int32_t* ci, int k, int kout,
-                       const double* H, const double* W, int act, const double* S,
-                       const double* X, const double* Z, const double* dHout, double* dH,
-                       double* dW) {
+static int va_backward_impl(int64_t n, const int64_t* rp, const int32_t* ci, int k, int kout,
+                            const double* H, const double* W, int act, const double* S,
+                            const double* X, const double* Z, const double* dHout, double* dH,
+                            double* dW, int bf16) {
   const int64_t nnz = rp[n];
   double* G = (double*)malloc(sizeof(double) * (size_t)(n * kout + 1));
   double* M = (double*)malloc(sizeof(double) * (size_t)(n * k + 1));
@@ -524,6 +550,7 @@ int oracle_va_backward(int64_t n, const int64_t* rp, const int32_t* ci, int k, i
   for (int64_t x = 0; x < n * kout; ++x) G[x] = dHout[x] * act_df(act, Z[x]);
   mm_tn(n, k, kout, X, G, dW);
   mm_nt(n, kout, k, G, W, M);
+  if (bf16) oracle_bf16_round(n * k, M);  /* BF16 mode (reading B2): M~ used throughout */
 #pragma omp parallel for schedule(dynamic, 64)
   for (int64_t i = 0; i < n; ++i)
     for (int64_t p = rp[i]; p < rp[i + 1]; ++p) {
@@ -546,6 +573,18 @@ int oracle_va_backward(int64_t n, const int64_t* rp, const int32_t* ci, int k, i
     }
   free(G); free(M); free(N); free(cp); free(pos); free(erow);
   return 0;
+}
+int oracle_va_backward(int64_t n, const int64_t* rp, const int32_t* ci, int k, int kout,
+                       const double* H, const double* W, int act, const double* S,
+                       const double* X, const double* Z, const double* dHout, double* dH,
+                       double* dW) {
+  return va_backward_impl(n, rp, ci, k, kout, H, W, act, S, X, Z, dHout, dH, dW, 0);
+}
+int oracle_va_backward_bf16(int64_t n, const int64_t* rp, const int32_t* ci, int k, int kout,
+                            const double* H, const double* W, int act, const double* S,
+                            const double* X, const double* Z, const double* dHout, double* dH,
+                            double* dW) {
+  return va_backward_impl(n, rp, ci, k, kout, H, W, act, S, X, Z, dHout, dH, dW, 1);
 }
 
 /* ================================================================== */

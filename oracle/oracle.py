@@ -120,9 +120,17 @@ def gat_backward(rp, ci, H, W, a, heads, fwd, dHout, slope=0.2, act="relu", bf16
     return out
 
 
-def agnn_forward(rp, ci, H, W, beta=1.0, eps=1e-12, act="relu"):
+def bf16_round(x):
+    """round(fp32(x)) to the nearest bfloat16 (ties to even), in the oracle's C."""
+    y = np.array(x, dtype=np.float64, copy=True, order="C")
+    lib().oracle_bf16_round(_i64(y.size), _p(y))
+    return y
+
+
+def agnn_forward(rp, ci, H, W, beta=1.0, eps=1e-12, act="relu", bf16=False):
+    """bf16: BF16 storage mode (reading B2): the layer computes on H~ = bf16(H)."""
     rp, ci, n, nnz = _csr(rp, ci)
-    H, W = _d(H), _d(W)
+    H, W = (bf16_round(H) if bf16 else _d(H)), _d(W)
     k, kout = W.shape
     out = {"nu": np.zeros(n), "alpha": np.zeros(nnz), "m": np.zeros(n), "l": np.zeros(n),
            "X": np.zeros((n, k)), "Z": np.zeros((n, kout)), "Hout": np.zeros((n, kout))}
@@ -136,12 +144,14 @@ def agnn_forward(rp, ci, H, W, beta=1.0, eps=1e-12, act="relu"):
     return out
 
 
-def agnn_backward(rp, ci, H, W, fwd, dHout, beta=1.0, eps=1e-12, act="relu"):
+def agnn_backward(rp, ci, H, W, fwd, dHout, beta=1.0, eps=1e-12, act="relu", bf16=False):
+    """bf16: BF16 storage mode (reading B2): H~ = bf16(H) and M~ = bf16(G W^T)."""
     rp, ci, n, nnz = _csr(rp, ci)
-    H, W, dHout = _d(H), _d(W), _d(dHout)
+    H, W, dHout = (bf16_round(H) if bf16 else _d(H)), _d(W), _d(dHout)
     k, kout = W.shape
     out = {"dH": np.zeros((n, k)), "dW": np.zeros((k, kout))}
-    rc = lib().oracle_agnn_backward(
+    fn = lib().oracle_agnn_backward_bf16 if bf16 else lib().oracle_agnn_backward
+    rc = fn(
         _i64(n), _p(rp), _p(ci), ctypes.c_int(k), ctypes.c_int(kout), _p(H), _p(W),
         ctypes.c_double(beta), ctypes.c_double(eps), ctypes.c_int(ACT[act]),
         _p(fwd["nu"]), _p(fwd["alpha"]), _p(fwd["X"]), _p(fwd["Z"]), _p(dHout),
@@ -151,9 +161,10 @@ def agnn_backward(rp, ci, H, W, fwd, dHout, beta=1.0, eps=1e-12, act="relu"):
     return out
 
 
-def va_forward(rp, ci, H, W, act="relu"):
+def va_forward(rp, ci, H, W, act="relu", bf16=False):
+    """bf16: BF16 storage mode (reading B2): the layer computes on H~ = bf16(H)."""
     rp, ci, n, nnz = _csr(rp, ci)
-    H, W = _d(H), _d(W)
+    H, W = (bf16_round(H) if bf16 else _d(H)), _d(W)
     k, kout = W.shape
     out = {"S": np.zeros(nnz), "X": np.zeros((n, k)), "Z": np.zeros((n, kout)),
            "Hout": np.zeros((n, kout))}
@@ -165,12 +176,14 @@ def va_forward(rp, ci, H, W, act="relu"):
     return out
 
 
-def va_backward(rp, ci, H, W, fwd, dHout, act="relu"):
+def va_backward(rp, ci, H, W, fwd, dHout, act="relu", bf16=False):
+    """bf16: BF16 storage mode (reading B2): H~ = bf16(H) and M~ = bf16(G W^T)."""
     rp, ci, n, nnz = _csr(rp, ci)
-    H, W, dHout = _d(H), _d(W), _d(dHout)
+    H, W, dHout = (bf16_round(H) if bf16 else _d(H)), _d(W), _d(dHout)
     k, kout = W.shape
     out = {"dH": np.zeros((n, k)), "dW": np.zeros((k, kout))}
-    rc = lib().oracle_va_backward(
+    fn = lib().oracle_va_backward_bf16 if bf16 else lib().oracle_va_backward
+    rc = fn(
         _i64(n), _p(rp), _p(ci), ctypes.c_int(k), ctypes.c_int(kout), _p(H), _p(W),
         ctypes.c_int(ACT[act]), _p(fwd["S"]), _p(fwd["X"]), _p(fwd["Z"]), _p(dHout),
         _p(out["dH"]), _p(out["dW"]))
@@ -219,11 +232,12 @@ def layer(model, rp, ci, H, W, a=None, heads=1, dHout=None, act="relu", slope=0.
         b = (gat_backward(rp, ci, H, W, a, heads, f, dHout, slope, act, bf16)
              if dHout is not None else None)
     elif model == "agnn":
-        f = agnn_forward(rp, ci, H, W, beta, eps, act)
-        b = agnn_backward(rp, ci, H, W, f, dHout, beta, eps, act) if dHout is not None else None
+        f = agnn_forward(rp, ci, H, W, beta, eps, act, bf16)
+        b = (agnn_backward(rp, ci, H, W, f, dHout, beta, eps, act, bf16)
+             if dHout is not None else None)
     elif model == "va":
-        f = va_forward(rp, ci, H, W, act)
-        b = va_backward(rp, ci, H, W, f, dHout, act) if dHout is not None else None
+        f = va_forward(rp, ci, H, W, act, bf16)
+        b = va_backward(rp, ci, H, W, f, dHout, act, bf16) if dHout is not None else None
     elif model == "cgnn":
         f = cgnn_forward(rp, ci, H, W, agg, act)
         b = cgnn_backward(rp, ci, H, W, f, dHout, agg, act) if dHout is not None else None

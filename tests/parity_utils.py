@@ -104,11 +104,13 @@ def oracle_step(w: gen.Workload, rp, ci, H, Ws, As, R):
                                     w.slope, w.act, bf16=w.prec == "bf16")
             das[l] = b["da"]
         elif w.model == "agnn":
-            b = oracle.agnn_backward(rp, ci, Hs[l], Ws[l], fwd[l], dHs[l + 1], w.beta, w.eps, w.act)
+            b = oracle.agnn_backward(rp, ci, Hs[l], Ws[l], fwd[l], dHs[l + 1], w.beta, w.eps, w.act,
+                                     bf16=w.prec == "bf16")
         elif w.model == "cgnn":
             b = oracle.cgnn_backward(rp, ci, Hs[l], Ws[l], fwd[l], dHs[l + 1], w.agg, w.act)
         else:
-            b = oracle.va_backward(rp, ci, Hs[l], Ws[l], fwd[l], dHs[l + 1], w.act)
+            b = oracle.va_backward(rp, ci, Hs[l], Ws[l], fwd[l], dHs[l + 1], w.act,
+                                   bf16=w.prec == "bf16")
         dHs[l], dWs[l] = b["dH"], b["dW"]
     return {"H": Hs, "fwd": fwd, "dH": dHs, "dW": dWs, "da": das}
 

@@ -574,3 +574,38 @@ def test_bf16_mode_within_the_north_star_bound():
     assert 0 < rel(f1["Z"], f0["Z"]) < 1e-2
     for key in ("dH", "dW"):
         assert 0 < rel(b1[key], b0[key]) < 1e-2
+
+
+@pytest.mark.parametrize("model", ["agnn", "va"])
+def test_agnn_va_bf16_mode_exact_when_representable(model):
+    """Reading B2 (AGNN / VA BF16 storage): the mode computes the fp64 layer on
+    H~ = bf16(H) with M~ = bf16(G W^T).  With H and M bf16-representable (H in
+    {-1, 0, 1}, W and R on a 2^-3 grid, act none, so G = R and M = R W^T lands on
+    the 2^-6 grid below 2^8) both roundings are exact and the mode IS the fp64 oracle."""
+    rng = np.random.default_rng(41)
+    n, k = 14, 8
+    rp, ci = rand_graph(n, 0.3, rng)
+    H = rng.integers(-1, 2, (n, k)).astype(np.float64)
+    W = rng.integers(-2, 3, (k, k)) * 0.125
+    R = rng.integers(-2, 3, (n, k)) * 0.125
+    f0, b0 = oracle.layer(model, rp, ci, H, W, dHout=R, act="none")
+    f1, b1 = oracle.layer(model, rp, ci, H, W, dHout=R, act="none", bf16=True)
+    for x, y in ((f0["Z"], f1["Z"]), (b0["dH"], b1["dH"]), (b0["dW"], b1["dW"])):
+        np.testing.assert_array_equal(x, y)
+
+
+@pytest.mark.parametrize("model", ["agnn", "va"])
+def test_agnn_va_bf16_mode_rounds_and_stays_within_bound(model):
+    """Generic inputs: the mode differs from the unrounded oracle (the rounding is
+    real) by far less than north_star's 1e-2, and equals the unrounded oracle run on
+    the rounded input H~ in the forward (only M's rounding is inside the backward)."""
+    rng = np.random.default_rng(42)
+    n, k = 16, 8
+    rp, ci = rand_graph(n, 0.3, rng)
+    H, W, _, R = rand_inputs(n, k, k, 1, rng)
+    f0, b0 = oracle.layer(model, rp, ci, H, W, dHout=R, act="elu")
+    f1, b1 = oracle.layer(model, rp, ci, H, W, dHout=R, act="elu", bf16=True)
+    fr, _ = oracle.layer(model, rp, ci, oracle.bf16_round(H), W, act="elu")
+    np.testing.assert_array_equal(f1["Z"], fr["Z"])
+    assert 1e-6 < rel(b1["dH"], b0["dH"]) < 1e-2
+    assert 1e-6 < rel(f1["Z"], f0["Z"]) < 1e-2
