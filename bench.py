@@ -67,7 +67,8 @@ def parse():
     p.add_argument("--no-bf16-line", action="store_true",
                    help="skip the extra BF16-storage measurement of GAT k'=128 workloads")
     p.add_argument("--prec", default="fp32", choices=["fp32", "bf16"],
-                   help="GAT feature storage: fp32, or bf16 (P and G stored as bfloat16, "
+                   help="feature storage: fp32, or bf16 (GAT: P and G, AGNN/VA: H and M stored "
+                        "as bfloat16, "
                         "fp32 arithmetic; include/agnn.h AGNN_PREC_BF16, reading B1)")
     p.add_argument("--scale", type=int, default=None,
                    help="override log2 n of the workload (same recipe and edge factor)")
@@ -339,7 +340,8 @@ def pass_bytes(w, m, n, factored_mode=1):
     GAT backward, unfactored: per edge 4 + P_i and G_i rows + rec_i and t_i
       (20 h); per row P_j, G_j read, dP_j written, record + t (20 h), row_ptr.
     AGNN/VA backward: per edge 4 + 2 k f (+16 AGNN record); per row H_j, M_j read,
-      dH_j written (3 k f) (+16) + 8.
+      dH_j written (3 k f) (+16) + 8.  BF16 storage (reading B2): H~, M~ rows are
+      2 k bytes (dH stays fp32).
     """
     f = 4
     out = {}
@@ -355,8 +357,9 @@ def pass_bytes(w, m, n, factored_mode=1):
             pe, pr = 4 + 2 * w.k * fs + 20 * w.heads, 2 * w.k * fs + w.k * f + 20 * w.heads + 8
         out["bwd"] = (pe * m + pr * n, pe, pr)
     else:
+        fs = 2 if w.prec == "bf16" else 4
         rec = 16 if w.model == "agnn" else 0
-        pe, pr = 4 + 2 * w.k * f + rec, 3 * w.k * f + rec + 8
+        pe, pr = 4 + 2 * w.k * fs + rec, 2 * w.k * fs + w.k * f + rec + 8
         out["bwd"] = (pe * m + pr * n, pe, pr)
     return out
 
@@ -695,7 +698,8 @@ def run_ours(args):
     # G stored as bfloat16 (include/agnn.h AGNN_PREC_BF16, reading B1: fp32
     # arithmetic, bf16 storage of the gathered rows), device-timed the same way.
     bf16 = None
-    if (w.model == "gat" and w.k == 128 and w.prec == "fp32" and not args.no_bf16_line
+    bf16_ok = ((w.model == "gat" and w.k == 128) or (w.model in ("agnn", "va") and w.k in (128, 256)))
+    if (bf16_ok and w.prec == "fp32" and not args.no_bf16_line
             and uid is None):  # (an NCCL unique id serves one communicator)
         import dataclasses
         w16 = dataclasses.replace(w, prec="bf16")
@@ -722,7 +726,9 @@ def run_ours(args):
             ms16 = float(t.item())
         bf16 = {"value": w.layers * m / (ms16 / 1e3 / args.steps), "unit": UNIT,
                 "ms_per_step": ms16 / args.steps, "dtype": "f32",
-                "storage": "bf16 P, G (fp32 arithmetic; AGNN_PREC_BF16, reading B1)",
+                "storage": ("bf16 P, G (fp32 arithmetic; AGNN_PREC_BF16, reading B1)"
+                            if w.model == "gat" else
+                            "bf16 H, M (fp32 arithmetic; AGNN_PREC_BF16, reading B2)"),
                 "tolerance": "1e-2 normwise (north_star 'BF16 projection')",
                 "roofline": roofline(args, w16, s16, prof16, world), "gpu_launches": l16,
                 "kernels": {k: {"launches": v[0], "ms_per_step": v[1] / args.steps}
@@ -736,8 +742,8 @@ def run_ours(args):
                 "dtype": "f32", "data": "synthetic",
                 "config": {"workload": args.config, "model": w.model, "graph": w.graph,
                            "n": n, "edges": m, "k": w.k, "heads": w.heads, "layers": w.layers,
-                           "storage": ("bf16 P, G (fp32 arithmetic; AGNN_PREC_BF16, tol 1e-2)"
-                                       if w.prec == "bf16" else "fp32"),
+                           "storage": ("bf16 gathered rows (fp32 arithmetic; AGNN_PREC_BF16, "
+                                       "tol 1e-2)" if w.prec == "bf16" else "fp32"),
                            "parallelism": f"1d-rowblock{world}",
                            "comm": (args.comm if world > 1 else None),
                            "l2_flush": "inputs > L2 (126 MB)" if not small else

@@ -97,7 +97,7 @@ typedef enum { AGNN_ACT_NONE = 0, AGNN_ACT_RELU = 1, AGNN_ACT_ELU = 2 } agnn_act
 
 /* precision mode.  Arithmetic is fp32 everywhere (dense projection: fp32 FFMA
  * or 3xTF32 on tcgen05, both fp32-accurate; sparse passes: fp32 FMA).
- * AGNN_PREC_BF16 (GAT only, k_out = 128, heads 1/2/4/8, symmetric pattern):
+ * AGNN_PREC_BF16 (GAT, k_out = 128, heads 1/2/4/8, symmetric pattern):
  * the gathered feature rows are STORED as bfloat16 — the projection P = HW
  * (rounded to nearest-even from the fp32 GEMM result; the scores s, t come from
  * the unrounded product, a' = Wa being its own GEMM column) and
@@ -105,11 +105,16 @@ typedef enum { AGNN_ACT_NONE = 0, AGNN_ACT_RELU = 1, AGNN_ACT_ELU = 2 } agnn_act
  * delta, dalpha, the aggregation of G).  Everything else (H, Z, H_out, dP, dW,
  * da, dH, the saved statistics) stays fp32.  This is north_star's "BF16
  * projection" mode, tolerance 1e-2 normwise (reading B1); it halves
- * the bytes of every gather.  Other shapes: AGNN_EUNSUPPORTED.             */
+ * the bytes of every gather.
+ * AGNN / VA (k_in = 128 / 256, symmetric pattern; reading B2): the gathered
+ * operands are the layer input and the backward's M = G W^T, so the layer
+ * computes on H~ = bf16(H) throughout (scores, norms nu, aggregation X = Psi H~)
+ * and the backward uses M~ = bf16(M) (rounded in the GEMM epilogue); X, Z, G,
+ * dW, dH and all statistics are fp32.  Other shapes: AGNN_EUNSUPPORTED.      */
 typedef enum {
   AGNN_PREC_FP32 = 0,    /* fp32 FFMA, or 3xTF32 on tcgen05 (fp32-accurate)  */
   AGNN_PREC_TF32X3 = 1,  /* same arithmetic as FP32 (the tcgen05 path is used wherever it has a shape) */
-  AGNN_PREC_BF16 = 2     /* GAT: P and G stored as bfloat16 (reading B1)      */
+  AGNN_PREC_BF16 = 2     /* GAT: P, G stored as bf16 (B1); AGNN/VA: H, M (B2) */
 } agnn_prec;
 
 /* agnn_csr.flags.

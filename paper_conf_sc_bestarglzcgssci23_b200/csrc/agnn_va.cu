@@ -173,6 +173,31 @@ nu_kernel(const float* __restrict__ H, int64_t n_local, float eps, float* __rest
   }
 }
 
+// BF16 storage (reading B2): H~ = bf16(H) of the local rows into the (replicated) H16
+// at their global offsets, and AGNN's nu_i = max(|H~_i|, eps) of the rounded row
+template <int K>
+__global__ void __launch_bounds__(kSparseThreads)
+av_round_kernel(const float* __restrict__ H, int64_t n_local, float eps, bf16* __restrict__ H16,
+                float* __restrict__ nu) {
+  using L = RowLayout<K, 1>;
+  const int lane = threadIdx.x & 31, g = lane / L::LANES, q = lane % L::LANES;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const int64_t slots = (n_local + L::GROUPS - 1) / L::GROUPS;
+  for (int64_t rs = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; rs < slots; rs += nw) {
+    const int64_t row = rs * L::GROUPS + g;
+    const bool ok = row < n_local;
+    float d[L::VPL];
+#pragma unroll
+    for (int v = 0; v < L::VPL; ++v) {
+      const float4 h = ok ? round_bf4(ldg4(H + row * K + L::col(v, q))) : f4(0.f);
+      if (ok) st4(H16 + row * K + L::col(v, q), h);
+      d[v] = dot4(h, h);
+    }
+    L::head_reduce(d);
+    if (ok && q == 0 && nu) nu[row] = fmaxf(sqrtf(d[0]), eps);
+  }
+}
+
 // ---------------------------------------------------------------- backward
 
 
@@ -194,7 +219,8 @@ __device__ __forceinline__ void bwd_store(const AvBwd& A, int64_t row, int64_t g
   float pr[L::VPL];
 #pragma unroll
   for (int v = 0; v < L::VPL; ++v) {
-    Hj[v] = ldg4(A.H + grow * K + L::col(v, q));
+    // (BF16 mode, heavy-row merge: the rounded row H~_j the layer computes on)
+    Hj[v] = A.H16 ? ldg4(A.H16 + grow * K + L::col(v, q)) : ldg4(A.H + grow * K + L::col(v, q));
     pr[v] = dot4(dh[v], Hj[v]);
   }
   L::head_reduce(pr);  // every lane participates (uniform)
@@ -377,10 +403,10 @@ __global__ void grad_act_kernel(const float* __restrict__ dHout, const float* __
   }
 }
 
-// rec_i = {nu_i, |beta|, 1/l_i, delta_i = M_i . X_i}   (AGNN)
-template <int K>
+// rec_i = {nu_i, |beta|, 1/l_i, delta_i = M_i . X_i}   (AGNN; TM = bf16: M~, reading B2)
+template <int K, typename TM = float>
 __global__ void __launch_bounds__(kSparseThreads)
-agnn_rec_kernel(int64_t n_local, int64_t row_begin, const float* __restrict__ M,
+agnn_rec_kernel(int64_t n_local, int64_t row_begin, const TM* __restrict__ M,
                 const float* __restrict__ X, const float* __restrict__ nu,
                 const float* __restrict__ l, float bound, float4* __restrict__ rec) {
   using L = RowLayout<K, 1>;
@@ -405,7 +431,8 @@ agnn_rec_kernel(int64_t n_local, int64_t row_begin, const float* __restrict__ M,
 
 __global__ void av_debug_kernel(const int64_t* __restrict__ rp, int64_t n_local,
                                 const int32_t* __restrict__ col, int64_t row_begin,
-                                const float* __restrict__ H, int K, const float* __restrict__ nu,
+                                const float* __restrict__ H, const bf16* __restrict__ H16, int K,
+                                const float* __restrict__ nu,
                                 const float* __restrict__ l, int model, float beta, float bound,
                                 const int64_t* __restrict__ pos, int64_t count,
                                 float* __restrict__ out) {
@@ -419,7 +446,11 @@ __global__ void av_debug_kernel(const int64_t* __restrict__ rp, int64_t n_local,
   }
   const int64_t i = row_begin + lo, j = col[e];
   float s = 0.f;
-  for (int c = 0; c < K; ++c) s = fmaf(H[i * K + c], H[j * K + c], s);
+  if (H16)
+    for (int c = 0; c < K; ++c)
+      s = fmaf(__bfloat162float(H16[i * K + c]), __bfloat162float(H16[j * K + c]), s);
+  else
+    for (int c = 0; c < K; ++c) s = fmaf(H[i * K + c], H[j * K + c], s);
   if (model == VA) {
     out[t] = s;
   } else {
@@ -427,13 +458,17 @@ __global__ void av_debug_kernel(const int64_t* __restrict__ rp, int64_t n_local,
   }
 }
 
+bool av_bf16(const agnn_layer_desc& d) { return d.prec == AGNN_PREC_BF16; }
+
 struct SavedAv {
   float *Hfull, *nu, *X, *Z, *l;
+  bf16* H16;  // BF16 mode (reading B2): H~ [n x k_in] (replicated), replaces Hfull
 };
 SavedAv carve_saved(const Plan& p, const agnn_layer_desc& d, void* base, size_t* total) {
   Carver c(base);
   SavedAv s;
-  s.Hfull = c.take<float>(p.world > 1 ? (size_t)p.n * d.k_in : 0);
+  s.H16 = c.take<bf16>(av_bf16(d) ? (size_t)p.n * d.k_in : 0);
+  s.Hfull = c.take<float>(p.world > 1 && !av_bf16(d) ? (size_t)p.n * d.k_in : 0);
   s.nu = c.take<float>(d.kind == AGNN_AGNN ? (size_t)p.n : 0);
   s.X = c.take<float>((size_t)p.n_local * d.k_in);
   s.Z = c.take<float>((size_t)p.n_local * d.k_out);
@@ -446,6 +481,7 @@ struct WsAv {
   float *pacc, *pl, *G, *M, *gemm, *WT, *dhp;
   float4* rec;
   void* saved_inf;
+  bf16* M16;  // BF16 mode (reading B2): M~ [n x k_in] (replicated), replaces M
 };
 WsAv carve_ws(const Plan& p, const agnn_layer_desc& d, void* base, size_t* total) {
   Carver c(base);
@@ -453,7 +489,9 @@ WsAv carve_ws(const Plan& p, const agnn_layer_desc& d, void* base, size_t* total
   size_t sv = 0;
   carve_saved(p, d, nullptr, &sv);
   // replicated (n-row) arrays first (same offsets on every rank; peer exchange)
-  w.M = c.take<float>((size_t)p.n * d.k_in);
+  w.M16 = c.take<bf16>(av_bf16(d) ? (size_t)p.n * d.k_in : 0);
+  // (BF16 mode: fp32 scratch of the local rows, used only by shapes without tcgen05)
+  w.M = c.take<float>(av_bf16(d) ? (size_t)p.n_local * d.k_in : (size_t)p.n * d.k_in);
   w.rec = c.take<float4>(d.kind == AGNN_AGNN ? (size_t)p.n : 0);
   w.saved_inf = c.take<char>(sv);  // its replicated prefix (H_full, nu) too
   w.pacc = c.take<float>((size_t)p.max_chunks() * 2 * d.k_in);
@@ -500,12 +538,24 @@ agnn_status av_forward(const Plan& p, const agnn_layer_desc& d, const float* W, 
   const bool ag = d.kind == AGNN_AGNN;
   agnn_status st;
   const float* Hf = H_in;
-  if (ag) {
+  const bool b16 = av_bf16(d);
+  if (b16) {
+    if (p.directed() || !(K_ == 128 || K_ == 256))
+      return fail(AGNN_EUNSUPPORTED, "AGNN/VA BF16: symmetric patterns with k_in = 128 / 256");
+    AGNN_AV_DISPATCH(K_, (av_round_kernel<K><<<grid_of(av_round_kernel<K>), kSparseThreads, 0, s>>>(
+                             H_in, p.n_local, d.eps, sv.H16 + p.row_begin * d.k_in,
+                             ag ? sv.nu + p.row_begin : nullptr)));
+    AGNN_LAUNCH_CHECK("av_round_kernel");
+    if (p.world > 1) {
+      const RowArray ra[2] = {{reinterpret_cast<float*>(sv.H16), d.k_in / 2}, {sv.nu, 1}};
+      if ((st = allgather_rows(p, ra, ag ? 2 : 1, s)) != AGNN_OK) return st;
+    }
+  } else if (ag) {
     AGNN_AV_DISPATCH(K_, (nu_kernel<K><<<grid_of(nu_kernel<K>), kSparseThreads, 0, s>>>(
                              H_in, p.n_local, d.eps, sv.nu + p.row_begin)));
     AGNN_LAUNCH_CHECK("nu_kernel");
   }
-  if (p.world > 1) {
+  if (p.world > 1 && !b16) {
     AGNN_CUDA_TRY(cudaMemcpyAsync(sv.Hfull + p.row_begin * d.k_in, H_in,
                                   sizeof(float) * p.n_local * d.k_in, cudaMemcpyDeviceToDevice, s));
     const RowArray ra[2] = {{sv.Hfull, d.k_in}, {sv.nu, 1}};
@@ -513,10 +563,10 @@ agnn_status av_forward(const Plan& p, const agnn_layer_desc& d, const float* W, 
     Hf = sv.Hfull;
   }
   Items it = items_of(p);
-  AvFwd A{Hf, sv.nu, d.beta, fabsf(d.beta), sv.X, sv.l, w.pacc, w.pl};
+  AvFwd A{Hf, b16 ? sv.H16 : nullptr, sv.nu, d.beta, fabsf(d.beta), sv.X, sv.l, w.pacc, w.pl};
   if (K_ == 128 || K_ == 256) {
     // gathered per entry: an H_j row (+ nu_j)
-    const Items ith = l2_hinted(it, p, 4 * (int64_t)K_ + (ag ? 4 : 0));
+    const Items ith = l2_hinted(it, p, (b16 ? 2 : 4) * (int64_t)K_ + (ag ? 4 : 0));
     if ((st = av_fwd_batched(ith, K_, ag, A, s)) != AGNN_OK) return st;
   } else if (it.n_chunks + it.n_light > 0) {
     if (ag) AGNN_AV_DISPATCH(K_, (av_fwd_kernel<K, AG, av_fwd_unroll<K>()>
@@ -562,23 +612,44 @@ agnn_status av_backward(const Plan& p, const agnn_layer_desc& d, const float* W,
   if (p.world > 1 && (st = allreduce_sum(p, dW, (int64_t)d.k_in * d.k_out, s)) != AGNN_OK) return st;
   if (!dH_in) return AGNN_OK;
   // M = G W^T (Eq. 12) for the local rows; with P > 1 the rows the other ranks
-  // reference (and AGNN's records) then go to their replicas (comm.cu)
-  float* Mloc = w.M + p.row_begin * d.k_in;
-  if ((st = gemm_rows(w.G, p.n_local, d.k_out, W, true, d.k_in, Mloc, d.k_in, nullptr, s)) !=
-      AGNN_OK)
-    return st;
-  if (ag) {
-    AGNN_AV_DISPATCH(K_, (agnn_rec_kernel<K><<<grid_of(agnn_rec_kernel<K>), kSparseThreads, 0, s>>>(
-                             p.n_local, p.row_begin, w.M, sv.X, sv.nu, sv.l, fabsf(d.beta), w.rec)));
-    AGNN_LAUNCH_CHECK("agnn_rec_kernel");
-  }
-  if (p.world > 1) {
-    const RowArray ra[2] = {{w.M, d.k_in}, {reinterpret_cast<float*>(w.rec), 4}};
-    if ((st = allgather_rows(p, ra, ag ? 2 : 1, s)) != AGNN_OK) return st;
+  // reference (and AGNN's records) then go to their replicas (comm.cu).  BF16 mode
+  // (reading B2): the GEMM epilogue stores M~ = bf16(M), used everywhere after.
+  const bool b16 = av_bf16(d);
+  if (b16) {
+    if ((st = gemm_rows_bf16(w.G, p.n_local, d.k_out, W, d.k_in, w.M16 + p.row_begin * d.k_in,
+                             d.k_in, nullptr, w.M, s)) != AGNN_OK)
+      return st;
+    if (ag) {
+      AGNN_AV_DISPATCH(K_, (agnn_rec_kernel<K, bf16><<<grid_of(agnn_rec_kernel<K, bf16>),
+                                                      kSparseThreads, 0, s>>>(
+                               p.n_local, p.row_begin, w.M16, sv.X, sv.nu, sv.l, fabsf(d.beta),
+                               w.rec)));
+      AGNN_LAUNCH_CHECK("agnn_rec_kernel");
+    }
+    if (p.world > 1) {
+      const RowArray ra[2] = {{reinterpret_cast<float*>(w.M16), d.k_in / 2},
+                              {reinterpret_cast<float*>(w.rec), 4}};
+      if ((st = allgather_rows(p, ra, ag ? 2 : 1, s)) != AGNN_OK) return st;
+    }
+  } else {
+    float* Mloc = w.M + p.row_begin * d.k_in;
+    if ((st = gemm_rows(w.G, p.n_local, d.k_out, W, true, d.k_in, Mloc, d.k_in, nullptr, s)) !=
+        AGNN_OK)
+      return st;
+    if (ag) {
+      AGNN_AV_DISPATCH(K_, (agnn_rec_kernel<K><<<grid_of(agnn_rec_kernel<K>), kSparseThreads, 0, s>>>(
+                               p.n_local, p.row_begin, w.M, sv.X, sv.nu, sv.l, fabsf(d.beta), w.rec)));
+      AGNN_LAUNCH_CHECK("agnn_rec_kernel");
+    }
+    if (p.world > 1) {
+      const RowArray ra[2] = {{w.M, d.k_in}, {reinterpret_cast<float*>(w.rec), 4}};
+      if ((st = allgather_rows(p, ra, ag ? 2 : 1, s)) != AGNN_OK) return st;
+    }
   }
   const float* Hf = p.world > 1 ? sv.Hfull : H_in;
   Items it = items_of(p);
-  AvBwd A{Hf, w.M, w.rec, d.beta, d.eps, dH_in, w.pacc, w.dhp};
+  AvBwd A{Hf, w.M, b16 ? sv.H16 : nullptr, b16 ? w.M16 : nullptr, w.rec, d.beta, d.eps, dH_in,
+          w.pacc, w.dhp};
   if (directed) {
 #define AV_PASS(ROLE_, ITEMS)                                                                      \
     do {                                                                                           \
@@ -607,7 +678,7 @@ agnn_status av_backward(const Plan& p, const agnn_layer_desc& d, const float* W,
   }
   if (K_ == 128 || K_ == 256) {
     // gathered per entry: the H_i and M_i rows (+ the record)
-    const Items ith = l2_hinted(it, p, 8 * (int64_t)K_ + (ag ? 16 : 0));
+    const Items ith = l2_hinted(it, p, (b16 ? 4 : 8) * (int64_t)K_ + (ag ? 16 : 0));
     if ((st = av_bwd_batched(ith, K_, ag, A, s)) != AGNN_OK) return st;
   } else if (it.n_chunks + it.n_light > 0) {
     if (ag) AGNN_AV_DISPATCH(K_, (av_bwd_kernel<K, AG, av_bwd_unroll<K>()>
@@ -635,9 +706,10 @@ agnn_status av_debug_attention(const Plan& p, const agnn_layer_desc& d, const vo
   if (count <= 0) return AGNN_OK;
   SavedAv sv = carve_saved(p, d, const_cast<void*>(saved), nullptr);
   const float* Hf = p.world > 1 ? sv.Hfull : H_in;
-  if (!Hf) return fail(AGNN_EINVAL, "debug_attention: AGNN/VA need H_in on one GPU");
+  const bf16* H16 = av_bf16(d) ? sv.H16 : nullptr;
+  if (!Hf && !H16) return fail(AGNN_EINVAL, "debug_attention: AGNN/VA need H_in on one GPU");
   av_debug_kernel<<<(unsigned)((count + 255) / 256), 256, 0, s>>>(
-      p.row_ptr, p.n_local, p.col_idx, p.row_begin, Hf, d.k_in, sv.nu, sv.l,
+      p.row_ptr, p.n_local, p.col_idx, p.row_begin, Hf, H16, d.k_in, sv.nu, sv.l,
       d.kind == AGNN_AGNN ? AG : VA, d.beta, fabsf(d.beta), pos, count, out);
   AGNN_LAUNCH_CHECK("av_debug_kernel");
   return AGNN_OK;

@@ -103,8 +103,11 @@ static agnn_status check_desc(const agnn_layer_desc& d) {
   if (d.prec < AGNN_PREC_FP32 || d.prec > AGNN_PREC_BF16) return fail(AGNN_EINVAL, "layer desc: prec");
   if (d.prec == AGNN_PREC_BF16 &&
       !(d.kind == AGNN_GAT && d.k_out == 128 &&
-        (d.heads == 1 || d.heads == 2 || d.heads == 4 || d.heads == 8)))
-    return fail(AGNN_EUNSUPPORTED, "AGNN_PREC_BF16: GAT with k_out = 128 and 1/2/4/8 heads only");
+        (d.heads == 1 || d.heads == 2 || d.heads == 4 || d.heads == 8)) &&
+      !((d.kind == AGNN_AGNN || d.kind == AGNN_VA) && (d.k_in == 128 || d.k_in == 256)))
+    return fail(AGNN_EUNSUPPORTED,
+                "AGNN_PREC_BF16: GAT with k_out = 128 and 1/2/4/8 heads, or AGNN / VA with "
+                "k_in = 128 / 256");
   if (d.kind == AGNN_GAT) {
     if (d.heads <= 0 || d.k_out % d.heads || (d.k_out / d.heads) % 4)
       return fail(AGNN_EINVAL, "GAT: k_out must split into heads of a multiple of 4 features");

@@ -7,6 +7,7 @@ namespace agnn {
 
 struct AvFwd {
   const float* H;     // [n_tot x K]  (replicated when world > 1)
+  const bf16* H16;    // BF16 mode (reading B2): H~ [n_tot x K] read instead of H
   const float* nu;    // [n_tot]      AGNN
   float beta, bound;  // bound = |beta|
   float* X;           // [n_local x K]
@@ -18,6 +19,8 @@ struct AvFwd {
 struct AvBwd {
   const float* H;      // [n_tot x K]
   const float* M;      // [n_tot x K]
+  const bf16* H16;     // BF16 mode (reading B2): H~, M~ [n_tot x K] read instead of H, M
+  const bf16* M16;
   const float4* rec;   // [n_tot] {nu, m, 1/l, delta}   AGNN
   float beta, eps;
   float* dH;           // [n_local x K]
@@ -29,6 +32,7 @@ enum { AV_VA = 0, AV_AG = 1 };
 
 // k = 128 / 256 batched lane-parallel kernels (av_batched.cu); symmetric patterns
 // (ROLE 0) only; AGNN_EUNSUPPORTED for other widths
+// (A.H16 != NULL: the BF16 storage variants, same arithmetic on the rounded rows)
 agnn_status av_fwd_batched(const Items& it, int k, bool agnn, const AvFwd& A, cudaStream_t s);
 agnn_status av_bwd_batched(const Items& it, int k, bool agnn, const AvBwd& A, cudaStream_t s);
 

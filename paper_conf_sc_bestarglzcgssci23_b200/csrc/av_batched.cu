@@ -22,11 +22,20 @@ using wb::FULL;
 using wb::item_of;
 using wb::Transpose;
 
-template <int B, int V>
+// TP = float (fp32 rows) or bf16 (BF16 storage, reading B2): the batches hold the raw
+// loaded slices and widen them at use, so a batch's loads stay in flight while the
+// previous batch is computed
+template <int B, int V, typename TP>
 struct FwdBatch {
-  float4 Hj[B][V];
+  typename Slice<TP>::raw Hj[B][V];
   float nuj;  // nu of the edge this lane owns after the reduction (AGNN)
 };
+template <typename TP>
+__device__ __forceinline__ const TP* pick_row(const float* f, const bf16* h);
+template <>
+__device__ __forceinline__ const float* pick_row<float>(const float* f, const bf16*) { return f; }
+template <>
+__device__ __forceinline__ const bf16* pick_row<bf16>(const float*, const bf16* h) { return h; }
 
 template <int V>
 __device__ __forceinline__ float dotv(const float4 (&a)[V], const float4 (&b)[V]) {
@@ -38,17 +47,19 @@ __device__ __forceinline__ float dotv(const float4 (&a)[V], const float4 (&b)[V]
 
 // X_i = sum_j w_ij H_j, w = exp(beta cos(H_i, H_j) - |beta|) (AGNN, l_i = sum w) or
 // w = H_i . H_j (VA)
-template <int K, int MODEL, int B, int MINB>
+template <int K, int MODEL, int B, int MINB, typename TP>
 __global__ void __launch_bounds__(256, MINB) av_fwd_batched_kernel(Items it, AvFwd A) {
   constexpr int V = K / 128;
   using TR = Transpose<B>;
+  using SL = Slice<TP>;
+  const TP* Hrow = pick_row<TP>(A.H, A.H16);
   const int lane = threadIdx.x & 31, cq = lane * 4;
   const int my_b = TR::edge_of(lane);
   const bool owner = (lane >> TR::T) == 0;
   const float beta = A.beta, bound = A.bound;
   const int64_t nitems = it.n_chunks + it.n_light;
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  const float* Hl = A.H + cq;
+  const TP* Hl = Hrow + cq;
   const Gath ga(it);  // L2 residency hints of the gathered rows (plan column classes)
   for (int64_t w = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; w < nitems; w += nw) {
     int64_t row, beg, end, slot;
@@ -57,12 +68,12 @@ __global__ void __launch_bounds__(256, MINB) av_fwd_batched_kernel(Items it, AvF
     float4 Hi[V], acc[V];
 #pragma unroll
     for (int v = 0; v < V; ++v) {
-      Hi[v] = ldg4(A.H + grow * K + v * 128 + cq);
+      Hi[v] = SL::f(SL::load(Hrow + grow * K + v * 128 + cq));
       acc[v] = f4(0.f);
     }
     const float scale_i = (MODEL == AV_AG) ? beta / __ldg(A.nu + grow) : 1.f;
     float lp = 0.f;
-    auto load = [&](FwdBatch<B, V>& q, int cidx, int off, int cnt) {
+    auto load = [&](FwdBatch<B, V, TP>& q, int cidx, int off, int cnt) {
 #pragma unroll
       for (int b = 0; b < B; ++b) {
         const int c = __shfl_sync(FULL, cidx, off + b);
@@ -70,17 +81,22 @@ __global__ void __launch_bounds__(256, MINB) av_fwd_batched_kernel(Items it, AvF
         const uint64_t pol = ga.policy(c);
 #pragma unroll
         for (int v = 0; v < V; ++v)
-          q.Hj[b][v] = b < cnt ? ldg4_pol(Hl + j * K + v * 128, pol) : f4(0.f);
+          q.Hj[b][v] = b < cnt ? SL::load(Hl + j * K + v * 128, pol) : SL::zero();
       }
       if (MODEL == AV_AG) {
         const int cm = __shfl_sync(FULL, cidx, off + my_b);
         q.nuj = my_b < cnt ? ldg1_pol(A.nu + ga.row(cm), ga.policy(cm)) : 1.f;
       }
     };
-    auto body = [&](const FwdBatch<B, V>& q, int cnt) {
+    auto body = [&](const FwdBatch<B, V, TP>& q, int cnt) {
+      float4 Hj[B][V];
+#pragma unroll
+      for (int b = 0; b < B; ++b)
+#pragma unroll
+        for (int v = 0; v < V; ++v) Hj[b][v] = SL::f(q.Hj[b][v]);
       float x[B];
 #pragma unroll
-      for (int b = 0; b < B; ++b) x[b] = dotv<V>(Hi, q.Hj[b]);
+      for (int b = 0; b < B; ++b) x[b] = dotv<V>(Hi, Hj[b]);
       TR::template reduce<32>(x, lane);
       float wgt;
       if (MODEL == AV_AG) wgt = ex2((scale_i * x[0] / q.nuj - bound) * kLog2e);  // exp(c_ij - |beta|)
@@ -91,14 +107,14 @@ __global__ void __launch_bounds__(256, MINB) av_fwd_batched_kernel(Items it, AvF
       for (int b = 0; b < B; ++b) {
         const float wbv = __shfl_sync(FULL, wgt, TR::lane_of(b));
 #pragma unroll
-        for (int v = 0; v < V; ++v) acc[v] = fma4(wbv, q.Hj[b][v], acc[v]);
+        for (int v = 0; v < V; ++v) acc[v] = fma4(wbv, Hj[b][v], acc[v]);
       }
     };
     for (int64_t w0 = beg; w0 < end; w0 += 32) {
       const int wcnt = (int)(end - w0 < 32 ? end - w0 : 32);
       const int cidx = lane < wcnt ? __ldg(it.col + w0 + lane) : 0;
       if (wcnt == 32) {
-        FwdBatch<B, V> qa, qb;
+        FwdBatch<B, V, TP> qa, qb;
         load(qa, cidx, 0, B);
 #pragma unroll
         for (int bb = 0; bb < 32 / B; bb += 2) {
@@ -109,7 +125,7 @@ __global__ void __launch_bounds__(256, MINB) av_fwd_batched_kernel(Items it, AvF
         }
       } else {
         for (int off = 0; off < wcnt; off += B) {
-          FwdBatch<B, V> q;
+          FwdBatch<B, V, TP> q;
           const int cnt = wcnt - off < B ? wcnt - off : B;
           load(q, cidx, off, cnt);
           body(q, cnt);
@@ -135,9 +151,9 @@ __global__ void __launch_bounds__(256, MINB) av_fwd_batched_kernel(Items it, AvF
   }
 }
 
-template <int B, int V>
+template <int B, int V, typename TP>
 struct BwdBatchAV {
-  float4 Hi[B][V], Mi[B][V];
+  typename Slice<TP>::raw Hi[B][V], Mi[B][V];
   float4 ri;  // record {nu, m, 1/l, delta} of the owned edge's vertex (AGNN)
 };
 
@@ -145,18 +161,21 @@ struct BwdBatchAV {
 //   VA   dH_j += (M_j.H_i + M_i.H_j) H_i + (H_i.H_j) M_i
 //   AGNN dH^_j += beta (a_ji (M_j.H_i - d_j) + a_ij (M_i.H_j - d_i)) H^_i,
 //        acc_j += a_ij M_i ;  dH_j = acc_j + (dH^_j - (dH^_j.H^_j) H^_j) / nu_j
-template <int K, int MODEL, int B, int MINB>
+template <int K, int MODEL, int B, int MINB, typename TP>
 __global__ void __launch_bounds__(256, MINB) av_bwd_batched_kernel(Items it, AvBwd A) {
   constexpr int V = K / 128;
   using TR = Transpose<B>;
+  using SL = Slice<TP>;
+  const TP* Hrow = pick_row<TP>(A.H, A.H16);
+  const TP* Mrow = pick_row<TP>(A.M, A.M16);
   const int lane = threadIdx.x & 31, cq = lane * 4;
   const int my_b = TR::edge_of(lane);
   const float beta = A.beta;
   const int64_t nitems = it.n_chunks + it.n_light;
   const Gath ga(it);
   const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  const float* Hl = A.H + cq;
-  const float* Ml = A.M + cq;
+  const TP* Hl = Hrow + cq;
+  const TP* Ml = Mrow + cq;
   for (int64_t w = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; w < nitems; w += nw) {
     int64_t row, beg, end, slot;
     item_of(it, w, row, beg, end, slot);
@@ -164,13 +183,13 @@ __global__ void __launch_bounds__(256, MINB) av_bwd_batched_kernel(Items it, AvB
     float4 Hj[V], Mj[V], dh[V], acc[V];
 #pragma unroll
     for (int v = 0; v < V; ++v) {
-      Hj[v] = ldg4(A.H + grow * K + v * 128 + cq);
-      Mj[v] = ldg4(A.M + grow * K + v * 128 + cq);
+      Hj[v] = SL::f(SL::load(Hrow + grow * K + v * 128 + cq));
+      Mj[v] = SL::f(SL::load(Mrow + grow * K + v * 128 + cq));
       dh[v] = acc[v] = f4(0.f);
     }
     const float4 rj = (MODEL == AV_AG) ? __ldg(A.rec + grow) : f4(1.f);
     const float sj = (MODEL == AV_AG) ? beta / rj.x : 0.f;
-    auto load = [&](BwdBatchAV<B, V>& q, int cidx, int off, int cnt) {
+    auto load = [&](BwdBatchAV<B, V, TP>& q, int cidx, int off, int cnt) {
 #pragma unroll
       for (int b = 0; b < B; ++b) {
         const int c = __shfl_sync(FULL, cidx, off + b);
@@ -179,10 +198,10 @@ __global__ void __launch_bounds__(256, MINB) av_bwd_batched_kernel(Items it, AvB
 #pragma unroll
         for (int v = 0; v < V; ++v) {
           if (b < cnt) {
-            q.Hi[b][v] = ldg4_pol(Hl + i * K + v * 128, pol);
-            q.Mi[b][v] = ldg4_pol(Ml + i * K + v * 128, pol);
+            q.Hi[b][v] = SL::load(Hl + i * K + v * 128, pol);
+            q.Mi[b][v] = SL::load(Ml + i * K + v * 128, pol);
           } else {
-            q.Hi[b][v] = q.Mi[b][v] = f4(0.f);
+            q.Hi[b][v] = q.Mi[b][v] = SL::zero();
           }
         }
       }
@@ -192,13 +211,21 @@ __global__ void __launch_bounds__(256, MINB) av_bwd_batched_kernel(Items it, AvB
                           : f4(1.f);
       }
     };
-    auto body = [&](const BwdBatchAV<B, V>& q, int cnt) {
+    auto body = [&](const BwdBatchAV<B, V, TP>& q, int cnt) {
+      float4 Hi[B][V], Mi[B][V];
+#pragma unroll
+      for (int b = 0; b < B; ++b)
+#pragma unroll
+        for (int v = 0; v < V; ++v) {
+          Hi[b][v] = SL::f(q.Hi[b][v]);
+          Mi[b][v] = SL::f(q.Mi[b][v]);
+        }
       float xs[B], x1[B], x2[B];
 #pragma unroll
       for (int b = 0; b < B; ++b) {
-        xs[b] = dotv<V>(Hj, q.Hi[b]);   // H_j . H_i
-        x1[b] = dotv<V>(Mj, q.Hi[b]);   // M_j . H_i  (row role)
-        x2[b] = dotv<V>(q.Mi[b], Hj);   // M_i . H_j  (column role)
+        xs[b] = dotv<V>(Hj, Hi[b]);   // H_j . H_i
+        x1[b] = dotv<V>(Mj, Hi[b]);   // M_j . H_i  (row role)
+        x2[b] = dotv<V>(Mi[b], Hj);   // M_i . H_j  (column role)
       }
       TR::template reduce<32>(xs, lane);
       TR::template reduce<32>(x1, lane);
@@ -223,9 +250,9 @@ __global__ void __launch_bounds__(256, MINB) av_bwd_batched_kernel(Items it, AvB
         const float cmb = __shfl_sync(FULL, cm, TR::lane_of(b));
 #pragma unroll
         for (int v = 0; v < V; ++v) {
-          dh[v] = fma4(chb, q.Hi[b][v], dh[v]);
-          if (MODEL == AV_VA) dh[v] = fma4(cmb, q.Mi[b][v], dh[v]);
-          else acc[v] = fma4(cmb, q.Mi[b][v], acc[v]);
+          dh[v] = fma4(chb, Hi[b][v], dh[v]);
+          if (MODEL == AV_VA) dh[v] = fma4(cmb, Mi[b][v], dh[v]);
+          else acc[v] = fma4(cmb, Mi[b][v], acc[v]);
         }
       }
     };
@@ -233,7 +260,7 @@ __global__ void __launch_bounds__(256, MINB) av_bwd_batched_kernel(Items it, AvB
       const int wcnt = (int)(end - w0 < 32 ? end - w0 : 32);
       const int cidx = lane < wcnt ? __ldg(it.col + w0 + lane) : 0;
       if (wcnt == 32) {
-        BwdBatchAV<B, V> qa, qb;
+        BwdBatchAV<B, V, TP> qa, qb;
         load(qa, cidx, 0, B);
 #pragma unroll
         for (int bb = 0; bb < 32 / B; bb += 2) {
@@ -244,7 +271,7 @@ __global__ void __launch_bounds__(256, MINB) av_bwd_batched_kernel(Items it, AvB
         }
       } else {
         for (int off = 0; off < wcnt; off += B) {
-          BwdBatchAV<B, V> q;
+          BwdBatchAV<B, V, TP> q;
           const int cnt = wcnt - off < B ? wcnt - off : B;
           load(q, cidx, off, cnt);
           body(q, cnt);
@@ -290,15 +317,26 @@ int grid_for(F* f) {
 // backward B = 4 (two batches of H_i, M_i in flight), 2 CTAs of 256 per SM; larger
 // batches or 3 CTAs per SM spill and lose 10-40 %.  k = 256 halves the batches
 // (same registers per batch).
+// (BF16 storage keeps the same batches: half the bytes per gathered row)
 template <int K, int MODEL>
 void launch_fwd(const Items& it, const AvFwd& A, cudaStream_t s) {
-  auto k = av_fwd_batched_kernel<K, MODEL, K == 128 ? 8 : 4, 2>;
-  k<<<grid_for(k), 256, 0, s>>>(it, A);
+  if (A.H16) {
+    auto k = av_fwd_batched_kernel<K, MODEL, K == 128 ? 8 : 4, 2, bf16>;
+    k<<<grid_for(k), 256, 0, s>>>(it, A);
+  } else {
+    auto k = av_fwd_batched_kernel<K, MODEL, K == 128 ? 8 : 4, 2, float>;
+    k<<<grid_for(k), 256, 0, s>>>(it, A);
+  }
 }
 template <int K, int MODEL>
 void launch_bwd(const Items& it, const AvBwd& A, cudaStream_t s) {
-  auto k = av_bwd_batched_kernel<K, MODEL, K == 128 ? 4 : 2, 2>;
-  k<<<grid_for(k), 256, 0, s>>>(it, A);
+  if (A.H16) {
+    auto k = av_bwd_batched_kernel<K, MODEL, K == 128 ? 4 : 2, 2, bf16>;
+    k<<<grid_for(k), 256, 0, s>>>(it, A);
+  } else {
+    auto k = av_bwd_batched_kernel<K, MODEL, K == 128 ? 4 : 2, 2, float>;
+    k<<<grid_for(k), 256, 0, s>>>(it, A);
+  }
 }
 
 }  // namespace

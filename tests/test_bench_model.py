@@ -48,6 +48,9 @@ def test_agnn_va_bytes(cfg, per_edge):
     b = _bench()
     w = gen.CONFIGS[cfg]
     assert b.pass_bytes(w, 1, 0)["bwd"][1] == per_edge
+    # BF16 storage (reading B2): the gathered H~, M~ rows at 2 bytes per feature
+    w16 = dataclasses.replace(w, prec="bf16")
+    assert b.pass_bytes(w16, 1, 0)["bwd"][1] == per_edge - 2 * w.k * 2
 
 
 def test_factored_mode_selection():

@@ -165,3 +165,59 @@ def test_bf16_unsupported_shapes_rejected(kind, k, heads):
     with pytest.raises(agnn.AgnnError) as e:
         agnn.Model(st.plan, [desc])
     assert e.value.status in (1, 5)  # EINVAL (k % heads) or EUNSUPPORTED
+
+
+# ------------------------------------------------------------------ AGNN / VA (reading B2)
+def WA(model, graph, scale, ef, k, layers=1, act="elu", n=None, samples=None):
+    n = n or (1 << scale)
+    return gen.Workload(f"{model}-bf16-{graph}{scale}-k{k}L{layers}-{act}", model, graph, scale, n,
+                        samples if samples is not None else ef * n, k, 1, layers, act=act,
+                        prec="bf16")
+
+
+AV_CASES = [
+    WA("agnn", "rmat", 13, 16, 128, layers=2),      # C3 shape (k = 128), heavy rows
+    WA("agnn", "kron", 12, 8, 256, act="none"),
+    WA("va", "kron", 12, 8, 256, act="none"),        # C4 shape (k = 256)
+    WA("va", "er", 0, 0, 128, n=3000, samples=30000, act="elu"),
+]
+
+
+@pytest.mark.parametrize("w", AV_CASES, ids=lambda w: w.name)
+def test_agnn_va_bf16_layer_parity(w):
+    """H~ = bf16(H) as the layer input and M~ = bf16(G W^T) (reading B2) against the
+    oracle's BF16 mode at north_star's 1e-2, the forward at the 2e-4 guard (the two
+    sides round the same fp32 input H, so H~ agrees exactly; later layers' inputs
+    differ by fp32 rounding)."""
+    src, dst, rp, ci = pu.host_graph(w)
+    g = pu.device_graph(w, src, dst)
+    H, Ws, As, R = w.host_inputs()
+    st = pu.gpu_step(w, graph=g, R=R)
+    ref = pu.oracle_step(w, rp, ci, H, Ws, As, R)
+    errs = pu.compare(w, st, ref, tol=pu.TOL_BF16)
+    fwd = {k: v for k, v in errs.items() if k.startswith("H") and not k.endswith(":row")}
+    assert max(fwd.values()) <= FWD_GUARD, errs
+    pu.compare_attention(w, st, ref)
+    ref32 = pu.oracle_step(dataclasses.replace(w, prec="fp32"), rp, ci, H, Ws, As, R)
+    assert pu.rel(st.dH[0].cpu().numpy(), ref32["dH"][0]) > 1e-5
+
+
+@pytest.mark.parametrize("model,k", [("agnn", 128), ("va", 256), ("agnn", 256)])
+def test_agnn_va_bf16_exact_operands_tight(model, k):
+    """H in {-1, 0, 1} and W, R in {-1, 0, 1} / 8 (act none): H~ = H and M~ = M exactly on
+    both sides, so the BF16 mode must meet 1e-4 on every output and row."""
+    w = WA(model, "kron", 12, 8, k, act="none")
+    src, dst, rp, ci = pu.host_graph(w)
+    g = pu.device_graph(w, src, dst)
+    rng = np.random.default_rng(9)
+    H = rng.integers(-1, 2, (w.n, k)).astype(np.float32)
+    Ws = [(rng.integers(-1, 2, (k, k)) * 0.125).astype(np.float32)]
+    R = (rng.integers(-1, 2, (w.n, k)) * 0.125).astype(np.float32)
+    st = runner.Stack(w, "cuda", graph=g)
+    st.H[0].copy_(torch.from_numpy(H))
+    st.W[0].copy_(torch.from_numpy(Ws[0]))
+    st.dH[1].copy_(torch.from_numpy(R))
+    st.step()
+    torch.cuda.synchronize()
+    ref = pu.oracle_step(w, rp, ci, H, Ws, [None], R)
+    pu.compare(w, st, ref, tol=EXACT_GUARD, all_rows=True, row_tol=1e-3)
