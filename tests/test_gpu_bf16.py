@@ -157,7 +157,8 @@ def test_bf16_saved_and_workspace_are_smaller():
     assert a.model.workspace_bytes(0) - b.model.workspace_bytes(0) >= 2 * n * k - 1024
 
 
-@pytest.mark.parametrize("kind,k,heads", [("agnn", 128, 1), ("gat", 64, 2), ("gat", 128, 3)])
+@pytest.mark.parametrize("kind,k,heads", [("agnn", 64, 1), ("va", 32, 1), ("cgnn", 128, 1),
+                                          ("gat", 64, 2), ("gat", 128, 3)])
 def test_bf16_unsupported_shapes_rejected(kind, k, heads):
     w = gen.CONFIGS["C1"]
     st = runner.Stack(w, "cuda")
