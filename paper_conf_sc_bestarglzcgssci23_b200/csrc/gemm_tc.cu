@@ -538,13 +538,19 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
 // Weight gradients Y = H^T dP / X^T G (PAPER.md:241 Eq. 5, :298 Eq. 13): the
 // reduction runs over the n rows, so both operands are MN-major for the MMA
 // (D[k1 x n] += A'[k1 x 8 rows] B'[8 rows x n]).  Each CTA reduces a contiguous
-// slab of rows: TMA brings 32-row chunks of A and B (128B-swizzled, MN-major
+// slab of rows: TMA brings TN_ROWS-row chunks of A and B (128B-swizzled, MN-major
 // atoms of 8 rows x 32 columns), threads split them 3xTF32, thread 0 issues
 // the MMAs; every TN_GROUP chunks the TMEM accumulator is drained into fp32
 // registers (one dW row per thread) so the tensor core's per-MMA rounding
-// never compounds over more than TN_GROUP * 12 accumulations.
-constexpr int TN_ROWS = 32;   // input rows per chunk
-constexpr int TN_GROUP = 2;   // chunks per TMEM drain
+// never compounds over more than TN_GROUP * 3 * TN_ROWS / 8 accumulations.
+// 16-row chunks (2 x 32 KB ring stages) so that three CTAs fit one SM (registers: the
+// 128-column fp32 dW row per thread): three independent TMA -> split -> MMA chains
+// per SM overlap each other's latencies.  Measured at M = 2^24, K1 = N = 128: 32-row
+// chunks with one CTA / SM 7.36 ms, 16-row chunks with 2 / SM 5.90 ms, with 3 / SM
+// 4.84 ms (scratch/time_gemm.py).
+constexpr int TN_ROWS = 16;   // input rows per chunk
+constexpr int TN_CTAS = 3;    // resident CTAs per SM
+constexpr int TN_GROUP = 2;   // chunks per TMEM drain (32 rows: 12 MMA accumulations)
 constexpr int64_t kTnMaxSlabs = 2048;  // fp32 partials per call (summed in fp64)
 
 // MN-major tf32 operands use the 128B swizzle with 32-byte atomicity (the only MN-major
@@ -557,7 +563,7 @@ __device__ __forceinline__ uint64_t sw128_mn_desc(uint32_t saddr, uint32_t lbo_b
 }
 
 template <int K1, int N>
-__global__ void __launch_bounds__(TC_THREADS, 1)
+__global__ void __launch_bounds__(TC_THREADS, TN_CTAS)
 gemm_tn_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                   int64_t M, int64_t rows_per_cta, float* __restrict__ part) {
   constexpr uint32_t LBO = TN_ROWS * 128;  // 32-column MN blocks (one TMA box each)
@@ -642,7 +648,7 @@ gemm_tn_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       const int li = isA ? i : i - A_BYTES / 16;
       uint8_t* hp = isA ? base + li * 16 : base + 2 * A_BYTES + li * 16;
       uint8_t* lp = hp + (isA ? A_BYTES : B_BYTES);
-      const int row = (li * 16 / 128) % TN_ROWS;   // 128-byte row inside a 32-row box
+      const int row = (li * 16 / 128) % TN_ROWS;   // 128-byte row inside a TN_ROWS-row box
       float4 x = *reinterpret_cast<const float4*>(hp);
       if (row >= valid_rows) x = f4(0.f);
       float4 hi, lo;
@@ -803,7 +809,7 @@ agnn_status launch_tn_tc(const float* A, int lda, int64_t M, const float* B, int
   rps = std::max<int64_t>(rps, 8192);
   rps = (rps + TN_ROWS - 1) / TN_ROWS * TN_ROWS;
   const int64_t nslabs = (M + rps - 1) / rps;
-  const int grid = (int)std::min<int64_t>(nslabs, sms);
+  const int grid = (int)std::min<int64_t>(nslabs, (int64_t)sms * TN_CTAS);
   gemm_tn_tc_kernel<K1, N><<<grid, TC_THREADS, smem, s>>>(ma, mb, M, rps, ws);
   AGNN_LAUNCH_CHECK("gemm_tn_kernel");
   const int64_t cnt = (int64_t)K1 * N;
