@@ -702,6 +702,218 @@ gemm_tn_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
                  : "memory");
 }
 
+// ---------------------------------------------------------------- C = A B^T, roles
+// Resident-B shapes (K <= 128): the same product as gemm_tc_kernel with every role
+// in its own warp(s), handing chunks on by mbarriers instead of a CTA barrier, so
+// no role waits for another's unrelated latency (the TMA issue no longer waits
+// behind the split, the split no longer waits for the MMA issue):
+//   warp 8  (producer, one lane): chunk g's TMA once the stage's previous MMAs are
+//           done (mma_bar), plus L2 prefetches further ahead;
+//   warps 0-3 (split): thread r splits row r of the landed chunk, hi in place, lo
+//           into a TMEM slot, then arrives on split_bar;
+//   warp 9  (MMA, one lane): the 12 tcgen05.mma of a chunk once it is split, into
+//           one of two TMEM accumulators (alternate tiles), commits mma_bar /
+//           acc_full;
+//   warps 4-7 (epilogue): drain the finished accumulator in 32-column parts and
+//           store, then release it (acc_empty) — the other accumulator keeps the
+//           tensor pipe busy meanwhile.
+// Accumulation groups: the tensor core rounds its fp32 accumulator once per MMA, so
+// where TMEM holds them (N <= 96: two buffers x two groups) the K chunks alternate
+// between NG = 2 accumulators summed by the epilogue; N = 128 / 144 keep one per
+// tile (the per-MMA rounding compounds over the tile's 48 MMAs: ~1e-6 normwise).
+constexpr int TCR_THREADS = 320;
+
+template <int N, int K, int S, int EPI>
+__global__ void __launch_bounds__(TCR_THREADS, 1)
+gemm_tc_roles_kernel(const __grid_constant__ CUtensorMap tmA, const float* __restrict__ B,
+                     int n_real, int64_t M, TcOut out) {
+  static_assert(N % 16 == 0 && N >= 16 && N <= 256, "UMMA N for M = 128");
+  static_assert(K % TC_KC == 0 && K <= 128, "resident B, K <= 128");
+  constexpr int KCH = K / TC_KC;
+  constexpr int A_BYTES = TC_BM * 128;
+  constexpr int BC_BYTES = N * 128;
+  constexpr int BRES = KCH * BC_BYTES;
+  // lo slots: as many as TMEM holds next to the two accumulators, and fewer than the
+  // stages (a slot's reuse waits on mma_bar of chunk g - LO_SLOTS, which must not have
+  // been reused by a later chunk yet: mbarrier parity tells only adjacent phases apart)
+  constexpr int NG = (KCH >= 2 && 4 * N + 2 * 32 <= 512) ? 2 : 1;
+  constexpr int LO_T = (2 * NG * N + 4 * 32 <= 512) ? 4 : 2;
+  constexpr int LO_SLOTS = LO_T < S - 1 ? LO_T : S - 1;
+  static_assert(LO_SLOTS >= 1, "lo slots");
+  constexpr uint32_t LO_COL = (uint32_t)(2 * NG * N);
+  constexpr uint32_t TMEM_NEED = (uint32_t)(2 * NG * N + 32 * LO_SLOTS);
+  static_assert(TMEM_NEED <= 512, "TMEM columns");
+  constexpr uint32_t TMEM_COLS = TMEM_NEED <= 32 ? 32 : TMEM_NEED <= 64 ? 64 : TMEM_NEED <= 128 ? 128
+                                 : TMEM_NEED <= 256 ? 256 : 512;
+  constexpr uint32_t IDESC = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(N >> 3) << 17) |
+                             ((uint32_t)(TC_BM >> 4) << 24);
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = smem_raw + ((1024u - (s_addr(smem_raw) & 1023u)) & 1023u);
+  uint8_t* Bh = smem;
+  uint8_t* Bl = smem + BRES;
+  uint8_t* ring = smem + 2 * BRES;
+  float* stg = reinterpret_cast<float*>(ring + S * A_BYTES);  // epilogue transpose, 4 x 32 x 36
+  __shared__ uint64_t tma_bar[S], mma_bar[S], split_bar[S], acc_full[2], acc_empty[2];
+  __shared__ uint32_t tmem_base_s;
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     s_addr(&tmem_base_s)),
+                 "r"(TMEM_COLS)
+                 : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+  }
+  if (tid == 0) {
+#pragma unroll
+    for (int i = 0; i < S; ++i) {
+      mbar_init(&tma_bar[i], 1);
+      mbar_init(&mma_bar[i], 1);
+      mbar_init(&split_bar[i], 128);
+    }
+    mbar_init(&acc_full[0], 1);
+    mbar_init(&acc_full[1], 1);
+    mbar_init(&acc_empty[0], 128);
+    mbar_init(&acc_empty[1], 128);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(&tmA) : "memory");
+  }
+  // B -> hi/lo tiles in the swizzled K-major layout (rows >= n_real are zero)
+  for (int idx = tid; idx < N * (K / 4); idx += TCR_THREADS) {
+    const int n = idx / (K / 4), c16 = idx % (K / 4), kc = c16 / 8, cc = c16 % 8;
+    float4 v = f4(0.f);
+    if (n < n_real) v = ldg4(B + (int64_t)n * K + c16 * 4);
+    float4 hi, lo;
+    split4(v, hi, lo);
+    const int off = kc * N * 128 + (n >> 3) * 1024 + (n & 7) * 128 + ((cc ^ (n & 7)) << 4);
+    *reinterpret_cast<float4*>(Bh + off) = hi;
+    *reinterpret_cast<float4*>(Bl + off) = lo;
+  }
+  fence_proxy_async();
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = tmem_base_s;
+  const int64_t ntiles = (M + TC_BM - 1) / TC_BM;
+  const int64_t first = blockIdx.x;
+  const int64_t my_tiles = first < ntiles ? (ntiles - 1 - first) / gridDim.x + 1 : 0;
+  const int64_t nchunks = my_tiles * KCH;
+
+  if (warp == 8) {  // ---------------------------------------------------- producer
+    if (lane == 0) {
+      for (int64_t g = 0; g < nchunks; ++g) {
+        const int st = (int)(g % S);
+        if (g >= S) mbar_wait(&mma_bar[st], (uint32_t)(((g - S) / S) & 1));
+        const int64_t t = first + (g / KCH) * gridDim.x;
+        mbar_expect_tx(&tma_bar[st], A_BYTES);
+        tma_load_2d(ring + st * A_BYTES, &tmA, &tma_bar[st], (int)(g % KCH) * TC_KC, (int)(t * TC_BM));
+        const int64_t gp = g + TC_PF;
+        if (gp < nchunks)
+          tma_prefetch_2d(&tmA, (int)(gp % KCH) * TC_KC, (int)((first + (gp / KCH) * gridDim.x) * TC_BM));
+      }
+    }
+  } else if (warp == 9) {  // ---------------------------------------------- MMA issue
+    if (lane == 0) {
+      for (int64_t g = 0; g < nchunks; ++g) {
+        const int st = (int)(g % S);
+        const int kc = (int)(g % KCH);
+        const int64_t tl = g / KCH;
+        const int b = (int)(tl & 1);
+        mbar_wait(&split_bar[st], (uint32_t)((g / S) & 1));
+        if (kc == 0 && tl >= 2) mbar_wait(&acc_empty[b], (uint32_t)(((tl - 2) >> 1) & 1));
+        tc_fence_after();
+        const uint32_t ah = s_addr(ring + st * A_BYTES);
+        const uint32_t bh = s_addr(Bh + kc * BC_BYTES), bl = s_addr(Bl + kc * BC_BYTES);
+        const uint32_t tacc = tmem + (uint32_t)((b * NG + kc % NG) * N);
+        const uint32_t lo_slot = LO_COL + (uint32_t)((g % LO_SLOTS) * 32);
+#pragma unroll
+        for (int ks = 0; ks < TC_KC / 8; ++ks) {
+          const uint32_t o = ks * 32;
+          const uint32_t acc0 = (kc >= NG || ks > 0) ? 1u : 0u;  // first MMA of the group
+          mma_tf32(tacc, sw128_desc(ah + o), sw128_desc(bh + o), IDESC, acc0);
+          mma_tf32(tacc, sw128_desc(ah + o), sw128_desc(bl + o), IDESC, 1u);
+          mma_tf32_ta(tacc, tmem + lo_slot + (uint32_t)(ks * 8), sw128_desc(bh + o), IDESC, 1u);
+        }
+        mma_commit(&mma_bar[st]);
+        if (kc == KCH - 1) mma_commit(&acc_full[b]);
+      }
+    }
+  } else if (warp < 4) {  // ------------------------------------------------- split
+    for (int64_t g = 0; g < nchunks; ++g) {
+      const int st = (int)(g % S);
+      mbar_wait(&tma_bar[st], (uint32_t)((g / S) & 1));
+      // the TMEM lo slot was last read by chunk g - LO_SLOTS's MMAs
+      if (g >= LO_SLOTS) mbar_wait(&mma_bar[(g - LO_SLOTS) % S], (uint32_t)(((g - LO_SLOTS) / S) & 1));
+      uint8_t* rowp = ring + st * A_BYTES + tid * 128;
+      float lo[32];
+#pragma unroll
+      for (int c = 0; c < 8; ++c) {
+        float4* q = reinterpret_cast<float4*>(rowp + ((c ^ (tid & 7)) << 4));
+        float4 hi, l4;
+        split4(*q, hi, l4);
+        *q = hi;
+        lo[4 * c] = l4.x;
+        lo[4 * c + 1] = l4.y;
+        lo[4 * c + 2] = l4.z;
+        lo[4 * c + 3] = l4.w;
+      }
+      tc_fence_after();
+      tmem_st32(tmem + ((uint32_t)(warp * 32) << 16) + LO_COL + (uint32_t)((g % LO_SLOTS) * 32), lo);
+      fence_proxy_async();
+      tc_fence_before();
+      mbar_arrive(&split_bar[st]);
+    }
+  } else {  // ------------------------------------------------------------- epilogue
+    const int ew = warp - 4;  // TMEM lanes 32 ew .. 32 ew + 31
+    float* wstg = stg + ew * 32 * 36;
+    for (int64_t tl = 0; tl < my_tiles; ++tl) {
+      const int b = (int)(tl & 1);
+      mbar_wait(&acc_full[b], (uint32_t)((tl >> 1) & 1));
+      tc_fence_after();
+      const uint32_t tbase = tmem + ((uint32_t)(ew * 32) << 16) + (uint32_t)(b * NG * N);
+      const int64_t t = first + tl * gridDim.x;
+      const int64_t row0 = t * TC_BM + ew * 32;
+      const int64_t row = row0 + lane;
+      const bool coal = (out.n_split & 3) == 0;
+#pragma unroll 1
+      for (int c0 = 0; c0 < N; c0 += 32) {
+        float q[32];
+#pragma unroll
+        for (int gi = 0; gi < NG; ++gi) {
+          uint32_t r[32];
+          tmem_ld16_issue(tbase + (uint32_t)(gi * N) + c0, r);
+          if (c0 + 16 < N) tmem_ld16_issue(tbase + (uint32_t)(gi * N) + c0 + 16, r + 16);
+          tmem_ld_wait();
+          tmem_reg_fence16(r);
+          if (c0 + 16 < N) tmem_reg_fence16(r + 16);
+#pragma unroll
+          for (int x = 0; x < 32; ++x) q[x] = gi == 0 ? __uint_as_float(r[x]) : q[x] + __uint_as_float(r[x]);
+        }
+        if (c0 + 32 <= N && coal && c0 + 32 <= out.n_split) {
+          store_block32<EPI>(out, row0, M, c0, q, wstg, lane);
+        } else if (row < M) {
+          float q16[16];
+#pragma unroll
+          for (int x = 0; x < 16; ++x) q16[x] = q[x];
+          store_row16<EPI>(out, row, c0, q16);
+          if (c0 + 16 < N) {
+#pragma unroll
+            for (int x = 0; x < 16; ++x) q16[x] = q[16 + x];
+            store_row16<EPI>(out, row, c0 + 16, q16);
+          }
+        }
+      }
+      tc_fence_before();
+      mbar_arrive(&acc_empty[b]);
+    }
+  }
+  __syncthreads();
+  if (warp == 0)
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem),
+                 "r"(TMEM_COLS)
+                 : "memory");
+}
+
 PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
   static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
   static std::once_flag once;
@@ -737,7 +949,32 @@ agnn_status launch_tc(const float* A, int64_t M, const float* B, int n_real, con
                 CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                 CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
     return fail(AGNN_ECUDA, "gemm_tc: tensor map encode failed");
-  if (!SB) mb = ma;  // unused
+  if constexpr (!SB) {
+    // resident B: the role-split kernel, as many 16 KB stages as fit next to B
+    constexpr int bres = 2 * (K / TC_KC) * N * 128;
+    constexpr int SR0 = (232448 - 2048 - bres - 4 * 32 * 36 * 4) / (TC_BM * 128);
+    constexpr int SR = SR0 > 8 ? 8 : SR0;
+    static_assert(SR >= 2, "ring stages");
+    constexpr int smem_r = bres + SR * TC_BM * 128 + 4 * 32 * 36 * 4 + 1024;
+    static bool attr_r = false;
+    if (!attr_r) {
+      cudaFuncSetAttribute(gemm_tc_roles_kernel<N, K, SR, EPI_PLAIN>,
+                           cudaFuncAttributeMaxDynamicSharedMemorySize, smem_r);
+      cudaFuncSetAttribute(gemm_tc_roles_kernel<N, K, SR, EPI_BF16>,
+                           cudaFuncAttributeMaxDynamicSharedMemorySize, smem_r);
+      attr_r = true;
+    }
+    int sms_r = kNumSMs, dev_r = 0;
+    if (cudaGetDevice(&dev_r) == cudaSuccess)
+      cudaDeviceGetAttribute(&sms_r, cudaDevAttrMultiProcessorCount, dev_r);
+    const int grid_r = (int)std::min<int64_t>((M + TC_BM - 1) / TC_BM, sms_r);
+    if (o.C0h)
+      gemm_tc_roles_kernel<N, K, SR, EPI_BF16><<<grid_r, TCR_THREADS, smem_r, s>>>(ma, B, n_real, M, o);
+    else
+      gemm_tc_roles_kernel<N, K, SR, EPI_PLAIN><<<grid_r, TCR_THREADS, smem_r, s>>>(ma, B, n_real, M, o);
+    AGNN_LAUNCH_CHECK("gemm_tc_kernel");
+    return AGNN_OK;
+  }
   constexpr int smem = (SB ? 0 : 2 * (K / TC_KC) * N * 128) +
                        S * (SB ? 2 * TC_BM * 128 + 2 * N * 128 : TC_BM * 128) + 4 * 32 * 36 * 4 +
                        1024;

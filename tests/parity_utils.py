@@ -86,6 +86,32 @@ def relu_kink_mask(w: gen.Workload, Z_last, R, rel_tau=1e-5):
     return R
 
 
+def tropical_tie_mask(w, rp, ci, Hin, R, rel_tau=1e-5):
+    """Multi-layer max/min C-GNN: zero the upstream gradient rows i whose layer-L
+    aggregation has a near tie (top-2 neighbour values of some feature within
+    rel_tau * rms of the layer input, decided by the ORACLE's layer input Hin).
+
+    The (sub)gradient of max/min goes to the arg neighbour (reading C4), a discrete
+    decision: the GPU's layer-L input differs from the oracle's by fp32 rounding
+    (~1e-6 relative), so a near tie can route the gradient of feature c of row i to
+    another neighbour — an O(1) change of that gradient, like the ReLU kink of
+    reading A6'.  R_i = 0 removes row i's routing from the comparison (a few hub rows)."""
+    if w.agg not in ("max", "min") or w.layers < 2:
+        return R
+    H = np.asarray(Hin, np.float64)
+    tau = rel_tau * np.sqrt(np.mean(H * H))
+    R = np.array(R, copy=True)
+    sgn = 1.0 if w.agg == "max" else -1.0
+    for i in range(len(rp) - 1):
+        nb = ci[rp[i]:rp[i + 1]]
+        if len(nb) < 2:
+            continue
+        v = np.sort(sgn * H[nb], axis=0)
+        if np.any(v[-1] - v[-2] < tau):
+            R[i] = 0.0
+    return R
+
+
 def oracle_step(w: gen.Workload, rp, ci, H, Ws, As, R):
     """L-layer forward then backward with the oracle; returns per-layer outputs."""
     Hs, fwd = [np.asarray(H, np.float64)], []

@@ -370,6 +370,8 @@ def _cgnn_check(w, rp, ci, g, symmetric=True, plan_options=None):
     if w.act == "relu":
         f0 = pu.oracle_step(w, rp, ci, H, Ws, As, R)["fwd"][-1]
         R = pu.relu_kink_mask(w, f0["Z"], R)
+    if w.agg in ("max", "min") and w.layers > 1:
+        R = pu.tropical_tie_mask(w, rp, ci, pu.oracle_step(w, rp, ci, H, Ws, As, R)["H"][-2], R)
     st = pu.gpu_step(w, graph=g, R=R, symmetric=symmetric, plan_options=plan_options)
     ref = pu.oracle_step(w, rp, ci, H, Ws, As, R)
     pu.compare(w, st, ref)
