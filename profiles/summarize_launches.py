@@ -29,7 +29,8 @@ ALIAS = {"gat_bwd_k128_kernel": "gat_bwd_kernel", "gat_bwd_k128f_kernel": "gat_b
          "gat_bwd_bundle_kernel": "gat_bwd_short_kernel", "gat_fwd_bundle_kernel": "gat_fwd_short_kernel", "gat_fwd_k128_kernel": "gat_fwd_kernel",
                   "av_bwd_k128_kernel": "av_bwd_kernel", "av_fwd_k128_kernel": "av_fwd_kernel",
          "av_bwd_batched_kernel": "av_bwd_kernel", "av_fwd_batched_kernel": "av_fwd_kernel",
-         "gemm_tn_tc_kernel": "gemm_tn_kernel", "tn_sum_kernel": "sum_splits_kernel"}
+         "gemm_tn_tc_kernel": "gemm_tn_kernel", "tn_sum_kernel": "sum_splits_kernel",
+         "gemm_tc_roles_kernel": "gemm_tc_kernel"}
 STEP = re.compile(r"(gat_|av_|gemm_|agnn_rec|nu_kernel|grad_act|sum_splits|tn_sum|sgd|transpose|to_bf16|cg_)")
 
 
