@@ -72,7 +72,7 @@ def parse():
                         "fp32 arithmetic; include/agnn.h AGNN_PREC_BF16, reading B1)")
     p.add_argument("--scale", type=int, default=None,
                    help="override log2 n of the workload (same recipe and edge factor)")
-    p.add_argument("--cpu-sample-scale", type=int, default=17,
+    p.add_argument("--cpu-sample-scale", type=int, default=19,
                    help="log2 n of the bounded oracle sample (same recipe as the workload)")
     p.add_argument("--weak", action="store_true",
                    help="weak scaling: n = 2^21 x N vertices (same recipe and edge factor)")
