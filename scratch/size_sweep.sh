@@ -5,6 +5,6 @@ for sc in 21 22 23 24; do
 import json,sys
 d=json.loads([l for l in sys.stdin if l.startswith('{')][-1])
 r=d['roofline']
-print('n=2^$sc', 'edges', d['config']['edges'], 'edges/s %.3e' % d['value'], 'ms/step %.2f' % d['ms_per_step'], 'dominant', r['pass'], 'alg frac %.2f' % r['frac'], 'clock', d['clocks']['sm_mhz'])
-" >> gpurun_out/size_sweep.txt
+print('n=2^$sc', 'edges', d['config']['edges'], 'edges/s %.3e' % d['value'], 'ms/step %.2f' % d['ms_per_step'], 'dominant', r['pass'], 'model frac %.2f' % r['model_frac'], 'clock', d['clocks']['sm_mhz'])
+" >> gpurun_out/r02_size_sweep.txt
 done
