@@ -69,12 +69,13 @@ struct BMap {
   int last;      // lane e: last entry of its row
   int c;         // lane e: column entry (with the L2 class bits)
   float sc[NH];  // lane r: per-head scalars of row r (st + soff)
+  float tj[NH];  // lane e: t_j of its column (forward; loaded a bundle ahead)
 };
 
-template <int NH>
+template <int NH, bool TJ = false>
 __device__ __forceinline__ void bmap(BMap<NH>& m, int4 B, int4 meta, const int32_t* __restrict__ col,
                                      const float* __restrict__ st, int64_t row_begin, int soff,
-                                     int lane) {
+                                     int lane, const Gath* ga = nullptr) {
   m.B = B;
   m.meta = meta;
   const bool isrow = lane < B.y;
@@ -99,6 +100,12 @@ __device__ __forceinline__ void bmap(BMap<NH>& m, int4 B, int4 meta, const int32
 #pragma unroll
   for (int h = 0; h < NH; ++h)
     m.sc[h] = isrow ? __ldg(st + (row_begin + meta.x) * (2 * NH) + soff + h) : 0.f;
+  if constexpr (TJ) {  // the entries' t_j (the forward's scores), one bundle ahead
+    const float* tp = st + ga->row(m.c) * (2 * NH) + NH;
+    const uint64_t pol = ga->policy(m.c);
+#pragma unroll
+    for (int h = 0; h < NH; ++h) m.tj[h] = valid ? ldg1_pol(tp + h, pol) : 0.f;
+  }
 }
 
 __device__ __forceinline__ int4 ld_rec(const int4* p, int64_t i, int64_t n) {
@@ -128,15 +135,15 @@ gat_fwd_bundle_kernel(Items it, const TP* __restrict__ P, const float* __restric
   BMap<NH> cur;
   {
     const int4 B0 = ld_rec(it.bundles, gw, nb);
-    bmap(cur, B0, lane < B0.y ? __ldg(it.short_meta + B0.x + lane) : make_int4(0, 0, 0, 0), it.col,
-         st, it.row_begin, 0, lane);
+    bmap<NH, true>(cur, B0, lane < B0.y ? __ldg(it.short_meta + B0.x + lane) : make_int4(0, 0, 0, 0),
+                   it.col, st, it.row_begin, 0, lane, &ga);
   }
   int4 Bn = ld_rec(it.bundles, gw + nw, nb);
   int4 Mn = lane < Bn.y ? __ldg(it.short_meta + Bn.x + lane) : make_int4(0, 0, 0, 0);
   int4 Bnn = ld_rec(it.bundles, gw + 2 * nw, nb);
   for (int64_t b = gw; b < nb; b += nw) {
     BMap<NH> nxt;
-    bmap(nxt, Bn, Mn, it.col, st, it.row_begin, 0, lane);
+    bmap<NH, true>(nxt, Bn, Mn, it.col, st, it.row_begin, 0, lane, &ga);
     Mn = lane < Bnn.y ? __ldg(it.short_meta + Bnn.x + lane) : make_int4(0, 0, 0, 0);
     Bn = Bnn;
     Bnn = ld_rec(it.bundles, b + 3 * nw, nb);
@@ -150,13 +157,7 @@ gat_fwd_bundle_kernel(Items it, const TP* __restrict__ P, const float* __restric
 #pragma unroll
     for (int u = 0; u < GR; ++u)
       qa[u] = u < ne ? SL::load(P + ga.row(sJ[wib][u]) * K + cq, ga.policy(sJ[wib][u])) : SL::zero();
-    float tj[NH];
-    {
-      const float* tp = st + ga.row(c) * (2 * NH) + NH;
-      const uint64_t pol = ga.policy(c);
-#pragma unroll
-      for (int h = 0; h < NH; ++h) tj[h] = valid ? ldg1_pol(tp + h, pol) : 0.f;
-    }
+    const float* tj = cur.tj;  // loaded a bundle ahead (bmap)
     const int src = valid ? rs : 0;
 #pragma unroll
     for (int h = 0; h < NH; ++h) {
