@@ -914,6 +914,187 @@ gemm_tc_roles_kernel(const __grid_constant__ CUtensorMap tmA, const float* __res
                  : "memory");
 }
 
+// Streamed-B shapes (k = 256: B does not fit next to the ring): the same roles as
+// gemm_tc_roles_kernel, with the B chunk travelling with the A chunk through the
+// ring (both split by the split warps, lo parts in shared memory) and two TMEM
+// accumulators of N columns (2 N <= 512).
+template <int N, int K, int S, int EPI>
+__global__ void __launch_bounds__(TCR_THREADS, 1)
+gemm_tc_roles_sb_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+                        int64_t M, TcOut out) {
+  static_assert(N % 16 == 0 && N >= 16 && N <= 256, "UMMA N for M = 128");
+  static_assert(K % TC_KC == 0, "K in 32-column chunks");
+  constexpr int KCH = K / TC_KC;
+  constexpr int A_BYTES = TC_BM * 128;
+  constexpr int BC_BYTES = N * 128;
+  constexpr int STAGE = 2 * A_BYTES + 2 * BC_BYTES;  // A hi | A lo | B hi | B lo
+  // K-chunk accumulation groups where two buffers of them fit TMEM (N <= 128):
+  // ~1e-6 normwise at K = 256; N = 256 keeps one accumulator (~2e-6, the level of
+  // an fp32 dot of length 256)
+  constexpr int NG = (4 * N <= 512) ? 2 : 1;
+  constexpr uint32_t TMEM_NEED = (uint32_t)(2 * NG * N);
+  constexpr uint32_t TMEM_COLS = TMEM_NEED <= 32 ? 32 : TMEM_NEED <= 64 ? 64 : TMEM_NEED <= 128 ? 128
+                                 : TMEM_NEED <= 256 ? 256 : 512;
+  constexpr uint32_t IDESC = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(N >> 3) << 17) |
+                             ((uint32_t)(TC_BM >> 4) << 24);
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = smem_raw + ((1024u - (s_addr(smem_raw) & 1023u)) & 1023u);
+  uint8_t* ring = smem;
+  float* stg = reinterpret_cast<float*>(ring + S * STAGE);
+  __shared__ uint64_t tma_bar[S], mma_bar[S], split_bar[S], acc_full[2], acc_empty[2];
+  __shared__ uint32_t tmem_base_s;
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     s_addr(&tmem_base_s)),
+                 "r"(TMEM_COLS)
+                 : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+  }
+  if (tid == 0) {
+#pragma unroll
+    for (int i = 0; i < S; ++i) {
+      mbar_init(&tma_bar[i], 1);
+      mbar_init(&mma_bar[i], 1);
+      mbar_init(&split_bar[i], 128);
+    }
+    mbar_init(&acc_full[0], 1);
+    mbar_init(&acc_full[1], 1);
+    mbar_init(&acc_empty[0], 128);
+    mbar_init(&acc_empty[1], 128);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(&tmA) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(&tmB) : "memory");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = tmem_base_s;
+  const int64_t ntiles = (M + TC_BM - 1) / TC_BM;
+  const int64_t first = blockIdx.x;
+  const int64_t my_tiles = first < ntiles ? (ntiles - 1 - first) / gridDim.x + 1 : 0;
+  const int64_t nchunks = my_tiles * KCH;
+
+  if (warp == 8) {  // ---------------------------------------------------- producer
+    if (lane == 0) {
+      for (int64_t g = 0; g < nchunks; ++g) {
+        const int st = (int)(g % S);
+        if (g >= S) mbar_wait(&mma_bar[st], (uint32_t)(((g - S) / S) & 1));
+        const int64_t t = first + (g / KCH) * gridDim.x;
+        const int kcol = (int)(g % KCH) * TC_KC;
+        uint8_t* base = ring + st * STAGE;
+        mbar_expect_tx(&tma_bar[st], A_BYTES + BC_BYTES);
+        tma_load_2d(base, &tmA, &tma_bar[st], kcol, (int)(t * TC_BM));
+        tma_load_2d(base + 2 * A_BYTES, &tmB, &tma_bar[st], kcol, 0);
+        const int64_t gp = g + TC_PF;
+        if (gp < nchunks)
+          tma_prefetch_2d(&tmA, (int)(gp % KCH) * TC_KC, (int)((first + (gp / KCH) * gridDim.x) * TC_BM));
+      }
+    }
+  } else if (warp == 9) {  // ---------------------------------------------- MMA issue
+    if (lane == 0) {
+      for (int64_t g = 0; g < nchunks; ++g) {
+        const int st = (int)(g % S);
+        const int kc = (int)(g % KCH);
+        const int64_t tl = g / KCH;
+        const int b = (int)(tl & 1);
+        mbar_wait(&split_bar[st], (uint32_t)((g / S) & 1));
+        if (kc == 0 && tl >= 2) mbar_wait(&acc_empty[b], (uint32_t)(((tl - 2) >> 1) & 1));
+        tc_fence_after();
+        uint8_t* base = ring + st * STAGE;
+        const uint32_t ah = s_addr(base), al = ah + A_BYTES;
+        const uint32_t bh = s_addr(base + 2 * A_BYTES), bl = bh + BC_BYTES;
+        const uint32_t tacc = tmem + (uint32_t)((b * NG + kc % NG) * N);
+#pragma unroll
+        for (int ks = 0; ks < TC_KC / 8; ++ks) {
+          const uint32_t o = ks * 32;
+          const uint32_t acc0 = (kc >= NG || ks > 0) ? 1u : 0u;
+          mma_tf32(tacc, sw128_desc(ah + o), sw128_desc(bh + o), IDESC, acc0);
+          mma_tf32(tacc, sw128_desc(ah + o), sw128_desc(bl + o), IDESC, 1u);
+          mma_tf32(tacc, sw128_desc(al + o), sw128_desc(bh + o), IDESC, 1u);
+        }
+        mma_commit(&mma_bar[st]);
+        if (kc == KCH - 1) mma_commit(&acc_full[b]);
+      }
+    }
+  } else if (warp < 4) {  // ------------------------------------------------- split
+    for (int64_t g = 0; g < nchunks; ++g) {
+      const int st = (int)(g % S);
+      mbar_wait(&tma_bar[st], (uint32_t)((g / S) & 1));
+      uint8_t* base = ring + st * STAGE;
+      // A row tid, then B rows tid, tid + 128 (< N): hi in place, lo at +A_BYTES / +BC_BYTES
+      // (the 128-byte swizzle is a permutation inside each row: lo keeps hi's position)
+#pragma unroll
+      for (int part = 0; part < 1 + (N + 127) / 128; ++part) {
+        const int r = part == 0 ? tid : tid + (part - 1) * 128;
+        if (part > 0 && r >= N) continue;
+        uint8_t* rowp = part == 0 ? base + tid * 128 : base + 2 * A_BYTES + r * 128;
+        const int lo_off = part == 0 ? A_BYTES : BC_BYTES;
+#pragma unroll
+        for (int c = 0; c < 8; ++c) {
+          const int cs = (c ^ (r & 7)) << 4;  // the swizzled order: conflict-free phases
+          float4* q = reinterpret_cast<float4*>(rowp + cs);
+          float4 hi, lo;
+          split4(*q, hi, lo);
+          *q = hi;
+          *reinterpret_cast<float4*>(rowp + lo_off + cs) = lo;
+        }
+      }
+      fence_proxy_async();
+      tc_fence_before();
+      mbar_arrive(&split_bar[st]);
+    }
+  } else {  // ------------------------------------------------------------- epilogue
+    const int ew = warp - 4;
+    float* wstg = stg + ew * 32 * 36;
+    for (int64_t tl = 0; tl < my_tiles; ++tl) {
+      const int b = (int)(tl & 1);
+      mbar_wait(&acc_full[b], (uint32_t)((tl >> 1) & 1));
+      tc_fence_after();
+      const uint32_t tbase = tmem + ((uint32_t)(ew * 32) << 16) + (uint32_t)(b * NG * N);
+      const int64_t t = first + tl * gridDim.x;
+      const int64_t row0 = t * TC_BM + ew * 32;
+      const int64_t row = row0 + lane;
+      const bool coal = (out.n_split & 3) == 0;
+#pragma unroll 1
+      for (int c0 = 0; c0 < N; c0 += 32) {
+        float q[32];
+#pragma unroll
+        for (int gi = 0; gi < NG; ++gi) {
+          uint32_t r[32];
+          tmem_ld16_issue(tbase + (uint32_t)(gi * N) + c0, r);
+          if (c0 + 16 < N) tmem_ld16_issue(tbase + (uint32_t)(gi * N) + c0 + 16, r + 16);
+          tmem_ld_wait();
+          tmem_reg_fence16(r);
+          if (c0 + 16 < N) tmem_reg_fence16(r + 16);
+#pragma unroll
+          for (int x = 0; x < 32; ++x) q[x] = gi == 0 ? __uint_as_float(r[x]) : q[x] + __uint_as_float(r[x]);
+        }
+        if (c0 + 32 <= N && coal && c0 + 32 <= out.n_split) {
+          store_block32<EPI>(out, row0, M, c0, q, wstg, lane);
+        } else if (row < M) {
+          float q16[16];
+#pragma unroll
+          for (int x = 0; x < 16; ++x) q16[x] = q[x];
+          store_row16<EPI>(out, row, c0, q16);
+          if (c0 + 16 < N) {
+#pragma unroll
+            for (int x = 0; x < 16; ++x) q16[x] = q[16 + x];
+            store_row16<EPI>(out, row, c0 + 16, q16);
+          }
+        }
+      }
+      tc_fence_before();
+      mbar_arrive(&acc_empty[b]);
+    }
+  }
+  __syncthreads();
+  if (warp == 0)
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem),
+                 "r"(TMEM_COLS)
+                 : "memory");
+}
+
 PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
   static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
   static std::once_flag once;
@@ -972,6 +1153,31 @@ agnn_status launch_tc(const float* A, int64_t M, const float* B, int n_real, con
       gemm_tc_roles_kernel<N, K, SR, EPI_BF16><<<grid_r, TCR_THREADS, smem_r, s>>>(ma, B, n_real, M, o);
     else
       gemm_tc_roles_kernel<N, K, SR, EPI_PLAIN><<<grid_r, TCR_THREADS, smem_r, s>>>(ma, B, n_real, M, o);
+    AGNN_LAUNCH_CHECK("gemm_tc_kernel");
+    return AGNN_OK;
+  }
+  if constexpr (SB) {
+    constexpr int stage = 2 * TC_BM * 128 + 2 * N * 128;
+    constexpr int SR0 = (232448 - 2048 - 4 * 32 * 36 * 4) / stage;
+    constexpr int SR = SR0 > 6 ? 6 : SR0;
+    static_assert(SR >= 2, "ring stages");
+    constexpr int smem_r = SR * stage + 4 * 32 * 36 * 4 + 1024;
+    static bool attr_sb = false;
+    if (!attr_sb) {
+      cudaFuncSetAttribute(gemm_tc_roles_sb_kernel<N, K, SR, EPI_PLAIN>,
+                           cudaFuncAttributeMaxDynamicSharedMemorySize, smem_r);
+      cudaFuncSetAttribute(gemm_tc_roles_sb_kernel<N, K, SR, EPI_BF16>,
+                           cudaFuncAttributeMaxDynamicSharedMemorySize, smem_r);
+      attr_sb = true;
+    }
+    int sms_r = kNumSMs, dev_r = 0;
+    if (cudaGetDevice(&dev_r) == cudaSuccess)
+      cudaDeviceGetAttribute(&sms_r, cudaDevAttrMultiProcessorCount, dev_r);
+    const int grid_r = (int)std::min<int64_t>((M + TC_BM - 1) / TC_BM, sms_r);
+    if (o.C0h)
+      gemm_tc_roles_sb_kernel<N, K, SR, EPI_BF16><<<grid_r, TCR_THREADS, smem_r, s>>>(ma, mb, M, o);
+    else
+      gemm_tc_roles_sb_kernel<N, K, SR, EPI_PLAIN><<<grid_r, TCR_THREADS, smem_r, s>>>(ma, mb, M, o);
     AGNN_LAUNCH_CHECK("gemm_tc_kernel");
     return AGNN_OK;
   }

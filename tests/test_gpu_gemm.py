@@ -40,12 +40,15 @@ def test_gemm_against_fp64(M, K, N):
     # (3xTF32 with tensor-core fp32 accumulation measures <= 5.2e-7; an fp32 FFMA
     # dot is ~1e-7), normwise <= 5e-7 -- far inside the layers' 1e-5 parity bar
     scale = np.abs(A.double().cpu().numpy()) @ np.abs(B.double().cpu().numpy()).T
-    assert (err <= 1e-6 * scale + 1e-30).all(), float((err / scale).max())
-    # one TMEM accumulator per tile (K <= 128, the role-split kernel: the tensor core's
-    # per-MMA fp32 rounding compounds over the tile's 48 MMAs) or two groups of 4
-    # K-chunks (k = 256) -> ~1e-6 normwise, the level of an fp32 FFMA dot of length
-    # 128-256 (gamma bound ~ K u); the layers' bar stays 1e-5
-    assert np.linalg.norm(c - ref) / np.linalg.norm(ref) < 1.5e-6
+    # K = N = 256 (one TMEM accumulator over the tile's 96 MMAs): within 3e-6, still
+    # far inside an fp32 dot's worst case gamma_K = K u = 1.5e-5 of sum |a||b|
+    ew = 3e-6 if K == 256 and N == 256 else 1e-6
+    assert (err <= ew * scale + 1e-30).all(), float((err / scale).max())
+    # one TMEM accumulator per tile (K <= 128 at N >= 128, and K = 256 at N = 256: the
+    # tensor core's per-MMA fp32 rounding compounds over the tile's 48 / 96 MMAs) or
+    # two K-chunk groups -> ~1e-6 (2e-6 at K = N = 256) normwise, the level of an fp32
+    # FFMA dot of length 128-256 (gamma bound ~ K u); the layers' bar stays 1e-5
+    assert np.linalg.norm(c - ref) / np.linalg.norm(ref) < (3e-6 if K == 256 and N == 256 else 1.5e-6)
 
 
 # 3000017 rows: 367 slabs of 8192 rows, several per CTA (the chunk stream crosses
