@@ -258,8 +258,9 @@ agnn_status transpose(const float* X, int rows, int cols, float* Y, cudaStream_t
 
 size_t gemm_tn_ws_floats(int K1, int N) {
   const size_t simt = (size_t)tn_splits(K1, N) * K1 * N;
-  // one partial per row slab of one <= 128 x 128 output block (gemm_tn_tc)
-  const size_t tc = (size_t)2048 * (K1 < 128 ? K1 : 128) * (N < 128 ? N : 128);
+  // one partial per (128 x 128 output block, row slab) (gemm_tn_tc)
+  const size_t blocks = (size_t)((K1 + 127) / 128) * ((N + 127) / 128);
+  const size_t tc = (size_t)2048 * (K1 < 128 ? K1 : 128) * (N < 128 ? N : 128) * blocks;
   return simt > tc ? simt : tc;
 }
 

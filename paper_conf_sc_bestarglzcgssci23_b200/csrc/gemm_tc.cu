@@ -565,7 +565,11 @@ __device__ __forceinline__ uint64_t sw128_mn_desc(uint32_t saddr, uint32_t lbo_b
 template <int K1, int N>
 __global__ void __launch_bounds__(TC_THREADS, TN_CTAS)
 gemm_tn_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-                  int64_t M, int64_t rows_per_cta, float* __restrict__ part) {
+                  int64_t M, int64_t rows_per_cta, float* __restrict__ part, int nbx) {
+  // output block (blockIdx.y) of a wider product: the K1 x N block at (qa K1, qb N) of
+  // A^T B — the CTAs of every block of one slab run together, so the A and B column
+  // blocks a slab shares come from DRAM once (L2 serves the other blocks)
+  const int qa = (int)blockIdx.y / nbx, qb = (int)blockIdx.y % nbx;
   constexpr uint32_t LBO = TN_ROWS * 128;  // 32-column MN blocks (one TMA box each)
   constexpr uint32_t SBO = 512;            // 4-row K groups
   static_assert(K1 == 128, "the MMA M is the K1 = 128 rows of dW");
@@ -614,10 +618,10 @@ gemm_tn_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
     mbar_expect_tx(&tma_bar[st], A_BYTES + B_BYTES);
 #pragma unroll
     for (int b = 0; b < K1 / 32; ++b)
-      tma_load_2d(base + b * (TN_ROWS * 128), &tmA, &tma_bar[st], b * 32, r);
+      tma_load_2d(base + b * (TN_ROWS * 128), &tmA, &tma_bar[st], qa * K1 + b * 32, r);
 #pragma unroll
     for (int b = 0; b < N / 32; ++b)
-      tma_load_2d(base + 2 * A_BYTES + b * (TN_ROWS * 128), &tmB, &tma_bar[st], b * 32, r);
+      tma_load_2d(base + 2 * A_BYTES + b * (TN_ROWS * 128), &tmB, &tma_bar[st], qb * N + b * 32, r);
   };
   if (tid == 0 && nch > 0) issue_tma(0, (int)(G0 & 1));
   for (int64_t g = 0; g < nch; ++g) {
@@ -626,9 +630,9 @@ gemm_tn_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
     if (tid == 0 && g + 1 + TC_PF / 2 < nch) {
       const int r = (int)(r_beg + (g + 1 + TC_PF / 2) * TN_ROWS);
 #pragma unroll
-      for (int b = 0; b < K1 / 32; ++b) tma_prefetch_2d(&tmA, b * 32, r);
+      for (int b = 0; b < K1 / 32; ++b) tma_prefetch_2d(&tmA, qa * K1 + b * 32, r);
 #pragma unroll
-      for (int b = 0; b < N / 32; ++b) tma_prefetch_2d(&tmB, b * 32, r);
+      for (int b = 0; b < N / 32; ++b) tma_prefetch_2d(&tmB, qb * N + b * 32, r);
     }
     if (tid == 0 && g + 1 < nch) {
       // stage st^1 held chunk G-1 (its MMAs must finish before the TMA overwrites it;
@@ -690,7 +694,8 @@ gemm_tn_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant
       __syncthreads();
     }
   }
-  float* out = part + slab * K1 * N + (int64_t)tid * N;  // dW row tid of this slab's partial
+  // dW row tid of this (block, slab)'s partial
+  float* out = part + ((int64_t)blockIdx.y * nslabs + slab) * K1 * N + (int64_t)tid * N;
 #pragma unroll
   for (int c = 0; c < N; c += 4) st4(out + c, make_float4(acc[c], acc[c + 1], acc[c + 2], acc[c + 3]));
   G0 += nch;
@@ -1218,24 +1223,29 @@ bool map_rows_box32(CUtensorMap* map, const float* base, int64_t rows, int cols,
              CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
-// C[r][c] (row stride ldc) = sum over the slab partials of part[p][r][c] (r < K1, c < N)
+// C block q (blockIdx.y; at rows (q / nbx) K1, columns (q % nbx) N; row stride ldc) =
+// sum over the slab partials of part[q][p][r][c] (r < K1, c < N)
 __global__ void tn_sum_kernel(const float* __restrict__ part, int splits, int K1, int N,
-                              float* __restrict__ C, int ldc) {
+                              float* __restrict__ C, int ldc, int nbx) {
   const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const int64_t count = (int64_t)K1 * N;
   if (i >= count) return;
+  const int q = (int)blockIdx.y;
+  const float* pq = part + (int64_t)q * splits * count;
   double s = 0.0;  // fixed order, fp64 across the slab partials
-  for (int p = 0; p < splits; ++p) s += (double)part[(int64_t)p * count + i];
-  C[(i / N) * ldc + (i % N)] = (float)s;
+  for (int p = 0; p < splits; ++p) s += (double)pq[(int64_t)p * count + i];
+  C[((int64_t)(q / nbx) * K1 + i / N) * ldc + (q % nbx) * N + (i % N)] = (float)s;
 }
 
 // C block [K1 x N] (row stride ldc) = A^T B over M rows; A, B column blocks of row
 // strides lda, ldb
+// C [nby K1 x nbx N] = A^T B over M rows in K1 x N blocks, one launch: A [M x nby K1],
+// B [M x nbx N] (row strides = their widths)
 template <int K1, int N>
-agnn_status launch_tn_tc(const float* A, int lda, int64_t M, const float* B, int ldb, float* C,
-                         int ldc, float* ws, cudaStream_t s) {
+agnn_status launch_tn_tc(const float* A, int nby, int64_t M, const float* B, int nbx, float* C,
+                         float* ws, cudaStream_t s) {
   CUtensorMap ma, mb;
-  if (!map_rows_box32(&ma, A, M, K1, lda) || !map_rows_box32(&mb, B, M, N, ldb))
+  if (!map_rows_box32(&ma, A, M, nby * K1, nby * K1) || !map_rows_box32(&mb, B, M, nbx * N, nbx * N))
     return fail(AGNN_ECUDA, "gemm_tn_tc: tensor map encode failed");
   constexpr int smem = 2 * (2 * TN_ROWS * K1 * 4 + 2 * TN_ROWS * N * 4) + 1024;
   static bool attr = false;
@@ -1247,21 +1257,22 @@ agnn_status launch_tn_tc(const float* A, int lda, int64_t M, const float* B, int
   int sms = kNumSMs, dev = 0;
   if (cudaGetDevice(&dev) == cudaSuccess)
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  // slabs of >= 8192 rows, at most kTnMaxSlabs of them; each slab leaves one fp32 partial
+  // slabs of >= 8192 rows, at most kTnMaxSlabs of them; each (block, slab) leaves one
+  // fp32 partial
   int64_t rps = (M + kTnMaxSlabs - 1) / kTnMaxSlabs;
   rps = std::max<int64_t>(rps, 8192);
   rps = (rps + TN_ROWS - 1) / TN_ROWS * TN_ROWS;
   const int64_t nslabs = (M + rps - 1) / rps;
-  const int grid = (int)std::min<int64_t>(nslabs, (int64_t)sms * TN_CTAS);
-  gemm_tn_tc_kernel<K1, N><<<grid, TC_THREADS, smem, s>>>(ma, mb, M, rps, ws);
+  const int nblk = nby * nbx;
+  const int gx = (int)std::min<int64_t>(nslabs, std::max<int64_t>(1, (int64_t)sms * TN_CTAS / nblk));
+  gemm_tn_tc_kernel<K1, N><<<dim3(gx, nblk), TC_THREADS, smem, s>>>(ma, mb, M, rps, ws, nbx);
   AGNN_LAUNCH_CHECK("gemm_tn_kernel");
   const int64_t cnt = (int64_t)K1 * N;
-  tn_sum_kernel<<<(unsigned)((cnt + 255) / 256), 256, 0, s>>>(ws, (int)nslabs, K1, N, C, ldc);
+  tn_sum_kernel<<<dim3((unsigned)((cnt + 255) / 256), nblk), 256, 0, s>>>(ws, (int)nslabs, K1, N, C,
+                                                                          nbx * N, nbx);
   AGNN_LAUNCH_CHECK("sum_splits_kernel");
   return AGNN_OK;
 }
-
-
 
 }  // namespace
 
@@ -1273,18 +1284,10 @@ agnn_status gemm_tn_tc(const float* A, int64_t M, int K1, const float* B, int N,
   if (M <= 0) return AGNN_EUNSUPPORTED;
   if ((reinterpret_cast<uintptr_t>(A) & 15) || (reinterpret_cast<uintptr_t>(B) & 15))
     return AGNN_EUNSUPPORTED;
-  if (K1 == 128 && N == 128) return launch_tn_tc<128, 128>(A, K1, M, B, N, C, N, ws, s);
-  if (K1 == 128 && N == 64) return launch_tn_tc<128, 64>(A, K1, M, B, N, C, N, ws, s);
-  if (K1 == 256 && (N == 256 || N == 128)) {
-    // 128 x 128 blocks of C, one pass each over the matching column blocks of A and B
-    for (int qa = 0; qa < K1 / 128; ++qa)
-      for (int qb = 0; qb < N / 128; ++qb) {
-        const agnn_status st = launch_tn_tc<128, 128>(A + qa * 128, K1, M, B + qb * 128, N,
-                                                      C + (int64_t)qa * 128 * N + qb * 128, N, ws, s);
-        if (st != AGNN_OK) return st;
-      }
-    return AGNN_OK;
-  }
+  if (K1 == 128 && N == 128) return launch_tn_tc<128, 128>(A, 1, M, B, 1, C, ws, s);
+  if (K1 == 128 && N == 64) return launch_tn_tc<128, 64>(A, 1, M, B, 1, C, ws, s);
+  // K1 = 256: 128 x 128 blocks of C in one launch
+  if (K1 == 256 && (N == 256 || N == 128)) return launch_tn_tc<128, 128>(A, 2, M, B, N / 128, C, ws, s);
   return AGNN_EUNSUPPORTED;
 }
 
