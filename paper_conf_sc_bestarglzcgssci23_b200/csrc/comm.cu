@@ -300,7 +300,47 @@ agnn_status peer_send_lists(Plan& p) {
     AGNN_CUDA_TRY(cudaMemcpy(p.send_idx, all.data(), sizeof(int32_t) * all.size(),
                              cudaMemcpyHostToDevice));
   }
+  // the same lists as a per-row bit mask over the compact peer order (rank order
+  // without this rank), for the producing kernels that store the rows themselves
+  std::vector<uint8_t> mask((size_t)std::max<int64_t>(p.n_local, 1), 0);
+  for (int q = 0, pi = 0; q < p.world; ++q) {
+    if (q == p.rank) continue;
+    for (int64_t x = p.send_off[q]; x < p.send_off[q + 1]; ++x)
+      mask[(size_t)(all[(size_t)x] - p.row_begin)] |= (uint8_t)(1u << pi);
+    ++pi;
+  }
+  if (p.send_mask) cudaFree(p.send_mask);
+  AGNN_CUDA_TRY(cudaMalloc(&p.send_mask, mask.size()));
+  AGNN_CUDA_TRY(cudaMemcpy(p.send_mask, mask.data(), mask.size(), cudaMemcpyHostToDevice));
   return AGNN_OK;
+}
+
+bool peer_rows(const Plan& p, const void* a, const void* b, PeerRows& out) {
+  out = PeerRows();
+  if (!p.peer || !p.peer_ready || p.world <= 1) return false;
+  PeerPtrs pa, pb;
+  if (!peer_lookup(p, a, pa) || (b && !peer_lookup(p, b, pb))) return false;
+  for (int q = 0; q < p.world; ++q) {
+    if (q == p.rank) continue;
+    out.a[out.n] = reinterpret_cast<float*>(pa.p[q]);
+    out.b[out.n] = b ? reinterpret_cast<float*>(pb.p[q]) : nullptr;
+    ++out.n;
+  }
+  out.mask = p.send_mask;
+  return true;
+}
+
+bool peer_out(const Plan& p, const void* c0, const void* c1, PeerOut& out) {
+  PeerRows r;
+  out = PeerOut();
+  if (!peer_rows(p, c0, c1, r)) return false;
+  out.n = r.n;
+  for (int i = 0; i < r.n; ++i) {
+    out.C0[i] = r.a[i];
+    out.C1[i] = r.b[i];
+  }
+  out.mask = r.mask;
+  return true;
 }
 
 agnn_status nccl_status(ncclResult_t r, const char* what) {
@@ -332,6 +372,8 @@ void comm_destroy(Plan& p) {
   p.regs = nullptr;
   if (p.send_idx) cudaFree(p.send_idx);
   p.send_idx = nullptr;
+  if (p.send_mask) cudaFree(p.send_mask);
+  p.send_mask = nullptr;
   if (p.ctl) cudaFree(p.ctl);
   p.ctl = nullptr;
 }

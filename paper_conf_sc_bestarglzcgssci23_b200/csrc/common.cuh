@@ -304,6 +304,7 @@ struct Plan {
   size_t want_off = 0;                // byte offset of this rank's wanted lists in ctl
   int64_t n_wanted = 0;               // columns of other blocks this rank's rows reference
   int32_t* send_idx = nullptr;        // device, plan-owned: rows to push, by peer
+  uint8_t* send_mask = nullptr;       // device [n_local]: bit pi = compact peer pi needs the row
   int64_t send_off[kMaxPeers + 1] = {};  // host: peer q's rows are send_idx[send_off[q] ..)
   mutable int64_t epoch = 0;          // barrier generation (host, in stream order)
   mutable int64_t red_calls = 0;      // all-reduce slot-set parity

@@ -557,15 +557,16 @@ gat_bwd_prologue_kernel(int64_t n_local, int64_t row_begin, const float* __restr
     for (int v = 0; v < L::VPL; ++v) {
       const int c = L::col(v, q), h = c / L::D;
       st4(G + grow * K + c, gv[v]);
-      for (int pi = 0; pi < peers.n; ++pi)  // peers' replicas (fused all-gather)
-        st4(reinterpret_cast<TG*>(peers.a[pi]) + grow * K + c, gv[v]);
+      const uint32_t pm = peers.n ? peers.mask[row] : 0u;
+      for (int pi = 0; pi < peers.n; ++pi)  // the peers whose rows reference this one
+        if ((pm >> pi) & 1u) st4(reinterpret_cast<TG*>(peers.a[pi]) + grow * K + c, gv[v]);
       if ((c % L::D) == 0) {
         const float lv = lrow[row * NH + h];
         const float4 r4 = make_float4(st[grow * 2 * NH + h], mrow[row * NH + h],
                                       lv > 0.f ? 1.f / lv : 0.f, dl[v]);
         rec[grow * NH + h] = r4;
         for (int pi = 0; pi < peers.n; ++pi)
-          reinterpret_cast<float4*>(peers.b[pi])[grow * NH + h] = r4;
+          if ((pm >> pi) & 1u) reinterpret_cast<float4*>(peers.b[pi])[grow * NH + h] = r4;
         if (Q) ds_row[row * NH + h] = dq[v];
       }
     }
@@ -796,13 +797,23 @@ agnn_status gat_forward(const Plan& p, const GatShape& g, const float* W, const 
     }
     return AGNN_OK;
   }
-  // P | s t for the local rows, written at their global offsets; with P > 1 the
-  // rows the other ranks reference are then pushed to their replicas (comm.cu)
+  // P | s t for the local rows, written at their global offsets.  With P > 1 over peer
+  // memory the GEMM epilogue also stores every row into the replicas of the peers whose
+  // CSR references it (fused GEMM -> needed-rows exchange, NVLink stores overlapping
+  // the next tiles), between an entry and an exit barrier; otherwise the rows are
+  // pushed after the GEMM (comm.cu)
   float* Ploc = sv.P + p.row_begin * g.k_out;
+  PeerOut po;
+  const bool fuse = p.world > 1 && peer_out(p, Ploc, stloc, po);
+  if (fuse && (st = peer_barrier(p, s)) != AGNN_OK) return st;
+  bool fused = false;
   if ((st = gemm_rows(H_in, p.n_local, g.k_in, w.Wext, true, NE, Ploc, g.k_out, stloc, s,
-                      nullptr, 0, NEs)) != AGNN_OK)
+                      nullptr, 0, NEs, fuse ? &po : nullptr, &fused)) != AGNN_OK)
     return st;
-  if (p.world > 1) {
+  if (fused) {
+    if ((st = peer_barrier(p, s)) != AGNN_OK) return st;
+  } else if (p.world > 1) {
+    if (fuse && (st = peer_barrier(p, s)) != AGNN_OK) return st;  // (same barrier count)
     const RowArray ra[2] = {{sv.P, g.k_out}, {sv.st, 2 * g.heads}};
     if ((st = allgather_rows(p, ra, 2, s)) != AGNN_OK) return st;
   }
@@ -846,7 +857,11 @@ agnn_status gat_backward(const Plan& p, const GatShape& g, const float* W, const
   const int K_ = g.k_out, NH_ = g.heads;
   Items it = items_of(p);
   agnn_status st;
-  const PeerRows pr;  // (no fused peer stores: the exchange below pushes the needed rows)
+  // peer memory: the prologue stores G | rec also into the replicas of the peers whose
+  // CSR references the row (fused prologue -> needed-rows exchange)
+  PeerRows pr;
+  const bool fuse_g = p.world > 1 && peer_rows(p, g.bf16 ? (void*)w.G16 : (void*)w.G, w.rec, pr);
+  if (fuse_g && (st = peer_barrier(p, s)) != AGNN_OK) return st;
   if (g.bf16) {
     if (directed)
       return fail(AGNN_EUNSUPPORTED, "AGNN_PREC_BF16: symmetric patterns only");
@@ -861,7 +876,9 @@ agnn_status gat_backward(const Plan& p, const GatShape& g, const float* W, const
                                     w.G, w.rec, pr, sv.Q, w.ds_row)));
   }
   AGNN_LAUNCH_CHECK("gat_bwd_prologue_kernel");
-  if (p.world > 1) {  // G | rec rows the other ranks reference -> their replicas
+  if (fuse_g) {  // exit barrier: the prologue's peer stores are visible
+    if ((st = peer_barrier(p, s)) != AGNN_OK) return st;
+  } else if (p.world > 1) {  // NCCL: G | rec blocks -> every replica
     const RowArray ra[2] = {{g.bf16 ? reinterpret_cast<float*>(w.G16) : w.G,
                              g.bf16 ? g.k_out / 2 : g.k_out},
                             {reinterpret_cast<float*>(w.rec), 4 * g.heads}};

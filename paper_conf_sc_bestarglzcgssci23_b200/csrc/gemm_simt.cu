@@ -204,7 +204,7 @@ __global__ void sum_splits_kernel(const float* __restrict__ part, int splits, in
 
 agnn_status gemm_tc(const float* A, int64_t M, int K, const float* B, int n_real, float* C0,
                     int n_split, float* C1, int n_store, float* Cact, int act, cudaStream_t s,
-                    bf16* C0h = nullptr);
+                    bf16* C0h = nullptr, const PeerOut* peers = nullptr);
 
 namespace {
 // Y[i] = bf16_rn(X[i]) over rows x cols (cols % 4 == 0)
@@ -234,11 +234,19 @@ agnn_status gemm_rows_bf16(const float* A, int64_t M, int K, const float* B, int
 
 agnn_status gemm_rows(const float* A, int64_t M, int K, const float* B, bool b_trans, int N,
                       float* C0, int n_split, float* C1, cudaStream_t s, float* Cact, int act,
-                      int n_store) {
+                      int n_store, const PeerOut* peers, bool* peers_done) {
+  if (peers_done) *peers_done = false;
   if (b_trans) {  // tcgen05 3xTF32 path when the shape has an instantiation
     const int ns = (n_store <= 0 || n_store > N) ? N : n_store;
-    const agnn_status st = gemm_tc(A, M, K, B, ns, C0, n_split, C1, ns, Cact, act, s);
-    if (st != AGNN_EUNSUPPORTED) return st;
+    agnn_status st = gemm_tc(A, M, K, B, ns, C0, n_split, C1, ns, Cact, act, s, nullptr, peers);
+    if (st != AGNN_EUNSUPPORTED) {
+      if (peers_done) *peers_done = peers != nullptr && st == AGNN_OK;
+      return st;
+    }
+    // no peer epilogue for this shape (the caller pushes the rows instead)
+    if (peers && (st = gemm_tc(A, M, K, B, ns, C0, n_split, C1, ns, Cact, act, s)) !=
+                     AGNN_EUNSUPPORTED)
+      return st;
   }
   if (M <= 0) return AGNN_OK;
   if (K % 4 || N % 4) return fail(AGNN_EINVAL, "gemm_rows: K and N must be multiples of 4");

@@ -188,10 +188,18 @@ struct TcOut {
   float* Cact;  // sigma(C) for columns < n_split (nullable)
   int n_split, n_store, act;
   bf16* C0h;    // EPI_BF16: columns [0, n_split) stored as bfloat16 here instead of C0
+  // EPI_PEER (fused GEMM -> needed-rows exchange): row r also goes to peer pi's
+  // replicas pC0[pi] / pC1[pi] (same offsets) when bit pi of pmask[r] is set
+  int npeer;
+  float* pC0[kMaxPeers - 1];
+  float* pC1[kMaxPeers - 1];
+  const uint8_t* pmask;
 };
 
-// epilogue variants (compile time, so the plain fp32 epilogue carries no bf16 code)
+// epilogue variants (compile time, so the plain fp32 epilogue carries no peer or
+// bf16 code)
 constexpr int EPI_PLAIN = 0;  // C0 | C1 fp32 (+ sigma copy)
+constexpr int EPI_PEER = 1;   // also the peers' replicas of the rows they reference
 constexpr int EPI_BF16 = 2;   // C0 columns rounded to bfloat16 into C0h (reading B1)
 
 // 16 consecutive columns c0.. of output row `row` (C0 | C1 split, optional sigma copy).
@@ -235,6 +243,12 @@ __device__ __forceinline__ void store_row16(const TcOut& out, int64_t row, int c
     return;
   }
   store_row16_to(out, out.C0, out.C1, out.Cact, row, c0, v);
+  if constexpr (EPI == EPI_PEER) {
+    const uint32_t m = out.pmask[row];
+#pragma unroll 1
+    for (int pi = 0; pi < out.npeer; ++pi)
+      if ((m >> pi) & 1u) store_row16_to(out, out.pC0[pi], out.pC1[pi], nullptr, row, c0, v);
+  }
 }
 
 // 32 columns [c0, c0+32) of the warp's 32 rows [row0, row0+32) through a per-warp
@@ -261,6 +275,12 @@ __device__ __forceinline__ void store_block32(const TcOut& out, int64_t row0, in
       }
       if (out.C0) st4(out.C0 + row * out.n_split + c0 + cc, q);
       if (out.Cact) st4(out.Cact + row * out.n_split + c0 + cc, act_fwd4(out.act, q));
+      if constexpr (EPI == EPI_PEER) {  // NVLink stores to the peers that need this row
+        const uint32_t m = out.pmask[row];
+#pragma unroll 1
+        for (int pi = 0; pi < out.npeer; ++pi)
+          if ((m >> pi) & 1u) st4(out.pC0[pi] + row * out.n_split + c0 + cc, q);
+      }
     }
   }
   __syncwarp();
@@ -1148,6 +1168,8 @@ agnn_status launch_tc(const float* A, int64_t M, const float* B, int n_real, con
                            cudaFuncAttributeMaxDynamicSharedMemorySize, smem_r);
       cudaFuncSetAttribute(gemm_tc_roles_kernel<N, K, SR, EPI_BF16>,
                            cudaFuncAttributeMaxDynamicSharedMemorySize, smem_r);
+      cudaFuncSetAttribute(gemm_tc_roles_kernel<N, K, SR, EPI_PEER>,
+                           cudaFuncAttributeMaxDynamicSharedMemorySize, smem_r);
       attr_r = true;
     }
     int sms_r = kNumSMs, dev_r = 0;
@@ -1156,6 +1178,8 @@ agnn_status launch_tc(const float* A, int64_t M, const float* B, int n_real, con
     const int grid_r = (int)std::min<int64_t>((M + TC_BM - 1) / TC_BM, sms_r);
     if (o.C0h)
       gemm_tc_roles_kernel<N, K, SR, EPI_BF16><<<grid_r, TCR_THREADS, smem_r, s>>>(ma, B, n_real, M, o);
+    else if (o.npeer > 0)
+      gemm_tc_roles_kernel<N, K, SR, EPI_PEER><<<grid_r, TCR_THREADS, smem_r, s>>>(ma, B, n_real, M, o);
     else
       gemm_tc_roles_kernel<N, K, SR, EPI_PLAIN><<<grid_r, TCR_THREADS, smem_r, s>>>(ma, B, n_real, M, o);
     AGNN_LAUNCH_CHECK("gemm_tc_kernel");
@@ -1295,16 +1319,27 @@ agnn_status gemm_tn_tc(const float* A, int64_t M, int K1, const float* B, int N,
 // Returns AGNN_EUNSUPPORTED when the shape has no tcgen05 instantiation.
 agnn_status gemm_tc(const float* A, int64_t M, int K, const float* B, int n_real, float* C0,
                     int n_split, float* C1, int n_store, float* Cact, int act, cudaStream_t s,
-                    bf16* C0h) {
+                    bf16* C0h, const PeerOut* peers) {
   if ((reinterpret_cast<uintptr_t>(A) & 15) || (K % 32)) return AGNN_EUNSUPPORTED;
   if (C0h && (Cact || (n_split & 3))) return AGNN_EUNSUPPORTED;
+  // the peer epilogue exists for the resident-B (K <= 128) kernel; the shape decides,
+  // so every rank agrees on whether the exchange was fused
+  if (peers && (K > 128 || C0h || !C0 || peers->n > kMaxPeers - 1)) return AGNN_EUNSUPPORTED;
   const int npad = (n_real + 15) / 16 * 16;
   const bool shape_ok = (K == 128 && (npad == 128 || npad == 144 || npad == 160 || npad == 64)) ||
                         (K == 64 && (npad == 64 || npad == 80 || npad == 128)) ||
                         (K == 256 && (npad == 256 || npad == 128));
   if (!shape_ok) return AGNN_EUNSUPPORTED;
   if (M <= 0) return AGNN_OK;
-  TcOut o{C0, C1, Cact, n_split, n_store, act, C0h};
+  TcOut o{C0, C1, Cact, n_split, n_store, act, C0h, 0, {}, {}, nullptr};
+  if (peers) {
+    o.npeer = peers->n;
+    o.pmask = peers->mask;
+    for (int i = 0; i < peers->n; ++i) {
+      o.pC0[i] = peers->C0[i];
+      o.pC1[i] = peers->C1[i];
+    }
+  }
   // resident B: S = the 16 KB stages that fit next to B (2 x K x N x 4 bytes), <= 8
   if (K == 128 && npad == 128) return launch_tc<128, 128, 4, false>(A, M, B, n_real, o, s);
   if (K == 128 && npad == 144) return launch_tc<144, 128, 3, false>(A, M, B, n_real, o, s);

@@ -77,15 +77,30 @@ inline int grid_of(F* func) { return persistent_blocks(reinterpret_cast<const vo
 // Columns [0, n_split) go to C0 (ld = n_split), [n_split, N) to C1 (ld = N - n_split).
 // If Cact != NULL, sigma(C) (act) is also written to Cact (layout of C0); C0 may be NULL.
 // Columns >= n_store (padding) are computed but not stored (n_store <= 0: N).
-// replicas of up to two row arrays in the other ranks (kernel argument; unused when n = 0)
+// replicas of up to two row arrays in the other ranks (compact peer order: rank order
+// without this rank) and the needed-rows mask: local row r goes to peer pi iff bit pi
+// of mask[r] is set (the fused exchange; kernel argument, unused when n = 0)
 struct PeerRows {
   int n = 0;
   float* a[kMaxPeers - 1] = {};
   float* b[kMaxPeers - 1] = {};
+  const uint8_t* mask = nullptr;
+};
+// the same for a GEMM's output column blocks C0 | C1 (gemm_rows)
+struct PeerOut {
+  int n = 0;
+  float* C0[kMaxPeers - 1] = {};
+  float* C1[kMaxPeers - 1] = {};
+  const uint8_t* mask = nullptr;
 };
 agnn_status gemm_rows(const float* A, int64_t M, int K, const float* B, bool b_trans, int N,
                       float* C0, int n_split, float* C1, cudaStream_t s, float* Cact = nullptr,
-                      int act = 0, int n_store = 0);
+                      int act = 0, int n_store = 0, const PeerOut* peers = nullptr,
+                      bool* peers_done = nullptr);
+// peer exchange: the fused-exchange descriptors of replicated arrays (compact peer
+// order + the plan's needed-rows mask); false if the plan has no peer exchange
+bool peer_rows(const Plan& p, const void* a, const void* b, PeerRows& out);
+bool peer_out(const Plan& p, const void* c0, const void* c1, PeerOut& out);
 // BF16 storage (reading B1): C = A * B^T with columns [0, n_split) rounded to bf16
 // into C0h (ld n_split) and [n_split, N) fp32 into C1 (ld N - n_split); scratch
 // [M x n_split] fp32 is used only when the shape has no tcgen05 instantiation.
