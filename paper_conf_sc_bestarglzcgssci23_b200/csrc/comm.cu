@@ -14,7 +14,9 @@
 //    agnn_plan_register).  An all-gather is a kernel that stores rows of this
 //    rank's block straight into every peer's replica, fenced by a flag barrier —
 //    only the rows the peer's own CSR references (its "wanted" columns in this
-//    block, exchanged once at agnn_plan_connect): the sparse kernels gather a
+//    block, exchanged once at agnn_plan_connect; the GAT projection GEMM epilogue
+//    and backward prologue store their rows to the peers themselves by a per-row
+//    peer mask, so those exchanges overlap their producers): the sparse kernels gather a
 //    replicated row only as the neighbour of a local row, so every row a rank
 //    reads arrives and the results are bitwise those of the full all-gather, at
 //    ~40-60 % of its NVLink bytes on the Kronecker graphs.  An
