@@ -74,6 +74,10 @@ def parse():
                    help="override log2 n of the workload (same recipe and edge factor)")
     p.add_argument("--cpu-sample-scale", type=int, default=19,
                    help="log2 n of the bounded oracle sample (same recipe as the workload)")
+    p.add_argument("--spmmm", type=int, default=-1, choices=[-1, 0, 1],
+                   help="AGNN/VA k = 128 forward: 1 = fused SpMMM kernel (aggregation and "
+                        "projection in one kernel, agnn_plan_options.spmmm), 0 = SpMM kernel + "
+                        "tcgen05 GEMM, -1 = the library default")
     p.add_argument("--weak", action="store_true",
                    help="weak scaling: n = 2^21 x N vertices (same recipe and edge factor)")
     return p.parse_args()
@@ -484,7 +488,8 @@ def run_ours(args):
         uid = obj[0]
 
     t_setup = time.perf_counter()
-    st = runner.Stack(w, dev, rank=rank, world=world, nccl_uid=uid)
+    popts = {"spmmm": args.spmmm} if args.spmmm >= 0 else None
+    st = runner.Stack(w, dev, rank=rank, world=world, nccl_uid=uid, plan_options=popts)
     torch.cuda.synchronize()
     setup_s = time.perf_counter() - t_setup
     m, n = st.graph.nnz, w.n
@@ -750,6 +755,8 @@ def run_ours(args):
                                        "256 MB buffer written between timed steps (per-step "
                                        "event pairs)",
                            "cuda_graph": use_graph, "eager_ms_per_step": eager_ms / args.steps,
+                           "spmmm": (args.spmmm if args.spmmm >= 0 else "library default")
+                                    if w.model in ("agnn", "va") and w.k == 128 else None,
                            "setup_s": setup_s},
                 "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
                 "clocks": ck, "kernels": kernels, "per_rank": per_rank}

@@ -157,6 +157,13 @@ typedef struct {
                              1 k_out = 128 only (default), 2 every width          */
   int32_t l2_hot_mb;      /* L2 budget (MB) of the evict_last gathers, 0 disables
                              the hints; default 96 (performance only, see below)  */
+  int32_t spmmm;          /* AGNN/VA forward with k_in = k_out = 128: 1 fuses the
+                             aggregation and the projection into one SpMMM kernel
+                             (Table 2; X = Psi H goes to the
+                             tensor core through shared memory, not HBM), 0 runs
+                             the SpMM kernel and then the tcgen05 GEMM; default 0
+                             (measured).  Outputs agree up to fp32
+                             rounding order.                                      */
 } agnn_plan_options;
 
 typedef struct {

@@ -55,11 +55,12 @@ class PlanOptions(ctypes.Structure):
     """agnn_plan_options (include/agnn.h); a field < 0 (0 for chunk_edges) = default."""
     _fields_ = [("chunk_edges", ctypes.c_int32), ("short_edges", ctypes.c_int32),
                 ("short_bundles", ctypes.c_int32), ("gat_factored", ctypes.c_int32),
-                ("l2_hot_mb", ctypes.c_int32)]
+                ("l2_hot_mb", ctypes.c_int32), ("spmmm", ctypes.c_int32)]
 
     @classmethod
-    def make(cls, chunk_edges=0, short_edges=-1, short_bundles=-1, gat_factored=-1, l2_hot_mb=-1):
-        return cls(chunk_edges, short_edges, short_bundles, gat_factored, l2_hot_mb)
+    def make(cls, chunk_edges=0, short_edges=-1, short_bundles=-1, gat_factored=-1, l2_hot_mb=-1,
+             spmmm=-1):
+        return cls(chunk_edges, short_edges, short_bundles, gat_factored, l2_hot_mb, spmmm)
 
 
 class Dist(ctypes.Structure):

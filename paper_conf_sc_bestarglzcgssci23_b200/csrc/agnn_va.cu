@@ -480,6 +480,7 @@ SavedAv carve_saved(const Plan& p, const agnn_layer_desc& d, void* base, size_t*
 struct WsAv {
   float *pacc, *pl, *G, *M, *gemm, *WT, *dhp;
   float4* rec;
+  int* hcnt;  // SpMMM: completed chunks per heavy row
   void* saved_inf;
   bf16* M16;  // BF16 mode (reading B2): M~ [n x k_in] (replicated), replaces M
 };
@@ -500,6 +501,7 @@ WsAv carve_ws(const Plan& p, const agnn_layer_desc& d, void* base, size_t* total
   w.G = c.take<float>((size_t)p.n_local * d.k_out);
   w.gemm = c.take<float>(gemm_tn_ws_floats(d.k_in, d.k_out));
   w.WT = c.take<float>((size_t)d.k_in * d.k_out);
+  w.hcnt = c.take<int>(p.spmmm ? (size_t)p.n_heavy : 0);
   if (total) *total = c.off + 256;
   return w;
 }
@@ -564,6 +566,13 @@ agnn_status av_forward(const Plan& p, const agnn_layer_desc& d, const float* W, 
   }
   Items it = items_of(p);
   AvFwd A{Hf, b16 ? sv.H16 : nullptr, sv.nu, d.beta, fabsf(d.beta), sv.X, sv.l, w.pacc, w.pl};
+  if (p.spmmm && K_ == 128 && d.k_out == 128) {
+    // SpMMM (S8(f) f2): aggregation (heavy-row chunks and their merge included) and
+    // the projection by W in one kernel, X staying on chip
+    const Items ith = l2_hinted(it, p, (b16 ? 2 : 4) * (int64_t)K_ + (ag ? 4 : 0));
+    return av_fwd_spmmm(ith, ag, A, W, saved ? sv.Z : nullptr, H_out, w.hcnt, (int)d.act,
+                        saved != nullptr, s);
+  }
   if (K_ == 128 || K_ == 256) {
     // gathered per entry: an H_j row (+ nu_j)
     const Items ith = l2_hinted(it, p, (b16 ? 2 : 4) * (int64_t)K_ + (ag ? 4 : 0));

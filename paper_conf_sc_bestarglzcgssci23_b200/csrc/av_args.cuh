@@ -34,6 +34,12 @@ enum { AV_VA = 0, AV_AG = 1 };
 // (ROLE 0) only; AGNN_EUNSUPPORTED for other widths
 // (A.H16 != NULL: the BF16 storage variants, same arithmetic on the rounded rows)
 agnn_status av_fwd_batched(const Items& it, int k, bool agnn, const AvFwd& A, cudaStream_t s);
+// SpMMM, k_in = k_out = 128: X = Psi H and
+// Z = X W in one kernel (av_batched.cu), heavy-row chunks and their merge included;
+// Z (nullable) and H_out = sigma(Z) are stored by row; store_x: X and l are stored
+// too (training: the backward reads them).  hcnt: [n_heavy] ints of workspace.
+agnn_status av_fwd_spmmm(const Items& it, bool agnn, const AvFwd& A, const float* W, float* Z,
+                         float* H_out, int* hcnt, int act, bool store_x, cudaStream_t s);
 agnn_status av_bwd_batched(const Items& it, int k, bool agnn, const AvBwd& A, cudaStream_t s);
 
 }  // namespace agnn

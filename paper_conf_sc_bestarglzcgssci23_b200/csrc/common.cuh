@@ -280,6 +280,7 @@ struct Plan {
   int gat_factored = 1;               // 0 never, 1 k' = 128 only, 2 every width
   int bundle_mode = 1;                // short-row bundles: 0 never, 1 fp32, 2 fp32 + bf16
   int64_t l2_hot_mb = 96;             // evict_last budget; 0: no column classes
+  int spmmm = 0;                      // AGNN/VA k = 128 forward: fused SpMMM kernel
   int64_t max_chunks() const { return n_chunks > c_chunks ? n_chunks : c_chunks; }
   // distribution
   int rank = 0, world = 1;

@@ -321,6 +321,10 @@ agnn_status plan_options(Plan& p, const agnn_plan_options* o) {
     p.gat_factored = o->gat_factored;
   }
   if (o->l2_hot_mb >= 0) p.l2_hot_mb = o->l2_hot_mb;
+  if (o->spmmm >= 0) {
+    if (o->spmmm > 1) return fail(AGNN_EINVAL, "agnn_plan_options: spmmm > 1");
+    p.spmmm = o->spmmm;
+  }
   return AGNN_OK;
 }
 
