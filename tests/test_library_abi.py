@@ -26,6 +26,17 @@ def test_header_and_binding_agree():
     assert declared_symbols() == sorted(agnn.EXPORTS)
 
 
+def test_plan_options_layout_matches_header():
+    """agnn_plan_options (include/agnn.h) and the ctypes binding: same fields, order, types."""
+    src = open(os.path.join(ROOT, "include", "agnn.h")).read()
+    end = src.index("} agnn_plan_options;")
+    body = src[src.rindex("typedef struct {", 0, end):end]
+    body = re.sub(r"/\*.*?\*/", "", body, flags=re.S)
+    fields = re.findall(r"int32_t\s+(\w+);", body)
+    assert fields == [f for f, _ in agnn.PlanOptions._fields_]
+    assert all(t is ctypes.c_int32 for _, t in agnn.PlanOptions._fields_)
+
+
 def test_library_exports_every_declared_symbol():
     L = agnn.lib()
     for name in declared_symbols():
