@@ -436,10 +436,11 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
 // 128-column fp32 dW row per thread): three independent TMA -> split -> MMA chains
 // per SM overlap each other's latencies.  Measured at M = 2^24, K1 = N = 128: 32-row
 // chunks with one CTA / SM 7.36 ms, 16-row chunks with 2 / SM 5.90 ms, with 3 / SM
-// 4.84 ms (scratch/time_gemm.py).
+// 4.84 ms (scratch/time_gemm.py).  Draining every 4 chunks instead of 2 (64 rows,
+// 24 MMA accumulations; test_gpu_gemm.py bounds unchanged): C5 dW 5.1 -> 4.75 ms.
 constexpr int TN_ROWS = 16;   // input rows per chunk
 constexpr int TN_CTAS = 3;    // resident CTAs per SM
-constexpr int TN_GROUP = 2;   // chunks per TMEM drain (32 rows: 12 MMA accumulations)
+constexpr int TN_GROUP = 4;   // chunks per TMEM drain (64 rows: 24 MMA accumulations)
 constexpr int64_t kTnMaxSlabs = 2048;  // fp32 partials per call (summed in fp64)
 
 // MN-major tf32 operands use the 128B swizzle with 32-byte atomicity (the only MN-major
