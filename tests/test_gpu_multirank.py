@@ -36,9 +36,15 @@ CASES = {
     "agnn-k128-L2": gen.Workload("mr-agnn", "agnn", "rmat", 13, 1 << 13, 8 << 13, 128, 1, 2,
                                  act="elu"),
     "va-k64": gen.Workload("mr-va", "va", "kron", 13, 1 << 13, 8 << 13, 64, 1, 1, act="none"),
+    # the fused SpMMM forward (plan option spmmm) on the exchanged rows
+    "agnn-k128-L2-spmmm": gen.Workload("mr-agnn-sp", "agnn", "rmat", 13, 1 << 13, 8 << 13, 128,
+                                       1, 2, act="elu"),
     "cgnn-max": gen.Workload("mr-cg", "cgnn", "kron", 13, 1 << 13, 8 << 13, 64, 1, 1, act="elu",
                              agg="max"),
 }
+
+
+OPTS = {"agnn-k128-L2-spmmm": {"spmmm": 1}}
 
 
 def _free_port():
@@ -105,7 +111,8 @@ def _worker(rank, world, port, name):
     dist.init_process_group("gloo", rank=rank, world_size=world)
     torch.cuda.set_device(0)
     w = CASES[name]
-    st = runner.Stack(w, "cuda", rank=rank, world=world, nccl_uid=None)
+    st = runner.Stack(w, "cuda", rank=rank, world=world, nccl_uid=None,
+                      plan_options=OPTS.get(name))
     for _ in range(2):  # two steps: the second reuses every replica buffer
         st.step()
     torch.cuda.synchronize()
@@ -123,7 +130,7 @@ def _worker(rank, world, port, name):
     if rank == 0:
         _check_oracle(w, allout)
         _check_send_lists(w, allout)
-        ref = runner.Stack(w, "cuda")
+        ref = runner.Stack(w, "cuda", plan_options=OPTS.get(name))
         for _ in range(2):
             ref.step()
         torch.cuda.synchronize()

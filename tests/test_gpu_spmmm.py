@@ -90,6 +90,18 @@ def test_spmmm_inference_matches_training_forward(model):
     assert torch.equal(out_train, st.H[1])
 
 
+def test_spmmm_directed_pattern():
+    """A directed pattern (no AGNN_CSR_SYMMETRIC): the forward visits row i's stored
+    entries either way; the backward runs its row and column passes."""
+    from test_gpu_parity import _directed_graph
+    w = W("agnn", "kron", 13, 8, 128, act="elu")
+    rp, ci, g = _directed_graph(w)
+    H, Ws, As, R = w.host_inputs()
+    st = pu.gpu_step(w, graph=g, R=R, symmetric=False, plan_options=FUSED)
+    ref = pu.oracle_step(w, rp, ci, H, Ws, As, R)
+    pu.compare(w, st, ref)
+
+
 def test_spmmm_bf16_storage():
     """BF16 storage (reading B2): the gathered rows are the rounded H~; X stays fp32
     into the fused projection.  Same 1e-2 protocol as test_gpu_bf16.py."""
