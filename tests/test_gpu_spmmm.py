@@ -111,6 +111,27 @@ def test_spmmm_bf16_storage():
     pu.compare(w, st, ref, tol=pu.TOL_BF16)
 
 
+def test_spmmm_empty_rows():
+    """Rows without stored entries (reading A7): X_i = 0, so Z_i = 0 and H_out_i = sigma(0)."""
+    n = 70
+    rng = np.random.default_rng(5)
+    A = rng.random((n, n)) < 0.1
+    A = A | A.T
+    np.fill_diagonal(A, False)
+    A[7, :] = A[:, 7] = False
+    A[40, :] = A[:, 40] = False
+    rp = np.concatenate([[0], np.cumsum(A.sum(1))]).astype(np.int64)
+    ci = np.concatenate([np.nonzero(A[i])[0] for i in range(n)]).astype(np.int32)
+    for model in ("agnn", "va"):
+        w = gen.Workload("edge-sp", model, "er", 0, n, 0, 128, 1, 1, act="elu")
+        g = runner.Graph(n, torch.from_numpy(rp).cuda(), torch.from_numpy(ci).cuda(), len(ci))
+        st = pu.gpu_step(w, graph=g, plan_options=FUSED)
+        H, Ws, As, R = w.host_inputs()
+        pu.compare(w, st, pu.oracle_step(w, rp, ci, H, Ws, As, R))
+        for r in (7, 40):
+            assert torch.all(st.H[1][r] == 0) and torch.all(st.dH[0][r] == 0)
+
+
 def test_spmmm_option_validated():
     w = W("agnn", "er", 0, 0, 128, n=64, samples=256)
     src, dst, rp, ci = pu.host_graph(w)
