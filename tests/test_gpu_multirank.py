@@ -164,3 +164,10 @@ def test_peer_exchange_three_ranks_one_gpu(name):
     """Three ranks: uneven row blocks and two peers per rank in every exchange."""
     import torch.multiprocessing as mp
     mp.spawn(_worker, args=(3, _free_port(), name), nprocs=3, join=True)
+
+
+@pytest.mark.parametrize("name", ["gat-k128h4", "agnn-k128-L2-spmmm"])
+def test_peer_exchange_four_ranks_one_gpu(name):
+    """Four ranks: three peers per rank, per-row peer masks with several bits set."""
+    import torch.multiprocessing as mp
+    mp.spawn(_worker, args=(4, _free_port(), name), nprocs=4, join=True)
