@@ -275,8 +275,9 @@ def test_directed_heavy_chunks():
         pu.compare(w, st, pu.oracle_step(w, rp, ci, H, Ws, As, R))
 
 
-@pytest.mark.parametrize("k", [64, 128])
-def test_agnn_eps_branch(k):
+@pytest.mark.parametrize("k,opts", [(64, None), (128, None), (128, {"spmmm": 1})],
+                         ids=["k64", "k128", "k128-spmmm"])
+def test_agnn_eps_branch(k, opts):
     """Reading A8 on the GPU: zero rows and rows of norm < eps = 1e-12 take
     nu_i = eps (constant), with the gradient dHhat_j / eps of the oracle
     (pinned in test_oracle_pins.py::test_agnn_eps_branch)."""
@@ -290,7 +291,7 @@ def test_agnn_eps_branch(k):
     H = H.copy()
     H[zero] = 0.0
     H[tiny] *= np.float32(1e-14)
-    st = runner.Stack(w, "cuda", graph=g)
+    st = runner.Stack(w, "cuda", graph=g, plan_options=opts)
     st.H[0].copy_(torch.from_numpy(H))
     st.dH[1].copy_(torch.from_numpy(R))
     st.step()
