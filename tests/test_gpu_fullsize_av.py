@@ -1,6 +1,7 @@
 """Full-size parity of the AGNN / VA path at the bench configurations C3 (AGNN,
-R-MAT 2^20, k = 128, 3 layers) and C4 (VA, Kronecker 2^22, k = 256), in the
-launch configuration bench.py times, on outputs the oracle computes from exact
+R-MAT 2^20, k = 128, 3 layers) and C4 (VA, Kronecker 2^22, k = 256), and of C5 in
+the BF16 storage mode (the bench line's `bf16_storage`, reading B1, bar 1e-2), in
+the launch configuration bench.py times, on outputs the oracle computes from exact
 local sub-problems (the argument of test_gpu_fullsize.py):
 
   * forward: row i of layer 0 depends only on H of N(i) u {i}, so the oracle runs
@@ -16,6 +17,8 @@ local sub-problems (the argument of test_gpu_fullsize.py):
 """
 from __future__ import annotations
 
+import dataclasses
+
 import numpy as np
 import pytest
 
@@ -29,9 +32,12 @@ from paper_conf_sc_bestarglzcgssci23_b200 import gen, runner  # noqa: E402
 from test_gpu_fullsize import _hub_rows, _neighbours, _subproblem  # noqa: E402
 
 
-@pytest.fixture(scope="module", params=["C3", "C4"])
+@pytest.fixture(scope="module", params=["C3", "C4", "C5-bf16"])
 def stack(request):
-    w = gen.CONFIGS[request.param]
+    if request.param == "C5-bf16":
+        w = dataclasses.replace(gen.CONFIGS["C5"], prec="bf16")
+    else:
+        w = gen.CONFIGS[request.param]
     st = runner.Stack(w, "cuda")
     st.forward()
     torch.cuda.synchronize()
@@ -43,15 +49,25 @@ def stack(request):
 
 def _layer0_inputs(w, sources):
     H = gen.fill_rows(w.seed, gen.STREAM_H, np.asarray(sources, np.int64), w.k, 1.0)
-    wshape, _ = w.weight_shapes(0)
-    W0 = gen.fill(w.seed, gen.STREAM_W(0), wshape, gen.glorot_bound(w.k, w.k))
-    return H, W0
+    wshape, ashape = w.weight_shapes(0)
+    bound = gen.glorot_bound(w.k, w.k)
+    W0 = gen.fill(w.seed, gen.STREAM_W(0), wshape, bound)
+    a0 = gen.fill(w.seed, gen.STREAM_A(0), ashape, bound) if ashape else None
+    return H, W0, a0
 
 
-def _oracle_forward(w, srp, sci, H, W0):
-    f, _ = oracle.layer(w.model, srp, sci, np.asarray(H, np.float64), W0, None, 1, act=w.act,
-                        slope=w.slope, beta=w.beta, eps=w.eps, agg=w.agg)
+def _oracle_forward(w, srp, sci, H, W0, a0):
+    f, _ = oracle.layer(w.model, srp, sci, np.asarray(H, np.float64), W0, a0, w.heads, act=w.act,
+                        slope=w.slope, beta=w.beta, eps=w.eps, agg=w.agg, bf16=w.prec == "bf16")
     return f
+
+
+def _bars(w):
+    """FP32: 1e-5 normwise + per-row bounds; BF16 storage: 1e-2 and forward rows only
+    (pu.rowwise_keys: one-ulp bf16 decisions move single backward rows)."""
+    if w.prec == "bf16":
+        return dict(tol=pu.TOL_BF16, row_tol=pu.BF16_ROW_TOL), False
+    return dict(tol=pu.TOL_FP32), True
 
 
 def test_forward_sampled_rows(stack):
@@ -66,13 +82,14 @@ def test_forward_sampled_rows(stack):
     nbs = _neighbours(st, rp, rows)
     sources = np.union1d(np.unique(np.concatenate(nbs)), rows)
     srp, sci = _subproblem(rp, nbs, rows, sources)
-    H, W0 = _layer0_inputs(w, sources)
-    f = _oracle_forward(w, srp, sci, H, W0)
+    H, W0, a0 = _layer0_inputs(w, sources)
+    f = _oracle_forward(w, srp, sci, H, W0, a0)
     pos = np.searchsorted(sources, rows)
     got = st.H[1][torch.from_numpy(rows).cuda()].cpu().numpy()
     hub = np.isin(rows, hubs)
+    bars, _ = _bars(w)
     pu.compare_arrays({"Hout": (got, f["Hout"][pos]), "Hout_hubs": (got[hub], f["Hout"][pos][hub])},
-                      rowwise=["Hout", "Hout_hubs"])
+                      rowwise=["Hout", "Hout_hubs"], **bars)
 
 
 def test_backward_exact_on_row_support(stack):
@@ -95,8 +112,8 @@ def test_backward_exact_on_row_support(stack):
     nbs = _neighbours(st, rp, S)
     sources = np.union1d(np.unique(np.concatenate(nbs)), S)  # S u N(S)
     srp, sci = _subproblem(rp, nbs, S, sources)
-    H, W0 = _layer0_inputs(w, sources)
-    f = _oracle_forward(w, srp, sci, H, W0)
+    H, W0, a0 = _layer0_inputs(w, sources)
+    f = _oracle_forward(w, srp, sci, H, W0, a0)
     posS = np.searchsorted(sources, S)
     # ReLU kink (reading A6'): zero R where the oracle's Z is within 1e-5 rms of 0
     RS = gen.fill_rows(w.seed, gen.STREAM_R, S, w.k, 1.0).astype(np.float64)
@@ -105,10 +122,13 @@ def test_backward_exact_on_row_support(stack):
     R = np.zeros((len(sources), w.k))
     R[posS] = RS
     Hs = np.asarray(H, np.float64)
+    bf = w.prec == "bf16"
     if w.model == "agnn":
-        b = oracle.agnn_backward(srp, sci, Hs, W0, f, R, w.beta, w.eps, w.act)
+        b = oracle.agnn_backward(srp, sci, Hs, W0, f, R, w.beta, w.eps, w.act, bf16=bf)
+    elif w.model == "gat":
+        b = oracle.gat_backward(srp, sci, Hs, W0, a0, w.heads, f, R, w.slope, w.act, bf16=bf)
     else:
-        b = oracle.va_backward(srp, sci, Hs, W0, f, R, w.act)
+        b = oracle.va_backward(srp, sci, Hs, W0, f, R, w.act, bf16=bf)
     # the GPU backward of layer 0 (forward state of the bench's stack) with that R
     dH1 = torch.zeros_like(st.dH[1])
     dH1[torch.from_numpy(S).cuda()] = torch.from_numpy(RS.astype(np.float32)).cuda()
@@ -121,7 +141,10 @@ def test_backward_exact_on_row_support(stack):
     outside = torch.ones(w.n, dtype=torch.bool, device="cuda")
     outside[src_t] = False
     nonzero_outside = int((dH[outside] != 0).any(dim=1).sum())
-    pu.compare_arrays({"dH_support": (got_dH, b["dH"]), "dH_S": (got_dH[posS], b["dH"][posS]),
-                       "dW": (st.dW[0].cpu().numpy(), b["dW"])},
-                      rowwise=["dH_support", "dH_S", "dW"])
+    pairs = {"dH_support": (got_dH, b["dH"]), "dH_S": (got_dH[posS], b["dH"][posS]),
+             "dW": (st.dW[0].cpu().numpy(), b["dW"])}
+    if w.model == "gat":
+        pairs["da"] = (st.da[0].cpu().numpy(), b["da"])
+    bars, rowwise = _bars(w)
+    pu.compare_arrays(pairs, rowwise=["dH_support", "dH_S", "dW"] if rowwise else [], **bars)
     assert nonzero_outside == 0, nonzero_outside
