@@ -429,6 +429,57 @@ def roofline(args, w, st, prof, world):
     return r
 
 
+# dense TF32 : BF16 tensor throughput (B200_PROFILING.md nominal dense peaks: 1.1 and
+# 2.25 PFLOP/s); the TF32 peak is the measured BF16 peak times this ratio
+TF32_PER_BF16 = 1.1 / 2.25
+
+
+def gemm_flops_bytes(w, n, spmmm=False):
+    """Algorithmic FLOPs (3xTF32: every MMA of the three-term split counted, S§8(d))
+    and bytes of the tcgen05 GEMMs of one fwd+bwd step, by profile name.
+    GAT: gemm_tc = projection [P|s|t] = H W_ext (N = k' + 2h) + dH = dP W^T;
+    gemm_tn = dW = H^T dP.  AGNN / VA: gemm_tc = Z = X W (unless the fused SpMMM
+    kernel does it) + M = G W^T; gemm_tn = dW = X^T G.  Bytes: operands read once,
+    outputs written once (P~ / M~ two bytes in BF16 storage)."""
+    k, L, fs = w.k, w.layers, (2 if w.prec == "bf16" else 4)
+    mm = lambda K, N: 3 * 2 * n * K * N  # noqa: E731
+    if w.model == "gat":
+        tc_f = mm(k, k + 2 * w.heads) + mm(k, k)
+        tc_b = n * k * 4 + n * (k * fs + 2 * w.heads * 4) + n * k * 4 + n * k * 4
+    else:
+        tc_f = mm(k, k) * (1 if spmmm else 2)
+        tc_b = n * k * fs + n * k * 4 + (0 if spmmm else n * k * 4 + 2 * n * k * 4)
+    tn_f, tn_b = mm(k, k), 2 * n * k * 4
+    return {"gemm_tc_kernel": (tc_f * L, tc_b * L), "gemm_tn_kernel": (tn_f * L, tn_b * L)}
+
+
+def gemm_roofline(args, w, st, prof):
+    """The tcgen05 GEMMs against the tensor-pipe peak (TF32) and the HBM peak
+    (north_star item 3; S§8(d) "report the GEMMs against HBM (primary) and against
+    the tensor pipe (secondary)"), from the live per-kernel event profile."""
+    peaks = measured_peaks()
+    bf16 = peaks.get("bf16_tflops")
+    tpeak = bf16 * TF32_PER_BF16 if bf16 else 1100.0
+    hbm = peaks.get("hbm_gbs") or 6650.0
+    out = {}
+    for name, (fl, by) in gemm_flops_bytes(w, st.n_local, "av_spmmm_kernel" in prof).items():
+        if name not in prof:
+            continue
+        ms = prof[name][1] / args.steps
+        tf = fl / (ms / 1e3) / 1e12
+        gb = by / (ms / 1e3) / 1e9
+        out[name] = {"ms_per_step": ms, "tflops": tf, "tensor_peak_tflops": tpeak,
+                     "tensor_frac": tf / tpeak, "hbm_gbs": gb, "hbm_frac": gb / hbm,
+                     "flops_per_step": fl, "bytes_per_step": by}
+    if not out:
+        return None
+    out["basis"] = ("3xTF32 FLOPs (three MMAs per product) and operand/output bytes per "
+                    "step / live CUDA-event time; tensor peak = MEASURED_PEAKS bf16_tflops "
+                    "x 1.1/2.25 (TF32:BF16 dense, B200_PROFILING.md)" if bf16 else
+                    "fallback peaks (B200_PROFILING.md)")
+    return out
+
+
 def comm_split(prof, steps):
     """ms per step of the exchange (peer barriers, pushes, reductions or NCCL) and of
     everything else, from the live per-kernel profile of this rank."""
@@ -758,7 +809,8 @@ def run_ours(args):
                            "spmmm": (args.spmmm if args.spmmm >= 0 else "library default")
                                     if w.model in ("agnn", "va") and w.k == 128 else None,
                            "setup_s": setup_s},
-                "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
+                "roofline": roof, "gemm_roofline": gemm_roofline(args, w, st, prof),
+                "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
                 "clocks": ck, "kernels": kernels, "per_rank": per_rank}
         if same_gpu and world > 1:
             line["note"] = ("AGNN_BENCH_SAME_GPU: every rank ran on cuda:0 (functional test of the "

@@ -108,3 +108,21 @@ def test_stale_ncu_capture_is_refused(tmp_path, monkeypatch):
     assert per is None and "stale" in why
     per, why = b.ncu_traffic("C4")
     assert per is None
+
+
+def test_gemm_flops_and_bytes():
+    """The GEMM roofline's work per step: 3xTF32 counts three MMAs per product
+    (S§8(d)); C5 projection N = k' + 2h = 136, dH and dW 128 x 128; AGNN/VA two
+    k x k products in gemm_tc (one when the SpMMM kernel does Z = X W)."""
+    b = _bench()
+    n = 1000
+    g = b.gemm_flops_bytes(gen.CONFIGS["C5"], n)
+    assert g["gemm_tc_kernel"][0] == 6 * n * 128 * 136 + 6 * n * 128 * 128
+    assert g["gemm_tn_kernel"] == (6 * n * 128 * 128, 2 * n * 128 * 4)
+    # H read, P|s|t written, dP read, dH written
+    assert g["gemm_tc_kernel"][1] == n * 128 * 4 + n * (128 * 4 + 8 * 4) + 2 * n * 128 * 4
+    c3 = gen.CONFIGS["C3"]
+    a = b.gemm_flops_bytes(c3, n)
+    f = b.gemm_flops_bytes(c3, n, spmmm=True)
+    assert a["gemm_tc_kernel"][0] == 2 * f["gemm_tc_kernel"][0] == 3 * 2 * 6 * n * 128 * 128
+    assert b.TF32_PER_BF16 == pytest.approx(1.1 / 2.25)
