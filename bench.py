@@ -657,6 +657,7 @@ def run_ours(args):
 
     # ---- roofline of the dominant kernel ----------------------------------------
     roof = roofline(args, w, st, prof, world)
+    groof = gemm_roofline(args, w, st, prof)
     kernels = {k: {"launches": v[0], "ms_per_step": v[1] / args.steps} for k, v in prof.items()}
     split = comm_split(prof, args.steps)
     per_rank = [split]
@@ -809,7 +810,7 @@ def run_ours(args):
                            "spmmm": (args.spmmm if args.spmmm >= 0 else "library default")
                                     if w.model in ("agnn", "va") and w.k == 128 else None,
                            "setup_s": setup_s},
-                "roofline": roof, "gemm_roofline": gemm_roofline(args, w, st, prof),
+                "roofline": roof, "gemm_roofline": groof,
                 "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
                 "clocks": ck, "kernels": kernels, "per_rank": per_rank}
         if same_gpu and world > 1:
