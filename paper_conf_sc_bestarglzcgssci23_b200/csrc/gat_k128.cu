@@ -11,6 +11,9 @@
 //   warp max; running max / rescale once per batch; p_ij = 2^(e_ij - m).
 //   Then the warp walks the batch: lane q owns columns 4q..4q+3 of P_j and
 //   accumulates p_ij(head(q)) P_j.  Per edge: one 16-byte gather and 4 FMAs.
+//   BF16 storage (256-byte rows): the half-warps take the even / odd entries, two
+//   rows per 16-byte-per-lane load instruction (gat_fwd_k128_pair_kernel, and
+//   gat_bwd_k128f_pair_kernel for the factored backward).
 // Factored backward (default, gat_args.cuh): the forward also accumulates Q_j, and
 //   the backward row kernel (gat_bwd_k128f_kernel) keeps only the column role —
 //   32-entry windows, lane-parallel alpha_ij / c'_ij from the gathered records,
@@ -261,6 +264,216 @@ gat_fwd_k128_kernel(Items it, const TP* __restrict__ P, const float* __restrict_
       if constexpr (QF) {
         const float r = lh > 0.f ? ch / lh : 0.f;
         st4(o.Q + row * K + cq, mul4(inv, fma4(-r, acc, accu)));
+      }
+      if (o.m && lane == 0) {
+#pragma unroll
+        for (int h = 0; h < NH; ++h) {
+          o.m[row * NH + h] = l[h] > 0.f ? mr[h] : 0.f;
+          o.l[row * NH + h] = l[h];
+        }
+      }
+    }
+  }
+}
+
+// BF16 storage (reading B1): the same forward with TWO gathered rows per warp load
+// instruction.  A bf16 row of k' = 128 is 256 bytes = 16 lanes x 16 bytes, so the
+// half-warps take the even and the odd entries of a batch (lane L: columns
+// 8 (L % 16) .. + 7 of entry 2p + L / 16); each half accumulates its entries, and
+// the halves are added (one xor-16 shuffle per column) at the end of the item.
+// Scores, softmax statistics and outputs are those of gat_fwd_k128_kernel; only
+// the summation order of the aggregation differs (even / odd entries, then both).
+__device__ __forceinline__ void bf8_to_f8(uint4 u, float (&x)[8]) {
+  x[0] = __uint_as_float(u.x << 16);
+  x[1] = __uint_as_float(u.x & 0xffff0000u);
+  x[2] = __uint_as_float(u.y << 16);
+  x[3] = __uint_as_float(u.y & 0xffff0000u);
+  x[4] = __uint_as_float(u.z << 16);
+  x[5] = __uint_as_float(u.z & 0xffff0000u);
+  x[6] = __uint_as_float(u.w << 16);
+  x[7] = __uint_as_float(u.w & 0xffff0000u);
+}
+
+template <int NH, int UP, int MINB, bool QF>
+__global__ void __launch_bounds__(256, MINB)
+gat_fwd_k128_pair_kernel(Items it, const bf16* __restrict__ P, const float* __restrict__ st,
+                         float slope, int act, GatFwdOut o) {
+  constexpr int D = K / NH, LPH = D / 8;  // lanes of a half per head (8 columns each)
+  static_assert(D % 8 == 0, "8 columns of one head per lane");
+  __shared__ float sPw[QF ? 1 : 8][NH][33];
+  __shared__ float2 sP2[QF ? 8 : 1][NH][33];
+  __shared__ int sJ[8][32];
+  const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  const int half = lane >> 4, q16 = lane & 15;
+  const int hv = q16 / LPH, c8 = q16 * 8;
+  const int64_t nitems = it.n_chunks + it.n_light;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const Gath ga(it);
+  const bf16* Pl = P + c8;
+  for (int64_t w = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; w < nitems; w += nw) {
+    int64_t row, beg, end, slot;
+    item_of(it, w, row, beg, end, slot);
+    const int64_t grow = it.row_begin + row;
+    float si[NH], mr[NH], lp[NH], lc[NH];
+    load_n<NH>(st + grow * (2 * NH), si);
+#pragma unroll
+    for (int h = 0; h < NH; ++h) {
+      mr[h] = -INFINITY;
+      lp[h] = 0.f;
+      lc[h] = 0.f;
+    }
+    float acc[8], accu[8];
+#pragma unroll
+    for (int c = 0; c < 8; ++c) acc[c] = accu[c] = 0.f;
+    int jpre = beg + lane < end ? __ldg(it.col + beg + lane) : 0;
+    for (int64_t b0 = beg; b0 < end; b0 += 32) {
+      const int cnt = (int)(end - b0 < 32 ? end - b0 : 32);
+      const bool valid = lane < cnt;
+      const int j = jpre;
+      jpre = b0 + 32 + lane < end ? __ldg(it.col + b0 + 32 + lane) : 0;
+      sJ[wib][lane] = j;
+      __syncwarp();
+      auto ld = [&](int e) -> uint4 {
+        if (e >= cnt) return make_uint4(0u, 0u, 0u, 0u);
+        const int c = sJ[wib][e];
+        return ldg16_pol(Pl + ga.row(c) * K, ga.policy(c));
+      };
+      // the first UP pairs in flight while the scores are computed
+      uint4 pv[UP];
+#pragma unroll
+      for (int u = 0; u < UP; ++u) pv[u] = ld(2 * u + half);
+      float tj[NH];
+      load_n<NH>(st + ga.row(j) * (2 * NH) + NH, tj, ga.policy(j));
+      float sch = 1.f;
+#pragma unroll
+      for (int h = 0; h < NH; ++h) {
+        const float pre = si[h] + tj[h];
+        const float e = valid ? fmaxf(pre, slope * pre) : -INFINITY;
+        float bm = e;
+#pragma unroll
+        for (int off = 16; off > 0; off >>= 1) bm = fmaxf(bm, __shfl_xor_sync(FULL, bm, off));
+        const float mn = fmaxf(mr[h], bm);
+        const float sc = ex2(mr[h] - mn);
+        lp[h] = __fmul_rn(lp[h], sc);
+        if (h == hv) sch = sc;
+        mr[h] = mn;
+        const float p = valid ? ex2(e - mn) : 0.f;
+        lp[h] = __fadd_rn(lp[h], p);
+        if constexpr (QF) {
+          const float pc = pre > 0.f ? p : p * slope;
+          lc[h] = __fadd_rn(__fmul_rn(lc[h], sc), pc);
+          sP2[wib][h][lane] = make_float2(p, pc);
+        } else {
+          sPw[wib][h][lane] = p;
+        }
+      }
+#pragma unroll
+      for (int c = 0; c < 8; ++c) {
+        acc[c] *= sch;
+        if constexpr (QF) accu[c] *= sch;
+      }
+      __syncwarp();
+      auto axpy = [&](int e, const uint4& r) {
+        float x[8];
+        bf8_to_f8(r, x);
+        if constexpr (QF) {
+          const float2 pw = sP2[wib][hv][e];
+#pragma unroll
+          for (int c = 0; c < 8; ++c) {
+            acc[c] = fmaf(pw.x, x[c], acc[c]);
+            accu[c] = fmaf(pw.y, x[c], accu[c]);
+          }
+        } else {
+          const float pw = sPw[wib][hv][e];
+#pragma unroll
+          for (int c = 0; c < 8; ++c) acc[c] = fmaf(pw, x[c], acc[c]);
+        }
+      };
+      if (cnt == 32) {
+        // 16 pairs: groups of UP pairs, the next group in flight during this one
+        constexpr int NG = 16 / UP;
+        uint4 qa[UP], qb[UP];
+#pragma unroll
+        for (int u = 0; u < UP; ++u) qa[u] = pv[u];
+#pragma unroll
+        for (int g = 0; g < NG; g += 2) {
+#pragma unroll
+          for (int u = 0; u < UP; ++u) qb[u] = ld(2 * (UP * (g + 1) + u) + half);
+#pragma unroll
+          for (int u = 0; u < UP; ++u) axpy(2 * (UP * g + u) + half, qa[u]);
+          if (g + 2 < NG) {
+#pragma unroll
+            for (int u = 0; u < UP; ++u) qa[u] = ld(2 * (UP * (g + 2) + u) + half);
+          }
+#pragma unroll
+          for (int u = 0; u < UP; ++u) axpy(2 * (UP * (g + 1) + u) + half, qb[u]);
+        }
+      } else {
+        const int npair = (cnt + 1) >> 1;
+        for (int k0 = 0; k0 < npair; k0 += UP) {
+          if (k0 > 0) {
+#pragma unroll
+            for (int u = 0; u < UP; ++u) pv[u] = ld(2 * (k0 + u) + half);
+          }
+#pragma unroll
+          for (int u = 0; u < UP; ++u) {
+            const int e = 2 * (k0 + u) + half;
+            if (e < cnt) axpy(e, pv[u]);
+          }
+        }
+      }
+      __syncwarp();
+    }
+    // the two halves' partial sums (even / odd entries)
+#pragma unroll
+    for (int c = 0; c < 8; ++c) {
+      acc[c] += __shfl_xor_sync(FULL, acc[c], 16);
+      if constexpr (QF) accu[c] += __shfl_xor_sync(FULL, accu[c], 16);
+    }
+    float l[NH], cs[NH];
+#pragma unroll
+    for (int h = 0; h < NH; ++h) {
+      float x = lp[h], y = lc[h];
+#pragma unroll
+      for (int off = 16; off > 0; off >>= 1) {
+        x += __shfl_xor_sync(FULL, x, off);
+        if constexpr (QF) y += __shfl_xor_sync(FULL, y, off);
+      }
+      l[h] = x;
+      cs[h] = y;
+    }
+    float lh = l[0], ch = cs[0];
+#pragma unroll
+    for (int h = 1; h < NH; ++h)
+      if (h == hv) {
+        lh = l[h];
+        ch = cs[h];
+      }
+    // lane L stores columns c8 + 4 (L / 16) .. + 3
+    const int co = c8 + 4 * half;
+    const float4 a4 = half ? make_float4(acc[4], acc[5], acc[6], acc[7])
+                           : make_float4(acc[0], acc[1], acc[2], acc[3]);
+    const float4 u4 = half ? make_float4(accu[4], accu[5], accu[6], accu[7])
+                           : make_float4(accu[0], accu[1], accu[2], accu[3]);
+    if (slot >= 0) {
+      st4(o.pacc + slot * K + co, a4);
+      if constexpr (QF) st4(o.pu + slot * K + co, u4);
+      if (lane == 0) {
+#pragma unroll
+        for (int h = 0; h < NH; ++h) {
+          o.pm[slot * NH + h] = mr[h];
+          o.pl[slot * NH + h] = l[h];
+          if constexpr (QF) o.pc[slot * NH + h] = cs[h];
+        }
+      }
+    } else {
+      const float inv = lh > 0.f ? 1.f / lh : 0.f;
+      const float4 z = mul4(inv, a4);
+      if (o.Z) st4(o.Z + row * K + co, z);
+      st4(o.Hout + row * K + co, act_fwd4(act, z));
+      if constexpr (QF) {
+        const float r = lh > 0.f ? ch / lh : 0.f;
+        st4(o.Q + row * K + co, mul4(inv, fma4(-r, a4, u4)));
       }
       if (o.m && lane == 0) {
 #pragma unroll
@@ -563,6 +776,159 @@ gat_bwd_k128f_kernel(Items it, GatBwdArgs A) {
   st4(A.da_part + gw * 2 * K + K + cq, da2);
 }
 
+// BF16 storage: the factored backward with two gathered G rows per warp load
+// instruction (the pairing of gat_fwd_k128_pair_kernel: half-warps take the even /
+// odd entries, 8 columns per lane, halves added at the end of the item).  Lane L
+// owns output columns co = 8 (L % 16) + 4 (L / 16) .. + 3 for dP, the chunk partials
+// and its da partial.
+template <int NH, int UP, int MINB>
+__global__ void __launch_bounds__(256, MINB)
+gat_bwd_k128f_pair_kernel(Items it, GatBwdArgs A) {
+  constexpr int D = K / NH, LPH = D / 8;
+  static_assert(D % 8 == 0, "8 columns of one head per lane");
+  __shared__ float2 sAC[8][NH][33];  // {alpha_ij, c'_ij}
+  __shared__ int sJ[8][32];
+  const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  const int half = lane >> 4, q16 = lane & 15;
+  const int hv = q16 / LPH, c8 = q16 * 8, co = c8 + 4 * half;
+  const int64_t nitems = it.n_chunks + it.n_light;
+  const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+  const bf16* Gl = A.G16 + c8;
+  const float slope = A.slope;
+  const Gath ga(it);
+  using SL = Slice<bf16>;
+  float4 da1 = f4(0.f), da2 = f4(0.f);
+  for (int64_t w = gw; w < nitems; w += nw) {
+    int64_t row, beg, end, slot;
+    item_of(it, w, row, beg, end, slot);
+    const int64_t grow = it.row_begin + row;
+    float tj[NH], sd[NH];
+    load_n<NH>(A.st + grow * (2 * NH) + NH, tj);
+#pragma unroll
+    for (int h = 0; h < NH; ++h) sd[h] = 0.f;
+    float acc[8], accv[8];
+#pragma unroll
+    for (int c = 0; c < 8; ++c) acc[c] = accv[c] = 0.f;
+    int jpre = beg + lane < end ? __ldg(it.col + beg + lane) : 0;
+    for (int64_t b0 = beg; b0 < end; b0 += 32) {
+      const int cnt = (int)(end - b0 < 32 ? end - b0 : 32);
+      const bool valid = lane < cnt;
+      const int j = jpre;
+      jpre = b0 + 32 + lane < end ? __ldg(it.col + b0 + 32 + lane) : 0;
+      sJ[wib][lane] = j;
+      __syncwarp();
+      auto ld = [&](int e) -> uint4 {
+        if (e >= cnt) return make_uint4(0u, 0u, 0u, 0u);
+        const int c = sJ[wib][e];
+        return ldg16_pol(Gl + ga.row(c) * K, ga.policy(c));
+      };
+      uint4 qa[UP], qb[UP];
+      // the first group of G row pairs is in flight while the weights are computed
+#pragma unroll
+      for (int u = 0; u < UP; ++u) qa[u] = ld(2 * u + half);
+      {
+        const int64_t ir = ga.row(j);
+        const uint64_t pol = ga.policy(j);
+#pragma unroll
+        for (int h = 0; h < NH; ++h) {
+          const float4 r = valid ? ldg4_pol(reinterpret_cast<const float*>(A.rec + ir * NH + h), pol)
+                                 : f4(0.f);  // {s_i, m_i, 1/l_i, delta_i}
+          const float pre = r.x + tj[h];
+          const float e = fmaxf(pre, slope * pre);
+          const float al = valid ? ex2(e - r.y) * r.z : 0.f;
+          const float cc = pre > 0.f ? al : al * slope;
+          sd[h] = fmaf(cc, r.w, sd[h]);
+          sAC[wib][h][lane] = make_float2(al, cc);
+        }
+      }
+      __syncwarp();
+      auto axpy = [&](int e, const uint4& r) {
+        float x[8];
+        bf8_to_f8(r, x);
+        const float2 ac = sAC[wib][hv][e];
+#pragma unroll
+        for (int c = 0; c < 8; ++c) {
+          acc[c] = fmaf(ac.x, x[c], acc[c]);
+          accv[c] = fmaf(ac.y, x[c], accv[c]);
+        }
+      };
+      if (cnt == 32) {
+        constexpr int NG = 16 / UP;
+#pragma unroll
+        for (int g = 0; g < NG; g += 2) {
+#pragma unroll
+          for (int u = 0; u < UP; ++u) qb[u] = ld(2 * (UP * (g + 1) + u) + half);
+#pragma unroll
+          for (int u = 0; u < UP; ++u) axpy(2 * (UP * g + u) + half, qa[u]);
+          if (g + 2 < NG) {
+#pragma unroll
+            for (int u = 0; u < UP; ++u) qa[u] = ld(2 * (UP * (g + 2) + u) + half);
+          }
+#pragma unroll
+          for (int u = 0; u < UP; ++u) axpy(2 * (UP * (g + 1) + u) + half, qb[u]);
+        }
+      } else {
+        const int npair = (cnt + 1) >> 1;
+        for (int k0 = 0; k0 < npair; k0 += UP) {
+          if (k0 > 0) {
+#pragma unroll
+            for (int u = 0; u < UP; ++u) qa[u] = ld(2 * (k0 + u) + half);
+          }
+#pragma unroll
+          for (int u = 0; u < UP; ++u) {
+            const int e = 2 * (k0 + u) + half;
+            if (e < cnt) axpy(e, qa[u]);
+          }
+        }
+      }
+      __syncwarp();
+    }
+#pragma unroll
+    for (int c = 0; c < 8; ++c) {
+      acc[c] += __shfl_xor_sync(FULL, acc[c], 16);
+      accv[c] += __shfl_xor_sync(FULL, accv[c], 16);
+    }
+    const float4 a4 = half ? make_float4(acc[4], acc[5], acc[6], acc[7])
+                           : make_float4(acc[0], acc[1], acc[2], acc[3]);
+    const float4 v4 = half ? make_float4(accv[4], accv[5], accv[6], accv[7])
+                           : make_float4(accv[0], accv[1], accv[2], accv[3]);
+    // per row: dt_j = P_j . v_j - sum_i c'_ij delta_i (head hv: lanes 4hv.. of both halves)
+    const float4 Pj = SL::f(SL::load(A.P16 + grow * K + co));
+    float x = dot4(Pj, v4);
+#pragma unroll
+    for (int o = 1; o < LPH; o <<= 1) x += __shfl_xor_sync(FULL, x, o);
+    x += __shfl_xor_sync(FULL, x, 16);
+    float sdh = 0.f;
+#pragma unroll
+    for (int h = 0; h < NH; ++h) {
+      float y = sd[h];
+#pragma unroll
+      for (int off = 16; off > 0; off >>= 1) y += __shfl_xor_sync(FULL, y, off);
+      if (h == hv) sdh = y;
+    }
+    const float dt = x - sdh;
+    if (slot >= 0) {
+      st4(A.pacc + slot * K + co, a4);
+      if (half == 0 && (q16 % LPH) == 0) {
+        A.pdt[slot * NH + hv] = dt;
+        A.pds[slot * NH + hv] = it.chunk_idx[slot] == 0 ? A.ds_row[row * NH + hv] : 0.f;
+      }
+    } else {
+      const float ds = A.ds_row[row * NH + hv];
+      const float4 a1v = ldg4(A.a + hv * 2 * D + co % D);
+      const float4 a2v = ldg4(A.a + hv * 2 * D + D + co % D);
+      float4 dp = fma4(ds, a1v, a4);
+      dp = fma4(dt, a2v, dp);
+      st4(A.dP + row * K + co, dp);
+      da1 = fma4(ds, Pj, da1);
+      da2 = fma4(dt, Pj, da2);
+    }
+  }
+  st4(A.da_part + gw * 2 * K + co, da1);
+  st4(A.da_part + gw * 2 * K + K + co, da2);
+}
+
 template <typename F>
 int grid_for(F* f) {
   return persistent_blocks(reinterpret_cast<const void*>(f));
@@ -618,8 +984,10 @@ agnn_status gat_fwd_k128_bf16(const Items& it_all, int heads, const bf16* P, con
   const Items it = long_items(it_all);
   if (it.n_chunks + it.n_light == 0) return AGNN_OK;
   AGNN_K128_DISPATCH(heads, ({
-    auto* kern = o.Q ? gat_fwd_k128_kernel<bf16, NH, 8, 3, true>
-                     : gat_fwd_k128_kernel<bf16, NH, 8, 3, false>;
+    // two rows per load instruction, 3 blocks / SM (measured C5 bf16: 53.3 -> 47.2 ms
+    // against gat_fwd_k128_kernel<bf16> with 8-row groups)
+    auto* kern = o.Q ? gat_fwd_k128_pair_kernel<NH, 4, 3, true>
+                     : gat_fwd_k128_pair_kernel<NH, 4, 3, false>;
     kern<<<grid_for(kern), 256, 0, s>>>(it, P, st, slope, act, o);
     AGNN_LAUNCH_CHECK("gat_fwd_kernel");
   }));
@@ -656,9 +1024,10 @@ agnn_status gat_bwd_k128f(const Items& it_all, int heads, const GatBwdArgs& A, i
   *warps = 0;
   const Items it = long_items(it_all);
   AGNN_K128_DISPATCH(heads, ({
-    // fp32: 2 blocks / SM; bf16: 3 blocks / SM (measured C5, round 1: fp32 73.5 -> 69.2 ms
-    // against 3 blocks; bf16 59.2 vs 64.7 ms against 2)
-    auto* kern = A.P16 ? (void (*)(Items, GatBwdArgs))gat_bwd_k128f_kernel<bf16, NH, 3>
+    // fp32: 2 blocks / SM (measured C5, round 1: 73.5 -> 69.2 ms against 3 blocks);
+    // bf16: two G rows per load instruction, 2 blocks / SM (C5: 58.6 -> 51.8 ms against
+    // gat_bwd_k128f_kernel<bf16> at 3 blocks; the pair kernel at 3 blocks spills, 55.3)
+    auto* kern = A.P16 ? (void (*)(Items, GatBwdArgs))gat_bwd_k128f_pair_kernel<NH, 4, 2>
                        : (void (*)(Items, GatBwdArgs))gat_bwd_k128f_kernel<float, NH, 2>;
     const int grid = grid_for(kern);
     kern<<<grid, 256, 0, s>>>(it, A);
