@@ -27,6 +27,8 @@ def _bench():
 ALIAS = {"gat_bwd_k128_kernel": "gat_bwd_kernel", "gat_bwd_k128f_kernel": "gat_bwd_kernel",
          "gat_bwd_short_f_kernel": "gat_bwd_short_kernel",
          "gat_bwd_bundle_kernel": "gat_bwd_short_kernel", "gat_fwd_bundle_kernel": "gat_fwd_short_kernel", "gat_fwd_k128_kernel": "gat_fwd_kernel",
+         "gat_fwd_k128_pair_kernel": "gat_fwd_kernel", "gat_bwd_k128f_pair_kernel": "gat_bwd_kernel",
+         "av_spmmm_kernel": "av_spmmm_kernel",
                   "av_bwd_k128_kernel": "av_bwd_kernel", "av_fwd_k128_kernel": "av_fwd_kernel",
          "av_bwd_batched_kernel": "av_bwd_kernel", "av_fwd_batched_kernel": "av_fwd_kernel",
          "gemm_tn_tc_kernel": "gemm_tn_kernel", "tn_sum_kernel": "sum_splits_kernel",
